@@ -1,0 +1,246 @@
+/*
+ * pl.h — C-ABI of the B200 enforced-waiting streaming-pipeline executor.
+ *
+ * Implements the data-parallel hot path of Plano & Buhler, "Enabling Real-Time
+ * Irregular Data-Flow Pipelines on SIMD Devices" (SRMPDS '21; PAPER.md):
+ *   - a linear pipeline of N nodes with per-edge queues, average gains g_i and a
+ *     stream of items arriving every tau0 = 1/rho0 time units     (§2.1)
+ *   - each node fires a SIMD vector of up to v items taking a fixed service time t_i
+ *                                                                  (§2.2)
+ *   - a per-item deadline D and the active-fraction objective      (§2.3)
+ *   - enforced waiting: node i waits w_i after every firing        (§4)
+ *   - the monolithic block-of-M baseline                           (§5)
+ *   - the optimisation problems of Fig. 1 (L139–L151) and Fig. 2 (L165–L180)
+ * plus the north_star's threshold/deadline-slack firing rule (DESIGN.md R-THRESH).
+ *
+ * Every call is synchronous on the host unless stated; no C++ exception crosses
+ * this boundary.  Every function returns PL_OK (0) or a negative pl_status and, on
+ * failure, sets a thread-local message readable with pl_last_error().
+ *
+ * Ownership: every array in pl_config / pl_workload is COPIED at create; the
+ * caller may free it afterwards.  The pipeline handle owns all device memory it
+ * allocates (cudaMalloc on cfg->device) and frees it in pl_pipeline_destroy.
+ * Result buffers are caller-allocated; pass buf == NULL to query the count.
+ *
+ * Time: all times are int64 "units".  With PL_CLOCK_LOGICAL the executor runs a
+ * conservative parallel discrete-event schedule as fast as the GPU allows; with
+ * PL_CLOCK_GLOBALTIMER one unit is cfg->ns_per_unit nanoseconds of %globaltimer
+ * (32 ns resolution on B200, measured) and firings are paced in real time.
+ */
+#ifndef PL_H
+#define PL_H
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define PL_MAX_STAGES 8
+#define PL_MAX_U 16            /* cap on outputs per input of any stage (u = 16) */
+
+typedef int32_t pl_status;
+#define PL_OK           0
+#define PL_EINVAL      -1      /* bad argument / unsupported configuration          */
+#define PL_ENOMEM      -2      /* device or pinned-host allocation failed           */
+#define PL_EDEVICE     -3      /* CUDA error (launch, copy, device fault)           */
+#define PL_EINFEASIBLE -4      /* solver: Fig. 1 / Fig. 2 has no feasible point     */
+#define PL_ESTATE      -5      /* call out of order (e.g. push after drain)         */
+#define PL_EAGAIN      -6      /* (reserved) non-blocking push would block          */
+#define PL_EOVERFLOW   -7      /* a queue or output buffer overflowed during a run  */
+
+/* Stage kinds.  DNA stages follow classic BLAST [1] (§6.1; readings
+ * R-S0..R-S3 in DESIGN.md); random-gain stages follow PAPER.md L210.            */
+enum pl_stage_kind {
+  PL_BERNOULLI = 0,        /* 1 output with prob. param (=g), else 0; hash-driven    */
+  PL_FIXED_GAIN = 1,       /* exactly (int)param outputs (<= max_out)               */
+  PL_POISSON_CAPPED = 2,   /* min(Poisson(param), max_out) outputs (L210, u=max_out) */
+  PL_SEED_LOOKUP = 3,      /* S0: keep DB position p iff its k-mer occurs in query   */
+  PL_HIT_ENUM = 4,         /* S1: p -> (p,q_j), j < min(count, max_out)             */
+  PL_UNGAPPED_WINDOW = 5,  /* S2: keep (p,q) iff k+best_left(W)+best_right(W) >= T2  */
+  PL_UNGAPPED_XDROP = 6,   /* S3: X-drop ungapped extension, emit pl_match if >= T3  */
+  PL_KEEP_EVERY = 7        /* deterministic filter: keep iff root % (int)param == 0  */
+};
+
+enum pl_policy {
+  PL_FIXED_WAIT = 0,       /* paper §4: fire every t_i + w_i, even when empty (L97)  */
+  PL_THRESHOLD_SLACK = 1,  /* north_star: fire when |Q| >= theta_i or slack forces it */
+  PL_MONOLITHIC = 2        /* paper §5: blocks of M, whole pipeline per block        */
+};
+
+enum pl_clock { PL_CLOCK_LOGICAL = 0, PL_CLOCK_GLOBALTIMER = 1 };
+
+/* pl_config.flags: optional per-root / per-firing records (parity & tracing).    */
+#define PL_REC_LATENCY  1u     /* lat[r]: per-root latency (model units; + ns if physical) */
+#define PL_REC_TRACE    2u     /* cnt[r][0..N]: per-root surviving-stage trace           */
+#define PL_REC_FIRINGS  4u     /* per-stream log of non-empty firings                    */
+
+typedef struct {
+  uint32_t kind;           /* enum pl_stage_kind                                        */
+  uint32_t max_out;        /* u: cap on outputs per input (1..PL_MAX_U)                 */
+  double   param;          /* g (Bernoulli), c (fixed gain), lambda (Poisson), modulus  */
+  int32_t  iparam[4];      /* DNA: S0 {k}, S1 {k,u}, S2 {k,W,T2}, S3 {k,X,T3}           */
+} pl_stage;
+
+typedef struct {
+  uint32_t n_stages;               /* N, 1..PL_MAX_STAGES; linear chain only (L61)      */
+  const pl_stage* stages;          /* [N]                                               */
+  const int64_t* service_time;     /* t_i [N] > 0                                       */
+  const double*  gain;             /* g_i [N-1] for the solvers; NULL -> measured       */
+  const uint32_t* b;               /* b_i [N] queue multipliers (L133); NULL -> all 1   */
+  uint32_t vector_width;           /* v: 32, 64, 128 or 256; N*v <= 992                 */
+  const int64_t*  wait_time;       /* w_i [N] (FIXED_WAIT) or NULL -> solve Fig. 1      */
+  const uint32_t* wait_threshold;  /* theta_i [N] (THRESHOLD_SLACK) or NULL -> derived  */
+  int64_t deadline;                /* D (L73)                                           */
+  int64_t interarrival;            /* tau0 = 1/rho0 (L63), >= 1                          */
+  int64_t slack_guard;             /* THRESHOLD_SLACK: extra reserve added to R_i        */
+  uint32_t policy;                 /* enum pl_policy                                    */
+  uint32_t clock;                  /* enum pl_clock                                     */
+  uint32_t block_size;             /* M (MONOLITHIC); 0 -> solve Fig. 2                 */
+  uint32_t mono_b;                 /* b of Fig. 2 (0 -> 1)                              */
+  double   mono_S;                 /* S of Fig. 2 (0 -> 1)                              */
+  uint32_t n_streams;              /* independent pipeline instances = CTAs (>= 1)      */
+  uint64_t n_roots;                /* random-gain stages: roots per stream;             */
+                                   /* DNA: 0 (roots are the DB positions [0, Ldb-k])    */
+  uint64_t seed;                   /* counter-based RNG seed of random-gain stages      */
+  int32_t  device;                 /* CUDA device ordinal                               */
+  double   ns_per_unit;            /* physical clock: ns per time unit (> 0)            */
+  uint32_t flags;                  /* PL_REC_* bits                                     */
+  uint32_t queue_capacity;         /* smem entries per edge (power of 2; 0 -> default)  */
+  uint32_t spill_capacity;         /* HBM overflow entries per edge per stream (2^k; 0->dflt) */
+  uint32_t firing_log_capacity;    /* records per stream when PL_REC_FIRINGS (0 -> dflt) */
+  uint64_t match_capacity;         /* pl_match records (0 -> default)                   */
+} pl_config;
+
+/* Workload of the DNA pipeline: the query is known up front; the database is the
+ * stream and arrives through pl_pipeline_push / pl_pipeline_bind_device.
+ * Both sequences are 2-bit packed: base j at bits 2*(j mod 16) of uint32 word j/16,
+ * A=0 C=1 G=2 T=3.  Ignored (may be NULL) for random-gain pipelines.            */
+typedef struct {
+  const uint32_t* query;           /* host pointer, ceil(q_len/16) words             */
+  uint64_t q_len;                  /* <= 65535                                       */
+  uint64_t db_len;                 /* total DB bases the stream will carry           */
+} pl_workload;
+
+/* One HSP emitted by the last DNA stage (reading R-S3).                          */
+typedef struct {
+  uint32_t p, q;                   /* seed position in DB / query (root = p)          */
+  uint32_t db_start, q_start;      /* left end of the extension                       */
+  uint32_t len;                    /* extension length                                */
+  int32_t  score;
+} pl_match;
+
+/* One non-empty firing (PL_REC_FIRINGS).                                         */
+typedef struct {
+  int64_t  start;                  /* logical start time (units)                      */
+  uint32_t node, n;                /* node index, inputs consumed (1..v)              */
+  uint32_t first_root, last_root;  /* roots of the first and last consumed entry      */
+  uint32_t stream, pad;
+} pl_firing;
+
+typedef struct {
+  uint32_t n_stages, n_streams;
+  uint64_t roots;                          /* roots processed (all streams)           */
+  uint64_t firings[PL_MAX_STAGES];         /* non-empty firings                       */
+  uint64_t empty_firings[PL_MAX_STAGES];   /* FIXED_WAIT firings skipped as empty     */
+  uint64_t consumed[PL_MAX_STAGES];
+  uint64_t produced[PL_MAX_STAGES];
+  int64_t  active_window[PL_MAX_STAGES];   /* sum |[s,s+t_i) ∩ [0,H)| over ALL firings */
+  int64_t  busy_ns[PL_MAX_STAGES];         /* physical: measured firing time (ns)     */
+  uint64_t spilled[PL_MAX_STAGES];         /* entries written to the HBM overflow ring */
+  uint64_t overruns[PL_MAX_STAGES];        /* physical: firings longer than t_i        */
+  int64_t  max_lateness_ns[PL_MAX_STAGES]; /* physical: max(actual - scheduled start)  */
+  uint64_t sched_cycles[PL_MAX_STAGES];    /* clock64 cycles spent deciding firings    */
+  uint64_t matches;
+  uint64_t miss_events;                    /* terminal events with latency > D        */
+  uint64_t misses;                         /* distinct roots (needs PL_REC_LATENCY)    */
+  int64_t  max_latency;                    /* model units (logical schedule)          */
+  int64_t  max_latency_ns;                 /* physical: measured                       */
+  int64_t  window;                         /* sum over streams of H = X*tau0           */
+  int64_t  t_end;                          /* sum over streams of the drain end time   */
+  double   active_fraction;                /* PAPER.md L75 over [0,H)                  */
+  double   active_fraction_nonempty;       /* same, charging non-empty firings only    */
+  double   hw_busy_fraction;               /* physical: busy_ns / (N * wall)           */
+  int64_t  wall_ns;                        /* max over streams of kernel-side runtime  */
+  uint32_t errors;                         /* PL_EOVERFLOW bits etc.                   */
+  uint32_t launches;                       /* executor launches so far                 */
+} pl_stats;
+
+typedef struct pl_pipeline pl_pipeline;
+
+/* Create a pipeline.  Validates cfg (PL_EINVAL), solves Fig. 1 / Fig. 2 when
+ * w / M are missing and gains are given (PL_EINFEASIBLE), allocates device memory
+ * (PL_ENOMEM) and uploads the query index.  *out is NULL on failure.            */
+pl_status pl_pipeline_create(const pl_config* cfg, const pl_workload* wl, pl_pipeline** out);
+
+/* Bind the CUDA stream (cudaStream_t passed as void*) every later launch and copy
+ * uses.  NULL = the legacy default stream.                                      */
+pl_status pl_pipeline_set_stream(pl_pipeline* pl, void* stream);
+
+/* Append n items from HOST memory: for DNA pipelines `items` holds n bases, 2-bit
+ * packed, and the running total must stay <= wl->db_len (every push but the last
+ * must be a multiple of 16 bases); the copy to HBM is enqueued on the bound stream
+ * before the call returns and `items` may be reused immediately.  For random-gain
+ * pipelines items must be NULL and n counts roots per stream (<= cfg->n_roots).
+ * After pl_pipeline_drain: PL_ESTATE until pl_pipeline_rewind.                  */
+pl_status pl_pipeline_push(pl_pipeline* pl, const void* items, uint64_t n);
+
+/* Use a caller-owned DEVICE buffer of n packed bases as the whole DB (no copy).
+ * The buffer must stay alive until the last launch using it has completed.      */
+pl_status pl_pipeline_bind_device(pl_pipeline* pl, const void* dev_items, uint64_t n);
+
+/* Enqueue one executor run over every item pushed so far on the bound stream and
+ * return immediately (asynchronous).  Resets per-run outputs first.             */
+pl_status pl_pipeline_launch(pl_pipeline* pl);
+
+/* Launch if nothing is in flight, then block until the run has completed; checks
+ * device-side error flags (PL_EOVERFLOW) and CUDA errors (PL_EDEVICE).          */
+pl_status pl_pipeline_drain(pl_pipeline* pl);
+
+/* Allow another push/launch cycle with the same pipeline (rewinds the stream).   */
+pl_status pl_pipeline_rewind(pl_pipeline* pl);
+
+/* Statistics of the last completed run (copies counters device->host).          */
+pl_status pl_pipeline_stats(pl_pipeline* pl, pl_stats* out);
+
+/* Matches of the last run, unsorted.  buf==NULL: *n = count.  Otherwise copies
+ * min(cap, count) records and sets *n to the number copied.                     */
+pl_status pl_pipeline_results(pl_pipeline* pl, pl_match* buf, uint64_t cap, uint64_t* n);
+
+/* Per-root latencies (needs PL_REC_LATENCY): lat_units[r] (logical schedule) and,
+ * if lat_ns != NULL and the clock is physical, measured ns.  -1 = no terminal event.
+ * Arrays have *n = total roots entries (query with lat_units == NULL).          */
+pl_status pl_pipeline_latency(pl_pipeline* pl, int64_t* lat_units, int64_t* lat_ns, uint64_t cap, uint64_t* n);
+
+/* Per-root trace (needs PL_REC_TRACE): cnt[r*(N+1)+i] = descendants of root r
+ * consumed by node i (i < N); cnt[r*(N+1)+N] = outputs emitted by node N-1.     */
+pl_status pl_pipeline_trace(pl_pipeline* pl, uint32_t* cnt, uint64_t cap, uint64_t* n);
+
+/* Non-empty firings of the last run (needs PL_REC_FIRINGS), grouped by stream.  */
+pl_status pl_pipeline_firings(pl_pipeline* pl, pl_firing* buf, uint64_t cap, uint64_t* n);
+
+/* The effective parameters in use (after solving): w_i, theta_i, M.            */
+pl_status pl_pipeline_params(const pl_pipeline* pl, int64_t* w_out, uint32_t* theta_out, uint32_t* M_out);
+
+void pl_pipeline_destroy(pl_pipeline* pl);
+
+/* Thread-local message for the last non-OK status of this thread ("" if none).  */
+const char* pl_last_error(void);
+
+/* Fig. 1: minimise (1/N) sum t_i/(t_i+w_i) s.t. stability
+ * (L125, L131) and sum b_i (t_i+w_i) <= D (L135), w_i >= 0 integer.  Needs
+ * cfg->gain.  Writes w_out[N], theta_out[N] (THRESHOLD mapping, may be NULL),
+ * *T_out (objective at the integer optimum) and T_cont (continuous optimum, may be NULL). */
+pl_status pl_solve_enforced_waits(const pl_config* cfg, int64_t* w_out, uint32_t* theta_out,
+                                  double* T_out, double* T_cont);
+
+/* Fig. 2: best block size M by exhaustive search.          */
+pl_status pl_solve_monolithic(const pl_config* cfg, uint32_t* M_out, double* T_out);
+
+/* Library build identity (for logs): "plgpu <version> sm_100a".                  */
+const char* pl_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* PL_H */

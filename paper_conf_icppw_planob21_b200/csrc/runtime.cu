@@ -1,0 +1,681 @@
+// runtime.cu — host implementation of the C-ABI in include/pl.h.
+//
+// Owns device memory, validates configurations, derives the schedule parameters
+// (periods P_i = t_i + w_i, thresholds theta_i, reserves R_i, block size M) —
+// solving Fig. 1 / Fig. 2 when they are not given — builds the query index
+// (direct-address k-mer table, reading R-S1), and launches the persistent
+// executor kernels in executor.cu.  No exceptions cross the ABI.
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <cmath>
+#include <cstdarg>
+#include <cstdio>
+#include <cstring>
+#include <new>
+#include <string>
+#include <vector>
+
+#include "pl_internal.h"
+
+extern "C" __global__ void pl_exec_enforced(const __grid_constant__ DevParams p);
+extern "C" __global__ void pl_exec_monolithic(const __grid_constant__ DevParams p);
+uint32_t pl_layout_enforced_host(const DevParams& p);
+
+namespace plsolve {
+int solve_fig1(int N, const int64_t* t, const double* g, const uint32_t* b, uint32_t v, int64_t tau, int64_t D,
+               double* Pc, double* Tc, int64_t* Pi, double* Ti);
+void thresholds(int N, const double* g, const int64_t* P, int64_t tau, uint32_t v, uint32_t* theta);
+int solve_fig2(int N, const int64_t* t, const double* g, uint32_t v, int64_t tau, int64_t D, double bb, double S,
+               uint32_t* M_out, double* T_out);
+}  // namespace plsolve
+
+namespace {
+
+thread_local std::string g_err;
+
+pl_status fail(pl_status st, const char* fmt, ...) {
+  char buf[512];
+  va_list ap;
+  va_start(ap, fmt);
+  vsnprintf(buf, sizeof buf, fmt, ap);
+  va_end(ap);
+  g_err = buf;
+  return st;
+}
+
+#define CUDA_TRY(x)                                                                              \
+  do {                                                                                           \
+    cudaError_t _e = (x);                                                                        \
+    if (_e != cudaSuccess) return fail(PL_EDEVICE, "%s: %s", #x, cudaGetErrorString(_e));        \
+  } while (0)
+
+uint32_t next_pow2(uint32_t x) {
+  uint32_t p = 1;
+  while (p < x) p <<= 1;
+  return p;
+}
+bool is_pow2(uint32_t x) { return x && !(x & (x - 1)); }
+
+bool is_dna(uint32_t kind) {
+  return kind == PL_SEED_LOOKUP || kind == PL_HIT_ENUM || kind == PL_UNGAPPED_WINDOW || kind == PL_UNGAPPED_XDROP;
+}
+
+// exact floor(p * 2^64) for p in [0,1], saturated at 2^64-1 (same rule as plgen.gaintab)
+uint64_t prob_to_u64(double p) {
+  if (!(p > 0)) return 0;
+  if (p >= 1.0) return ~0ull;
+  int e;
+  double m = std::frexp(p, &e);             // p = m 2^e, m in [0.5, 1)
+  uint64_t mant = (uint64_t)std::ldexp(m, 53);   // exact 53-bit integer
+  int sh = 64 + e - 53;                     // p 2^64 = mant 2^(64+e-53)
+  if (sh >= 0) return sh >= 11 + 53 ? ~0ull : (mant << sh);
+  return mant >> (-sh);
+}
+
+double poisson_cdf(double lam, int k) {
+  double term = std::exp(-lam), acc = term;
+  for (int j = 1; j <= k; ++j) {
+    term *= lam / j;
+    acc += term;
+  }
+  return acc < 1.0 ? acc : 1.0;
+}
+
+}  // namespace
+
+struct pl_pipeline {
+  pl_config cfg;
+  pl_stage stages[PL_MAX_STAGES];
+  int64_t t[PL_MAX_STAGES], w[PL_MAX_STAGES];
+  double g[PL_MAX_STAGES];
+  bool have_g = false;
+  uint32_t b[PL_MAX_STAGES], theta[PL_MAX_STAGES];
+  uint32_t M = 0;
+  bool dna = false;
+  int k = 0;
+  uint64_t q_len = 0, db_len = 0;
+  std::vector<uint32_t> query;
+  DevParams dp;
+  uint32_t smem = 0, block = 0;
+  cudaStream_t stream = nullptr;
+  // device buffers
+  uint32_t* d_db = nullptr;
+  const uint32_t* d_db_bound = nullptr;   // caller-owned
+  uint16_t *d_qoff = nullptr, *d_qpos = nullptr;
+  uint32_t* d_qw = nullptr;
+  uint2* d_spill = nullptr;
+  uint2* d_mono = nullptr;
+  int64_t *d_lat = nullptr, *d_lat_ns = nullptr;
+  uint32_t* d_trace = nullptr;
+  pl_match* d_matches = nullptr;
+  unsigned long long* d_match_count = nullptr;
+  pl_firing* d_flog = nullptr;
+  CtaStats* d_stats = nullptr;
+  uint64_t roots_cap = 0;   // per-root arrays sized for this many roots
+  // host state
+  uint64_t pushed = 0;      // DNA: bases; gain: roots per stream
+  bool in_flight = false, drained = false;
+  uint32_t launches = 0;
+  int device = 0;
+};
+
+namespace {
+
+void free_all(pl_pipeline* pl) {
+  void* ptrs[] = {pl->d_db, pl->d_qoff, pl->d_qpos, pl->d_qw, pl->d_spill, pl->d_mono, pl->d_lat, pl->d_lat_ns,
+                  pl->d_trace, pl->d_matches, pl->d_match_count, pl->d_flog, pl->d_stats};
+  for (void* p : ptrs)
+    if (p) cudaFree(p);
+}
+
+pl_status validate(const pl_config* c, const pl_workload* wl) {
+  if (!c) return fail(PL_EINVAL, "cfg is NULL");
+  const uint32_t N = c->n_stages;
+  if (N < 1 || N > PL_MAX_STAGES) return fail(PL_EINVAL, "n_stages %u not in [1, %d]", N, PL_MAX_STAGES);
+  if (!c->stages || !c->service_time) return fail(PL_EINVAL, "stages / service_time missing");
+  const uint32_t v = c->vector_width;
+  if (v != 32 && v != 64 && v != 128 && v != 256) return fail(PL_EINVAL, "vector_width %u not in {32,64,128,256}", v);
+  if (N * v > 1024) return fail(PL_EINVAL, "N*v = %u exceeds 1024 threads", N * v);
+  if (c->interarrival < 1) return fail(PL_EINVAL, "interarrival must be >= 1");
+  if (c->deadline < 1) return fail(PL_EINVAL, "deadline must be >= 1");
+  if (c->policy > PL_MONOLITHIC) return fail(PL_EINVAL, "bad policy %u", c->policy);
+  if (c->clock > PL_CLOCK_GLOBALTIMER) return fail(PL_EINVAL, "bad clock %u", c->clock);
+  if (c->clock == PL_CLOCK_GLOBALTIMER && !(c->ns_per_unit > 0)) return fail(PL_EINVAL, "ns_per_unit must be > 0");
+  if (c->n_streams < 1 || c->n_streams > (1u << 20)) return fail(PL_EINVAL, "n_streams %u", c->n_streams);
+  bool dna = is_dna(c->stages[0].kind);
+  for (uint32_t i = 0; i < N; ++i) {
+    const pl_stage& s = c->stages[i];
+    if (c->service_time[i] < 1) return fail(PL_EINVAL, "service_time[%u] must be >= 1", i);
+    if (s.kind > PL_KEEP_EVERY) return fail(PL_EINVAL, "stage %u: bad kind %u", i, s.kind);
+    if (is_dna(s.kind) != dna) return fail(PL_EINVAL, "stage %u mixes DNA and random-gain kinds", i);
+    if (s.max_out < 1 || s.max_out > PL_MAX_U) return fail(PL_EINVAL, "stage %u: max_out %u", i, s.max_out);
+    if (s.kind == PL_FIXED_GAIN && ((int)s.param < 0 || (uint32_t)s.param > s.max_out))
+      return fail(PL_EINVAL, "stage %u: fixed gain %g exceeds max_out", i, s.param);
+    if (s.kind == PL_KEEP_EVERY && (int)s.param < 1) return fail(PL_EINVAL, "stage %u: modulus < 1", i);
+    if (s.kind == PL_BERNOULLI && !(s.param >= 0 && s.param <= 1)) return fail(PL_EINVAL, "stage %u: g not in [0,1]", i);
+    if (s.kind == PL_POISSON_CAPPED && !(s.param >= 0)) return fail(PL_EINVAL, "stage %u: lambda < 0", i);
+    if (s.kind != PL_FIXED_GAIN && s.kind != PL_POISSON_CAPPED && s.kind != PL_HIT_ENUM && s.max_out != 1)
+      return fail(PL_EINVAL, "stage %u: filter stages have max_out 1", i);
+  }
+  if (c->wait_time)
+    for (uint32_t i = 0; i < N; ++i)
+      if (c->wait_time[i] < 0) return fail(PL_EINVAL, "wait_time[%u] < 0", i);
+  if (c->wait_threshold)
+    for (uint32_t i = 0; i < N; ++i)
+      if (c->wait_threshold[i] < 1 || c->wait_threshold[i] > v) return fail(PL_EINVAL, "wait_threshold[%u] not in [1,v]", i);
+  if (dna) {
+    if (!wl || !wl->query) return fail(PL_EINVAL, "DNA pipeline needs a workload with a query");
+    int k = c->stages[0].iparam[0];
+    if (k < 1 || k > PL_MAX_K) return fail(PL_EINVAL, "k = %d not in [1, %d]", k, PL_MAX_K);
+    for (uint32_t i = 0; i < N; ++i)
+      if (c->stages[i].iparam[0] != k) return fail(PL_EINVAL, "stage %u: k differs", i);
+    if (wl->q_len < (uint64_t)k || wl->q_len > 65535) return fail(PL_EINVAL, "q_len %llu", (unsigned long long)wl->q_len);
+    if (wl->db_len >= (1ull << 32)) return fail(PL_EINVAL, "db_len must be < 2^32");
+  } else {
+    if (c->n_roots >= (1ull << 32) / c->n_streams) return fail(PL_EINVAL, "n_roots * n_streams must be < 2^32");
+  }
+  return PL_OK;
+}
+
+}  // namespace
+
+extern "C" {
+
+const char* pl_last_error(void) { return g_err.c_str(); }
+const char* pl_version(void) { return "plgpu 0.1 sm_100a"; }
+
+pl_status pl_solve_enforced_waits(const pl_config* cfg, int64_t* w_out, uint32_t* theta_out, double* T_out,
+                                  double* T_cont) {
+  if (!cfg || !cfg->service_time || !w_out) return fail(PL_EINVAL, "NULL argument");
+  if (!cfg->gain && cfg->n_stages > 1) return fail(PL_EINVAL, "solver needs gains");
+  const int N = (int)cfg->n_stages;
+  if (N < 1 || N > PL_MAX_STAGES) return fail(PL_EINVAL, "n_stages");
+  uint32_t b[PL_MAX_STAGES];
+  for (int i = 0; i < N; ++i) b[i] = cfg->b ? cfg->b[i] : 1u;
+  double g[PL_MAX_STAGES] = {0};
+  for (int i = 0; i + 1 < N; ++i) g[i] = cfg->gain[i];
+  double Pc[PL_MAX_STAGES], Tc, Ti;
+  int64_t Pi[PL_MAX_STAGES];
+  int st = plsolve::solve_fig1(N, cfg->service_time, g, b, cfg->vector_width, cfg->interarrival, cfg->deadline, Pc,
+                               &Tc, Pi, &Ti);
+  if (st == PL_EINVAL) return fail(PL_EINVAL, "gains must be > 0");
+  if (st != PL_OK) return fail(PL_EINFEASIBLE, "Fig. 1 infeasible at tau0=%lld D=%lld", (long long)cfg->interarrival,
+                               (long long)cfg->deadline);
+  for (int i = 0; i < N; ++i) w_out[i] = Pi[i] - cfg->service_time[i];
+  if (theta_out) plsolve::thresholds(N, g, Pi, cfg->interarrival, cfg->vector_width, theta_out);
+  if (T_out) *T_out = Ti;
+  if (T_cont) *T_cont = Tc;
+  return PL_OK;
+}
+
+pl_status pl_solve_monolithic(const pl_config* cfg, uint32_t* M_out, double* T_out) {
+  if (!cfg || !cfg->service_time || !M_out) return fail(PL_EINVAL, "NULL argument");
+  if (!cfg->gain && cfg->n_stages > 1) return fail(PL_EINVAL, "solver needs gains");
+  const int N = (int)cfg->n_stages;
+  double g[PL_MAX_STAGES] = {0};
+  for (int i = 0; i + 1 < N; ++i) g[i] = cfg->gain[i];
+  double T;
+  int st = plsolve::solve_fig2(N, cfg->service_time, g, cfg->vector_width, cfg->interarrival, cfg->deadline,
+                               cfg->mono_b ? (double)cfg->mono_b : 1.0, cfg->mono_S > 0 ? cfg->mono_S : 1.0, M_out, &T);
+  if (st != PL_OK) return fail(PL_EINFEASIBLE, "Fig. 2 infeasible at tau0=%lld D=%lld", (long long)cfg->interarrival,
+                               (long long)cfg->deadline);
+  if (T_out) *T_out = T;
+  return PL_OK;
+}
+
+pl_status pl_pipeline_create(const pl_config* cfg, const pl_workload* wl, pl_pipeline** out) {
+  if (!out) return fail(PL_EINVAL, "out is NULL");
+  *out = nullptr;
+  pl_status st = validate(cfg, wl);
+  if (st != PL_OK) return st;
+  pl_pipeline* pl = new (std::nothrow) pl_pipeline();
+  if (!pl) return fail(PL_ENOMEM, "host allocation failed");
+  const uint32_t N = cfg->n_stages;
+  pl->cfg = *cfg;
+  for (uint32_t i = 0; i < N; ++i) {
+    pl->stages[i] = cfg->stages[i];
+    pl->t[i] = cfg->service_time[i];
+    pl->b[i] = cfg->b ? cfg->b[i] : 1u;
+  }
+  pl->cfg.stages = pl->stages;
+  pl->cfg.service_time = pl->t;
+  pl->cfg.b = pl->b;
+  pl->have_g = cfg->gain != nullptr;
+  for (uint32_t i = 0; i + 1 < N; ++i) pl->g[i] = cfg->gain ? cfg->gain[i] : 0.0;
+  pl->cfg.gain = pl->have_g ? pl->g : nullptr;
+  pl->dna = is_dna(cfg->stages[0].kind);
+  pl->device = cfg->device;
+  auto bail = [&](pl_status s) {
+    std::string keep = g_err;
+    free_all(pl);
+    delete pl;
+    g_err = keep;
+    return s;
+  };
+  // ---- schedule parameters
+  const uint32_t v = cfg->vector_width;
+  if (cfg->policy == PL_FIXED_WAIT || cfg->policy == PL_THRESHOLD_SLACK) {
+    if (cfg->wait_time) {
+      for (uint32_t i = 0; i < N; ++i) pl->w[i] = cfg->wait_time[i];
+    } else if (cfg->policy == PL_FIXED_WAIT || !cfg->wait_threshold) {
+      if (!pl->have_g && N > 1) return bail(fail(PL_EINVAL, "wait_time missing and no gains to solve Fig. 1"));
+      double T;
+      st = pl_solve_enforced_waits(&pl->cfg, pl->w, nullptr, &T, nullptr);
+      if (st != PL_OK) return bail(st);
+    }
+    if (cfg->wait_threshold) {
+      for (uint32_t i = 0; i < N; ++i) pl->theta[i] = cfg->wait_threshold[i];
+    } else if (cfg->policy == PL_THRESHOLD_SLACK) {
+      if (!pl->have_g && N > 1) return bail(fail(PL_EINVAL, "wait_threshold missing and no gains"));
+      int64_t P[PL_MAX_STAGES];
+      for (uint32_t i = 0; i < N; ++i) P[i] = pl->t[i] + pl->w[i];
+      plsolve::thresholds((int)N, pl->g, P, cfg->interarrival, v, pl->theta);
+    }
+  } else {
+    pl->M = cfg->block_size;
+    if (!pl->M) {
+      if (!pl->have_g && N > 1) return bail(fail(PL_EINVAL, "block_size missing and no gains to solve Fig. 2"));
+      double T;
+      st = pl_solve_monolithic(&pl->cfg, &pl->M, &T);
+      if (st != PL_OK) return bail(st);
+    }
+  }
+  pl->cfg.wait_time = pl->w;
+  pl->cfg.wait_threshold = pl->theta;
+  // ---- device
+  int ndev = 0;
+  if (cudaGetDeviceCount(&ndev) != cudaSuccess || ndev == 0) return bail(fail(PL_EDEVICE, "no CUDA device"));
+  if (cfg->device < 0 || cfg->device >= ndev) return bail(fail(PL_EINVAL, "device %d of %d", cfg->device, ndev));
+  if (cudaSetDevice(cfg->device) != cudaSuccess) return bail(fail(PL_EDEVICE, "cudaSetDevice failed"));
+  cudaDeviceProp prop;
+  cudaGetDeviceProperties(&prop, cfg->device);
+  if (prop.major != 10) return bail(fail(PL_EDEVICE, "built for sm_100a; device is sm_%d%d", prop.major, prop.minor));
+
+  DevParams& d = pl->dp;
+  std::memset(&d, 0, sizeof d);
+  d.N = (int)N;
+  d.v = (int)v;
+  d.policy = (int)cfg->policy;
+  d.clock = (int)cfg->clock;
+  for (uint32_t i = 0; i < N; ++i) {
+    d.t[i] = pl->t[i];
+    d.P[i] = pl->t[i] + pl->w[i];
+    d.theta[i] = pl->theta[i] ? pl->theta[i] : 1u;
+    int64_t r = pl->t[i];
+    for (uint32_t j = i + 1; j < N; ++j) r += 2 * pl->t[j];   // R_i = t_i + 2 sum_{j>i} t_j (R-THRESH)
+    d.R[i] = r + cfg->slack_guard;
+  }
+  d.D = cfg->deadline;
+  d.tau = cfg->interarrival;
+  d.M = pl->M;
+  d.ns_per_unit = cfg->clock == PL_CLOCK_GLOBALTIMER ? cfg->ns_per_unit : 1.0;
+  d.seed = cfg->seed;
+  d.n_streams = (int)cfg->n_streams;
+  d.flags = cfg->flags;
+  for (uint32_t i = 0; i < N; ++i) {
+    const pl_stage& s = pl->stages[i];
+    DevStage& ds = d.st[i];
+    ds.kind = s.kind;
+    ds.max_out = s.max_out;
+    for (int j = 0; j < 4; ++j) ds.ip[j] = s.iparam[j];
+    ds.cfix = (s.kind == PL_FIXED_GAIN || s.kind == PL_KEEP_EVERY) ? (uint32_t)s.param : 0u;
+    if (s.kind == PL_BERNOULLI) ds.thr[0] = prob_to_u64(s.param);
+    if (s.kind == PL_POISSON_CAPPED)
+      for (uint32_t j = 0; j < s.max_out; ++j) ds.thr[j] = prob_to_u64(poisson_cdf(s.param, (int)j));
+  }
+  // ---- DNA: query index (direct-address k-mer table; counting sort keeps q ascending)
+  if (pl->dna) {
+    pl->k = cfg->stages[0].iparam[0];
+    pl->q_len = wl->q_len;
+    pl->db_len = wl->db_len;
+    const uint32_t nqw = (uint32_t)((wl->q_len + 15) / 16);
+    pl->query.assign(wl->query, wl->query + nqw);
+    const uint32_t K = 1u << (2 * pl->k);
+    const uint32_t nq = (uint32_t)(wl->q_len - pl->k + 1);
+    std::vector<uint16_t> off(K + 1, 0), pos(nq);
+    std::vector<uint32_t> keys(nq);
+    auto qb = [&](uint64_t j) { return (pl->query[j >> 4] >> ((j & 15) * 2)) & 3u; };
+    for (uint32_t q = 0; q < nq; ++q) {
+      uint32_t key = 0;
+      for (int j = 0; j < pl->k; ++j) key = (key << 2) | qb(q + j);
+      keys[q] = key;
+      off[key + 1]++;
+    }
+    for (uint32_t j = 0; j < K; ++j) off[j + 1] += off[j];
+    std::vector<uint16_t> fill(off.begin(), off.end() - 1);
+    for (uint32_t q = 0; q < nq; ++q) pos[fill[keys[q]]++] = (uint16_t)q;
+    if (cudaMalloc(&pl->d_qoff, (K + 1) * 2) != cudaSuccess || cudaMalloc(&pl->d_qpos, nq * 2) != cudaSuccess ||
+        cudaMalloc(&pl->d_qw, nqw * 4) != cudaSuccess)
+      return bail(fail(PL_ENOMEM, "query index allocation"));
+    cudaMemcpy(pl->d_qoff, off.data(), (K + 1) * 2, cudaMemcpyHostToDevice);
+    cudaMemcpy(pl->d_qpos, pos.data(), nq * 2, cudaMemcpyHostToDevice);
+    cudaMemcpy(pl->d_qw, pl->query.data(), nqw * 4, cudaMemcpyHostToDevice);
+    d.k = pl->k;
+    d.q_len = (int)wl->q_len;
+    d.qoff = pl->d_qoff;
+    d.qpos = pl->d_qpos;
+    d.qwords = pl->d_qw;
+    const uint64_t dbw = (wl->db_len + 15) / 16 + 1;
+    if (cudaMalloc(&pl->d_db, dbw * 4) != cudaSuccess) return bail(fail(PL_ENOMEM, "DB allocation"));
+    cudaMemset(pl->d_db, 0, dbw * 4);
+    pl->roots_cap = wl->db_len >= (uint64_t)pl->k ? wl->db_len - pl->k + 1 : 0;
+  } else {
+    pl->roots_cap = cfg->n_roots * cfg->n_streams;
+  }
+  // ---- queues
+  const uint32_t S = cfg->n_streams;
+  d.segcap = next_pow2(2 * v);
+  uint32_t maxu = 1;
+  for (uint32_t i = 1; i < N; ++i) {
+    const uint32_t u = pl->stages[i - 1].max_out;
+    if (u > maxu) maxu = u;
+    uint32_t cap = cfg->queue_capacity ? cfg->queue_capacity : next_pow2(std::max(4 * v, v * (u + 1)));
+    if (!is_pow2(cap)) return bail(fail(PL_EINVAL, "queue_capacity must be a power of 2"));
+    d.cap_s[i] = cap;
+  }
+  d.cap_g = cfg->spill_capacity ? cfg->spill_capacity : (1u << 15);
+  if (!is_pow2(d.cap_g)) return bail(fail(PL_EINVAL, "spill_capacity must be a power of 2"));
+  if (d.cap_g < v * (maxu + 1)) return bail(fail(PL_EINVAL, "spill_capacity < v*(u+1) can deadlock"));
+  for (uint32_t i = 1; i < N; ++i)
+    if (d.cap_g < d.cap_s[i]) return bail(fail(PL_EINVAL, "spill_capacity smaller than the smem ring"));
+  if (cfg->policy == PL_MONOLITHIC) {
+    for (uint32_t i = 0; i < PL_MAX_STAGES; ++i) d.cap_s[i] = 0;
+    d.segcap = 0;
+    uint64_t mx = pl->M, cur = pl->M;
+    for (uint32_t i = 0; i + 1 < N; ++i) {
+      cur *= pl->stages[i].max_out;
+      mx = std::max(mx, cur);
+    }
+    d.mono_cap = (uint32_t)std::min<uint64_t>(mx, 1u << 24);
+    if (cudaMalloc(&pl->d_mono, (size_t)S * 2 * d.mono_cap * sizeof(uint2)) != cudaSuccess)
+      return bail(fail(PL_ENOMEM, "monolithic buffers"));
+    pl->block = std::min<uint32_t>(N * v, 1024);
+  } else {
+    if (N > 1 && cudaMalloc(&pl->d_spill, (size_t)S * N * d.cap_g * sizeof(uint2)) != cudaSuccess)
+      return bail(fail(PL_ENOMEM, "spill rings (%u streams x %u edges x %u)", S, N, d.cap_g));
+    pl->block = N * v;
+  }
+  d.spill = pl->d_spill;
+  d.mono_buf = pl->d_mono;
+  pl->smem = pl_layout_enforced_host(d);
+  if (pl->smem > 200 * 1024) return bail(fail(PL_EINVAL, "smem layout %u B exceeds budget; lower queue_capacity", pl->smem));
+  // ---- outputs
+  const uint64_t R = std::max<uint64_t>(pl->roots_cap, 1);
+  if (cfg->flags & PL_REC_LATENCY) {
+    if (cudaMalloc(&pl->d_lat, R * 8) != cudaSuccess || cudaMalloc(&pl->d_lat_ns, R * 8) != cudaSuccess)
+      return bail(fail(PL_ENOMEM, "latency arrays"));
+  }
+  if (cfg->flags & PL_REC_TRACE) {
+    if (cudaMalloc(&pl->d_trace, R * (N + 1) * 4) != cudaSuccess) return bail(fail(PL_ENOMEM, "trace array"));
+  }
+  d.log_cap = (cfg->flags & PL_REC_FIRINGS) ? (cfg->firing_log_capacity ? cfg->firing_log_capacity : (1u << 16)) : 0u;
+  if (d.log_cap && cudaMalloc(&pl->d_flog, (size_t)S * d.log_cap * sizeof(pl_firing)) != cudaSuccess)
+    return bail(fail(PL_ENOMEM, "firing log"));
+  d.match_cap = cfg->match_capacity ? cfg->match_capacity : (1ull << 20);
+  if (!pl->dna) d.match_cap = 1;
+  if (cudaMalloc(&pl->d_matches, d.match_cap * sizeof(pl_match)) != cudaSuccess ||
+      cudaMalloc(&pl->d_match_count, 8) != cudaSuccess || cudaMalloc(&pl->d_stats, S * sizeof(CtaStats)) != cudaSuccess)
+    return bail(fail(PL_ENOMEM, "output buffers"));
+  cudaMemset(pl->d_match_count, 0, 8);
+  cudaMemset(pl->d_stats, 0, S * sizeof(CtaStats));
+  d.lat = pl->d_lat;
+  d.lat_ns = cfg->clock == PL_CLOCK_GLOBALTIMER ? pl->d_lat_ns : nullptr;
+  if (!(cfg->flags & PL_REC_LATENCY)) d.lat_ns = nullptr;
+  d.trace = pl->d_trace;
+  d.matches = pl->d_matches;
+  d.match_count = pl->d_match_count;
+  d.flog = pl->d_flog;
+  d.stats = pl->d_stats;
+  cudaError_t e1 = cudaFuncSetAttribute(pl_exec_enforced, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024);
+  cudaError_t e2 = cudaFuncSetAttribute(pl_exec_monolithic, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024);
+  if (e1 != cudaSuccess || e2 != cudaSuccess)
+    return bail(fail(PL_EDEVICE, "cudaFuncSetAttribute: %s", cudaGetErrorString(e1 != cudaSuccess ? e1 : e2)));
+  cudaError_t e = cudaDeviceSynchronize();
+  if (e != cudaSuccess) return bail(fail(PL_EDEVICE, "create: %s", cudaGetErrorString(e)));
+  *out = pl;
+  return PL_OK;
+}
+
+pl_status pl_pipeline_set_stream(pl_pipeline* pl, void* stream) {
+  if (!pl) return fail(PL_EINVAL, "NULL pipeline");
+  pl->stream = (cudaStream_t)stream;
+  return PL_OK;
+}
+
+pl_status pl_pipeline_push(pl_pipeline* pl, const void* items, uint64_t n) {
+  if (!pl) return fail(PL_EINVAL, "NULL pipeline");
+  if (pl->drained) return fail(PL_ESTATE, "push after drain; call pl_pipeline_rewind");
+  if (pl->dna) {
+    if (!items) return fail(PL_EINVAL, "DNA push needs items");
+    if (pl->d_db_bound) return fail(PL_ESTATE, "a device DB is bound");
+    if (pl->pushed % 16) return fail(PL_EINVAL, "previous push was not a multiple of 16 bases");
+    if (pl->pushed + n > pl->db_len) return fail(PL_EINVAL, "push exceeds db_len");
+    cudaSetDevice(pl->device);
+    const uint64_t words = (n + 15) / 16;
+    CUDA_TRY(cudaMemcpyAsync(pl->d_db + pl->pushed / 16, items, words * 4, cudaMemcpyHostToDevice, pl->stream));
+    pl->pushed += n;
+  } else {
+    if (items) return fail(PL_EINVAL, "random-gain push takes items == NULL");
+    if (pl->pushed + n > pl->cfg.n_roots) return fail(PL_EINVAL, "push exceeds n_roots");
+    pl->pushed += n;
+  }
+  return PL_OK;
+}
+
+pl_status pl_pipeline_bind_device(pl_pipeline* pl, const void* dev_items, uint64_t n) {
+  if (!pl || !dev_items) return fail(PL_EINVAL, "NULL argument");
+  if (!pl->dna) return fail(PL_EINVAL, "bind_device is for DNA pipelines");
+  if (n > pl->db_len) return fail(PL_EINVAL, "bound DB longer than db_len");
+  pl->d_db_bound = (const uint32_t*)dev_items;
+  pl->pushed = n;
+  return PL_OK;
+}
+
+pl_status pl_pipeline_launch(pl_pipeline* pl) {
+  if (!pl) return fail(PL_EINVAL, "NULL pipeline");
+  cudaSetDevice(pl->device);
+  DevParams& d = pl->dp;
+  if (pl->dna) {
+    d.db = pl->d_db_bound ? pl->d_db_bound : pl->d_db;
+    d.db_len = pl->pushed;
+    d.db_words = (uint32_t)((pl->pushed + 15) / 16);
+    d.total_roots = pl->pushed >= (uint64_t)pl->k ? pl->pushed - pl->k + 1 : 0;
+  } else {
+    d.total_roots = pl->pushed * pl->cfg.n_streams;
+  }
+  if (d.total_roots > pl->roots_cap) return fail(PL_EINVAL, "more roots than allocated");
+  CUDA_TRY(cudaMemsetAsync(pl->d_match_count, 0, 8, pl->stream));
+  const dim3 grid(pl->cfg.n_streams), block(pl->block);
+  if (pl->cfg.policy == PL_MONOLITHIC) pl_exec_monolithic<<<grid, block, pl->smem, pl->stream>>>(d);
+  else pl_exec_enforced<<<grid, block, pl->smem, pl->stream>>>(d);
+  CUDA_TRY(cudaGetLastError());
+  pl->in_flight = true;
+  pl->launches++;
+  return PL_OK;
+}
+
+pl_status pl_pipeline_drain(pl_pipeline* pl) {
+  if (!pl) return fail(PL_EINVAL, "NULL pipeline");
+  if (!pl->in_flight) {
+    pl_status s = pl_pipeline_launch(pl);
+    if (s != PL_OK) return s;
+  }
+  CUDA_TRY(cudaStreamSynchronize(pl->stream));
+  pl->in_flight = false;
+  pl->drained = true;
+  std::vector<CtaStats> cs(pl->cfg.n_streams);
+  CUDA_TRY(cudaMemcpy(cs.data(), pl->d_stats, cs.size() * sizeof(CtaStats), cudaMemcpyDeviceToHost));
+  uint32_t err = 0;
+  for (auto& s : cs) err |= s.errors;
+  if (err) return fail(PL_EOVERFLOW, "device reported overflow bits 0x%x (queue=1 match=2 log=4 seg=8)", err);
+  return PL_OK;
+}
+
+pl_status pl_pipeline_rewind(pl_pipeline* pl) {
+  if (!pl) return fail(PL_EINVAL, "NULL pipeline");
+  pl->drained = false;
+  if (!pl->d_db_bound) pl->pushed = 0;
+  return PL_OK;
+}
+
+pl_status pl_pipeline_stats(pl_pipeline* pl, pl_stats* out) {
+  if (!pl || !out) return fail(PL_EINVAL, "NULL argument");
+  cudaSetDevice(pl->device);
+  CUDA_TRY(cudaStreamSynchronize(pl->stream));
+  const uint32_t S = pl->cfg.n_streams, N = pl->cfg.n_stages;
+  std::vector<CtaStats> cs(S);
+  CUDA_TRY(cudaMemcpy(cs.data(), pl->d_stats, S * sizeof(CtaStats), cudaMemcpyDeviceToHost));
+  std::memset(out, 0, sizeof *out);
+  out->n_stages = N;
+  out->n_streams = S;
+  const int64_t tau = pl->cfg.interarrival;
+  for (const CtaStats& s : cs) {
+    out->roots += s.n_roots;
+    const int64_t H = (int64_t)s.n_roots * tau;
+    out->window += H;
+    out->t_end += s.t_end;
+    for (uint32_t i = 0; i < N; ++i) {
+      out->firings[i] += s.firings[i];
+      out->empty_firings[i] += s.empty[i];
+      out->consumed[i] += s.consumed[i];
+      out->produced[i] += s.produced[i];
+      out->busy_ns[i] += s.busy_ns[i];
+      out->spilled[i] += s.spilled[i];
+      out->overruns[i] += s.overruns[i];
+      out->max_lateness_ns[i] = std::max(out->max_lateness_ns[i], s.lateness[i]);
+      out->sched_cycles[i] += s.sched_cycles[i];
+      if (pl->cfg.policy == PL_FIXED_WAIT) {   // every firing m*P_i < H is charged (L97, R-WINDOW)
+        const int64_t P = pl->dp.P[i], t = pl->t[i];
+        out->active_window[i] += (H / P) * t + std::min(t, H % P);
+      } else {
+        out->active_window[i] += s.active_ne[i];
+      }
+    }
+    out->miss_events += s.miss_events;
+    out->max_latency = std::max(out->max_latency, s.max_lat);
+    out->max_latency_ns = std::max(out->max_latency_ns, s.max_lat_ns);
+    out->wall_ns = std::max(out->wall_ns, s.wall_ns);
+    out->errors |= s.errors;
+  }
+  unsigned long long mc = 0;
+  CUDA_TRY(cudaMemcpy(&mc, pl->d_match_count, 8, cudaMemcpyDeviceToHost));
+  out->matches = std::min<uint64_t>(mc, pl->dp.match_cap);
+  double act = 0, act_ne = 0, busy = 0;
+  for (uint32_t i = 0; i < N; ++i) {
+    act += (double)out->active_window[i];
+    busy += (double)out->busy_ns[i];
+  }
+  for (const CtaStats& s : cs)
+    for (uint32_t i = 0; i < N; ++i) act_ne += (double)s.active_ne[i];
+  const double denom = pl->cfg.policy == PL_MONOLITHIC ? (double)out->window : (double)N * (double)out->window;
+  out->active_fraction = out->window ? act / denom : 0.0;
+  out->active_fraction_nonempty = out->window ? act_ne / denom : 0.0;
+  if (out->wall_ns > 0) {
+    const double procs = pl->cfg.policy == PL_MONOLITHIC ? 1.0 : (double)N;
+    out->hw_busy_fraction = busy / (procs * (double)out->wall_ns * (double)S);
+  }
+  if ((pl->cfg.flags & PL_REC_LATENCY) && pl->d_lat) {
+    std::vector<int64_t> lat(pl->dp.total_roots);
+    if (!lat.empty()) {
+      CUDA_TRY(cudaMemcpy(lat.data(), pl->d_lat, lat.size() * 8, cudaMemcpyDeviceToHost));
+      std::vector<int64_t> latn;
+      const bool phys = pl->cfg.clock == PL_CLOCK_GLOBALTIMER;
+      if (phys) {
+        latn.resize(lat.size());
+        CUDA_TRY(cudaMemcpy(latn.data(), pl->d_lat_ns, latn.size() * 8, cudaMemcpyDeviceToHost));
+      }
+      const double Dns = (double)pl->cfg.deadline * pl->dp.ns_per_unit;
+      for (size_t r = 0; r < lat.size(); ++r)
+        out->misses += phys ? ((double)latn[r] > Dns) : (lat[r] > pl->cfg.deadline);
+    }
+  }
+  out->launches = pl->launches;
+  return PL_OK;
+}
+
+pl_status pl_pipeline_results(pl_pipeline* pl, pl_match* buf, uint64_t cap, uint64_t* n) {
+  if (!pl || !n) return fail(PL_EINVAL, "NULL argument");
+  cudaSetDevice(pl->device);
+  CUDA_TRY(cudaStreamSynchronize(pl->stream));
+  unsigned long long mc = 0;
+  CUDA_TRY(cudaMemcpy(&mc, pl->d_match_count, 8, cudaMemcpyDeviceToHost));
+  uint64_t cnt = std::min<uint64_t>(mc, pl->dp.match_cap);
+  if (!buf) { *n = cnt; return PL_OK; }
+  cnt = std::min(cnt, cap);
+  if (cnt) CUDA_TRY(cudaMemcpy(buf, pl->d_matches, cnt * sizeof(pl_match), cudaMemcpyDeviceToHost));
+  *n = cnt;
+  return PL_OK;
+}
+
+pl_status pl_pipeline_latency(pl_pipeline* pl, int64_t* lat_units, int64_t* lat_ns, uint64_t cap, uint64_t* n) {
+  if (!pl || !n) return fail(PL_EINVAL, "NULL argument");
+  if (!(pl->cfg.flags & PL_REC_LATENCY)) return fail(PL_ESTATE, "PL_REC_LATENCY not enabled");
+  cudaSetDevice(pl->device);
+  CUDA_TRY(cudaStreamSynchronize(pl->stream));
+  uint64_t R = pl->dp.total_roots;
+  if (!lat_units) { *n = R; return PL_OK; }
+  R = std::min(R, cap);
+  if (R) CUDA_TRY(cudaMemcpy(lat_units, pl->d_lat, R * 8, cudaMemcpyDeviceToHost));
+  if (lat_ns && R) {
+    if (pl->cfg.clock == PL_CLOCK_GLOBALTIMER) CUDA_TRY(cudaMemcpy(lat_ns, pl->d_lat_ns, R * 8, cudaMemcpyDeviceToHost));
+    else for (uint64_t r = 0; r < R; ++r) lat_ns[r] = -1;
+  }
+  *n = R;
+  return PL_OK;
+}
+
+pl_status pl_pipeline_trace(pl_pipeline* pl, uint32_t* cnt, uint64_t cap, uint64_t* n) {
+  if (!pl || !n) return fail(PL_EINVAL, "NULL argument");
+  if (!(pl->cfg.flags & PL_REC_TRACE)) return fail(PL_ESTATE, "PL_REC_TRACE not enabled");
+  cudaSetDevice(pl->device);
+  CUDA_TRY(cudaStreamSynchronize(pl->stream));
+  uint64_t E = pl->dp.total_roots * (pl->cfg.n_stages + 1);
+  if (!cnt) { *n = E; return PL_OK; }
+  E = std::min(E, cap);
+  if (E) CUDA_TRY(cudaMemcpy(cnt, pl->d_trace, E * 4, cudaMemcpyDeviceToHost));
+  *n = E;
+  return PL_OK;
+}
+
+pl_status pl_pipeline_firings(pl_pipeline* pl, pl_firing* buf, uint64_t cap, uint64_t* n) {
+  if (!pl || !n) return fail(PL_EINVAL, "NULL argument");
+  if (!(pl->cfg.flags & PL_REC_FIRINGS)) return fail(PL_ESTATE, "PL_REC_FIRINGS not enabled");
+  cudaSetDevice(pl->device);
+  CUDA_TRY(cudaStreamSynchronize(pl->stream));
+  const uint32_t S = pl->cfg.n_streams;
+  std::vector<CtaStats> cs(S);
+  CUDA_TRY(cudaMemcpy(cs.data(), pl->d_stats, S * sizeof(CtaStats), cudaMemcpyDeviceToHost));
+  uint64_t total = 0;
+  for (auto& s : cs) total += s.n_log;
+  if (!buf) { *n = total; return PL_OK; }
+  uint64_t w = 0;
+  for (uint32_t s = 0; s < S && w < cap; ++s) {
+    const uint64_t c = std::min<uint64_t>(cs[s].n_log, cap - w);
+    if (c) CUDA_TRY(cudaMemcpy(buf + w, pl->d_flog + (uint64_t)s * pl->dp.log_cap, c * sizeof(pl_firing),
+                               cudaMemcpyDeviceToHost));
+    w += c;
+  }
+  *n = w;
+  return PL_OK;
+}
+
+pl_status pl_pipeline_params(const pl_pipeline* pl, int64_t* w_out, uint32_t* theta_out, uint32_t* M_out) {
+  if (!pl) return fail(PL_EINVAL, "NULL pipeline");
+  for (uint32_t i = 0; i < pl->cfg.n_stages; ++i) {
+    if (w_out) w_out[i] = pl->w[i];
+    if (theta_out) theta_out[i] = pl->dp.theta[i];
+  }
+  if (M_out) *M_out = pl->M;
+  return PL_OK;
+}
+
+void pl_pipeline_destroy(pl_pipeline* pl) {
+  if (!pl) return;
+  cudaSetDevice(pl->device);
+  cudaStreamSynchronize(pl->stream);
+  free_all(pl);
+  delete pl;
+}
+
+}  // extern "C"

@@ -1,0 +1,72 @@
+"""Shared helpers for the GPU parity tests: run the CUDA path (through the C-ABI)
+and the oracle on the same seeded inputs and compare element by element."""
+from __future__ import annotations
+
+import numpy as np
+
+from plgen import configs as C
+from plgen import dna as G
+
+
+def workload_for(cfg):
+    if cfg.dna is None:
+        return None
+    return G.make_dna(cfg.seed, **cfg.dna)
+
+
+def run_gpu(cfg, wl, flags=7, **over):
+    from paper_conf_icppw_planob21_b200 import Pipeline
+    pl = Pipeline(cfg, wl, flags=flags, **over)
+    if wl is not None:
+        pl.push(wl.db, wl.db_len)
+    else:
+        pl.push(None, cfg.n_roots)
+    pl.drain()
+    out = dict(stats=pl.stats(), matches=pl.results() if wl is not None else [])
+    if flags & 1:
+        out["lat"], out["lat_ns"] = pl.latency()
+    if flags & 2:
+        out["trace"] = pl.trace()
+    if flags & 4:
+        out["firings"] = pl.firings()
+    out["params"] = pl.params()
+    pl.close()
+    return out
+
+
+def run_oracle(cfg, wl, streams=None):
+    from oracle import des
+    return des.run(cfg, wl, streams=streams)
+
+
+def oracle_firings(res, stream_ids=None):
+    out = []
+    for k, s in enumerate(res.streams):
+        sid = stream_ids[k] if stream_ids is not None else k
+        for (i, st, n, a, b) in s.firings:
+            out.append((sid, i, st, n, a, b))
+    return sorted(out)
+
+
+def compare(cfg, g, o, check_firings=True):
+    """Assert bit-exact agreement of everything the logical schedule determines."""
+    N = cfg.n_stages
+    st = g["stats"]
+    assert st["errors"] == 0, st["errors"]
+    assert g["matches"] == [tuple(m) for m in o.matches]
+    if "lat" in g:
+        assert np.array_equal(g["lat"], np.asarray(o.lat, dtype=np.int64))
+    if "trace" in g:
+        assert np.array_equal(g["trace"], np.asarray(o.trace, dtype=np.uint32))
+    if check_firings and "firings" in g:
+        assert sorted(g["firings"]) == oracle_firings(o)
+    for i in range(N):
+        assert st["consumed"][i] == sum(s.consumed[i] for s in o.streams), i
+        assert st["produced"][i] == sum(s.produced[i] for s in o.streams), i
+        ne = sum(1 for s in o.streams for f in s.firings if f[0] == i)
+        assert st["firings"][i] == ne, i
+        assert st["active_window"][i] == sum(s.active_H[i] for s in o.streams), i
+    assert st["t_end"] == sum(s.T_end for s in o.streams)
+    assert st["max_latency"] == max(o.lat)
+    assert st["misses"] == o.misses(cfg.deadline)
+    assert abs(st["active_fraction"] - o.active_fraction(cfg.policy)) < 1e-12
