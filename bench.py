@@ -1,0 +1,379 @@
+#!/usr/bin/env python
+"""bench.py — sustained items/s at zero deadline misses of the enforced-waiting executor.
+
+Metric (BASELINE.json): "items/s at 0 deadline misses; SM utilisation vs no-wait baseline".
+Workload (BASELINE.json configs[1]): the BLAST-style 4-stage pipeline
+(seed lookup -> hit enumeration -> ungapped window filter -> X-drop extension) on a seeded
+synthetic 1 Mbp DB with a 1 kbp query and 64 planted matches, split into 148 independent
+streams (one CTA each) on one B200; the physical %globaltimer clock (1 unit = 1 ns).
+
+One step = one executor launch over the whole c2 DB (all streams).  Before timing:
+  1. gains g_i from a logical-clock run; service-time budgets t_i from a physical run
+     with generous budgets (longest firing x 1.25 + 256 ns);
+  2. the deadline D (default 350 us = the paper's largest D, 3.5e5 units, L212) and
+     b = (1, 3, 9, 6) (L230); Fig. 1 solved by the library for w_i;
+  3. tau0 = the smallest inter-arrival (ns) whose physical run has zero deadline misses,
+     zero budget overruns and no queue overflow.
+value = roots processed / device time of the timed launches (CUDA events on the launch
+stream, L2 flushed between steps), whole job over all ranks (max-over-ranks time).
+The monolithic no-internal-wait baseline (§5, Fig. 2) runs at the same tau0, D.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import math
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+from plgen import configs as C  # noqa: E402
+from plgen import dna as G  # noqa: E402
+
+METRIC = "items/s at 0 deadline misses; SM utilisation vs no-wait baseline"
+WORKLOAD = ("c2: BLAST seed-lookup -> hit-enumeration -> ungapped-window -> x-drop, 1 Mbp synthetic DB "
+            "(seed 2 + rank), 1 kbp query, 64 planted matches, 148 streams (1 CTA each) per GPU")
+
+
+def parse():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=20)
+    ap.add_argument("--warmup", type=int, default=5)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--deadline-ns", type=int, default=350_000)
+    ap.add_argument("--streams", type=int, default=148)
+    ap.add_argument("--cpu-sample-streams", type=int, default=148)
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-e2e", action="store_true")
+    return ap.parse_args()
+
+
+# ------------------------------------------------------------------ clocks
+class ClockSampler:
+    """nvidia-smi clocks/throttle sampling during the timed region (B200_PROFILING.md)."""
+    Q = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.hw_slowdown,"
+         "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
+         "clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, device):
+        self.device = device
+        self.rows = []
+        self.proc = None
+
+    def start(self):
+        try:
+            self.proc = subprocess.Popen(["nvidia-smi", f"--query-gpu={self.Q}", "--format=csv,noheader,nounits",
+                                          "-lms", "100", "-i", str(self.device)], stdout=subprocess.PIPE,
+                                         stderr=subprocess.DEVNULL, text=True)
+            self.th = threading.Thread(target=self._read, daemon=True)
+            self.th.start()
+        except OSError:
+            self.proc = None
+
+    def _read(self):
+        for line in self.proc.stdout:
+            self.rows.append([x.strip() for x in line.split(",")])
+
+    def stop(self):
+        if self.proc is None:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        time.sleep(0.25)
+        self.proc.terminate()
+        try:
+            self.proc.wait(timeout=2)
+        except subprocess.TimeoutExpired:
+            self.proc.kill()
+        sm = [float(r[1]) for r in self.rows if len(r) >= 8 and r[1].replace(".", "").isdigit()]
+        mx = [float(r[2]) for r in self.rows if len(r) >= 8 and r[2].replace(".", "").isdigit()]
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        reasons = sorted({names[k] for r in self.rows if len(r) >= 8 for k in range(4) if r[4 + k] == "Active"})
+        return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": max(mx) if mx else None,
+                "reasons": reasons, "samples": len(self.rows)}
+
+
+def peaks():
+    try:
+        with open(os.path.join(ROOT, "MEASURED_PEAKS.json")) as f:
+            return json.load(f)["hbm_gbs"], "measured (MEASURED_PEAKS.json)"
+    except (OSError, KeyError, ValueError):
+        return 6650.0, "fallback (B200_PROFILING.md)"
+
+
+def ncu_traffic():
+    """dram bytes per launch of the executor from the committed ncu --set full capture."""
+    try:
+        with open(os.path.join(ROOT, "profiles", "ncu_summary.json")) as f:
+            return json.load(f).get("dram_bytes_per_launch")
+    except (OSError, ValueError):
+        return None
+
+
+# --------------------------------------------------------------- oracle leg
+def _oracle_stream(args):
+    cfg, lo, hi = args
+    from oracle import des
+    wl = _ORACLE_WL
+    from oracle import stages as S
+    ctx = S.DnaContext(wl.db, wl.db_len, wl.query, wl.q_len, cfg.stages[0].iparam[0])
+    fns = des.make_stage_fns(cfg, ctx)
+    r = des.simulate_stream(cfg, fns, lo, hi)
+    return hi - lo, r.lat and max(r.lat)
+
+
+_ORACLE_WL = None
+
+
+def oracle_rate(cfg, wl, n_streams, procs=None):
+    """The oracle DES (as it stands) on `n_streams` streams of the workload, over a
+    process pool on the host cores.  Returns (items/s, cores, seconds, roots)."""
+    global _ORACLE_WL
+    import multiprocessing as mp
+    _ORACLE_WL = wl
+    from oracle import des
+    k = cfg.stages[0].iparam[0]
+    total = wl.db_len - k + 1
+    rng = des.stream_ranges(cfg, total)[:n_streams]
+    cores = procs or len(os.sched_getaffinity(0))
+    t0 = time.perf_counter()
+    with mp.get_context("fork").Pool(cores) as pool:
+        res = pool.map(_oracle_stream, [(cfg, lo, hi) for lo, hi in rng], chunksize=1)
+    dt = time.perf_counter() - t0
+    roots = sum(r[0] for r in res)
+    return roots / dt, cores, dt, roots
+
+
+def logical_cfg(base):
+    from paper_conf_icppw_planob21_b200 import solve_enforced_waits
+    w, th, T, Tc = solve_enforced_waits(base.replace(gain=C.TABLE1_G))
+    return base.replace(wait_time=tuple(w), gain=C.TABLE1_G)
+
+
+# -------------------------------------------------------------- reference arm
+def run_reference(a):
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return
+    base = C.c2(n_streams=a.streams)
+    wl = G.make_dna(base.seed, **base.dna)
+    cfg = logical_cfg(base)
+    n = min(a.cpu_sample_streams, a.streams)
+    for _ in range(a.warmup):
+        oracle_rate(cfg, wl, max(1, n // 8))
+    times, roots = [], 0
+    for _ in range(a.steps):
+        rate, cores, dt, r = oracle_rate(cfg, wl, n)
+        times.append(dt)
+        roots = r
+    V = roots * a.steps / sum(times)
+    line = {"metric": METRIC, "value": V, "unit": "items/s", "n_gpus": a.gpus, "steps": a.steps,
+            "warmup": a.warmup, "ms_per_step": 1e3 * sum(times) / a.steps, "higher_is_better": True,
+            "scaling": "weak", "vs_baseline": None, "dtype": "int64", "data": "synthetic",
+            "impl": "reference",
+            "config": {"workload": WORKLOAD, "policy": "FIXED_WAIT", "clock": "logical (oracle DES)"},
+            "cpu_baseline": {"value": V, "unit": "items/s", "cores": cores, "kind": "oracle",
+                             "sample": f"{n} of {a.streams} c2 streams ({roots} roots) per step"},
+            "e2e": {"value": V, "unit": "items/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+
+
+# ------------------------------------------------------------------ our arm
+def main():
+    a = parse()
+    if a.impl == "reference":
+        run_reference(a)
+        return
+    import torch
+    import torch.distributed as dist
+    from paper_conf_icppw_planob21_b200 import Pipeline, realtime
+    from paper_conf_icppw_planob21_b200.dist import allreduce_stats
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=dev)
+    log = (lambda d: print(json.dumps(d), file=sys.stderr, flush=True)) if rank == 0 else (lambda d: None)
+
+    base = C.c2(n_streams=a.streams, seed=2 + rank)
+    wl = G.make_dna(base.seed, **base.dna)
+    db_dev = torch.from_numpy(wl.db.view("int32")).to(dev)
+    db_ptr = db_dev.data_ptr()
+    stream = torch.cuda.current_stream(dev)
+
+    # 1. gains (logical run) and budgets (physical run)
+    gains = realtime.measure_gains(base.replace(wait_time=(0,) * 4), wl, db_ptr, stream=stream)
+    budgets, cal = realtime.calibrate_budgets(base, wl, db_ptr, stream=stream)
+    if world > 1:   # every rank runs the same schedule: max budgets / min gains are conservative
+        t = torch.tensor(budgets, dtype=torch.int64, device=dev)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        budgets = tuple(int(x) for x in t.tolist())
+    log({"gains": gains, "budgets_ns": budgets, "cal_max_fire_ns": cal["max_fire_ns"]})
+    cfg = base.replace(clock=1, ns_per_unit=1.0, service_time=budgets, gain=gains, deadline=a.deadline_ns,
+                       b=C.PAPER_B)
+    # 2./3. the fastest miss-free rate
+    tau, w, th, T, st_ok = realtime.find_rate(cfg, wl, db_ptr, stream=stream, log=log)
+    if world > 1:
+        t = torch.tensor([tau], dtype=torch.int64, device=dev)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        if int(t.item()) != tau:
+            tau = int(t.item())
+            w, th, T = realtime.solve_at(cfg, tau)
+    run_cfg = cfg.replace(interarrival=tau, wait_time=tuple(w))
+    pl = Pipeline(run_cfg, wl, flags=0, stream=stream)
+    pl.bind_device(db_ptr, wl.db_len)
+    flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)
+
+    for _ in range(a.warmup):
+        pl.launch()
+    torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    clocks = ClockSampler(local)
+    clocks.start()
+    ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(a.steps)]
+    misses = 0
+    overruns = 0
+    errors = 0
+    roots = 0
+    torch.cuda.synchronize()
+    for k in range(a.steps):
+        flush.zero_()                                  # L2 flush, outside the timed region
+        ev[k][0].record(stream)
+        pl.launch()
+        ev[k][1].record(stream)
+        st = pl.stats()                                # syncs; outside the timed region
+        misses += st["miss_events"]
+        overruns += sum(st["overruns"])
+        errors |= st["errors"]
+        roots += st["roots"]
+    torch.cuda.synchronize()
+    clk = clocks.stop()
+    step_ms = [e0.elapsed_time(e1) for e0, e1 in ev]
+    tot_ms = sum(step_ms)
+    if world > 1:
+        dist.barrier()
+    st_last = allreduce_stats(dict(st, policy=0), device=dev)
+    tt = torch.tensor([tot_ms], dtype=torch.float64, device=dev)
+    cnt = torch.tensor([roots, misses, overruns], dtype=torch.int64, device=dev)
+    if world > 1:
+        dist.all_reduce(tt, op=dist.ReduceOp.MAX)
+        dist.all_reduce(cnt, op=dist.ReduceOp.SUM)
+    tot_ms = float(tt.item())
+    roots_all, misses_all, overruns_all = (int(x) for x in cnt.tolist())
+    value = roots_all / (tot_ms * 1e-3)
+
+    # logical-clock throughput of the same executor (no real-time pacing)
+    lc = logical_cfg(base)
+    pll = Pipeline(lc, wl, flags=0, stream=stream)
+    pll.bind_device(db_ptr, wl.db_len)
+    for _ in range(3):
+        pll.launch()
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    torch.cuda.synchronize()
+    e0.record(stream)
+    for _ in range(5):
+        pll.launch()
+    e1.record(stream)
+    torch.cuda.synchronize()
+    logical_ips = 5 * pll.stats()["roots"] / (e0.elapsed_time(e1) * 1e-3)
+    pll.close()
+
+    # monolithic baseline at the same (tau0, D)
+    mono = {}
+    Mr = realtime.monolithic_at(cfg, tau)
+    if Mr is not None:
+        M, Tm = Mr
+        plm = Pipeline(cfg.replace(interarrival=tau, policy=2, block_size=M), wl, flags=1, stream=stream)
+        plm.bind_device(db_ptr, wl.db_len)
+        plm.drain()
+        sm = plm.stats()
+        plm.close()
+        mono = {"M": M, "fig2_objective": Tm, "active_fraction": sm["active_fraction"],
+                "hw_busy_fraction": sm["hw_busy_fraction"], "misses": sm["misses"],
+                "max_latency_ns": sm["max_latency_ns"]}
+    else:
+        mono = {"feasible": False}
+
+    # e2e through the C-ABI with host buffers (H2D of the DB and D2H of the stats each step)
+    e2e = None
+    if not a.no_e2e:
+        host = torch.from_numpy(wl.db.view("int32")).pin_memory()
+        ple = Pipeline(run_cfg, wl, flags=0, stream=stream)
+        for _ in range(2):
+            ple.push_ptr(host.data_ptr(), wl.db_len)
+            ple.drain()
+            ple.stats()
+            ple.rewind()
+        s0 = ple.stats()
+        torch.cuda.synchronize()
+        t0 = time.perf_counter()
+        e_roots = 0
+        for _ in range(a.steps):
+            ple.push_ptr(host.data_ptr(), wl.db_len)
+            ple.drain()
+            se = ple.stats()
+            e_roots += se["roots"]
+            ple.rewind()
+        e_dt = time.perf_counter() - t0
+        s1 = ple.stats()
+        ple.close()
+        et = torch.tensor([e_dt], dtype=torch.float64, device=dev)
+        er = torch.tensor([e_roots], dtype=torch.int64, device=dev)
+        if world > 1:
+            dist.all_reduce(et, op=dist.ReduceOp.MAX)
+            dist.all_reduce(er, op=dist.ReduceOp.SUM)
+        e2e = {"value": int(er.item()) / float(et.item()), "unit": "items/s",
+               "h2d_bytes_per_step": (s1["h2d_bytes"] - s0["h2d_bytes"]) // a.steps,
+               "d2h_bytes_per_step": (s1["d2h_bytes"] - s0["d2h_bytes"]) // a.steps}
+
+    # roofline of the dominant kernel (the executor): algorithmic bytes / launch time
+    pk, pk_src = peaks()
+    bytes_per_launch = 0.25 * st_last["roots"] / max(1, world) + 24.0 * st["matches"]
+    achieved = bytes_per_launch / (tot_ms / a.steps * 1e-3) / 1e9
+    cpu = None
+    if rank == 0 and not a.no_cpu_baseline:
+        rate, cores, dt, r = oracle_rate(logical_cfg(base), wl, min(a.cpu_sample_streams, a.streams))
+        cpu = {"value": rate, "unit": "items/s", "cores": cores, "kind": "oracle",
+               "sample": f"{min(a.cpu_sample_streams, a.streams)} of {a.streams} c2 streams ({r} roots), "
+                         f"logical clock, Table-1 timing, {dt:.1f} s"}
+    if rank == 0:
+        line = {
+            "metric": METRIC, "value": value, "unit": "items/s", "n_gpus": world, "steps": a.steps,
+            "warmup": a.warmup, "ms_per_step": tot_ms / a.steps, "higher_is_better": True, "scaling": "weak",
+            "vs_baseline": None, "dtype": "int32", "data": "synthetic",
+            "config": {"workload": WORKLOAD, "policy": "FIXED_WAIT", "clock": "globaltimer (1 unit = 1 ns)",
+                       "deadline_ns": a.deadline_ns, "tau0_ns": tau, "b": list(C.PAPER_B),
+                       "budgets_ns": list(budgets), "w_ns": list(w), "gains": [round(g, 5) for g in gains],
+                       "streams_per_gpu": a.streams, "l2": "flushed between timed steps (256 MiB memset)",
+                       "parallelism": f"{a.streams} streams x {world} GPUs (independent; NCCL stats all-reduce)"},
+            "misses": misses_all, "overruns": overruns_all, "errors": errors,
+            "sustained_items_per_s": world * a.streams * 1e9 / tau,
+            "logical_items_per_s": logical_ips,
+            "utilisation": {"enforced_model": st_last["active_fraction"], "enforced_fig1_T": T,
+                            "enforced_hw_busy": st["hw_busy_fraction"], "monolithic": mono},
+            "clocks": clk,
+            "e2e": e2e,
+            "gpu_launches": a.steps,
+            "roofline": {"bound": "hbm", "achieved": achieved, "peak": pk, "unit": "GB/s", "frac": achieved / pk,
+                         "traffic": ncu_traffic(), "peak_source": pk_src,
+                         "algorithmic_bytes_per_launch": bytes_per_launch},
+            "cpu_baseline": cpu,
+        }
+        print(json.dumps(line), flush=True)
+    pl.close()
+    if world > 1:
+        dist.barrier()
+        dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

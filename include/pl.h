@@ -151,6 +151,11 @@ typedef struct {
   uint64_t overruns[PL_MAX_STAGES];        /* physical: firings longer than t_i        */
   int64_t  max_lateness_ns[PL_MAX_STAGES]; /* physical: max(actual - scheduled start)  */
   uint64_t sched_cycles[PL_MAX_STAGES];    /* clock64 cycles spent deciding firings    */
+  int64_t  max_fire_ns[PL_MAX_STAGES];     /* physical: longest firing (start->publish) */
+  /* leader-lane clock64 cycles per phase of a firing, summed over firings:
+   * [0] decide (scheduler), [1] release barrier, [2] load+stage+scan,
+   * [3] records+reserve, [4] output writes, [5] publish                        */
+  uint64_t phase_cycles[PL_MAX_STAGES][6];
   uint64_t matches;
   uint64_t miss_events;                    /* terminal events with latency > D        */
   uint64_t misses;                         /* distinct roots (needs PL_REC_LATENCY)    */
@@ -164,6 +169,8 @@ typedef struct {
   int64_t  wall_ns;                        /* max over streams of kernel-side runtime  */
   uint32_t errors;                         /* PL_EOVERFLOW bits etc.                   */
   uint32_t launches;                       /* executor launches so far                 */
+  uint64_t h2d_bytes;                      /* host->device bytes copied by this handle (cumulative) */
+  uint64_t d2h_bytes;                      /* device->host bytes copied by this handle (cumulative) */
 } pl_stats;
 
 typedef struct pl_pipeline pl_pipeline;

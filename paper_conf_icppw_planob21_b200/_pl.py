@@ -61,19 +61,23 @@ class pl_stats(C.Structure):
     _fields_ = [("n_stages", C.c_uint32), ("n_streams", C.c_uint32), ("roots", C.c_uint64),
                 ("firings", _A8), ("empty_firings", _A8), ("consumed", _A8), ("produced", _A8),
                 ("active_window", _I8), ("busy_ns", _I8), ("spilled", _A8), ("overruns", _A8),
-                ("max_lateness_ns", _I8), ("sched_cycles", _A8), ("matches", C.c_uint64),
+                ("max_lateness_ns", _I8), ("sched_cycles", _A8), ("max_fire_ns", _I8),
+                ("phase_cycles", (C.c_uint64 * 6) * PL_MAX_STAGES), ("matches", C.c_uint64),
                 ("miss_events", C.c_uint64), ("misses", C.c_uint64), ("max_latency", C.c_int64),
                 ("max_latency_ns", C.c_int64), ("window", C.c_int64), ("t_end", C.c_int64),
                 ("active_fraction", C.c_double), ("active_fraction_nonempty", C.c_double),
                 ("hw_busy_fraction", C.c_double), ("wall_ns", C.c_int64), ("errors", C.c_uint32),
-                ("launches", C.c_uint32)]
+                ("launches", C.c_uint32), ("h2d_bytes", C.c_uint64), ("d2h_bytes", C.c_uint64)]
 
     def as_dict(self):
         N = self.n_stages
         out = {}
         for name, _ in self._fields_:
             val = getattr(self, name)
-            out[name] = list(val)[:N] if hasattr(val, "__len__") else val
+            if name == "phase_cycles":
+                out[name] = [list(val[i]) for i in range(N)]
+            else:
+                out[name] = list(val)[:N] if hasattr(val, "__len__") else val
         return out
 
 

@@ -54,53 +54,89 @@ __device__ __forceinline__ uint64_t gain_hash(uint64_t seed, uint32_t stage, uin
 }
 
 // ------------------------------------------------------------------ DNA access
+// The DB is read through a per-stream smem window (staged by a TMA bulk copy at
+// CTA start, cta_setup) with an __ldg fallback outside it.  Extensions compare 16
+// bases per step: XOR of two 2-bit-packed 32-bit windows gives a mismatch mask.
 struct Dna {
-  const uint32_t* db;
+  const uint32_t* db;      // packed DB (global)
   uint32_t nwords;
   uint64_t db_len;
-  const uint32_t* qw;      // query words (smem)
+  const uint32_t* win;     // smem copy of DB words [win_lo, win_lo + win_n)
+  int64_t win_lo;
+  uint32_t win_n;
+  const uint32_t* qw;      // query words (smem), nqw valid words
+  uint32_t nqw;
   const uint16_t* qoff;    // smem
   const uint16_t* qpos;    // smem
   int k, q_len;
-  __device__ __forceinline__ uint32_t dbw(uint32_t w) const { return w < nwords ? __ldg(db + w) : 0u; }
-  __device__ __forceinline__ uint32_t dbase(uint32_t j) const { return (dbw(j >> 4) >> ((j & 15) * 2)) & 3u; }
-  __device__ __forceinline__ uint32_t qbase(uint32_t j) const { return (qw[j >> 4] >> ((j & 15) * 2)) & 3u; }
+  __device__ __forceinline__ uint32_t dbw(int64_t w) const {
+    const uint64_t r = (uint64_t)(w - win_lo);
+    if (r < win_n) return win[r];
+    return (w >= 0 && w < (int64_t)nwords) ? __ldg(db + w) : 0u;
+  }
+  __device__ __forceinline__ uint32_t qww(int64_t w) const { return (w >= 0 && w < (int64_t)nqw) ? qw[w] : 0u; }
+  // bases s..s+15 (base s in bits 0-1); s may be negative (out-of-range bases read as 0)
+  __device__ __forceinline__ uint32_t db16(int64_t s) const {
+    const int64_t w = s >> 4;
+    return __funnelshift_r(dbw(w), dbw(w + 1), (uint32_t)(s & 15) * 2u);
+  }
+  __device__ __forceinline__ uint32_t q16(int64_t s) const {
+    const int64_t w = s >> 4;
+    return __funnelshift_r(qww(w), qww(w + 1), (uint32_t)(s & 15) * 2u);
+  }
   // key(db, p) = sum_{j<k} db[p+j] 4^(k-1-j)  (first base most significant; R-S0)
   __device__ __forceinline__ uint32_t key(uint32_t p) const {
-    uint64_t x = (((uint64_t)dbw((p >> 4) + 1) << 32) | dbw(p >> 4)) >> ((p & 15) * 2);
+    const uint32_t x = db16(p);
     uint32_t key = 0;
-#pragma unroll 7
+#pragma unroll
     for (int j = 0; j < PL_MAX_K; ++j)
-      if (j < k) key = (key << 2) | (uint32_t)((x >> (2 * j)) & 3u);
+      if (j < k) key = (key << 2) | ((x >> (2 * j)) & 3u);
     return key;
   }
-  // best extension to the right of the seed (db[p+k-1+d] vs query[q+k-1+d]), d <= W
-  // or X-drop (W < 0).  Returns best score (>= 0) and smallest d attaining it.
-  __device__ __forceinline__ int ext_right(uint32_t p, uint32_t q, int W, int X, int* dbest) const {
+  // Walk d = 1..limit away from the seed scoring +1/-3 (R-S2/R-S3); stop early on
+  // X-drop (X > 0: score <= best - X).  Returns best (>= 0) and the smallest d
+  // attaining it.  dir = +1: db[p+k-1+d] vs query[q+k-1+d]; dir = -1: db[p-d] vs query[q-d].
+  __device__ __forceinline__ int extend(uint32_t p, uint32_t q, int dir, int64_t limit, int X, int* dbest) const {
     int score = 0, best = 0, db_ = 0;
-    uint64_t i = (uint64_t)p + k, j = (uint64_t)q + k;   // first position right of the seed
-    for (int d = 1;; ++d, ++i, ++j) {
-      if (W >= 0 && d > W) break;
-      if (i >= db_len || j >= (uint64_t)q_len) break;
-      score += (dbase((uint32_t)i) == qbase((uint32_t)j)) ? 1 : -3;
-      if (score > best) { best = score; db_ = d; }
-      if (X > 0 && score <= best - X) break;
+    int64_t d = 0;
+    while (d < limit) {
+      const int64_t n = (limit - d) < 16 ? (limit - d) : 16;
+      uint32_t mm;   // bit 2e set <=> mismatch at step d+1+e
+      if (dir > 0) {
+        const uint32_t x = db16((int64_t)p + k + d) ^ q16((int64_t)q + k + d);
+        mm = (x | (x >> 1)) & 0x55555555u;
+      } else {
+        // window ending at p-d-1: step d+1+e is window position 15-e -> bit-reverse the pairs
+        const uint32_t x = db16((int64_t)p - d - 16) ^ q16((int64_t)q - d - 16);
+        mm = __brev((x | (x >> 1)) & 0x55555555u) >> 1;
+      }
+      // Between mismatches the score rises by 1 per step, so the running best can
+      // only be set just before a mismatch (or at the chunk end) and an x-drop can
+      // only happen just after one: visit the mismatch steps only.
+      uint32_t mmv = mm & (n >= 16 ? 0xffffffffu : ((1u << (2 * n)) - 1u));
+      int last = 0;                      // steps of this chunk already scored
+      while (mmv) {
+        const int e = (__ffs(mmv) - 1) >> 1;   // mismatch at step d+1+e
+        mmv &= mmv - 1;
+        score += e - last;               // matches at steps last+1 .. e (1-based within chunk)
+        if (score > best) { best = score; db_ = (int)(d + e); }
+        score -= 3;
+        last = e + 1;
+        if (X > 0 && score <= best - X) { *dbest = db_; return best; }
+      }
+      score += (int)n - last;
+      if (score > best) { best = score; db_ = (int)(d + n); }
+      d += n;
     }
     *dbest = db_;
     return best;
   }
-  __device__ __forceinline__ int ext_left(uint32_t p, uint32_t q, int W, int X, int* dbest) const {
-    int score = 0, best = 0, db_ = 0;
-    for (int d = 1;; ++d) {
-      if (W >= 0 && d > W) break;
-      if ((uint32_t)d > p || (uint32_t)d > q) break;
-      score += (dbase(p - d) == qbase(q - d)) ? 1 : -3;
-      if (score > best) { best = score; db_ = d; }
-      if (X > 0 && score <= best - X) break;
-    }
-    *dbest = db_;
-    return best;
+  __device__ __forceinline__ int64_t right_limit(uint32_t p, uint32_t q) const {
+    const int64_t a = (int64_t)db_len - ((int64_t)p + k), b = (int64_t)q_len - ((int64_t)q + k);
+    const int64_t m = a < b ? a : b;
+    return m > 0 ? m : 0;
   }
+  __device__ __forceinline__ int64_t left_limit(uint32_t p, uint32_t q) const { return p < q ? p : q; }
 };
 
 // --------------------------------------------------------------- shared state
@@ -130,6 +166,7 @@ struct Shared {
   uint32_t errors;
   uint32_t log_count;       // firing-log records reserved by all nodes of this stream
   uint64_t T0;
+  alignas(8) uint64_t mbar; // TMA completion barrier for the DB window
 };
 
 struct Ctx {
@@ -145,78 +182,137 @@ struct Ctx {
 
 __device__ __forceinline__ int64_t arrival(const Ctx& c, uint32_t root) { return (int64_t)(root - c.lo) * c.p->tau; }
 
-// location of sequence number s of edge i: spilled iff it lies in a spilled segment
-__device__ __forceinline__ uint2 load_entry(const Ctx& c, int i, uint32_t s, uint32_t segh, uint32_t st,
-                                            uint32_t spill_end) {
+// floor(a / b) for a >= 0, b > 0 without a 64-bit integer division (double estimate + fix-up)
+__device__ __forceinline__ int64_t fdiv(int64_t a, int64_t b) {
+  int64_t q = (int64_t)((double)a / (double)b);
+  while (q > 0 && q * b > a) --q;
+  while ((q + 1) * b <= a) ++q;
+  return q;
+}
+__device__ __forceinline__ int64_t cdiv(int64_t a, int64_t b) { return a <= 0 ? 0 : fdiv(a - 1, b) + 1; }
+
+// Per-node constants, built once per warp group and kept in registers.
+struct Node {
+  int i, N, v;
+  bool sink, phys, fixed;
+  int64_t t, P, R, D, tau, X, H;
+  uint32_t theta;
+  uint64_t lo;
+  double nspu;
+  uint32_t segmask, capg;
+  EdgeCtl* Ein;                 // input edge (i > 0)
+  const uint2* in_ent;
+  const Seg* in_seg;
+  const uint2* in_spill;
+  uint32_t in_mask;
+  EdgeCtl* Eout;                // output edge (i < N-1)
+  uint2* out_ent;
+  Seg* out_seg;
+  uint2* out_spill;
+  uint32_t out_cap;
+  uint32_t kind, max_out, cfix, umax;
+  int32_t ip1, ip2;
+  __device__ __forceinline__ int64_t arrival(uint32_t root) const { return (int64_t)(root - lo) * tau; }
+};
+
+__device__ __forceinline__ Node make_node(const Ctx& c, int i) {
   const DevParams& p = *c.p;
-  if ((int32_t)(s - spill_end) >= 0) return c.ent[i][s & (p.cap_s[i] - 1)];
-  // binary search the live segments [segh, st) for the first with end > s
+  Node n;
+  n.i = i; n.N = p.N; n.v = p.v;
+  n.sink = i == p.N - 1;
+  n.phys = p.clock == PL_CLOCK_GLOBALTIMER;
+  n.fixed = p.policy == PL_FIXED_WAIT;
+  n.t = p.t[i]; n.P = p.P[i]; n.R = p.R[i]; n.D = p.D; n.tau = p.tau; n.X = c.X; n.H = c.H;
+  n.theta = p.theta[i];
+  n.lo = c.lo;
+  n.nspu = p.ns_per_unit;
+  n.segmask = p.segcap - 1;
+  n.capg = p.cap_g;
+  n.Ein = &c.sh->e[i];
+  n.in_ent = c.ent[i]; n.in_seg = c.seg[i]; n.in_spill = c.spill[i];
+  n.in_mask = p.cap_s[i] ? p.cap_s[i] - 1 : 0;
+  const int o = i + 1 < p.N ? i + 1 : i;
+  n.Eout = &c.sh->e[o];
+  n.out_ent = c.ent[o]; n.out_seg = c.seg[o]; n.out_spill = c.spill[o];
+  n.out_cap = p.cap_s[o];
+  const DevStage& s = p.st[i];
+  n.kind = s.kind; n.max_out = s.max_out; n.cfix = s.cfix;
+  n.umax = s.kind == PL_FIXED_GAIN ? s.cfix : s.max_out;
+  n.ip1 = s.ip[1]; n.ip2 = s.ip[2];
+  return n;
+}
+
+// Entry with sequence number s of the node's input edge: spilled iff it lies in
+// a spilled segment (binary search of the live segments [segh, st)).
+__device__ __forceinline__ uint2 load_entry(const Node& nd, uint32_t s, uint32_t segh, uint32_t st,
+                                            uint32_t spill_end) {
+  if ((int32_t)(s - spill_end) >= 0) return nd.in_ent[s & nd.in_mask];
   uint32_t lo = segh, hi = st;
   while (lo < hi) {
-    uint32_t mid = lo + ((hi - lo) >> 1);
-    if ((int32_t)(c.seg[i][mid & (p.segcap - 1)].end - s) > 0) hi = mid; else lo = mid + 1;
+    const uint32_t mid = lo + ((hi - lo) >> 1);
+    if ((int32_t)(nd.in_seg[mid & nd.segmask].end - s) > 0) hi = mid; else lo = mid + 1;
   }
-  if (c.seg[i][lo & (p.segcap - 1)].loc == LOC_SPILL) return __ldcg(c.spill[i] + (s & (p.cap_g - 1)));
-  return c.ent[i][s & (p.cap_s[i] - 1)];
+  if (nd.in_seg[lo & nd.segmask].loc == LOC_SPILL) return __ldcg(nd.in_spill + (s & (nd.capg - 1)));
+  return nd.in_ent[s & nd.in_mask];
 }
 
 // ------------------------------------------------------------ stage functions
 // Phase A: number of outputs of one input entry (and per-lane state for phase B).
 struct LaneOut {
   uint32_t c;       // outputs
-  uint32_t a, b;    // kind-specific state (S1: off; S3: db_start|len ...)
-  int32_t score;
+  uint32_t a;       // S1: offset into the query position list; S3: db_start
+  int32_t score;    // S3
   uint32_t q_start, len;
 };
 
-__device__ __forceinline__ LaneOut stage_count(const Ctx& c, int i, uint2 e) {
-  const DevParams& p = *c.p;
-  const DevStage& s = p.st[i];
+__device__ __forceinline__ LaneOut stage_count(const Node& nd, const Dna& dna, const DevParams& p, uint2 e) {
   LaneOut o;
-  o.c = 0; o.a = 0; o.b = 0; o.score = 0; o.q_start = 0; o.len = 0;
-  switch (s.kind) {
-    case PL_BERNOULLI: o.c = gain_hash(p.seed, i, e.x, e.y) < s.thr[0] ? 1u : 0u; break;
-    case PL_FIXED_GAIN: o.c = s.cfix; break;
+  o.c = 0; o.a = 0; o.score = 0; o.q_start = 0; o.len = 0;
+  switch (nd.kind) {
+    case PL_BERNOULLI: o.c = gain_hash(p.seed, nd.i, e.x, e.y) < p.st[nd.i].thr[0] ? 1u : 0u; break;
+    case PL_FIXED_GAIN: o.c = nd.cfix; break;
     case PL_POISSON_CAPPED: {
-      uint64_t h = gain_hash(p.seed, i, e.x, e.y);
+      const uint64_t h = gain_hash(p.seed, nd.i, e.x, e.y);
       uint32_t n = 0;
-      for (uint32_t k = 0; k < s.max_out; ++k) n += (h >= s.thr[k]) ? 1u : 0u;
+      for (uint32_t k = 0; k < nd.max_out; ++k) n += (h >= p.st[nd.i].thr[k]) ? 1u : 0u;
       o.c = n;
       break;
     }
-    case PL_KEEP_EVERY: o.c = (e.x % s.cfix) == 0 ? 1u : 0u; break;
+    case PL_KEEP_EVERY: o.c = (e.x % nd.cfix) == 0 ? 1u : 0u; break;
     case PL_SEED_LOOKUP: {
-      uint32_t key = c.dna.key(e.x);
-      o.c = c.dna.qoff[key + 1] > c.dna.qoff[key] ? 1u : 0u;
+      const uint32_t key = dna.key(e.x);
+      o.c = dna.qoff[key + 1] > dna.qoff[key] ? 1u : 0u;
       break;
     }
     case PL_HIT_ENUM: {
-      uint32_t key = c.dna.key(e.x);
-      uint32_t off = c.dna.qoff[key], cnt = c.dna.qoff[key + 1] - off;
+      const uint32_t key = dna.key(e.x);
+      const uint32_t off = dna.qoff[key], cnt = dna.qoff[key + 1] - off;
       o.a = off;
-      o.c = cnt < s.max_out ? cnt : s.max_out;
+      o.c = cnt < nd.max_out ? cnt : nd.max_out;
       break;
     }
     case PL_UNGAPPED_WINDOW: {
-      uint32_t q = e.y & 0xffffu;
+      const uint32_t q = e.y & 0xffffu;
+      const int64_t W = nd.ip1;
       int d;
-      int bl = c.dna.ext_left(e.x, q, s.ip[1], 0, &d);
-      int br = c.dna.ext_right(e.x, q, s.ip[1], 0, &d);
-      o.c = (c.dna.k + bl + br >= s.ip[2]) ? 1u : 0u;
+      const int64_t ll = dna.left_limit(e.x, q), rl = dna.right_limit(e.x, q);
+      const int bl = dna.extend(e.x, q, -1, ll < W ? ll : W, 0, &d);
+      const int br = dna.extend(e.x, q, +1, rl < W ? rl : W, 0, &d);
+      o.c = (dna.k + bl + br >= nd.ip2) ? 1u : 0u;
       break;
     }
     case PL_UNGAPPED_XDROP: {
-      uint32_t q = e.y & 0xffffu;
+      const uint32_t q = e.y & 0xffffu;
       int dl, dr;
-      int bl = c.dna.ext_left(e.x, q, -1, s.ip[1], &dl);
-      int br = c.dna.ext_right(e.x, q, -1, s.ip[1], &dr);
-      int score = c.dna.k + bl + br;
-      if (score >= s.ip[2]) {
+      const int bl = dna.extend(e.x, q, -1, dna.left_limit(e.x, q), nd.ip1, &dl);
+      const int br = dna.extend(e.x, q, +1, dna.right_limit(e.x, q), nd.ip1, &dr);
+      const int score = dna.k + bl + br;
+      if (score >= nd.ip2) {
         o.c = 1;
         o.score = score;
         o.a = e.x - dl;
         o.q_start = q - dl;
-        o.len = c.dna.k + dl + dr;
+        o.len = dna.k + dl + dr;
       }
       break;
     }
@@ -225,12 +321,11 @@ __device__ __forceinline__ LaneOut stage_count(const Ctx& c, int i, uint2 e) {
 }
 
 // Phase B: output j of an entry (non-sink nodes).
-__device__ __forceinline__ uint2 stage_output(const Ctx& c, int i, uint2 e, const LaneOut& o, uint32_t j) {
-  const DevStage& s = c.p->st[i];
-  switch (s.kind) {
-    case PL_FIXED_GAIN: return make_uint2(e.x, e.y * s.cfix + j);
-    case PL_POISSON_CAPPED: return make_uint2(e.x, e.y * s.max_out + j);
-    case PL_HIT_ENUM: return make_uint2(e.x, (uint32_t)c.dna.qpos[o.a + j] | (j << 16));
+__device__ __forceinline__ uint2 stage_output(const Node& nd, const Dna& dna, uint2 e, const LaneOut& o, uint32_t j) {
+  switch (nd.kind) {
+    case PL_FIXED_GAIN: return make_uint2(e.x, e.y * nd.cfix + j);
+    case PL_POISSON_CAPPED: return make_uint2(e.x, e.y * nd.max_out + j);
+    case PL_HIT_ENUM: return make_uint2(e.x, (uint32_t)dna.qpos[o.a + j] | (j << 16));
     default: return e;
   }
 }
@@ -246,19 +341,18 @@ struct Leader {   // leader-private schedule state of one node
   int64_t m;      // FIXED_WAIT: index of the next firing
   int64_t B;      // THRESHOLD_SLACK: busy until
   uint64_t c0;    // node 0: roots consumed
-  uint32_t head, segh;      // consumer side of the input edge
+  uint32_t head, segh;          // consumer side of the input edge
   uint32_t out_tail, out_segt;  // producer side of the output edge
   int64_t W_pub;
   uint64_t empties;
-  uint64_t sched_cycles;
 };
 
-__device__ __forceinline__ void publish_W(Ctx& c, int i, Leader& L, int64_t w) {
-  if (i + 1 >= c.p->N) return;
+__device__ __forceinline__ void publish_W(const Node& nd, Leader& L, int64_t w) {
+  if (nd.sink) return;
   if (w > L.W_pub) {
     L.W_pub = w;
     __threadfence_block();
-    vst(&c.sh->e[i + 1].W, w);
+    vst(&nd.Eout->W, w);
   }
 }
 
@@ -268,142 +362,134 @@ __device__ __forceinline__ void backoff(int& spins) {
   ++spins;
 }
 
-// number of entries of edge i with ready <= T among the published ones (stops at v)
-__device__ __forceinline__ uint32_t count_le(const Ctx& c, int i, const Leader& L, uint32_t st, int64_t T,
-                                             uint32_t v) {
+// number of entries of the input edge with ready <= T among the published ones (stops at v)
+__device__ __forceinline__ uint32_t count_le(const Node& nd, const Leader& L, uint32_t st, int64_t T) {
   uint32_t end = L.head;
   for (uint32_t k = L.segh; k != st; ++k) {
-    const Seg& sg = c.seg[i][k & (c.p->segcap - 1)];
+    const Seg& sg = nd.in_seg[k & nd.segmask];
     if (sg.ready > T) break;
     end = sg.end;
-    if (end - L.head >= v) break;
+    if (end - L.head >= (uint32_t)nd.v) break;
   }
   return end - L.head;
 }
 
-__device__ Decision decide(Ctx& c, int i, Leader& L) {
-  const DevParams& p = *c.p;
-  const uint32_t v = (uint32_t)p.v;
-  const int64_t t_i = p.t[i];
+__device__ Decision decide(const Node& nd, Leader& L) {
+  const uint32_t v = (uint32_t)nd.v;
   Decision d;
   d.done = false; d.T = 0; d.n = 0;
   int spins = 0;
-  const bool fixed = p.policy == PL_FIXED_WAIT;
   for (;;) {
-    if (i == 0) {
-      // arrivals are fully known: root lo+r arrives at r*tau0 (L63)
-      const int64_t X = c.X;
-      if ((int64_t)L.c0 >= X) { d.done = true; return d; }
-      if (fixed) {
-        const int64_t P = p.P[0];
-        int64_t T = L.m * P;
-        int64_t arrived = T / p.tau + 1; if (arrived > X) arrived = X;
-        int64_t avail = arrived - (int64_t)L.c0;
-        if (avail <= 0) {   // empty firings until the next root has arrived
-          int64_t m2 = ceil_div64((int64_t)L.c0 * p.tau, P);
+    if (nd.i == 0) {
+      // arrivals are fully known: root lo+r arrives at r*tau0
+      if ((int64_t)L.c0 >= nd.X) { d.done = true; return d; }
+      int64_t T;
+      if (nd.fixed) {
+        T = L.m * nd.P;
+        if (T < (int64_t)L.c0 * nd.tau) {   // empty firings until the next root has arrived
+          const int64_t m2 = cdiv((int64_t)L.c0 * nd.tau, nd.P);
           L.empties += (uint64_t)(m2 - L.m);
           L.m = m2;
-          continue;
+          T = L.m * nd.P;
         }
-        d.T = T; d.n = (uint32_t)(avail < (int64_t)v ? avail : v);
-        return d;
       } else {
-        int64_t Tth = ((int64_t)L.c0 + p.theta[0] - 1 < X) ? ((int64_t)L.c0 + p.theta[0] - 1) * p.tau : PL_INF64;
-        int64_t ah = (int64_t)L.c0 * p.tau;
-        int64_t Tf = ah + p.D - p.R[0]; if (Tf < ah) Tf = ah;
-        int64_t T = Tth < Tf ? Tth : Tf; if (T < L.B) T = L.B;
-        int64_t arrived = T / p.tau + 1; if (arrived > X) arrived = X;
-        int64_t avail = arrived - (int64_t)L.c0;
-        d.T = T; d.n = (uint32_t)(avail < (int64_t)v ? avail : v);
-        return d;
+        const int64_t ah = (int64_t)L.c0 * nd.tau;
+        const int64_t Tth = ((int64_t)L.c0 + nd.theta - 1 < nd.X) ? ah + (int64_t)(nd.theta - 1) * nd.tau : PL_INF64;
+        int64_t Tf = ah + nd.D - nd.R;
+        if (Tf < ah) Tf = ah;
+        T = Tth < Tf ? Tth : Tf;
+        if (T < L.B) T = L.B;
       }
+      int64_t arrived = fdiv(T, nd.tau) + 1;
+      if (arrived > nd.X) arrived = nd.X;
+      const int64_t avail = arrived - (int64_t)L.c0;
+      d.T = T;
+      d.n = (uint32_t)(avail < (int64_t)v ? avail : v);
+      return d;
     }
     // node i >= 1: read the upstream watermark first, then the published segments
-    EdgeCtl& E = c.sh->e[i];
-    const int64_t Wup = vld(&E.W);
+    const int64_t Wup = vld(&nd.Ein->W);
     __threadfence_block();
-    const uint32_t st = vld(&E.seg_tail);
-    const uint32_t tail_known = (st != L.segh) ? c.seg[i][(st - 1) & (p.segcap - 1)].end : L.head;
+    const uint32_t st = vld(&nd.Ein->seg_tail);
+    const uint32_t tail_known = (st != L.segh) ? nd.in_seg[(st - 1) & nd.segmask].end : L.head;
     const bool any = tail_known != L.head;
-    if (fixed) {
-      const int64_t P = p.P[i];
-      const int64_t T = L.m * P;
-      uint32_t cnt = count_le(c, i, L, st, T, v);
+    if (nd.fixed) {
+      const int64_t T = L.m * nd.P;
+      const uint32_t cnt = count_le(nd, L, st, T);
       if (cnt >= v || Wup > T) {
         if (cnt > 0) { d.T = T; d.n = cnt < v ? cnt : v; return d; }
         if (!any && Wup == PL_INF64) { d.done = true; return d; }
-        int64_t r = any ? c.seg[i][L.segh & (p.segcap - 1)].ready : Wup;
-        int64_t m2 = ceil_div64(r, P);
+        const int64_t r = any ? nd.in_seg[L.segh & nd.segmask].ready : Wup;
+        int64_t m2 = cdiv(r, nd.P);
         if (m2 < L.m + 1) m2 = L.m + 1;
         L.empties += (uint64_t)(m2 - L.m);
         L.m = m2;
-        publish_W(c, i, L, L.m * P + t_i);
+        publish_W(nd, L, L.m * nd.P + nd.t);
         spins = 0;
         continue;
       }
-      publish_W(c, i, L, T + t_i);
+      publish_W(nd, L, T + nd.t);
       backoff(spins);
       continue;
     }
     // THRESHOLD_SLACK
     if (!any) {
       if (Wup == PL_INF64) { d.done = true; return d; }
-      int64_t lb = Wup > L.B ? Wup : L.B;
-      publish_W(c, i, L, lb + t_i);
+      publish_W(nd, L, (Wup > L.B ? Wup : L.B) + nd.t);
       backoff(spins);
       continue;
     }
-    const Seg& hs = c.seg[i][L.segh & (p.segcap - 1)];
+    const Seg& hs = nd.in_seg[L.segh & nd.segmask];
     __threadfence_block();
-    uint2 he = load_entry(c, i, L.head, L.segh, st, vld(&E.spill_end));
-    int64_t Tf = arrival(c, he.x) + p.D - p.R[i];
+    const uint2 he = load_entry(nd, L.head, L.segh, st, vld(&nd.Ein->spill_end));
+    int64_t Tf = nd.arrival(he.x) + nd.D - nd.R;
     if (Tf < hs.ready) Tf = hs.ready;
-    const uint32_t kth = L.head + p.theta[i] - 1;
+    const uint32_t kth = L.head + nd.theta - 1;
     const bool th_known = (int32_t)(tail_known - kth) > 0;
     int64_t Tth = PL_INF64;
     if (th_known) {
       for (uint32_t k = L.segh; k != st; ++k) {
-        const Seg& sg = c.seg[i][k & (p.segcap - 1)];
+        const Seg& sg = nd.in_seg[k & nd.segmask];
         if ((int32_t)(sg.end - kth) > 0) { Tth = sg.ready; break; }
       }
     }
     int64_t Tk = Tth < Tf ? Tth : Tf;
     if (Tk < L.B) Tk = L.B;
     if (th_known || Tk < Wup) {
-      uint32_t cnt = count_le(c, i, L, st, Tk, v);
+      const uint32_t cnt = count_le(nd, L, st, Tk);
       if (Wup > Tk || cnt >= v) { d.T = Tk; d.n = cnt < v ? cnt : v; return d; }
     }
     int64_t lb = Tk < Wup ? Tk : Wup;
     if (lb < L.B) lb = L.B;
-    publish_W(c, i, L, lb + t_i);
+    publish_W(nd, L, lb + nd.t);
     backoff(spins);
   }
 }
 
-// reserve `total` entries on the output edge of node i; returns location or ~0u on overflow
-__device__ uint32_t reserve_out(Ctx& c, int i, Leader& L, uint32_t total) {
-  const DevParams& p = *c.p;
-  EdgeCtl& E = c.sh->e[i + 1];
+// Reserve room for `worst` outputs on the output edge (worst case n*u, decided
+// before the stage runs so that no extra barrier is needed).  Returns the
+// location, or ~0u on overflow (physical mode only; logical mode back-pressures).
+__device__ uint32_t reserve_out(const Node& nd, Leader& L, uint32_t worst, uint32_t* errors) {
   int spins = 0;
   for (;;) {
-    const uint32_t h = vld(&E.head), sh = vld(&E.seg_head);
-    const bool seg_ok = (L.out_segt - sh) < p.segcap;
-    const uint32_t need = L.out_tail + total - h;
-    if (seg_ok && need <= p.cap_s[i + 1]) return LOC_SMEM;
-    if (seg_ok && need <= p.cap_g) return LOC_SPILL;
-    if (p.clock == PL_CLOCK_GLOBALTIMER) {
-      atomicOr(&c.sh->errors, seg_ok ? PL_ERR_QUEUE_OVERFLOW : PL_ERR_SEG_OVERFLOW);
+    const uint32_t h = vld(&nd.Eout->head), sh = vld(&nd.Eout->seg_head);
+    const bool seg_ok = (L.out_segt - sh) <= nd.segmask;
+    const uint32_t need = L.out_tail + worst - h;
+    if (seg_ok && need <= nd.out_cap) return LOC_SMEM;
+    if (seg_ok && need <= nd.capg) return LOC_SPILL;
+    if (nd.phys) {
+      atomicOr(errors, seg_ok ? PL_ERR_QUEUE_OVERFLOW : PL_ERR_SEG_OVERFLOW);
       return ~0u;
     }
     backoff(spins);   // logical mode: back-pressure (deadlock-free)
   }
 }
 
-__device__ __forceinline__ void pace(Ctx& c, int64_t T, uint64_t* start_ns, int64_t* late) {
-  const uint64_t target = c.sh->T0 + (uint64_t)((double)T * c.p->ns_per_unit);
+__device__ __forceinline__ void pace(uint64_t T0, double nspu, int64_t T, uint64_t* start_ns, int64_t* late) {
+  const uint64_t target = T0 + (uint64_t)((double)T * nspu);
   uint64_t now = gtimer();
   while (now < target) {
-    uint64_t rem = target - now;
+    const uint64_t rem = target - now;
     __nanosleep(rem > 2048 ? 1024 : (rem > 256 ? 128 : 0));
     now = gtimer();
   }
@@ -411,22 +497,27 @@ __device__ __forceinline__ void pace(Ctx& c, int64_t T, uint64_t* start_ns, int6
   *late = (int64_t)(now - target);
 }
 
-
 // exclusive scan of per-lane output counts over the node's v lanes (warp shuffles
 // + one named barrier); returns the lane's offset and the group total.
-__device__ __forceinline__ uint32_t group_scan(GroupCtl& G, uint32_t x, uint32_t* total, int gtid, int v, int bid) {
+__device__ __forceinline__ uint32_t group_scan(GroupCtl& G, uint32_t x, uint32_t* total, int gtid, int v, int bid,
+                                               bool binary) {
   const int lane = gtid & 31, w = gtid >> 5;
-  uint32_t inc = x;
+  uint32_t inc;
+  if (binary) {   // 0/1 outputs per lane: one ballot instead of five shuffles
+    inc = __popc(__ballot_sync(0xffffffffu, x != 0u) & (0xffffffffu >> (31 - lane)));
+  } else {
+    inc = x;
 #pragma unroll
-  for (int o = 1; o < 32; o <<= 1) {
-    uint32_t y = __shfl_up_sync(0xffffffffu, inc, o);
-    if (lane >= o) inc += y;
+    for (int o = 1; o < 32; o <<= 1) {
+      const uint32_t y = __shfl_up_sync(0xffffffffu, inc, o);
+      if (lane >= o) inc += y;
+    }
   }
   if (lane == 31) G.wtot[w] = inc;
   bar_sync(bid, v);                                                    // B2
   uint32_t pre = 0, tot = 0;
   for (int k = 0; k < (v >> 5); ++k) {
-    uint32_t t = G.wtot[k];
+    const uint32_t t = G.wtot[k];
     pre += (k < w) ? t : 0u;
     tot += t;
   }
@@ -435,61 +526,76 @@ __device__ __forceinline__ uint32_t group_scan(GroupCtl& G, uint32_t x, uint32_t
 }
 
 __device__ __forceinline__ int64_t overlap(int64_t s, int64_t e, int64_t lo, int64_t hi) {
-  int64_t a = s > lo ? s : lo, b = e < hi ? e : hi;
+  const int64_t a = s > lo ? s : lo, b = e < hi ? e : hi;
   return b > a ? b - a : 0;
 }
 
+__device__ __forceinline__ void bar_arrive(int id, int n) {
+  asm volatile("bar.arrive %0, %1;" ::"r"(id), "r"(n) : "memory");
+}
+
 // ------------------------------------------------------------------- node loop
-__device__ void run_node(Ctx& c, int i, int gtid) {
+// Per firing: leader decides (+ reserves output room, + paces in physical mode)
+// -> B1 -> lanes load / run the stage / scan (B2) -> leader releases the input
+// slots -> lanes compact their outputs -> B4 (arrive; the leader's warp syncs)
+// -> leader publishes the segment and its watermark.
+__device__ void run_node(Ctx& c, const Dna dna, int i, int gtid) {
   const DevParams& p = *c.p;
-  const int v = p.v, N = p.N;
+  const Node nd = make_node(c, i);
+  const int v = nd.v, N = nd.N;
   const bool leader = gtid == 0;
-  const bool sink = i == N - 1;
-  const int bid = 1 + i;
-  const bool phys = p.clock == PL_CLOCK_GLOBALTIMER;
-  const int64_t t_i = p.t[i];
+  const int bidA = 1 + i;
+  const int bidB = (i < 7) ? 9 + i : bidA;       // barrier ids 9..15 for the output barrier
   GroupCtl& G = c.sh->g[i];
   const uint32_t stream = blockIdx.x;
   const uint32_t rec = p.flags;
+  const uint64_t T0 = c.sh->T0;
 
   Leader L;
   L.m = 0; L.B = 0; L.c0 = 0; L.head = 0; L.segh = 0; L.out_tail = 0; L.out_segt = 0;
-  L.W_pub = -1; L.empties = 0; L.sched_cycles = 0;
+  L.W_pub = -1; L.empties = 0;
   uint64_t firings = 0, consumed = 0, produced = 0, spilled = 0, overruns = 0;
-  int64_t active = 0, busy_ns = 0, lateness = 0, t_end = 0;
-  uint32_t n_log = 0;
+  int64_t active = 0, busy_ns = 0, lateness = 0, t_end = 0, max_fire = 0;
   uint64_t start_ns = 0, end_ns_prev = 0;
   uint32_t pend_root = NO_ROOT;          // lane: physical terminal event awaiting its end time
-  uint32_t out_loc = LOC_SMEM;
+  uint64_t ph[6] = {0, 0, 0, 0, 0, 0};   // leader: per-phase clock64 cycles
+  long long tc = 0;
 
   for (;;) {
     if (leader) {
-      long long c0 = clock64();
-      Decision d = decide(c, i, L);
-      L.sched_cycles += (uint64_t)(clock64() - c0);
+      const long long c0 = clock64();
+      const Decision d = decide(nd, L);
       G.done = d.done ? 1u : 0u;
       G.T = d.T;
       G.n = d.n;
       G.head = (i == 0) ? (uint32_t)L.c0 : L.head;
       G.segh = L.segh;
       if (i > 0) {
-        G.st = vld(&c.sh->e[i].seg_tail);
+        G.st = vld(&nd.Ein->seg_tail);
         __threadfence_block();
-        G.in_spill_end = vld(&c.sh->e[i].spill_end);
+        G.in_spill_end = vld(&nd.Ein->spill_end);
       }
       G.end_ns_prev = end_ns_prev;
-      if (!d.done && (rec & PL_REC_FIRINGS)) G.log_idx = atomicAdd(&c.sh->log_count, 1u);
-      if (d.done) {
-        publish_W(c, i, L, PL_INF64);
-      } else if (phys) {
+      if (!d.done) {
+        if (rec & PL_REC_FIRINGS) G.log_idx = atomicAdd(&c.sh->log_count, 1u);
+        G.out_loc = nd.sink ? LOC_SMEM : reserve_out(nd, L, d.n * nd.umax, &c.sh->errors);
+        G.out_base = L.out_tail;
+      } else {
+        publish_W(nd, L, PL_INF64);
+      }
+      tc = clock64();
+      ph[0] += (uint64_t)(tc - c0);
+      if (!d.done && nd.phys) {
         int64_t late;
-        pace(c, d.T, &start_ns, &late);
+        pace(T0, nd.nspu, d.T, &start_ns, &late);
         if (late > lateness) lateness = late;
+        tc = clock64();
       }
     }
-    bar_sync(bid, v);                                                  // B1: decision
+    bar_sync(bidA, v);                                                 // B1: decision
+    if (leader) { const long long t2 = clock64(); ph[1] += (uint64_t)(t2 - tc); tc = t2; }
     if (pend_root != NO_ROOT) {          // deferred physical latency of the previous firing
-      const uint64_t a_ns = c.sh->T0 + (uint64_t)((double)arrival(c, pend_root) * p.ns_per_unit);
+      const uint64_t a_ns = T0 + (uint64_t)((double)nd.arrival(pend_root) * nd.nspu);
       const int64_t l = (int64_t)G.end_ns_prev - (int64_t)a_ns;
       if (rec & PL_REC_LATENCY) atomicMax((long long*)&p.lat_ns[pend_root], (long long)l);
       atomicMax(&c.sh->max_lat_ns, (unsigned long long)(l > 0 ? l : 0));
@@ -501,26 +607,35 @@ __device__ void run_node(Ctx& c, int i, int gtid) {
     const bool act = (uint32_t)gtid < n;
     uint2 e = make_uint2(0u, 0u);
     if (act) {
-      if (i == 0) e = make_uint2((uint32_t)(c.lo + head + gtid), 0u);
-      else e = load_entry(c, i, head + gtid, G.segh, G.st, G.in_spill_end);
+      if (i == 0) e = make_uint2((uint32_t)(nd.lo + head + gtid), 0u);
+      else e = load_entry(nd, head + gtid, G.segh, G.st, G.in_spill_end);
     }
     LaneOut o;
-    if (act) o = stage_count(c, i, e);
-    else { o.c = 0; o.a = 0; o.b = 0; o.score = 0; o.q_start = 0; o.len = 0; }
+    if (act) o = stage_count(nd, dna, p, e);
+    else { o.c = 0; o.a = 0; o.score = 0; o.q_start = 0; o.len = 0; }
     uint32_t total;
-    const uint32_t off = group_scan(G, o.c, &total, gtid, v, bid);   // B2 inside
+    const uint32_t off = group_scan(G, o.c, &total, gtid, v, bidA, nd.umax <= 1);   // B2 inside
+    if (leader) { const long long t2 = clock64(); ph[2] += (uint64_t)(t2 - tc); tc = t2; }
+    // --- release the input slots (every lane has loaded its entry: B2 passed)
+    if (leader && i > 0) {
+      L.head = head + n;
+      const uint32_t st = G.st;
+      while (L.segh != st && (int32_t)(nd.in_seg[L.segh & nd.segmask].end - L.head) <= 0) ++L.segh;
+      __threadfence_block();
+      vst(&nd.Ein->head, L.head);
+      vst(&nd.Ein->seg_head, L.segh);
+    }
     // --- per-item records: trace, terminal events (reading R-DONE)
+    const bool term = act && (nd.sink || o.c == 0);
+    const int64_t lat = term ? T + nd.t - nd.arrival(e.x) : 0;
     if (act) {
       if (rec & PL_REC_TRACE) {
         atomicAdd(&p.trace[(uint64_t)e.x * (N + 1) + i], 1u);
-        if (sink && o.c) atomicAdd(&p.trace[(uint64_t)e.x * (N + 1) + N], o.c);
+        if (nd.sink && o.c) atomicAdd(&p.trace[(uint64_t)e.x * (N + 1) + N], o.c);
       }
-      if (sink || o.c == 0) {
-        const int64_t l = T + t_i - arrival(c, e.x);
-        if (rec & PL_REC_LATENCY) atomicMax((long long*)&p.lat[e.x], (long long)l);
-        atomicMax(&c.sh->max_lat, (unsigned long long)l);
-        if (l > p.D) atomicAdd(&c.sh->miss_events, 1ull);
-        if (phys) pend_root = e.x;
+      if (term) {
+        if (rec & PL_REC_LATENCY) atomicMax((long long*)&p.lat[e.x], (long long)lat);
+        if (nd.phys) pend_root = e.x;
       }
       if ((rec & PL_REC_FIRINGS) && (gtid == 0 || (uint32_t)gtid == n - 1)) {
         const uint32_t li = G.log_idx;
@@ -532,84 +647,84 @@ __device__ void run_node(Ctx& c, int i, int gtid) {
           atomicOr(&c.sh->errors, PL_ERR_LOG_OVERFLOW);
         }
       }
-      if (sink && o.c && p.st[i].kind == PL_UNGAPPED_XDROP) {
-        unsigned long long mi = atomicAdd(p.match_count, 1ull);
-        if (mi < p.match_cap) {
-          pl_match mt;
-          mt.p = e.x; mt.q = e.y & 0xffffu; mt.db_start = o.a; mt.q_start = o.q_start;
-          mt.len = o.len; mt.score = o.score;
-          p.matches[mi] = mt;
-        } else {
-          atomicOr(&c.sh->errors, PL_ERR_MATCH_OVERFLOW);
+    }
+    {   // per-stream max latency / deadline misses / matches: one atomic per warp
+      const uint32_t lmax = __reduce_max_sync(0xffffffffu, (uint32_t)(lat > 0 ? (lat < 0xffffffffll ? lat : 0xffffffffll) : 0));
+      const uint32_t missb = __ballot_sync(0xffffffffu, term && lat > nd.D);
+      if ((gtid & 31) == 0) {
+        if (lmax) atomicMax(&c.sh->max_lat, (unsigned long long)lmax);
+        if (missb) atomicAdd(&c.sh->miss_events, (unsigned long long)__popc(missb));
+      }
+      if (nd.sink && nd.kind == PL_UNGAPPED_XDROP) {
+        const uint32_t mb = __ballot_sync(0xffffffffu, act && o.c);
+        if (mb) {
+          unsigned long long base = 0;
+          if ((gtid & 31) == 0) base = atomicAdd(p.match_count, (unsigned long long)__popc(mb));
+          base = __shfl_sync(0xffffffffu, base, 0);
+          if (act && o.c) {
+            const unsigned long long mi = base + __popc(mb & ((1u << (gtid & 31)) - 1u));
+            if (mi < p.match_cap) {
+              pl_match mt;
+              mt.p = e.x; mt.q = e.y & 0xffffu; mt.db_start = o.a; mt.q_start = o.q_start;
+              mt.len = o.len; mt.score = o.score;
+              p.matches[mi] = mt;
+            } else {
+              atomicOr(&c.sh->errors, PL_ERR_MATCH_OVERFLOW);
+            }
+          }
         }
       }
     }
-    // --- release the input slots (every lane has loaded its entry: B2 passed)
-    if (leader) {
-      if (i == 0) {
-        L.c0 += n;
-      } else {
-        L.head = head + n;
-        const uint32_t st = G.st;
-        while (L.segh != st && (int32_t)(c.seg[i][L.segh & (p.segcap - 1)].end - L.head) <= 0) ++L.segh;
-        __threadfence_block();
-        vst(&c.sh->e[i].head, L.head);
-        vst(&c.sh->e[i].seg_head, L.segh);
-      }
-    }
+    if (leader) { const long long t2 = clock64(); ph[3] += (uint64_t)(t2 - tc); tc = t2; }
     // --- compaction into the next queue (stable: lane order, then child order)
-    if (!sink && total > 0) {
-      if (leader) {
-        G.out_loc = reserve_out(c, i, L, total);
-        G.out_base = L.out_tail;
-      }
-      bar_sync(bid, v);                                                // B3: output slot
-      out_loc = G.out_loc;
-      const uint32_t base = G.out_base;
-      if (act && out_loc != ~0u) {
-        for (uint32_t j = 0; j < o.c; ++j) {
-          const uint32_t s = base + off + j;
-          const uint2 val = stage_output(c, i, e, o, j);
-          if (out_loc == LOC_SMEM) c.ent[i + 1][s & (p.cap_s[i + 1] - 1)] = val;
-          else __stcg(c.spill[i + 1] + (s & (p.cap_g - 1)), val);
-        }
+    const uint32_t out_loc = G.out_loc;
+    if (!nd.sink && act && o.c && out_loc != ~0u) {
+      const uint32_t base = G.out_base + off;
+      for (uint32_t j = 0; j < o.c; ++j) {
+        const uint32_t s = base + j;
+        const uint2 val = stage_output(nd, dna, e, o, j);
+        if (out_loc == LOC_SMEM) nd.out_ent[s & (nd.out_cap - 1)] = val;
+        else __stcg(nd.out_spill + (s & (nd.capg - 1)), val);
       }
     }
-    bar_sync(bid, v);                                                  // B4: outputs written
+    if (gtid < 32) bar_sync(bidB, v);                                  // B4: outputs written
+    else bar_arrive(bidB, v);
     if (leader) {
-      if (phys) {
+      { const long long t2 = clock64(); ph[4] += (uint64_t)(t2 - tc); tc = t2; }
+      if (nd.phys) {
         const uint64_t en = gtimer();
         busy_ns += (int64_t)(en - start_ns);
-        if ((double)(en - start_ns) > (double)t_i * p.ns_per_unit) ++overruns;
+        if ((int64_t)(en - start_ns) > max_fire) max_fire = (int64_t)(en - start_ns);
+        if ((double)(en - start_ns) > (double)nd.t * nd.nspu) ++overruns;
         end_ns_prev = en;
       }
       ++firings;
       consumed += n;
       produced += total;
-      active += overlap(T, T + t_i, 0, c.H);
-      if (T + t_i > t_end) t_end = T + t_i;
-      if (rec & PL_REC_FIRINGS) ++n_log;
-      if (!sink && total > 0 && out_loc != ~0u) {
-        EdgeCtl& E = c.sh->e[i + 1];
+      active += overlap(T, T + nd.t, 0, nd.H);
+      if (T + nd.t > t_end) t_end = T + nd.t;
+      if (!nd.sink && total > 0 && out_loc != ~0u) {
         Seg sg;
-        sg.ready = T + t_i;
+        sg.ready = T + nd.t;
         sg.end = L.out_tail + total;
         sg.loc = out_loc;
-        c.seg[i + 1][L.out_segt & (p.segcap - 1)] = sg;
-        if (out_loc == LOC_SPILL) { vst(&E.spill_end, sg.end); spilled += total; }
+        nd.out_seg[L.out_segt & nd.segmask] = sg;
+        if (out_loc == LOC_SPILL) { vst(&nd.Eout->spill_end, sg.end); spilled += total; }
         __threadfence_block();
         ++L.out_segt;
         L.out_tail += total;
-        vst(&E.seg_tail, L.out_segt);
-        vst(&E.tail, L.out_tail);
+        vst(&nd.Eout->seg_tail, L.out_segt);
+        vst(&nd.Eout->tail, L.out_tail);
       }
-      if (p.policy == PL_FIXED_WAIT) {
+      if (i == 0) L.c0 += n;
+      if (nd.fixed) {
         ++L.m;
-        publish_W(c, i, L, L.m * p.P[i] + t_i);
+        publish_W(nd, L, L.m * nd.P + nd.t);
       } else {
-        L.B = T + t_i;
-        publish_W(c, i, L, L.B + t_i);
+        L.B = T + nd.t;
+        publish_W(nd, L, L.B + nd.t);
       }
+      ph[5] += (uint64_t)(clock64() - tc);
     }
   }
   if (leader) {
@@ -623,8 +738,9 @@ __device__ void run_node(Ctx& c, int i, int gtid) {
     S.spilled[i] = spilled;
     S.overruns[i] = overruns;
     S.lateness[i] = lateness;
-    S.sched_cycles[i] = L.sched_cycles;
-    (void)n_log;
+    S.sched_cycles[i] = ph[0];
+    S.max_fire_ns[i] = max_fire;
+    for (int k = 0; k < 6; ++k) S.phase_cycles[i][k] = ph[k];
     atomicMax((long long*)&S.t_end, (long long)t_end);
   }
 }
@@ -645,6 +761,8 @@ __host__ __device__ inline uint32_t layout_enforced(const DevParams& p, SmemLayo
   off += dna ? (((uint32_t)(p.q_len - p.k + 1) * 2u) + 15u) & ~15u : 0u;
   L->off_qw = off;
   off += dna ? (((uint32_t)(p.q_len + 15) / 16u) * 4u + 15u) & ~15u : 0u;
+  L->off_win = off;
+  off += p.win_cap * 4u;
   L->total = off;
   return off;
 }
@@ -672,6 +790,44 @@ __device__ void cta_setup(Ctx& c, Shared& sh, unsigned char* dsm, const DevParam
   c.dna.qoff = (const uint16_t*)(dsm + Lo.off_qoff);
   c.dna.qpos = (const uint16_t*)(dsm + Lo.off_qpos);
   c.dna.qw = (const uint32_t*)(dsm + Lo.off_qw);
+  c.dna.nqw = (uint32_t)(p.q_len + 15) / 16u;
+  c.dna.win = (const uint32_t*)(dsm + Lo.off_win);
+  c.dna.win_lo = 0;
+  c.dna.win_n = 0;
+  if (p.k > 0 && p.win_cap > 0 && c.hi > c.lo) {
+    // this stream's DB window: roots [lo, hi) plus the k-1 overlap and a halo for
+    // the extensions, in 16-byte units (4 words) so that one TMA bulk copy moves it
+    int64_t wlo = ((int64_t)c.lo - (int64_t)p.win_halo) >> 4;
+    int64_t whi = (((int64_t)c.hi + p.k + (int64_t)p.win_halo) >> 4) + 1;
+    wlo = wlo < 0 ? 0 : (wlo & ~3ll);
+    whi = (whi + 3) & ~3ll;
+    if (whi > (int64_t)p.db_alloc_words) whi = (int64_t)p.db_alloc_words & ~3ll;
+    if (whi - wlo > (int64_t)p.win_cap) whi = wlo + p.win_cap;
+    c.dna.win_lo = wlo;
+    c.dna.win_n = whi > wlo ? (uint32_t)(whi - wlo) : 0u;
+    uint32_t* win = (uint32_t*)(dsm + Lo.off_win);
+    if (p.db_tma && c.dna.win_n) {
+      if (tid == 0) {
+        const uint32_t bar = (uint32_t)__cvta_generic_to_shared(&sh.mbar);
+        const uint32_t bytes = c.dna.win_n * 4u;
+        asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(bar));
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+        asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(bar), "r"(bytes) : "memory");
+        const uint32_t dst = (uint32_t)__cvta_generic_to_shared(win);
+        asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
+                     ::"r"(dst), "l"(p.db + wlo), "r"(bytes), "r"(bar) : "memory");
+        uint32_t done = 0;
+        while (!done)
+          asm volatile("{ .reg .pred q; mbarrier.try_wait.parity.shared::cta.b64 q, [%1], 0; selp.u32 %0, 1, 0, q; }"
+                       : "=r"(done) : "r"(bar) : "memory");
+      }
+    } else {
+      for (uint32_t j = tid; j < c.dna.win_n; j += nt) {
+        const int64_t w = wlo + j;
+        win[j] = w < (int64_t)p.db_words ? p.db[w] : 0u;
+      }
+    }
+  }
   if (p.k > 0) {   // query index -> smem
     uint16_t* qo = (uint16_t*)(dsm + Lo.off_qoff);
     uint16_t* qp = (uint16_t*)(dsm + Lo.off_qpos);
@@ -760,7 +916,7 @@ __device__ void run_monolithic(Ctx& c) {
     if (phys) {
       if (tid == 0) {
         uint64_t s_ns; int64_t late;
-        pace(c, ready, &s_ns, &late);      // the block is complete in real time
+        pace(c.sh->T0, p.ns_per_unit, ready, &s_ns, &late);   // the block is complete in real time
         sh_start_ns = s_ns;
       }
       __syncthreads();
@@ -770,6 +926,7 @@ __device__ void run_monolithic(Ctx& c) {
     uint32_t ncur = (uint32_t)(b1 - b0);
     for (int i = 0; i < N && ncur > 0; ++i) {
       const bool sink = i == N - 1;
+      const Node nd = make_node(c, i);
       const int64_t t_i = p.t[i];
       const uint32_t nf = (ncur + v - 1) / v;
       uint32_t nxt_count = 0;
@@ -779,8 +936,8 @@ __device__ void run_monolithic(Ctx& c) {
         uint2 e = make_uint2(0u, 0u);
         if (act) e = (i == 0) ? make_uint2((uint32_t)(c.lo + b0 + idx), 0u) : cur[idx];
         LaneOut o;
-        if (act) o = stage_count(c, i, e);
-        else { o.c = 0; o.a = 0; o.b = 0; o.score = 0; o.q_start = 0; o.len = 0; }
+        if (act) o = stage_count(nd, c.dna, p, e);
+        else { o.c = 0; o.a = 0; o.score = 0; o.q_start = 0; o.len = 0; }
         uint32_t total;
         const uint32_t off = block_scan(o.c, &total, wt);
         if (act) {
@@ -831,7 +988,7 @@ __device__ void run_monolithic(Ctx& c) {
           if (!sink) {
             for (uint32_t j = 0; j < o.c; ++j) {
               const uint32_t s = nxt_count + off + j;
-              if (s < p.mono_cap) nxt[s] = stage_output(c, i, e, o, j);
+              if (s < p.mono_cap) nxt[s] = stage_output(nd, c.dna, e, o, j);
               else atomicOr(&c.sh->errors, PL_ERR_QUEUE_OVERFLOW);
             }
           }
@@ -862,7 +1019,8 @@ __device__ void run_monolithic(Ctx& c) {
     for (int i = 0; i < PL_MAX_STAGES; ++i) {
       S.firings[i] = firings[i]; S.empty[i] = 0; S.consumed[i] = consumed[i]; S.produced[i] = produced[i];
       S.active_ne[i] = active[i]; S.busy_ns[i] = i == 0 ? busy_ns : 0; S.spilled[i] = 0; S.overruns[i] = 0;
-      S.lateness[i] = 0; S.sched_cycles[i] = 0;
+      S.lateness[i] = 0; S.sched_cycles[i] = 0; S.max_fire_ns[i] = 0;
+      for (int k = 0; k < 6; ++k) S.phase_cycles[i][k] = 0;
     }
     S.t_end = t_end;
   }
@@ -871,7 +1029,8 @@ __device__ void run_monolithic(Ctx& c) {
 }  // namespace
 
 // FIXED_WAIT / THRESHOLD_SLACK executor: grid = n_streams, block = N*v threads.
-extern "C" __global__ void __launch_bounds__(1024, 1) pl_exec_enforced(const __grid_constant__ DevParams p) {
+template <int MAXT>
+__global__ void __launch_bounds__(MAXT, 1) pl_exec_enforced(const __grid_constant__ DevParams p) {
   extern __shared__ __align__(16) unsigned char dsm[];
   __shared__ Shared sh;
   Ctx c;
@@ -880,7 +1039,7 @@ extern "C" __global__ void __launch_bounds__(1024, 1) pl_exec_enforced(const __g
   if (threadIdx.x == 0) sh.T0 = gtimer();
   __syncthreads();
   const int gi = threadIdx.x / p.v;
-  if (gi < p.N) run_node(c, gi, threadIdx.x % p.v);
+  if (gi < p.N) run_node(c, c.dna, gi, threadIdx.x % p.v);
   __syncthreads();
   cta_finish(c, sh, p);
 }
@@ -891,7 +1050,8 @@ uint32_t pl_layout_enforced_host(const DevParams& p) {
 }
 
 // MONOLITHIC executor: grid = n_streams, block = any multiple of 32 (N*v by default).
-extern "C" __global__ void __launch_bounds__(1024, 1) pl_exec_monolithic(const __grid_constant__ DevParams p) {
+template <int MAXT>
+__global__ void __launch_bounds__(MAXT, 1) pl_exec_monolithic(const __grid_constant__ DevParams p) {
   extern __shared__ __align__(16) unsigned char dsm[];
   __shared__ Shared sh;
   Ctx c;
@@ -902,4 +1062,25 @@ extern "C" __global__ void __launch_bounds__(1024, 1) pl_exec_monolithic(const _
   run_monolithic(c);
   __syncthreads();
   cta_finish(c, sh, p);
+}
+
+// host-side launchers (the kernels are templates on the block-size bound)
+cudaError_t pl_launch(const DevParams& p, unsigned grid, unsigned block, unsigned smem, cudaStream_t st) {
+  const bool mono = p.policy == PL_MONOLITHIC;
+  if (block <= 512) {
+    if (mono) pl_exec_monolithic<512><<<grid, block, smem, st>>>(p);
+    else pl_exec_enforced<512><<<grid, block, smem, st>>>(p);
+  } else {
+    if (mono) pl_exec_monolithic<1024><<<grid, block, smem, st>>>(p);
+    else pl_exec_enforced<1024><<<grid, block, smem, st>>>(p);
+  }
+  return cudaGetLastError();
+}
+
+cudaError_t pl_kernel_attributes(unsigned max_smem) {
+  cudaError_t e;
+  if ((e = cudaFuncSetAttribute(pl_exec_enforced<512>, cudaFuncAttributeMaxDynamicSharedMemorySize, max_smem))) return e;
+  if ((e = cudaFuncSetAttribute(pl_exec_enforced<1024>, cudaFuncAttributeMaxDynamicSharedMemorySize, max_smem))) return e;
+  if ((e = cudaFuncSetAttribute(pl_exec_monolithic<512>, cudaFuncAttributeMaxDynamicSharedMemorySize, max_smem))) return e;
+  return cudaFuncSetAttribute(pl_exec_monolithic<1024>, cudaFuncAttributeMaxDynamicSharedMemorySize, max_smem);
 }

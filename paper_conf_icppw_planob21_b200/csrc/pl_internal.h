@@ -42,6 +42,8 @@ struct CtaStats {
   uint64_t overruns[PL_MAX_STAGES];
   int64_t  lateness[PL_MAX_STAGES];
   uint64_t sched_cycles[PL_MAX_STAGES];
+  int64_t  max_fire_ns[PL_MAX_STAGES];
+  uint64_t phase_cycles[PL_MAX_STAGES][6];
   uint64_t miss_events;
   int64_t  max_lat;                     // model units
   int64_t  max_lat_ns;
@@ -73,6 +75,10 @@ struct DevParams {
   const uint16_t* qoff;                 // [4^k + 1]
   const uint16_t* qpos;                 // [q_len - k + 1]
   const uint32_t* qwords;               // [ceil(q_len/16)]
+  uint32_t win_cap;                     // smem DB window capacity (words, multiple of 4; 0 = off)
+  uint32_t win_halo;                    // bases staged beyond the stream's roots on each side
+  uint64_t db_alloc_words;              // readable words at db (>= db_words)
+  uint32_t db_tma;                      // db is 16-byte aligned and padded: stage with cp.async.bulk
   // queues
   uint32_t cap_s[PL_MAX_STAGES];        // smem entries of the edge INTO node i (pow2), i >= 1
   uint32_t cap_g;                       // spill entries per edge per stream (pow2)
@@ -97,7 +103,7 @@ struct DevParams {
 struct SmemLayout {
   uint32_t off_ent[PL_MAX_STAGES];      // uint2 rings, edge into node i (i >= 1)
   uint32_t off_seg[PL_MAX_STAGES];
-  uint32_t off_qoff, off_qpos, off_qw;
+  uint32_t off_qoff, off_qpos, off_qw, off_win;
   uint32_t total;
 };
 

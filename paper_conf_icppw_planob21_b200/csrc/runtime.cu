@@ -18,8 +18,8 @@
 
 #include "pl_internal.h"
 
-extern "C" __global__ void pl_exec_enforced(const __grid_constant__ DevParams p);
-extern "C" __global__ void pl_exec_monolithic(const __grid_constant__ DevParams p);
+cudaError_t pl_launch(const DevParams& p, unsigned grid, unsigned block, unsigned smem, cudaStream_t st);
+cudaError_t pl_kernel_attributes(unsigned max_smem);
 uint32_t pl_layout_enforced_host(const DevParams& p);
 
 namespace plsolve {
@@ -113,11 +113,13 @@ struct pl_pipeline {
   pl_firing* d_flog = nullptr;
   CtaStats* d_stats = nullptr;
   uint64_t roots_cap = 0;   // per-root arrays sized for this many roots
+  uint64_t db_alloc_words = 0;
   // host state
   uint64_t pushed = 0;      // DNA: bases; gain: roots per stream
   bool in_flight = false, drained = false;
   uint32_t launches = 0;
   int device = 0;
+  uint64_t h2d = 0, d2h = 0;  // bytes moved across the host boundary (cumulative)
 };
 
 namespace {
@@ -356,9 +358,17 @@ pl_status pl_pipeline_create(const pl_config* cfg, const pl_workload* wl, pl_pip
     d.qoff = pl->d_qoff;
     d.qpos = pl->d_qpos;
     d.qwords = pl->d_qw;
-    const uint64_t dbw = (wl->db_len + 15) / 16 + 1;
+    const uint64_t dbw = (wl->db_len + 15) / 16 + 8;     // padded: TMA copies whole 16-byte units
     if (cudaMalloc(&pl->d_db, dbw * 4) != cudaSuccess) return bail(fail(PL_ENOMEM, "DB allocation"));
     cudaMemset(pl->d_db, 0, dbw * 4);
+    pl->db_alloc_words = dbw;
+    // smem DB window per stream: its roots + k-1 overlap + halo on both sides (capped at 64 KB)
+    const uint64_t R = wl->db_len >= (uint64_t)pl->k ? wl->db_len - pl->k + 1 : 0;
+    const uint64_t per = (R + cfg->n_streams - 1) / cfg->n_streams;
+    d.win_halo = 512;
+    uint64_t words = (per + pl->k + 2 * d.win_halo) / 16 + 8;
+    words = (words + 3) & ~3ull;
+    d.win_cap = (uint32_t)std::min<uint64_t>(words, 16384);
     pl->roots_cap = wl->db_len >= (uint64_t)pl->k ? wl->db_len - pl->k + 1 : 0;
   } else {
     pl->roots_cap = cfg->n_roots * cfg->n_streams;
@@ -427,10 +437,8 @@ pl_status pl_pipeline_create(const pl_config* cfg, const pl_workload* wl, pl_pip
   d.match_count = pl->d_match_count;
   d.flog = pl->d_flog;
   d.stats = pl->d_stats;
-  cudaError_t e1 = cudaFuncSetAttribute(pl_exec_enforced, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024);
-  cudaError_t e2 = cudaFuncSetAttribute(pl_exec_monolithic, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024);
-  if (e1 != cudaSuccess || e2 != cudaSuccess)
-    return bail(fail(PL_EDEVICE, "cudaFuncSetAttribute: %s", cudaGetErrorString(e1 != cudaSuccess ? e1 : e2)));
+  cudaError_t e1 = pl_kernel_attributes(200 * 1024);
+  if (e1 != cudaSuccess) return bail(fail(PL_EDEVICE, "cudaFuncSetAttribute: %s", cudaGetErrorString(e1)));
   cudaError_t e = cudaDeviceSynchronize();
   if (e != cudaSuccess) return bail(fail(PL_EDEVICE, "create: %s", cudaGetErrorString(e)));
   *out = pl;
@@ -454,6 +462,7 @@ pl_status pl_pipeline_push(pl_pipeline* pl, const void* items, uint64_t n) {
     cudaSetDevice(pl->device);
     const uint64_t words = (n + 15) / 16;
     CUDA_TRY(cudaMemcpyAsync(pl->d_db + pl->pushed / 16, items, words * 4, cudaMemcpyHostToDevice, pl->stream));
+    pl->h2d += words * 4;
     pl->pushed += n;
   } else {
     if (items) return fail(PL_EINVAL, "random-gain push takes items == NULL");
@@ -480,16 +489,15 @@ pl_status pl_pipeline_launch(pl_pipeline* pl) {
     d.db = pl->d_db_bound ? pl->d_db_bound : pl->d_db;
     d.db_len = pl->pushed;
     d.db_words = (uint32_t)((pl->pushed + 15) / 16);
+    d.db_alloc_words = pl->d_db_bound ? d.db_words : pl->db_alloc_words;
+    d.db_tma = pl->d_db_bound ? (((uintptr_t)pl->d_db_bound & 15u) == 0u) : 1u;
     d.total_roots = pl->pushed >= (uint64_t)pl->k ? pl->pushed - pl->k + 1 : 0;
   } else {
     d.total_roots = pl->pushed * pl->cfg.n_streams;
   }
   if (d.total_roots > pl->roots_cap) return fail(PL_EINVAL, "more roots than allocated");
   CUDA_TRY(cudaMemsetAsync(pl->d_match_count, 0, 8, pl->stream));
-  const dim3 grid(pl->cfg.n_streams), block(pl->block);
-  if (pl->cfg.policy == PL_MONOLITHIC) pl_exec_monolithic<<<grid, block, pl->smem, pl->stream>>>(d);
-  else pl_exec_enforced<<<grid, block, pl->smem, pl->stream>>>(d);
-  CUDA_TRY(cudaGetLastError());
+  CUDA_TRY(pl_launch(d, pl->cfg.n_streams, pl->block, pl->smem, pl->stream));
   pl->in_flight = true;
   pl->launches++;
   return PL_OK;
@@ -506,6 +514,7 @@ pl_status pl_pipeline_drain(pl_pipeline* pl) {
   pl->drained = true;
   std::vector<CtaStats> cs(pl->cfg.n_streams);
   CUDA_TRY(cudaMemcpy(cs.data(), pl->d_stats, cs.size() * sizeof(CtaStats), cudaMemcpyDeviceToHost));
+  pl->d2h += cs.size() * sizeof(CtaStats);
   uint32_t err = 0;
   for (auto& s : cs) err |= s.errors;
   if (err) return fail(PL_EOVERFLOW, "device reported overflow bits 0x%x (queue=1 match=2 log=4 seg=8)", err);
@@ -526,6 +535,7 @@ pl_status pl_pipeline_stats(pl_pipeline* pl, pl_stats* out) {
   const uint32_t S = pl->cfg.n_streams, N = pl->cfg.n_stages;
   std::vector<CtaStats> cs(S);
   CUDA_TRY(cudaMemcpy(cs.data(), pl->d_stats, S * sizeof(CtaStats), cudaMemcpyDeviceToHost));
+  pl->d2h += S * sizeof(CtaStats);
   std::memset(out, 0, sizeof *out);
   out->n_stages = N;
   out->n_streams = S;
@@ -545,6 +555,8 @@ pl_status pl_pipeline_stats(pl_pipeline* pl, pl_stats* out) {
       out->overruns[i] += s.overruns[i];
       out->max_lateness_ns[i] = std::max(out->max_lateness_ns[i], s.lateness[i]);
       out->sched_cycles[i] += s.sched_cycles[i];
+      out->max_fire_ns[i] = std::max(out->max_fire_ns[i], s.max_fire_ns[i]);
+      for (int k = 0; k < 6; ++k) out->phase_cycles[i][k] += s.phase_cycles[i][k];
       if (pl->cfg.policy == PL_FIXED_WAIT) {   // every firing m*P_i < H is charged (L97, R-WINDOW)
         const int64_t P = pl->dp.P[i], t = pl->t[i];
         out->active_window[i] += (H / P) * t + std::min(t, H % P);
@@ -560,6 +572,7 @@ pl_status pl_pipeline_stats(pl_pipeline* pl, pl_stats* out) {
   }
   unsigned long long mc = 0;
   CUDA_TRY(cudaMemcpy(&mc, pl->d_match_count, 8, cudaMemcpyDeviceToHost));
+  pl->d2h += 8;
   out->matches = std::min<uint64_t>(mc, pl->dp.match_cap);
   double act = 0, act_ne = 0, busy = 0;
   for (uint32_t i = 0; i < N; ++i) {
@@ -591,6 +604,8 @@ pl_status pl_pipeline_stats(pl_pipeline* pl, pl_stats* out) {
     }
   }
   out->launches = pl->launches;
+  out->h2d_bytes = pl->h2d;
+  out->d2h_bytes = pl->d2h;
   return PL_OK;
 }
 
@@ -604,6 +619,7 @@ pl_status pl_pipeline_results(pl_pipeline* pl, pl_match* buf, uint64_t cap, uint
   if (!buf) { *n = cnt; return PL_OK; }
   cnt = std::min(cnt, cap);
   if (cnt) CUDA_TRY(cudaMemcpy(buf, pl->d_matches, cnt * sizeof(pl_match), cudaMemcpyDeviceToHost));
+  pl->d2h += 8 + cnt * sizeof(pl_match);
   *n = cnt;
   return PL_OK;
 }

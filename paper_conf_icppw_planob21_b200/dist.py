@@ -1,0 +1,56 @@
+"""Cross-GPU reduction of executor statistics.
+
+Streams are independent pipeline instances (§2.2: one processor per
+application instance), so ranks share no data; the only collective is one
+all-reduce of the int64 counter vector (SUM) and one of the maxima (MAX), over
+NCCL on NVLink/NVSwitch (gloo on CPU for tests).
+"""
+from __future__ import annotations
+
+SUM_KEYS = ("roots", "firings", "empty_firings", "consumed", "produced", "active_window", "busy_ns",
+            "spilled", "overruns", "matches", "miss_events", "misses", "window", "t_end")
+MAX_KEYS = ("max_lateness_ns", "max_fire_ns", "max_latency", "max_latency_ns", "wall_ns", "errors")
+
+
+def _flatten(st, keys):
+    out = []
+    for k in keys:
+        v = st[k]
+        out.extend(int(x) for x in (v if isinstance(v, (list, tuple)) else [v]))
+    return out
+
+
+def _unflatten(st, keys, vals):
+    res = dict(st)
+    i = 0
+    for k in keys:
+        v = st[k]
+        if isinstance(v, (list, tuple)):
+            res[k] = [int(x) for x in vals[i:i + len(v)]]
+            i += len(v)
+        else:
+            res[k] = int(vals[i])
+            i += 1
+    return res
+
+
+def allreduce_stats(st: dict, device=None) -> dict:
+    """SUM the counters and MAX the maxima of a pl_stats dict over all ranks.
+    The active fractions are recomputed from the reduced sums."""
+    import torch
+    import torch.distributed as dist
+    if not (dist.is_available() and dist.is_initialized()) or dist.get_world_size() == 1:
+        return st
+    s = torch.tensor(_flatten(st, SUM_KEYS), dtype=torch.int64, device=device)
+    m = torch.tensor(_flatten(st, MAX_KEYS), dtype=torch.int64, device=device)
+    dist.all_reduce(s, op=dist.ReduceOp.SUM)
+    dist.all_reduce(m, op=dist.ReduceOp.MAX)
+    res = _unflatten(st, SUM_KEYS, s.tolist())
+    res = _unflatten(res, MAX_KEYS, m.tolist())
+    N = st["n_stages"]
+    mono = st.get("policy") == 2
+    if res["window"]:
+        act = sum(res["active_window"][:N])
+        res["active_fraction"] = act / (res["window"] * (1 if mono else N))
+    res["n_ranks"] = dist.get_world_size()
+    return res
