@@ -74,6 +74,8 @@ enum pl_clock { PL_CLOCK_LOGICAL = 0, PL_CLOCK_GLOBALTIMER = 1 };
 #define PL_REC_LATENCY  1u     /* lat[r]: per-root latency (model units; + ns if physical) */
 #define PL_REC_TRACE    2u     /* cnt[r][0..N]: per-root surviving-stage trace           */
 #define PL_REC_FIRINGS  4u     /* per-stream log of non-empty firings                    */
+#define PL_FIXED_SERVICE 8u    /* physical clock: publish a firing's outputs at start + t_i,
+                                  the paper's fixed service time (L69), not as soon as done */
 
 typedef struct {
   uint32_t kind;           /* enum pl_stage_kind                                        */

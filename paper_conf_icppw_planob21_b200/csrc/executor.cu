@@ -24,6 +24,9 @@ namespace {
 
 constexpr uint32_t LOC_SMEM = 0, LOC_SPILL = 1;
 constexpr uint32_t NO_ROOT = 0xffffffffu;
+// physical clock: a stream's time origin is set this far after its CTA starts, so that
+// every warp group is resident and warm before the first arrival (absorbs start-up lateness)
+constexpr uint64_t PL_T0_OFFSET_NS = 2048;
 
 __device__ __forceinline__ uint64_t gtimer() {
   uint64_t t;
@@ -488,9 +491,9 @@ __device__ uint32_t reserve_out(const Node& nd, Leader& L, uint32_t worst, uint3
 __device__ __forceinline__ void pace(uint64_t T0, double nspu, int64_t T, uint64_t* start_ns, int64_t* late) {
   const uint64_t target = T0 + (uint64_t)((double)T * nspu);
   uint64_t now = gtimer();
-  while (now < target) {
+  while (now < target) {   // __nanosleep rounds up to powers of two: sleep at most ~rem/4
     const uint64_t rem = target - now;
-    __nanosleep(rem > 2048 ? 1024 : (rem > 256 ? 128 : 0));
+    __nanosleep(rem > 4096 ? 1024 : (rem > 1024 ? 256 : (rem > 256 ? 64 : 0)));
     now = gtimer();
   }
   *start_ns = now;
@@ -692,10 +695,17 @@ __device__ void run_node(Ctx& c, const Dna dna, int i, int gtid) {
     if (leader) {
       { const long long t2 = clock64(); ph[4] += (uint64_t)(t2 - tc); tc = t2; }
       if (nd.phys) {
-        const uint64_t en = gtimer();
-        busy_ns += (int64_t)(en - start_ns);
+        uint64_t en = gtimer();
+        const uint64_t due = T0 + (uint64_t)((double)(T + nd.t) * nd.nspu);
+        if ((double)(en - start_ns) > (double)nd.t * nd.nspu) ++overruns;   // work outlasted t_i
         if ((int64_t)(en - start_ns) > max_fire) max_fire = (int64_t)(en - start_ns);
-        if ((double)(en - start_ns) > (double)nd.t * nd.nspu) ++overruns;
+        if (rec & PL_FIXED_SERVICE) {   // hold the outputs until start + t_i (L69)
+          while (en < due) {
+            __nanosleep(due - en > 256 ? 128 : 0);
+            en = gtimer();
+          }
+        }
+        busy_ns += (int64_t)(en - start_ns);
         end_ns_prev = en;
       }
       ++firings;
@@ -1036,7 +1046,7 @@ __global__ void __launch_bounds__(MAXT, 1) pl_exec_enforced(const __grid_constan
   Ctx c;
   cta_setup(c, sh, dsm, p);
   __syncthreads();
-  if (threadIdx.x == 0) sh.T0 = gtimer();
+  if (threadIdx.x == 0) sh.T0 = gtimer() + (p.clock == PL_CLOCK_GLOBALTIMER ? PL_T0_OFFSET_NS : 0);
   __syncthreads();
   const int gi = threadIdx.x / p.v;
   if (gi < p.N) run_node(c, c.dna, gi, threadIdx.x % p.v);
@@ -1057,7 +1067,7 @@ __global__ void __launch_bounds__(MAXT, 1) pl_exec_monolithic(const __grid_const
   Ctx c;
   cta_setup(c, sh, dsm, p);
   __syncthreads();
-  if (threadIdx.x == 0) sh.T0 = gtimer();
+  if (threadIdx.x == 0) sh.T0 = gtimer() + (p.clock == PL_CLOCK_GLOBALTIMER ? PL_T0_OFFSET_NS : 0);
   __syncthreads();
   run_monolithic(c);
   __syncthreads();

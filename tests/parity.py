@@ -70,3 +70,41 @@ def compare(cfg, g, o, check_firings=True):
     assert st["max_latency"] == max(o.lat)
     assert st["misses"] == o.misses(cfg.deadline)
     assert abs(st["active_fraction"] - o.active_fraction(cfg.policy)) < 1e-12
+
+
+_WL = None
+
+
+def _oracle_one(args):
+    cfg, lo, hi, kw = args
+    from oracle import des
+    from oracle import stages as S
+    ctx = None
+    if _WL is not None:
+        ctx = S.DnaContext(_WL.db, _WL.db_len, _WL.query, _WL.q_len, cfg.stages[0].iparam[0])
+    fns = des.make_stage_fns(cfg, ctx)
+    return des.simulate_stream(cfg, fns, lo, hi, **kw)
+
+
+def run_oracle_parallel(cfg, wl, streams=None, **kw):
+    """oracle.des.run over a fork process pool (same result as run_oracle)."""
+    global _WL
+    import multiprocessing as mp
+    import os
+    from oracle import des
+    _WL = wl
+    if wl is not None:
+        total = wl.db_len - cfg.stages[0].iparam[0] + 1
+    else:
+        total = cfg.n_roots * cfg.n_streams
+    rng = des.stream_ranges(cfg, total)
+    idx = list(range(len(rng))) if streams is None else list(streams)
+    with mp.get_context("fork").Pool(min(len(idx), len(os.sched_getaffinity(0)))) as pool:
+        res = pool.map(_oracle_one, [(cfg, rng[s][0], rng[s][1], kw) for s in idx], chunksize=1)
+    lat, trace, matches = [], [], []
+    for r in res:
+        lat += r.lat
+        trace += r.trace
+        matches += r.matches
+    matches.sort()
+    return des.Result(res, lat, trace, matches, cfg.n_stages)
