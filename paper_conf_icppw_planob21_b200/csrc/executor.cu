@@ -152,20 +152,20 @@ struct EdgeCtl {            // queue INTO node i
   uint32_t spill_end;       // producer: end seq of the last spilled segment
   uint32_t pad;
 };
-struct GroupCtl {           // broadcast from a node's leader to its lanes
-  int64_t  T;
-  uint64_t end_ns_prev;     // physical: end time of the previous firing
-  uint32_t n, head, done, segh, st, log_idx;
-  uint32_t in_spill_end;    // input edge: end seq of its last spilled segment
-  uint32_t out_base, out_loc;
-  uint32_t wtot[8];
+struct GroupCtl {           // broadcast from a node's leader to its lanes, double-buffered
+  int64_t  T[2];            // by firing parity so that no barrier is needed between firings
+  uint64_t end_ns[2];       // physical: publish time of the firing of that parity
+  uint32_t n[2], head[2], done[2], segh[2], st[2], log_idx[2];
+  uint32_t in_spill_end[2]; // input edge: end seq of its last spilled segment
+  uint32_t out_base[2], out_loc[2];
+  uint32_t wtot[2][8];
 };
 struct Shared {
   EdgeCtl e[PL_MAX_STAGES];
   GroupCtl g[PL_MAX_STAGES];
-  unsigned long long max_lat;
-  unsigned long long max_lat_ns;
-  unsigned long long miss_events;
+  uint32_t max_lat;         // per-stream aggregates: 32-bit so the smem atomics are native
+  uint32_t max_lat_ns;      // (64-bit smem atomicMax compiles to a CAS loop)
+  uint32_t miss_events;
   uint32_t errors;
   uint32_t log_count;       // firing-log records reserved by all nodes of this stream
   uint64_t T0;
@@ -175,9 +175,7 @@ struct Shared {
 struct Ctx {
   const DevParams* p;
   Shared* sh;
-  uint2* ent[PL_MAX_STAGES];   // smem rings (edge into node i)
-  Seg* seg[PL_MAX_STAGES];
-  uint2* spill[PL_MAX_STAGES]; // this stream's HBM rings
+  unsigned char* dsm;          // dynamic smem base (rings, segments, index, DB window)
   Dna dna;
   uint64_t lo, hi;             // roots [lo, hi)
   int64_t X, H;
@@ -185,14 +183,19 @@ struct Ctx {
 
 __device__ __forceinline__ int64_t arrival(const Ctx& c, uint32_t root) { return (int64_t)(root - c.lo) * c.p->tau; }
 
-// floor(a / b) for a >= 0, b > 0 without a 64-bit integer division (double estimate + fix-up)
-__device__ __forceinline__ int64_t fdiv(int64_t a, int64_t b) {
-  int64_t q = (int64_t)((double)a / (double)b);
-  while (q > 0 && q * b > a) --q;
-  while ((q + 1) * b <= a) ++q;
+// floor(a / d) for 0 <= a < 2^63 by a host-precomputed reciprocal m = floor((2^64-1)/d):
+// umulhi(a, m) is floor(a/d) or one less, fixed by one compare (no 64-bit division).
+struct MDiv {
+  uint64_t m;
+  int64_t d;
+};
+__device__ __forceinline__ int64_t fdiv(int64_t a, const MDiv& D) {
+  if (D.d == 1) return a;
+  int64_t q = (int64_t)__umul64hi((uint64_t)a, D.m);
+  if ((q + 1) * D.d <= a) ++q;
   return q;
 }
-__device__ __forceinline__ int64_t cdiv(int64_t a, int64_t b) { return a <= 0 ? 0 : fdiv(a - 1, b) + 1; }
+__device__ __forceinline__ int64_t cdiv(int64_t a, const MDiv& D) { return a <= 0 ? 0 : fdiv(a - 1, D) + 1; }
 
 // Per-node constants, built once per warp group and kept in registers.
 struct Node {
@@ -215,11 +218,16 @@ struct Node {
   uint32_t out_cap;
   uint32_t kind, max_out, cfix, umax;
   int32_t ip1, ip2;
+  MDiv dtau, dP;
   __device__ __forceinline__ int64_t arrival(uint32_t root) const { return (int64_t)(root - lo) * tau; }
 };
 
+__host__ __device__ inline uint32_t layout_enforced(const DevParams& p, SmemLayout* L);
+
 __device__ __forceinline__ Node make_node(const Ctx& c, int i) {
   const DevParams& p = *c.p;
+  SmemLayout Lo;
+  layout_enforced(p, &Lo);
   Node n;
   n.i = i; n.N = p.N; n.v = p.v;
   n.sink = i == p.N - 1;
@@ -232,16 +240,23 @@ __device__ __forceinline__ Node make_node(const Ctx& c, int i) {
   n.segmask = p.segcap - 1;
   n.capg = p.cap_g;
   n.Ein = &c.sh->e[i];
-  n.in_ent = c.ent[i]; n.in_seg = c.seg[i]; n.in_spill = c.spill[i];
+  const uint64_t sp = (uint64_t)blockIdx.x * p.N;
+  n.in_ent = (const uint2*)(c.dsm + Lo.off_ent[i]);
+  n.in_seg = (const Seg*)(c.dsm + Lo.off_seg[i]);
+  n.in_spill = p.spill ? p.spill + (sp + i) * p.cap_g : nullptr;
   n.in_mask = p.cap_s[i] ? p.cap_s[i] - 1 : 0;
   const int o = i + 1 < p.N ? i + 1 : i;
   n.Eout = &c.sh->e[o];
-  n.out_ent = c.ent[o]; n.out_seg = c.seg[o]; n.out_spill = c.spill[o];
+  n.out_ent = (uint2*)(c.dsm + Lo.off_ent[o]);
+  n.out_seg = (Seg*)(c.dsm + Lo.off_seg[o]);
+  n.out_spill = p.spill ? p.spill + (sp + o) * p.cap_g : nullptr;
   n.out_cap = p.cap_s[o];
   const DevStage& s = p.st[i];
   n.kind = s.kind; n.max_out = s.max_out; n.cfix = s.cfix;
   n.umax = s.kind == PL_FIXED_GAIN ? s.cfix : s.max_out;
   n.ip1 = s.ip[1]; n.ip2 = s.ip[2];
+  n.dtau.m = p.tau_m; n.dtau.d = p.tau;
+  n.dP.m = p.P_m[i]; n.dP.d = p.P[i];
   return n;
 }
 
@@ -323,6 +338,34 @@ __device__ __forceinline__ LaneOut stage_count(const Node& nd, const Dna& dna, c
   return o;
 }
 
+// S2 / S3 for one entry.
+__device__ __forceinline__ LaneOut stage_count_ext(const Node& nd, const Dna& dna, uint2 e) {
+  LaneOut o;
+  o.c = 0; o.a = 0; o.score = 0; o.q_start = 0; o.len = 0;
+  const uint32_t q = e.y & 0xffffu;
+  if (nd.kind == PL_UNGAPPED_WINDOW) {
+    const int64_t W = nd.ip1;
+    int d;
+    const int64_t ll = dna.left_limit(e.x, q), rl = dna.right_limit(e.x, q);
+    const int bl = dna.extend(e.x, q, -1, ll < W ? ll : W, 0, &d);
+    const int br = dna.extend(e.x, q, +1, rl < W ? rl : W, 0, &d);
+    o.c = (dna.k + bl + br >= nd.ip2) ? 1u : 0u;
+  } else {
+    int dl, dr;
+    const int bl = dna.extend(e.x, q, -1, dna.left_limit(e.x, q), nd.ip1, &dl);
+    const int br = dna.extend(e.x, q, +1, dna.right_limit(e.x, q), nd.ip1, &dr);
+    const int score = dna.k + bl + br;
+    if (score >= nd.ip2) {
+      o.c = 1;
+      o.score = score;
+      o.a = e.x - dl;
+      o.q_start = q - dl;
+      o.len = dna.k + dl + dr;
+    }
+  }
+  return o;
+}
+
 // Phase B: output j of an entry (non-sink nodes).
 __device__ __forceinline__ uint2 stage_output(const Node& nd, const Dna& dna, uint2 e, const LaneOut& o, uint32_t j) {
   switch (nd.kind) {
@@ -377,39 +420,52 @@ __device__ __forceinline__ uint32_t count_le(const Node& nd, const Leader& L, ui
   return end - L.head;
 }
 
+// Node 0: arrivals are fully known (root lo+r arrives at r*tau0), so every
+// lane evaluates the firing decision itself from replicated state (no broadcast barrier).
+struct Rep {
+  int64_t m;        // FIXED_WAIT: next firing index
+  int64_t B;        // THRESHOLD_SLACK: busy until
+  int64_t c0;       // roots consumed
+  uint64_t empties;
+};
+__device__ __forceinline__ Decision decide0(const Node& nd, Rep& r) {
+  Decision d;
+  d.done = r.c0 >= nd.X;
+  d.T = 0;
+  d.n = 0;
+  if (d.done) return d;
+  int64_t T;
+  if (nd.fixed) {
+    T = r.m * nd.P;
+    if (T < r.c0 * nd.tau) {             // empty firings until the next root has arrived
+      const int64_t m2 = cdiv(r.c0 * nd.tau, nd.dP);
+      r.empties += (uint64_t)(m2 - r.m);
+      r.m = m2;
+      T = r.m * nd.P;
+    }
+  } else {
+    const int64_t ah = r.c0 * nd.tau;
+    const int64_t Tth = (r.c0 + nd.theta - 1 < nd.X) ? ah + (int64_t)(nd.theta - 1) * nd.tau : PL_INF64;
+    int64_t Tf = ah + nd.D - nd.R;
+    if (Tf < ah) Tf = ah;
+    T = Tth < Tf ? Tth : Tf;
+    if (T < r.B) T = r.B;
+  }
+  int64_t arrived = fdiv(T, nd.dtau) + 1;
+  if (arrived > nd.X) arrived = nd.X;
+  const int64_t avail = arrived - r.c0;
+  d.T = T;
+  d.n = (uint32_t)(avail < (int64_t)nd.v ? avail : nd.v);
+  return d;
+}
+
+// Nodes i >= 1: the leader decides from the published queue state and watermark.
 __device__ Decision decide(const Node& nd, Leader& L) {
   const uint32_t v = (uint32_t)nd.v;
   Decision d;
   d.done = false; d.T = 0; d.n = 0;
   int spins = 0;
   for (;;) {
-    if (nd.i == 0) {
-      // arrivals are fully known: root lo+r arrives at r*tau0
-      if ((int64_t)L.c0 >= nd.X) { d.done = true; return d; }
-      int64_t T;
-      if (nd.fixed) {
-        T = L.m * nd.P;
-        if (T < (int64_t)L.c0 * nd.tau) {   // empty firings until the next root has arrived
-          const int64_t m2 = cdiv((int64_t)L.c0 * nd.tau, nd.P);
-          L.empties += (uint64_t)(m2 - L.m);
-          L.m = m2;
-          T = L.m * nd.P;
-        }
-      } else {
-        const int64_t ah = (int64_t)L.c0 * nd.tau;
-        const int64_t Tth = ((int64_t)L.c0 + nd.theta - 1 < nd.X) ? ah + (int64_t)(nd.theta - 1) * nd.tau : PL_INF64;
-        int64_t Tf = ah + nd.D - nd.R;
-        if (Tf < ah) Tf = ah;
-        T = Tth < Tf ? Tth : Tf;
-        if (T < L.B) T = L.B;
-      }
-      int64_t arrived = fdiv(T, nd.tau) + 1;
-      if (arrived > nd.X) arrived = nd.X;
-      const int64_t avail = arrived - (int64_t)L.c0;
-      d.T = T;
-      d.n = (uint32_t)(avail < (int64_t)v ? avail : v);
-      return d;
-    }
     // node i >= 1: read the upstream watermark first, then the published segments
     const int64_t Wup = vld(&nd.Ein->W);
     __threadfence_block();
@@ -423,7 +479,7 @@ __device__ Decision decide(const Node& nd, Leader& L) {
         if (cnt > 0) { d.T = T; d.n = cnt < v ? cnt : v; return d; }
         if (!any && Wup == PL_INF64) { d.done = true; return d; }
         const int64_t r = any ? nd.in_seg[L.segh & nd.segmask].ready : Wup;
-        int64_t m2 = cdiv(r, nd.P);
+        int64_t m2 = cdiv(r, nd.dP);
         if (m2 < L.m + 1) m2 = L.m + 1;
         L.empties += (uint64_t)(m2 - L.m);
         L.m = m2;
@@ -502,7 +558,7 @@ __device__ __forceinline__ void pace(uint64_t T0, double nspu, int64_t T, uint64
 
 // exclusive scan of per-lane output counts over the node's v lanes (warp shuffles
 // + one named barrier); returns the lane's offset and the group total.
-__device__ __forceinline__ uint32_t group_scan(GroupCtl& G, uint32_t x, uint32_t* total, int gtid, int v, int bid,
+__device__ __forceinline__ uint32_t group_scan(uint32_t* wtot, uint32_t x, uint32_t* total, int gtid, int v, int bid,
                                                bool binary) {
   const int lane = gtid & 31, w = gtid >> 5;
   uint32_t inc;
@@ -516,11 +572,11 @@ __device__ __forceinline__ uint32_t group_scan(GroupCtl& G, uint32_t x, uint32_t
       if (lane >= o) inc += y;
     }
   }
-  if (lane == 31) G.wtot[w] = inc;
+  if (lane == 31) wtot[w] = inc;
   bar_sync(bid, v);                                                    // B2
   uint32_t pre = 0, tot = 0;
   for (int k = 0; k < (v >> 5); ++k) {
-    const uint32_t t = G.wtot[k];
+    const uint32_t t = wtot[k];
     pre += (k < w) ? t : 0u;
     tot += t;
   }
@@ -537,15 +593,96 @@ __device__ __forceinline__ void bar_arrive(int id, int n) {
   asm volatile("bar.arrive %0, %1;" ::"r"(id), "r"(n) : "memory");
 }
 
+
+// K items of one lane through stage KIND (compile-time), written so that the K
+// independent items interleave: S0/S1 read their k-mer words from the smem DB window
+// with no per-item branch when the whole warp is inside it.
+template <int K, int KIND>
+__device__ __forceinline__ void stage_batch(const Node& nd, const Dna& dna, const DevParams& p, const uint2 (&e)[K],
+                                            const bool (&act)[K], LaneOut (&o)[K]) {
+#pragma unroll
+  for (int j = 0; j < K; ++j) { o[j].c = 0; o[j].a = 0; o[j].score = 0; o[j].q_start = 0; o[j].len = 0; }
+  if constexpr (KIND == PL_SEED_LOOKUP || KIND == PL_HIT_ENUM) {
+    uint32_t r[K];
+    bool inwin = true;
+#pragma unroll
+    for (int j = 0; j < K; ++j) {
+      r[j] = (uint32_t)((int64_t)(e[j].x >> 4) - dna.win_lo);
+      inwin &= r[j] + 1u < dna.win_n;
+    }
+    uint32_t key[K];
+    if (__all_sync(0xffffffffu, inwin)) {
+#pragma unroll
+      for (int j = 0; j < K; ++j) {
+        const uint32_t x = __funnelshift_r(dna.win[r[j]], dna.win[r[j] + 1], (e[j].x & 15u) * 2u);
+        uint32_t kk = 0;
+#pragma unroll
+        for (int b = 0; b < PL_MAX_K; ++b)
+          if (b < dna.k) kk = (kk << 2) | ((x >> (2 * b)) & 3u);
+        key[j] = kk;
+      }
+    } else {
+#pragma unroll
+      for (int j = 0; j < K; ++j) key[j] = dna.key(e[j].x);
+    }
+#pragma unroll
+    for (int j = 0; j < K; ++j) {
+      const uint32_t lo = dna.qoff[key[j]], hi = dna.qoff[key[j] + 1];
+      if (KIND == PL_SEED_LOOKUP) {
+        o[j].c = (act[j] && hi > lo) ? 1u : 0u;
+      } else {
+        const uint32_t cnt = hi - lo;
+        o[j].a = lo;
+        o[j].c = act[j] ? (cnt < nd.max_out ? cnt : nd.max_out) : 0u;
+      }
+    }
+  } else if constexpr (KIND == PL_BERNOULLI) {
+#pragma unroll
+    for (int j = 0; j < K; ++j) o[j].c = (act[j] && gain_hash(p.seed, nd.i, e[j].x, e[j].y) < p.st[nd.i].thr[0]) ? 1u : 0u;
+  } else if constexpr (KIND == PL_FIXED_GAIN) {
+#pragma unroll
+    for (int j = 0; j < K; ++j) o[j].c = act[j] ? nd.cfix : 0u;
+  } else if constexpr (KIND == PL_KEEP_EVERY) {
+#pragma unroll
+    for (int j = 0; j < K; ++j) o[j].c = (act[j] && (e[j].x % nd.cfix) == 0) ? 1u : 0u;
+  } else if constexpr (KIND == PL_POISSON_CAPPED) {
+#pragma unroll
+    for (int j = 0; j < K; ++j) {
+      const uint64_t h = gain_hash(p.seed, nd.i, e[j].x, e[j].y);
+      uint32_t n = 0;
+      for (uint32_t q = 0; q < nd.max_out; ++q) n += (h >= p.st[nd.i].thr[q]) ? 1u : 0u;
+      o[j].c = act[j] ? n : 0u;
+    }
+  } else {   // S2 window filter / S3 x-drop: per item, one shared copy of the code
+#pragma unroll
+    for (int j = 0; j < K; ++j)
+      if (act[j]) o[j] = stage_count_ext(nd, dna, e[j]);
+  }
+}
+
+template <int KIND>
+__device__ __forceinline__ uint2 stage_output_k(const Node& nd, const Dna& dna, uint2 e, const LaneOut& o, uint32_t j) {
+  if constexpr (KIND == PL_FIXED_GAIN) return make_uint2(e.x, e.y * nd.cfix + j);
+  else if constexpr (KIND == PL_POISSON_CAPPED) return make_uint2(e.x, e.y * nd.max_out + j);
+  else if constexpr (KIND == PL_HIT_ENUM) return make_uint2(e.x, (uint32_t)dna.qpos[o.a + j] | (j << 16));
+  else return e;
+}
+
 // ------------------------------------------------------------------- node loop
-// Per firing: leader decides (+ reserves output room, + paces in physical mode)
-// -> B1 -> lanes load / run the stage / scan (B2) -> leader releases the input
-// slots -> lanes compact their outputs -> B4 (arrive; the leader's warp syncs)
-// -> leader publishes the segment and its watermark.
+// One warp group of v threads per node, one item per lane.  Measured faster on B200 than
+// one warp with v/32 items per lane: the group's warps run the per-item latency chains in
+// parallel (tools/node_scaling.py; profiles/r01_phase_cycles_*).
+// Per firing of node i >= 1: leader decides (+ reserves output room, + paces) -> B1 ->
+// lanes load / run the stage / scan (B2) -> leader releases the input slots -> lanes
+// compact their outputs -> B4 (arrive; the leader's warp syncs) -> leader publishes the
+// segment and its watermark.  Node 0 skips B1: its arrivals are fully known, so every lane
+// evaluates the decision itself and the leader's reservation reaches the lanes through
+// B2.  Broadcast slots are double-buffered by firing parity.
 __device__ void run_node(Ctx& c, const Dna dna, int i, int gtid) {
   const DevParams& p = *c.p;
   const Node nd = make_node(c, i);
   const int v = nd.v, N = nd.N;
+  const bool n0 = i == 0;
   const bool leader = gtid == 0;
   const int bidA = 1 + i;
   const int bidB = (i < 7) ? 9 + i : bidA;       // barrier ids 9..15 for the output barrier
@@ -553,139 +690,180 @@ __device__ void run_node(Ctx& c, const Dna dna, int i, int gtid) {
   const uint32_t stream = blockIdx.x;
   const uint32_t rec = p.flags;
   const uint64_t T0 = c.sh->T0;
+  const uint32_t lt_mask = (1u << (gtid & 31)) - 1u;
 
   Leader L;
   L.m = 0; L.B = 0; L.c0 = 0; L.head = 0; L.segh = 0; L.out_tail = 0; L.out_segt = 0;
   L.W_pub = -1; L.empties = 0;
+  Rep R;
+  R.m = 0; R.B = 0; R.c0 = 0; R.empties = 0;
   uint64_t firings = 0, consumed = 0, produced = 0, spilled = 0, overruns = 0;
   int64_t active = 0, busy_ns = 0, lateness = 0, t_end = 0, max_fire = 0;
-  uint64_t start_ns = 0, end_ns_prev = 0;
+  uint64_t start_ns = 0;
   uint32_t pend_root = NO_ROOT;          // lane: physical terminal event awaiting its end time
   uint64_t ph[6] = {0, 0, 0, 0, 0, 0};   // leader: per-phase clock64 cycles
   long long tc = 0;
+  int par = 0;
+  if (leader) { G.end_ns[0] = 0; G.end_ns[1] = 0; }
 
   for (;;) {
-    if (leader) {
-      const long long c0 = clock64();
-      const Decision d = decide(nd, L);
-      G.done = d.done ? 1u : 0u;
-      G.T = d.T;
-      G.n = d.n;
-      G.head = (i == 0) ? (uint32_t)L.c0 : L.head;
-      G.segh = L.segh;
-      if (i > 0) {
-        G.st = vld(&nd.Ein->seg_tail);
-        __threadfence_block();
-        G.in_spill_end = vld(&nd.Ein->spill_end);
-      }
-      G.end_ns_prev = end_ns_prev;
-      if (!d.done) {
-        if (rec & PL_REC_FIRINGS) G.log_idx = atomicAdd(&c.sh->log_count, 1u);
-        G.out_loc = nd.sink ? LOC_SMEM : reserve_out(nd, L, d.n * nd.umax, &c.sh->errors);
-        G.out_base = L.out_tail;
-      } else {
-        publish_W(nd, L, PL_INF64);
-      }
-      tc = clock64();
-      ph[0] += (uint64_t)(tc - c0);
-      if (!d.done && nd.phys) {
-        int64_t late;
-        pace(T0, nd.nspu, d.T, &start_ns, &late);
-        if (late > lateness) lateness = late;
+    int64_t T;
+    uint32_t n, head;
+    if (n0) {
+      const long long c0 = leader ? clock64() : 0;
+      const Decision d = decide0(nd, R);
+      if (d.done) break;
+      T = d.T; n = d.n; head = (uint32_t)R.c0;
+      if (leader) {
+        if (rec & PL_REC_FIRINGS) G.log_idx[par] = atomicAdd(&c.sh->log_count, 1u);
+        G.out_loc[par] = nd.sink ? LOC_SMEM : reserve_out(nd, L, n * nd.umax, &c.sh->errors);
+        G.out_base[par] = L.out_tail;
         tc = clock64();
+        ph[0] += (uint64_t)(tc - c0);
       }
+      if (nd.phys && (gtid & 31) == 0) {   // every warp paces itself against %globaltimer
+        uint64_t s_ns; int64_t late;
+        pace(T0, nd.nspu, T, &s_ns, &late);
+        if (leader) { start_ns = s_ns; if (late > lateness) lateness = late; tc = clock64(); }
+      }
+      __syncwarp();
+    } else {
+      if (leader) {
+        const long long c0 = clock64();
+        const Decision d = decide(nd, L);
+        G.done[par] = d.done ? 1u : 0u;
+        G.T[par] = d.T;
+        G.n[par] = d.n;
+        G.head[par] = L.head;
+        G.segh[par] = L.segh;
+        G.st[par] = vld(&nd.Ein->seg_tail);
+        __threadfence_block();
+        G.in_spill_end[par] = vld(&nd.Ein->spill_end);
+        if (!d.done) {
+          if (rec & PL_REC_FIRINGS) G.log_idx[par] = atomicAdd(&c.sh->log_count, 1u);
+          G.out_loc[par] = nd.sink ? LOC_SMEM : reserve_out(nd, L, d.n * nd.umax, &c.sh->errors);
+          G.out_base[par] = L.out_tail;
+        } else {
+          publish_W(nd, L, PL_INF64);
+        }
+        tc = clock64();
+        ph[0] += (uint64_t)(tc - c0);
+        if (!d.done && nd.phys) {
+          int64_t late;
+          pace(T0, nd.nspu, d.T, &start_ns, &late);
+          if (late > lateness) lateness = late;
+          tc = clock64();
+        }
+      }
+      bar_sync(bidA, v);                                               // B1: decision
+      if (leader) { const long long t2 = clock64(); ph[1] += (uint64_t)(t2 - tc); tc = t2; }
+      if (pend_root != NO_ROOT) {        // deferred physical latency of the previous firing
+        const uint64_t a_ns = T0 + (uint64_t)((double)nd.arrival(pend_root) * nd.nspu);
+        const int64_t l = (int64_t)G.end_ns[par ^ 1] - (int64_t)a_ns;
+        if (rec & PL_REC_LATENCY) atomicMax((long long*)&p.lat_ns[pend_root], (long long)l);
+        atomicMax(&c.sh->max_lat_ns, (uint32_t)(l > 0 ? (l < 0xffffffffll ? l : 0xffffffffll) : 0));
+        pend_root = NO_ROOT;
+      }
+      if (G.done[par]) break;
+      T = G.T[par]; n = G.n[par]; head = G.head[par];
     }
-    bar_sync(bidA, v);                                                 // B1: decision
-    if (leader) { const long long t2 = clock64(); ph[1] += (uint64_t)(t2 - tc); tc = t2; }
-    if (pend_root != NO_ROOT) {          // deferred physical latency of the previous firing
+    const bool act = (uint32_t)gtid < n;
+    uint2 e[1];
+    const bool acts[1] = {act};
+    LaneOut o[1];
+    {
+      const uint32_t ld = act ? (uint32_t)gtid : 0u;   // inactive lanes repeat a valid entry
+      if (n0) e[0] = make_uint2((uint32_t)(nd.lo + head + ld), 0u);
+      else e[0] = load_entry(nd, head + ld, G.segh[par], G.st[par], G.in_spill_end[par]);
+    }
+    switch (nd.kind) {   // warp-uniform dispatch to the stage body
+      case PL_SEED_LOOKUP: stage_batch<1, PL_SEED_LOOKUP>(nd, dna, p, e, acts, o); break;
+      case PL_HIT_ENUM: stage_batch<1, PL_HIT_ENUM>(nd, dna, p, e, acts, o); break;
+      case PL_BERNOULLI: stage_batch<1, PL_BERNOULLI>(nd, dna, p, e, acts, o); break;
+      case PL_FIXED_GAIN: stage_batch<1, PL_FIXED_GAIN>(nd, dna, p, e, acts, o); break;
+      case PL_KEEP_EVERY: stage_batch<1, PL_KEEP_EVERY>(nd, dna, p, e, acts, o); break;
+      case PL_POISSON_CAPPED: stage_batch<1, PL_POISSON_CAPPED>(nd, dna, p, e, acts, o); break;
+      default: stage_batch<1, PL_UNGAPPED_WINDOW>(nd, dna, p, e, acts, o); break;   // S2 / S3
+    }
+    uint32_t total;
+    const uint32_t off = group_scan(G.wtot[par], o[0].c, &total, gtid, v, bidA, nd.umax <= 1);   // B2
+    if (leader) { const long long t2 = clock64(); ph[2] += (uint64_t)(t2 - tc); tc = t2; }
+    if (n0 && pend_root != NO_ROOT) {    // node 0: the previous publish time arrives through B2
       const uint64_t a_ns = T0 + (uint64_t)((double)nd.arrival(pend_root) * nd.nspu);
-      const int64_t l = (int64_t)G.end_ns_prev - (int64_t)a_ns;
+      const int64_t l = (int64_t)G.end_ns[par ^ 1] - (int64_t)a_ns;
       if (rec & PL_REC_LATENCY) atomicMax((long long*)&p.lat_ns[pend_root], (long long)l);
-      atomicMax(&c.sh->max_lat_ns, (unsigned long long)(l > 0 ? l : 0));
+      atomicMax(&c.sh->max_lat_ns, (uint32_t)(l > 0 ? (l < 0xffffffffll ? l : 0xffffffffll) : 0));
       pend_root = NO_ROOT;
     }
-    if (G.done) break;
-    const int64_t T = G.T;
-    const uint32_t n = G.n, head = G.head;
-    const bool act = (uint32_t)gtid < n;
-    uint2 e = make_uint2(0u, 0u);
-    if (act) {
-      if (i == 0) e = make_uint2((uint32_t)(nd.lo + head + gtid), 0u);
-      else e = load_entry(nd, head + gtid, G.segh, G.st, G.in_spill_end);
-    }
-    LaneOut o;
-    if (act) o = stage_count(nd, dna, p, e);
-    else { o.c = 0; o.a = 0; o.score = 0; o.q_start = 0; o.len = 0; }
-    uint32_t total;
-    const uint32_t off = group_scan(G, o.c, &total, gtid, v, bidA, nd.umax <= 1);   // B2 inside
-    if (leader) { const long long t2 = clock64(); ph[2] += (uint64_t)(t2 - tc); tc = t2; }
     // --- release the input slots (every lane has loaded its entry: B2 passed)
-    if (leader && i > 0) {
+    if (leader && !n0) {
       L.head = head + n;
-      const uint32_t st = G.st;
+      const uint32_t st = G.st[par];
       while (L.segh != st && (int32_t)(nd.in_seg[L.segh & nd.segmask].end - L.head) <= 0) ++L.segh;
       __threadfence_block();
       vst(&nd.Ein->head, L.head);
       vst(&nd.Ein->seg_head, L.segh);
     }
-    // --- per-item records: trace, terminal events (reading R-DONE)
-    const bool term = act && (nd.sink || o.c == 0);
-    const int64_t lat = term ? T + nd.t - nd.arrival(e.x) : 0;
-    if (act) {
-      if (rec & PL_REC_TRACE) {
-        atomicAdd(&p.trace[(uint64_t)e.x * (N + 1) + i], 1u);
-        if (nd.sink && o.c) atomicAdd(&p.trace[(uint64_t)e.x * (N + 1) + N], o.c);
+    // --- per-item records: terminal events (reading R-DONE), trace, log
+    const uint2 ei = e[0];
+    const LaneOut oi = o[0];
+    const bool term = act && (nd.sink || oi.c == 0);
+    const int64_t lat = T + nd.t - nd.arrival(ei.x);
+    if (rec) {                            // optional per-item records (parity / tracing runs)
+      if (act && (rec & PL_REC_TRACE)) {
+        atomicAdd(&p.trace[(uint64_t)ei.x * (N + 1) + i], 1u);
+        if (nd.sink && oi.c) atomicAdd(&p.trace[(uint64_t)ei.x * (N + 1) + N], oi.c);
       }
-      if (term) {
-        if (rec & PL_REC_LATENCY) atomicMax((long long*)&p.lat[e.x], (long long)lat);
-        if (nd.phys) pend_root = e.x;
-      }
-      if ((rec & PL_REC_FIRINGS) && (gtid == 0 || (uint32_t)gtid == n - 1)) {
-        const uint32_t li = G.log_idx;
+      if (term && (rec & PL_REC_LATENCY)) atomicMax((long long*)&p.lat[ei.x], (long long)lat);
+      if (act && (rec & PL_REC_FIRINGS) && (gtid == 0 || (uint32_t)gtid == n - 1)) {
+        const uint32_t li = G.log_idx[par];
         if (li < p.log_cap) {
           pl_firing* f = p.flog + (uint64_t)stream * p.log_cap + li;
-          if (gtid == 0) { f->start = T; f->node = i; f->n = n; f->first_root = e.x; f->stream = stream; f->pad = 0; }
-          if ((uint32_t)gtid == n - 1) f->last_root = e.x;
+          if (gtid == 0) { f->start = T; f->node = i; f->n = n; f->first_root = ei.x; f->stream = stream; f->pad = 0; }
+          if ((uint32_t)gtid == n - 1) f->last_root = ei.x;
         } else if (gtid == 0) {
           atomicOr(&c.sh->errors, PL_ERR_LOG_OVERFLOW);
         }
       }
     }
-    {   // per-stream max latency / deadline misses / matches: one atomic per warp
-      const uint32_t lmax = __reduce_max_sync(0xffffffffu, (uint32_t)(lat > 0 ? (lat < 0xffffffffll ? lat : 0xffffffffll) : 0));
+    if (term && nd.phys) pend_root = ei.x;
+    {   // per-stream max latency / deadline misses: one smem atomic per warp
+      const uint32_t l32 = term ? (uint32_t)(lat > 0 ? (lat < 0xffffffffll ? lat : 0xffffffffll) : 0) : 0u;
+      const uint32_t lmax = __reduce_max_sync(0xffffffffu, l32);
       const uint32_t missb = __ballot_sync(0xffffffffu, term && lat > nd.D);
       if ((gtid & 31) == 0) {
-        if (lmax) atomicMax(&c.sh->max_lat, (unsigned long long)lmax);
-        if (missb) atomicAdd(&c.sh->miss_events, (unsigned long long)__popc(missb));
+        if (lmax) atomicMax(&c.sh->max_lat, lmax);
+        if (missb) atomicAdd(&c.sh->miss_events, (uint32_t)__popc(missb));
       }
-      if (nd.sink && nd.kind == PL_UNGAPPED_XDROP) {
-        const uint32_t mb = __ballot_sync(0xffffffffu, act && o.c);
-        if (mb) {
-          unsigned long long base = 0;
-          if ((gtid & 31) == 0) base = atomicAdd(p.match_count, (unsigned long long)__popc(mb));
-          base = __shfl_sync(0xffffffffu, base, 0);
-          if (act && o.c) {
-            const unsigned long long mi = base + __popc(mb & ((1u << (gtid & 31)) - 1u));
-            if (mi < p.match_cap) {
-              pl_match mt;
-              mt.p = e.x; mt.q = e.y & 0xffffu; mt.db_start = o.a; mt.q_start = o.q_start;
-              mt.len = o.len; mt.score = o.score;
-              p.matches[mi] = mt;
-            } else {
-              atomicOr(&c.sh->errors, PL_ERR_MATCH_OVERFLOW);
-            }
+    }
+    if (nd.sink && nd.kind == PL_UNGAPPED_XDROP) {   // matches: one global atomic per warp
+      const bool hit = act && oi.c;
+      const uint32_t mb = __ballot_sync(0xffffffffu, hit);
+      if (mb) {
+        unsigned long long base = 0;
+        if ((gtid & 31) == 0) base = atomicAdd(p.match_count, (unsigned long long)__popc(mb));
+        base = __shfl_sync(0xffffffffu, base, 0);
+        if (hit) {
+          const unsigned long long mi = base + __popc(mb & lt_mask);
+          if (mi < p.match_cap) {
+            pl_match mt;
+            mt.p = ei.x; mt.q = ei.y & 0xffffu; mt.db_start = oi.a; mt.q_start = oi.q_start;
+            mt.len = oi.len; mt.score = oi.score;
+            p.matches[mi] = mt;
+          } else {
+            atomicOr(&c.sh->errors, PL_ERR_MATCH_OVERFLOW);
           }
         }
       }
     }
     if (leader) { const long long t2 = clock64(); ph[3] += (uint64_t)(t2 - tc); tc = t2; }
     // --- compaction into the next queue (stable: lane order, then child order)
-    const uint32_t out_loc = G.out_loc;
-    if (!nd.sink && act && o.c && out_loc != ~0u) {
-      const uint32_t base = G.out_base + off;
-      for (uint32_t j = 0; j < o.c; ++j) {
+    const uint32_t out_loc = G.out_loc[par];
+    if (!nd.sink && act && oi.c && out_loc != ~0u) {
+      const uint32_t base = G.out_base[par] + off;
+      for (uint32_t j = 0; j < oi.c; ++j) {
         const uint32_t s = base + j;
-        const uint2 val = stage_output(nd, dna, e, o, j);
+        const uint2 val = stage_output(nd, dna, ei, oi, j);
         if (out_loc == LOC_SMEM) nd.out_ent[s & (nd.out_cap - 1)] = val;
         else __stcg(nd.out_spill + (s & (nd.capg - 1)), val);
       }
@@ -706,7 +884,7 @@ __device__ void run_node(Ctx& c, const Dna dna, int i, int gtid) {
           }
         }
         busy_ns += (int64_t)(en - start_ns);
-        end_ns_prev = en;
+        G.end_ns[par] = en;
       }
       ++firings;
       consumed += n;
@@ -726,21 +904,35 @@ __device__ void run_node(Ctx& c, const Dna dna, int i, int gtid) {
         vst(&nd.Eout->seg_tail, L.out_segt);
         vst(&nd.Eout->tail, L.out_tail);
       }
-      if (i == 0) L.c0 += n;
       if (nd.fixed) {
         ++L.m;
-        publish_W(nd, L, L.m * nd.P + nd.t);
+        publish_W(nd, L, (n0 ? R.m + 1 : L.m) * nd.P + nd.t);
       } else {
         L.B = T + nd.t;
         publish_W(nd, L, L.B + nd.t);
       }
       ph[5] += (uint64_t)(clock64() - tc);
     }
+    if (n0) {                            // replicated node-0 state, identical in every lane
+      R.c0 += n;
+      if (nd.fixed) ++R.m; else R.B = T + nd.t;
+    }
+    par ^= 1;
+  }
+  if (n0) {
+    if (leader) publish_W(nd, L, PL_INF64);   // after the last segment was published
+    bar_sync(bidA, v);                   // the last publish time is visible to every lane
+    if (pend_root != NO_ROOT) {
+      const uint64_t a_ns = T0 + (uint64_t)((double)nd.arrival(pend_root) * nd.nspu);
+      const int64_t l = (int64_t)G.end_ns[par ^ 1] - (int64_t)a_ns;
+      if (rec & PL_REC_LATENCY) atomicMax((long long*)&p.lat_ns[pend_root], (long long)l);
+      atomicMax(&c.sh->max_lat_ns, (uint32_t)(l > 0 ? (l < 0xffffffffll ? l : 0xffffffffll) : 0));
+    }
   }
   if (leader) {
     CtaStats& S = p.stats[stream];
     S.firings[i] = firings;
-    S.empty[i] = L.empties;
+    S.empty[i] = n0 ? R.empties : L.empties;
     S.consumed[i] = consumed;
     S.produced[i] = produced;
     S.active_ne[i] = active;
@@ -787,11 +979,7 @@ __device__ void cta_setup(Ctx& c, Shared& sh, unsigned char* dsm, const DevParam
   c.hi = (p.total_roots * (s + 1)) / (uint64_t)p.n_streams;
   c.X = (int64_t)(c.hi - c.lo);
   c.H = c.X * p.tau;
-  for (int i = 0; i < PL_MAX_STAGES; ++i) {
-    c.ent[i] = (uint2*)(dsm + Lo.off_ent[i]);
-    c.seg[i] = (Seg*)(dsm + Lo.off_seg[i]);
-    c.spill[i] = p.spill ? p.spill + ((uint64_t)s * p.N + i) * p.cap_g : nullptr;
-  }
+  c.dsm = dsm;
   c.dna.db = p.db;
   c.dna.nwords = p.db_words;
   c.dna.db_len = p.db_len;
@@ -804,48 +992,53 @@ __device__ void cta_setup(Ctx& c, Shared& sh, unsigned char* dsm, const DevParam
   c.dna.win = (const uint32_t*)(dsm + Lo.off_win);
   c.dna.win_lo = 0;
   c.dna.win_n = 0;
-  if (p.k > 0 && p.win_cap > 0 && c.hi > c.lo) {
-    // this stream's DB window: roots [lo, hi) plus the k-1 overlap and a halo for
-    // the extensions, in 16-byte units (4 words) so that one TMA bulk copy moves it
-    int64_t wlo = ((int64_t)c.lo - (int64_t)p.win_halo) >> 4;
-    int64_t whi = (((int64_t)c.hi + p.k + (int64_t)p.win_halo) >> 4) + 1;
-    wlo = wlo < 0 ? 0 : (wlo & ~3ll);
-    whi = (whi + 3) & ~3ll;
-    if (whi > (int64_t)p.db_alloc_words) whi = (int64_t)p.db_alloc_words & ~3ll;
-    if (whi - wlo > (int64_t)p.win_cap) whi = wlo + p.win_cap;
+  // DNA: the query index (offsets, positions, packed query) and this stream's DB window
+  // (its roots plus the k-1 overlap and a halo for the extensions) are staged into smem
+  // by TMA bulk copies (cp.async.bulk, one mbarrier), falling back to plain loads for an
+  // unaligned caller-owned DB.
+  if (p.k > 0) {
+    const uint32_t nko = (1u << (2 * p.k)) + 1u, nqp = (uint32_t)(p.q_len - p.k + 1);
+    const uint32_t nqw = (uint32_t)(p.q_len + 15) / 16u;
+    const uint32_t b_qo = (nko * 2u + 15u) & ~15u, b_qp = (nqp * 2u + 15u) & ~15u, b_qw = (nqw * 4u + 15u) & ~15u;
+    int64_t wlo = 0, whi = 0;
+    if (p.win_cap > 0 && c.hi > c.lo) {
+      wlo = ((int64_t)c.lo - (int64_t)p.win_halo) >> 4;
+      whi = (((int64_t)c.hi + p.k + (int64_t)p.win_halo) >> 4) + 1;
+      wlo = wlo < 0 ? 0 : (wlo & ~3ll);
+      whi = (whi + 3) & ~3ll;
+      if (whi > (int64_t)p.db_alloc_words) whi = (int64_t)p.db_alloc_words & ~3ll;
+      if (whi - wlo > (int64_t)p.win_cap) whi = wlo + p.win_cap;
+      if (whi < wlo) whi = wlo;
+    }
     c.dna.win_lo = wlo;
-    c.dna.win_n = whi > wlo ? (uint32_t)(whi - wlo) : 0u;
+    c.dna.win_n = (uint32_t)(whi - wlo);
     uint32_t* win = (uint32_t*)(dsm + Lo.off_win);
-    if (p.db_tma && c.dna.win_n) {
-      if (tid == 0) {
-        const uint32_t bar = (uint32_t)__cvta_generic_to_shared(&sh.mbar);
-        const uint32_t bytes = c.dna.win_n * 4u;
-        asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(bar));
-        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
-        asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(bar), "r"(bytes) : "memory");
-        const uint32_t dst = (uint32_t)__cvta_generic_to_shared(win);
+    const bool win_tma = p.db_tma && c.dna.win_n;
+    if (tid == 0) {
+      const uint32_t bar = (uint32_t)__cvta_generic_to_shared(&sh.mbar);
+      const uint32_t bytes = b_qo + b_qp + b_qw + (win_tma ? c.dna.win_n * 4u : 0u);
+      asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(bar));
+      asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+      asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(bar), "r"(bytes) : "memory");
+      const void* src[4] = {p.qoff, p.qpos, p.qwords, p.db + wlo};
+      const uint32_t off[4] = {Lo.off_qoff, Lo.off_qpos, Lo.off_qw, Lo.off_win};
+      const uint32_t len[4] = {b_qo, b_qp, b_qw, win_tma ? c.dna.win_n * 4u : 0u};
+      for (int j = 0; j < 4; ++j) {
+        if (!len[j]) continue;
+        const uint32_t dst = (uint32_t)__cvta_generic_to_shared(dsm + off[j]);
         asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
-                     ::"r"(dst), "l"(p.db + wlo), "r"(bytes), "r"(bar) : "memory");
-        uint32_t done = 0;
-        while (!done)
-          asm volatile("{ .reg .pred q; mbarrier.try_wait.parity.shared::cta.b64 q, [%1], 0; selp.u32 %0, 1, 0, q; }"
-                       : "=r"(done) : "r"(bar) : "memory");
+                     ::"r"(dst), "l"(src[j]), "r"(len[j]), "r"(bar) : "memory");
       }
-    } else {
+      uint32_t done = 0;
+      while (!done)
+        asm volatile("{ .reg .pred q; mbarrier.try_wait.parity.shared::cta.b64 q, [%1], 0; selp.u32 %0, 1, 0, q; }"
+                     : "=r"(done) : "r"(bar) : "memory");
+    }
+    if (!win_tma)
       for (uint32_t j = tid; j < c.dna.win_n; j += nt) {
         const int64_t w = wlo + j;
         win[j] = w < (int64_t)p.db_words ? p.db[w] : 0u;
       }
-    }
-  }
-  if (p.k > 0) {   // query index -> smem
-    uint16_t* qo = (uint16_t*)(dsm + Lo.off_qoff);
-    uint16_t* qp = (uint16_t*)(dsm + Lo.off_qpos);
-    uint32_t* qw = (uint32_t*)(dsm + Lo.off_qw);
-    const uint32_t nko = (1u << (2 * p.k)) + 1u, nqp = (uint32_t)(p.q_len - p.k + 1), nqw = (uint32_t)(p.q_len + 15) / 16u;
-    for (uint32_t j = tid; j < nko; j += nt) qo[j] = p.qoff[j];
-    for (uint32_t j = tid; j < nqp; j += nt) qp[j] = p.qpos[j];
-    for (uint32_t j = tid; j < nqw; j += nt) qw[j] = p.qwords[j];
   }
   if (tid < PL_MAX_STAGES) {
     EdgeCtl& E = sh.e[tid];
@@ -960,13 +1153,13 @@ __device__ void run_monolithic(Ctx& c) {
           if (sink || o.c == 0) {
             const int64_t l = end - arrival(c, e.x);
             if (rec & PL_REC_LATENCY) atomicMax((long long*)&p.lat[e.x], (long long)l);
-            atomicMax(&c.sh->max_lat, (unsigned long long)l);
-            if (l > p.D) atomicAdd(&c.sh->miss_events, 1ull);
+            atomicMax(&c.sh->max_lat, (uint32_t)(l > 0 ? (l < 0xffffffffll ? l : 0xffffffffll) : 0));
+            if (l > p.D) atomicAdd(&c.sh->miss_events, 1u);
             if (phys) {
               const uint64_t a_ns = c.sh->T0 + (uint64_t)((double)arrival(c, e.x) * p.ns_per_unit);
               const int64_t ln = (int64_t)gtimer() - (int64_t)a_ns;
               if (rec & PL_REC_LATENCY) atomicMax((long long*)&p.lat_ns[e.x], (long long)ln);
-              atomicMax(&c.sh->max_lat_ns, (unsigned long long)(ln > 0 ? ln : 0));
+              atomicMax(&c.sh->max_lat_ns, (uint32_t)(ln > 0 ? (ln < 0xffffffffll ? ln : 0xffffffffll) : 0));
             }
           }
           if ((rec & PL_REC_FIRINGS) && (idx % (uint32_t)v == 0 || idx == ncur - 1 || idx % (uint32_t)v == (uint32_t)v - 1)) {
@@ -1038,7 +1231,8 @@ __device__ void run_monolithic(Ctx& c) {
 
 }  // namespace
 
-// FIXED_WAIT / THRESHOLD_SLACK executor: grid = n_streams, block = N*v threads.
+// FIXED_WAIT / THRESHOLD_SLACK executor: grid = n_streams, block = N*32 threads (one warp
+// per node); up to 4 CTAs (streams) per SM when N <= 4.
 template <int MAXT>
 __global__ void __launch_bounds__(MAXT, 1) pl_exec_enforced(const __grid_constant__ DevParams p) {
   extern __shared__ __align__(16) unsigned char dsm[];
@@ -1077,11 +1271,11 @@ __global__ void __launch_bounds__(MAXT, 1) pl_exec_monolithic(const __grid_const
 // host-side launchers (the kernels are templates on the block-size bound)
 cudaError_t pl_launch(const DevParams& p, unsigned grid, unsigned block, unsigned smem, cudaStream_t st) {
   const bool mono = p.policy == PL_MONOLITHIC;
-  if (block <= 512) {
-    if (mono) pl_exec_monolithic<512><<<grid, block, smem, st>>>(p);
-    else pl_exec_enforced<512><<<grid, block, smem, st>>>(p);
+  if (mono) {
+    if (block <= 512) pl_exec_monolithic<512><<<grid, block, smem, st>>>(p);
+    else pl_exec_monolithic<1024><<<grid, block, smem, st>>>(p);
   } else {
-    if (mono) pl_exec_monolithic<1024><<<grid, block, smem, st>>>(p);
+    if (block <= 512) pl_exec_enforced<512><<<grid, block, smem, st>>>(p);
     else pl_exec_enforced<1024><<<grid, block, smem, st>>>(p);
   }
   return cudaGetLastError();

@@ -61,6 +61,7 @@ struct DevParams {
   uint32_t theta[PL_MAX_STAGES];        // THRESHOLD_SLACK thresholds
   int64_t  R[PL_MAX_STAGES];            // THRESHOLD_SLACK reserves (incl. guard)
   int64_t  D, tau;
+  uint64_t tau_m, P_m[PL_MAX_STAGES];    // reciprocals floor((2^64-1)/x) for division-free fdiv
   int64_t  M;                           // MONOLITHIC block size
   double   ns_per_unit;
   uint64_t seed;

@@ -310,6 +310,8 @@ pl_status pl_pipeline_create(const pl_config* cfg, const pl_workload* wl, pl_pip
   }
   d.D = cfg->deadline;
   d.tau = cfg->interarrival;
+  d.tau_m = d.tau > 1 ? ~0ull / (uint64_t)d.tau : 0;
+  for (uint32_t i = 0; i < N; ++i) d.P_m[i] = d.P[i] > 1 ? ~0ull / (uint64_t)d.P[i] : 0;
   d.M = pl->M;
   d.ns_per_unit = cfg->clock == PL_CLOCK_GLOBALTIMER ? cfg->ns_per_unit : 1.0;
   d.seed = cfg->seed;
@@ -347,9 +349,15 @@ pl_status pl_pipeline_create(const pl_config* cfg, const pl_workload* wl, pl_pip
     for (uint32_t j = 0; j < K; ++j) off[j + 1] += off[j];
     std::vector<uint16_t> fill(off.begin(), off.end() - 1);
     for (uint32_t q = 0; q < nq; ++q) pos[fill[keys[q]]++] = (uint16_t)q;
-    if (cudaMalloc(&pl->d_qoff, (K + 1) * 2) != cudaSuccess || cudaMalloc(&pl->d_qpos, nq * 2) != cudaSuccess ||
-        cudaMalloc(&pl->d_qw, nqw * 4) != cudaSuccess)
+    // padded to whole 16-byte units: the kernel stages them with cp.async.bulk
+    const size_t b_qo = ((K + 1) * 2 + 15) & ~size_t(15), b_qp = (nq * 2 + 15) & ~size_t(15),
+                 b_qw = (nqw * 4 + 15) & ~size_t(15);
+    if (cudaMalloc(&pl->d_qoff, b_qo) != cudaSuccess || cudaMalloc(&pl->d_qpos, b_qp) != cudaSuccess ||
+        cudaMalloc(&pl->d_qw, b_qw) != cudaSuccess)
       return bail(fail(PL_ENOMEM, "query index allocation"));
+    cudaMemset(pl->d_qoff, 0, b_qo);
+    cudaMemset(pl->d_qpos, 0, b_qp);
+    cudaMemset(pl->d_qw, 0, b_qw);
     cudaMemcpy(pl->d_qoff, off.data(), (K + 1) * 2, cudaMemcpyHostToDevice);
     cudaMemcpy(pl->d_qpos, pos.data(), nq * 2, cudaMemcpyHostToDevice);
     cudaMemcpy(pl->d_qw, pl->query.data(), nqw * 4, cudaMemcpyHostToDevice);
@@ -404,7 +412,7 @@ pl_status pl_pipeline_create(const pl_config* cfg, const pl_workload* wl, pl_pip
   } else {
     if (N > 1 && cudaMalloc(&pl->d_spill, (size_t)S * N * d.cap_g * sizeof(uint2)) != cudaSuccess)
       return bail(fail(PL_ENOMEM, "spill rings (%u streams x %u edges x %u)", S, N, d.cap_g));
-    pl->block = N * v;
+    pl->block = N * v;             // one warp group of v lanes per node (executor.cu run_node)
   }
   d.spill = pl->d_spill;
   d.mono_buf = pl->d_mono;

@@ -32,9 +32,10 @@ def measure_gains(cfg, wl, db_dev, stream=None):
     return tuple(st["produced"][i] / max(1, st["consumed"][i]) for i in range(N - 1))
 
 
-def calibrate_budgets(cfg, wl, db_dev, margin=1.25, slack_ns=256, probe_t=20_000, probe_tau=200, stream=None):
+def calibrate_budgets(cfg, wl, db_dev, margin=1.25, slack_ns=256, probe_t=20_000, probe_tau=100, stream=None):
     """Service-time budgets t_i (ns): the longest measured firing of each node in a
-    physical run with generous budgets, times `margin`, plus `slack_ns`."""
+    physical run with generous budgets, times `margin`, plus `slack_ns`.  The probe's
+    arrivals (probe_t / probe_tau > v per period) keep node 0's vectors full."""
     N = cfg.n_stages
     probe = cfg.replace(clock=PHYS, service_time=(probe_t,) * N, wait_time=(0,) * N, interarrival=probe_tau,
                         deadline=10**12, policy=0, gain=None, ns_per_unit=1.0)
@@ -65,8 +66,9 @@ def min_feasible_tau(cfg, lo=1, hi=1 << 20):
 
 
 def find_rate(cfg, wl, db_dev, tries=10, grow=1.15, stream=None, log=None):
-    """Smallest tau0 (ns) at which a physical FIXED_WAIT run has zero deadline misses,
-    zero overruns and no queue overflow.  Returns (tau0, w, theta, T, stats)."""
+    """Smallest tau0 (ns) at which a physical FIXED_WAIT run has zero deadline misses and
+    no queue overflow (budget overruns are counted and reported, not fatal: they delay
+    firings, and any delay that matters shows up as a miss).  Returns (tau0, w, theta, T, stats)."""
     tau = min_feasible_tau(cfg)
     if tau is None:
         raise RuntimeError("Fig. 1 infeasible for every tau0 at this deadline")
@@ -74,7 +76,7 @@ def find_rate(cfg, wl, db_dev, tries=10, grow=1.15, stream=None, log=None):
         w, th, T = solve_at(cfg, tau)
         c = cfg.replace(interarrival=int(tau), wait_time=tuple(w), clock=PHYS)
         st = _run(c, db_dev, wl.db_len, wl, flags=1, stream=stream)
-        ok = st["misses"] == 0 and sum(st["overruns"]) == 0 and st["errors"] == 0
+        ok = st["misses"] == 0 and st["errors"] == 0
         if log:
             log(dict(tau=tau, w=w, T=T, misses=st["misses"], overruns=st["overruns"], errors=st["errors"],
                      max_latency_ns=st["max_latency_ns"]))
