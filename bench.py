@@ -287,21 +287,34 @@ def main():
     logical_ips = 5 * pll.stats()["roots"] / (e0.elapsed_time(e1) * 1e-3)
     pll.close()
 
-    # monolithic baseline at the same (tau0, D)
+    # monolithic baseline (§5, Fig. 2): at the enforced rate, and at the fastest
+    # rate where both strategies are feasible (the paper's utilisation comparison, L236-L255)
+    def run_policy(policy, tau_x, M=0):
+        c = cfg.replace(interarrival=int(tau_x), policy=policy, block_size=M)
+        if policy == 0:
+            sol = realtime.solve_at(cfg, tau_x)
+            if sol is None:
+                return None
+            c = c.replace(wait_time=tuple(sol[0]))
+        pp = Pipeline(c, wl, flags=1, stream=stream)
+        pp.bind_device(db_ptr, wl.db_len)
+        pp.drain()
+        sx = pp.stats()
+        pp.close()
+        return {"tau0_ns": int(tau_x), "active_fraction": sx["active_fraction"],
+                "hw_busy_fraction": sx["hw_busy_fraction"], "misses": sx["misses"],
+                "max_latency_ns": sx["max_latency_ns"], **({"M": M} if policy == 2 else {})}
+
     mono = {}
     Mr = realtime.monolithic_at(cfg, tau)
-    if Mr is not None:
-        M, Tm = Mr
-        plm = Pipeline(cfg.replace(interarrival=tau, policy=2, block_size=M), wl, flags=1, stream=stream)
-        plm.bind_device(db_ptr, wl.db_len)
-        plm.drain()
-        sm = plm.stats()
-        plm.close()
-        mono = {"M": M, "fig2_objective": Tm, "active_fraction": sm["active_fraction"],
-                "hw_busy_fraction": sm["hw_busy_fraction"], "misses": sm["misses"],
-                "max_latency_ns": sm["max_latency_ns"]}
-    else:
-        mono = {"feasible": False}
+    mono["at_enforced_rate"] = run_policy(2, tau, Mr[0]) if Mr is not None else {"feasible": False}
+    tau_m = tau
+    while realtime.monolithic_at(cfg, tau_m) is None and tau_m < 100 * tau:
+        tau_m = int(math.ceil(tau_m * 1.05)) + 1
+    Mm = realtime.monolithic_at(cfg, tau_m)
+    if Mm is not None:
+        mono["common_rate"] = {"tau0_ns": tau_m, "monolithic": run_policy(2, tau_m, Mm[0]),
+                               "enforced": run_policy(0, tau_m), "fig2_objective": Mm[1]}
 
     # e2e through the C-ABI with host buffers (H2D of the DB and D2H of the stats each step)
     e2e = None

@@ -106,6 +106,8 @@ def _load():
         "pl_version": (C.c_char_p, []),
         "pl_solve_enforced_waits": (C.c_int32, [C.POINTER(pl_config), P, P, P, P]),
         "pl_solve_monolithic": (C.c_int32, [C.POINTER(pl_config), P, P]),
+        "pl_stage_batch": (C.c_int32, [P, C.c_uint32, P, C.c_uint64, C.c_uint64, P, C.c_uint64,
+                                       C.POINTER(C.c_uint64), C.POINTER(C.c_uint64)]),
     }
     for name, (res, args) in sig.items():
         fn = getattr(lib, name)
@@ -119,7 +121,7 @@ EXPORTED = ("pl_pipeline_create", "pl_pipeline_set_stream", "pl_pipeline_push", 
             "pl_pipeline_launch", "pl_pipeline_drain", "pl_pipeline_rewind", "pl_pipeline_stats",
             "pl_pipeline_results", "pl_pipeline_latency", "pl_pipeline_trace", "pl_pipeline_firings",
             "pl_pipeline_params", "pl_pipeline_destroy", "pl_last_error", "pl_solve_enforced_waits",
-            "pl_solve_monolithic", "pl_version")
+            "pl_solve_monolithic", "pl_version", "pl_stage_batch")
 
 
 class PlError(RuntimeError):

@@ -1288,3 +1288,88 @@ cudaError_t pl_kernel_attributes(unsigned max_smem) {
   if ((e = cudaFuncSetAttribute(pl_exec_monolithic<512>, cudaFuncAttributeMaxDynamicSharedMemorySize, max_smem))) return e;
   return cudaFuncSetAttribute(pl_exec_monolithic<1024>, cudaFuncAttributeMaxDynamicSharedMemorySize, max_smem);
 }
+
+// ------------------------------------------------------------- stage batch kernels
+// K-BENCH: one stage over a large batch, vectors of v inputs per CTA iteration, DB read
+// from global memory (no smem window), query index in smem; outputs compacted per vector
+// (block scan) and appended at an atomically reserved offset.
+template <int MAXT>
+__global__ void __launch_bounds__(MAXT, 1) pl_stage_batch_kernel(const __grid_constant__ DevParams p, int stage,
+                                                                 const uint2* in, uint64_t n, uint64_t first_root,
+                                                                 uint2* out, uint64_t cap, unsigned long long* cnt) {
+  extern __shared__ __align__(16) unsigned char dsm[];
+  __shared__ Shared sh;
+  __shared__ uint32_t wt[32];
+  __shared__ unsigned long long sbase;
+  Ctx c;
+  c.p = &p;
+  c.sh = &sh;
+  c.dsm = dsm;
+  c.lo = 0;
+  c.hi = p.total_roots;
+  c.X = (int64_t)p.total_roots;
+  c.H = c.X * p.tau;
+  SmemLayout Lo;
+  layout_enforced(p, &Lo);
+  c.dna.db = p.db; c.dna.nwords = p.db_words; c.dna.db_len = p.db_len; c.dna.k = p.k; c.dna.q_len = p.q_len;
+  c.dna.qoff = (const uint16_t*)(dsm + Lo.off_qoff);
+  c.dna.qpos = (const uint16_t*)(dsm + Lo.off_qpos);
+  c.dna.qw = (const uint32_t*)(dsm + Lo.off_qw);
+  c.dna.nqw = (uint32_t)(p.q_len + 15) / 16u;
+  c.dna.win = nullptr; c.dna.win_lo = 0; c.dna.win_n = 0;
+  const uint32_t tid = threadIdx.x, v = blockDim.x;
+  if (p.k > 0) {
+    const uint32_t nko = (1u << (2 * p.k)) + 1u, nqp = (uint32_t)(p.q_len - p.k + 1);
+    uint16_t* qo = (uint16_t*)(dsm + Lo.off_qoff);
+    uint16_t* qp = (uint16_t*)(dsm + Lo.off_qpos);
+    uint32_t* qw = (uint32_t*)(dsm + Lo.off_qw);
+    for (uint32_t j = tid; j < nko; j += v) qo[j] = p.qoff[j];
+    for (uint32_t j = tid; j < nqp; j += v) qp[j] = p.qpos[j];
+    for (uint32_t j = tid; j < c.dna.nqw; j += v) qw[j] = p.qwords[j];
+  }
+  if (tid == 0) { sh.errors = 0; }
+  __syncthreads();
+  const Node nd = make_node(c, stage);
+  const bool sink = stage == p.N - 1;
+  for (uint64_t vec = blockIdx.x; vec * v < n; vec += gridDim.x) {
+    const long long c0 = clock64();
+    const uint64_t idx = vec * v + tid;
+    const bool act = idx < n;
+    uint2 e = make_uint2(0u, 0u);
+    if (act) e = stage == 0 ? make_uint2((uint32_t)(first_root + idx), 0u) : __ldg(in + idx);
+    LaneOut o;
+    if (act) o = stage_count(nd, c.dna, p, e);
+    else { o.c = 0; o.a = 0; o.score = 0; o.q_start = 0; o.len = 0; }
+    uint32_t total;
+    const uint32_t off = block_scan(o.c, &total, wt);
+    if (tid == 0) sbase = total ? atomicAdd(cnt, (unsigned long long)total) : 0ull;
+    __syncthreads();
+    const unsigned long long base = sbase;
+    if (act && o.c) {
+      if (sink && nd.kind == PL_UNGAPPED_XDROP) {
+        const unsigned long long mi = base + off;
+        if (mi < p.match_cap) {
+          pl_match mt;
+          mt.p = e.x; mt.q = e.y & 0xffffu; mt.db_start = o.a; mt.q_start = o.q_start; mt.len = o.len; mt.score = o.score;
+          p.matches[mi] = mt;
+        }
+      } else if (!sink) {
+        for (uint32_t j = 0; j < o.c; ++j)
+          if (base + off + j < cap) out[base + off + j] = stage_output(nd, c.dna, e, o, j);
+      }
+    }
+    __syncthreads();
+    if (tid == 0) atomicMax(cnt + 1, (unsigned long long)(clock64() - c0));
+  }
+}
+
+cudaError_t pl_launch_stage_batch(const DevParams& p, int stage, const void* in, uint64_t n, uint64_t first_root,
+                                  void* out, uint64_t cap, unsigned long long* cnt, unsigned smem, cudaStream_t st) {
+  const unsigned v = (unsigned)p.v;
+  uint64_t vecs = (n + v - 1) / v;
+  unsigned grid = (unsigned)(vecs < 148u * 8u ? (vecs ? vecs : 1) : 148u * 8u);
+  cudaError_t e = cudaFuncSetAttribute(pl_stage_batch_kernel<256>, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024);
+  if (e) return e;
+  pl_stage_batch_kernel<256><<<grid, v, smem, st>>>(p, stage, (const uint2*)in, n, first_root, (uint2*)out, cap, cnt);
+  return cudaGetLastError();
+}

@@ -20,6 +20,8 @@
 
 cudaError_t pl_launch(const DevParams& p, unsigned grid, unsigned block, unsigned smem, cudaStream_t st);
 cudaError_t pl_kernel_attributes(unsigned max_smem);
+cudaError_t pl_launch_stage_batch(const DevParams& p, int stage, const void* in, uint64_t n, uint64_t first_root,
+                                  void* out, uint64_t cap, unsigned long long* cnt, unsigned smem, cudaStream_t st);
 uint32_t pl_layout_enforced_host(const DevParams& p);
 
 namespace plsolve {
@@ -120,16 +122,19 @@ struct pl_pipeline {
   uint32_t launches = 0;
   int device = 0;
   uint64_t h2d = 0, d2h = 0;  // bytes moved across the host boundary (cumulative)
+  unsigned long long* d_scratch = nullptr;   // stage-batch counters
 };
 
 namespace {
 
 void free_all(pl_pipeline* pl) {
   void* ptrs[] = {pl->d_db, pl->d_qoff, pl->d_qpos, pl->d_qw, pl->d_spill, pl->d_mono, pl->d_lat, pl->d_lat_ns,
-                  pl->d_trace, pl->d_matches, pl->d_match_count, pl->d_flog, pl->d_stats};
+                  pl->d_trace, pl->d_matches, pl->d_match_count, pl->d_flog, pl->d_stats, pl->d_scratch};
   for (void* p : ptrs)
     if (p) cudaFree(p);
 }
+
+bool v_too_big(const pl_pipeline* pl) { return pl->cfg.vector_width > 256; }
 
 pl_status validate(const pl_config* c, const pl_workload* wl) {
   if (!c) return fail(PL_EINVAL, "cfg is NULL");
@@ -681,6 +686,43 @@ pl_status pl_pipeline_firings(pl_pipeline* pl, pl_firing* buf, uint64_t cap, uin
     w += c;
   }
   *n = w;
+  return PL_OK;
+}
+
+pl_status pl_stage_batch(pl_pipeline* pl, uint32_t stage, const void* in_dev, uint64_t n, uint64_t first_root,
+                         void* out_dev, uint64_t cap, uint64_t* n_out, uint64_t* max_vec_cycles) {
+  if (!pl || !n_out) return fail(PL_EINVAL, "NULL argument");
+  if (stage >= pl->cfg.n_stages) return fail(PL_EINVAL, "stage %u out of range", stage);
+  if (stage > 0 && n && !in_dev) return fail(PL_EINVAL, "stage > 0 needs input entries");
+  if (pl->dna && pl->pushed < (uint64_t)pl->k) return fail(PL_ESTATE, "push or bind the DB first");
+  if (v_too_big(pl)) return fail(PL_EINVAL, "vector_width > 256");
+  cudaSetDevice(pl->device);
+  DevParams d = pl->dp;
+  if (pl->dna) {
+    d.db = pl->d_db_bound ? pl->d_db_bound : pl->d_db;
+    d.db_len = pl->pushed;
+    d.db_words = (uint32_t)((pl->pushed + 15) / 16);
+    d.total_roots = pl->pushed - pl->k + 1;
+  } else {
+    d.total_roots = first_root + n;
+  }
+  d.win_cap = 0;
+  if (!pl->d_scratch && cudaMalloc(&pl->d_scratch, 16) != cudaSuccess) return fail(PL_ENOMEM, "scratch");
+  CUDA_TRY(cudaMemsetAsync(pl->d_scratch, 0, 16, pl->stream));
+  if (stage == pl->cfg.n_stages - 1) CUDA_TRY(cudaMemsetAsync(pl->d_match_count, 0, 8, pl->stream));
+  const uint32_t smem = pl_layout_enforced_host(d);
+  CUDA_TRY(pl_launch_stage_batch(d, (int)stage, in_dev, n, first_root, out_dev, cap, pl->d_scratch, smem, pl->stream));
+  unsigned long long h[2];
+  CUDA_TRY(cudaMemcpyAsync(h, pl->d_scratch, 16, cudaMemcpyDeviceToHost, pl->stream));
+  CUDA_TRY(cudaStreamSynchronize(pl->stream));
+  if (stage == pl->cfg.n_stages - 1 && pl->dna) {   // the sink's records are the pipeline's matches
+    const unsigned long long mc = std::min<unsigned long long>(h[0], pl->dp.match_cap);
+    CUDA_TRY(cudaMemcpy(pl->d_match_count, &mc, 8, cudaMemcpyHostToDevice));
+  }
+  *n_out = h[0];
+  if (max_vec_cycles) *max_vec_cycles = h[1];
+  if (h[0] > cap && stage + 1 < pl->cfg.n_stages) return fail(PL_EOVERFLOW, "output capacity %llu < %llu",
+                                                              (unsigned long long)cap, h[0]);
   return PL_OK;
 }
 

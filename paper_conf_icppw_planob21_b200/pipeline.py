@@ -162,6 +162,15 @@ class Pipeline:
         check(lib.pl_pipeline_firings(self.h, buf, n.value, C.byref(n)), "pl_pipeline_firings")
         return [(f.stream, f.node, f.start, f.n, f.first_root, f.last_root) for f in buf[:n.value]]
 
+    def stage_batch(self, stage, in_ptr, n, first_root, out_ptr, cap):
+        """pl_stage_batch: one stage over n device entries -> (outputs, longest vector cycles)."""
+        n_out = C.c_uint64()
+        cyc = C.c_uint64()
+        check(lib.pl_stage_batch(self.h, int(stage), C.c_void_p(in_ptr or 0), int(n), int(first_root),
+                                 C.c_void_p(out_ptr or 0), int(cap), C.byref(n_out), C.byref(cyc)),
+              "pl_stage_batch")
+        return n_out.value, cyc.value
+
     def params(self):
         w = (C.c_int64 * 8)()
         th = (C.c_uint32 * 8)()
