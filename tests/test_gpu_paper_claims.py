@@ -1,0 +1,53 @@
+"""The paper's empirical claims re-measured on the GPU executor (logical clock), on its own
+random-gain BLAST model (Table 1), 100 streams x 50,000 items per point
+(= 100 seeds x 50,000-input streams, L227-L230)."""
+import numpy as np
+import pytest
+
+from plgen import configs as C
+
+pytestmark = pytest.mark.gpu
+S, X = 100, 50_000
+
+
+def _run(cfg):
+    from paper_conf_icppw_planob21_b200 import Pipeline
+    pl = Pipeline(cfg, None, flags=1)
+    pl.push(None, cfg.n_roots)
+    pl.drain()
+    st = pl.stats()
+    lat, _ = pl.latency()
+    pl.close()
+    miss_free = int(((lat.reshape(cfg.n_streams, -1) > cfg.deadline).sum(axis=1) == 0).sum())
+    return st, miss_free
+
+
+@pytest.mark.parametrize("tau,D", [(10, 50_000), (20, 100_000), (50, 25_000), (100, 350_000), (5, 200_000)])
+def test_enforced_waits_miss_free_and_match_optimiser(tau, D):
+    """L230: with b = (1,3,9,6) >= 95 % of trials are miss-free; L227: simulated active
+    fraction closely matches the optimiser (Fig. 1)."""
+    from paper_conf_icppw_planob21_b200 import solve_enforced_waits
+    cfg = C.gain_model_blast(interarrival=tau, deadline=D, n_streams=S, n_roots=X, seed=11)
+    w, th, T, Tc = solve_enforced_waits(cfg)
+    st, mf = _run(cfg.replace(wait_time=tuple(w)))
+    assert mf >= 95
+    assert abs(st["active_fraction"] - T) < 0.01
+
+
+def test_fig4_complementary_strengths():
+    """L249: enforced waits win by >= 0.4 at fast arrivals with deadline slack; monolithic
+    wins by a similar margin at slow arrivals with little slack."""
+    from paper_conf_icppw_planob21_b200 import solve_enforced_waits, solve_monolithic
+
+    def both(tau, D):
+        cfg = C.gain_model_blast(interarrival=tau, deadline=D, n_streams=S, n_roots=X, seed=12)
+        w, th, T, Tc = solve_enforced_waits(cfg)
+        se, _ = _run(cfg.replace(wait_time=tuple(w)))
+        M, Tm = solve_monolithic(cfg)
+        sm, _ = _run(cfg.replace(policy=C.MONOLITHIC, block_size=M))
+        return se["active_fraction"], sm["active_fraction"]
+
+    e, m = both(10, 100_000)
+    assert m - e >= 0.4
+    e, m = both(100, 25_000)
+    assert e - m >= 0.4
