@@ -151,6 +151,7 @@ typedef struct {
   int64_t  busy_ns[PL_MAX_STAGES];         /* physical: measured firing time (ns)     */
   uint64_t spilled[PL_MAX_STAGES];         /* entries written to the HBM overflow ring */
   uint64_t overruns[PL_MAX_STAGES];        /* physical: firings longer than t_i        */
+  uint64_t stalls[PL_MAX_STAGES];          /* firings that waited for room in the next queue */
   int64_t  max_lateness_ns[PL_MAX_STAGES]; /* physical: max(actual - scheduled start)  */
   uint64_t sched_cycles[PL_MAX_STAGES];    /* clock64 cycles spent deciding firings    */
   int64_t  max_fire_ns[PL_MAX_STAGES];     /* physical: longest firing (start->publish) */

@@ -60,7 +60,7 @@ _I8 = C.c_int64 * PL_MAX_STAGES
 class pl_stats(C.Structure):
     _fields_ = [("n_stages", C.c_uint32), ("n_streams", C.c_uint32), ("roots", C.c_uint64),
                 ("firings", _A8), ("empty_firings", _A8), ("consumed", _A8), ("produced", _A8),
-                ("active_window", _I8), ("busy_ns", _I8), ("spilled", _A8), ("overruns", _A8),
+                ("active_window", _I8), ("busy_ns", _I8), ("spilled", _A8), ("overruns", _A8), ("stalls", _A8),
                 ("max_lateness_ns", _I8), ("sched_cycles", _A8), ("max_fire_ns", _I8),
                 ("phase_cycles", (C.c_uint64 * 6) * PL_MAX_STAGES), ("matches", C.c_uint64),
                 ("miss_events", C.c_uint64), ("misses", C.c_uint64), ("max_latency", C.c_int64),

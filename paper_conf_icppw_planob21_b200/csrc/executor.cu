@@ -525,10 +525,11 @@ __device__ Decision decide(const Node& nd, Leader& L) {
   }
 }
 
-// Reserve room for `worst` outputs on the output edge (worst case n*u, decided
-// before the stage runs so that no extra barrier is needed).  Returns the
-// location, or ~0u on overflow (physical mode only; logical mode back-pressures).
-__device__ uint32_t reserve_out(const Node& nd, Leader& L, uint32_t worst, uint32_t* errors) {
+// Reserve room for `worst` outputs on the output edge (worst case n*u, decided before the
+// stage runs so that no extra barrier is needed).  Returns the location.  A full queue
+// back-pressures the producer in both clock modes (deadlock-free):
+// in physical mode the wait shows up as lateness and, if it matters, as deadline misses.
+__device__ uint32_t reserve_out(const Node& nd, Leader& L, uint32_t worst, uint64_t* stalls) {
   int spins = 0;
   for (;;) {
     const uint32_t h = vld(&nd.Eout->head), sh = vld(&nd.Eout->seg_head);
@@ -536,11 +537,8 @@ __device__ uint32_t reserve_out(const Node& nd, Leader& L, uint32_t worst, uint3
     const uint32_t need = L.out_tail + worst - h;
     if (seg_ok && need <= nd.out_cap) return LOC_SMEM;
     if (seg_ok && need <= nd.capg) return LOC_SPILL;
-    if (nd.phys) {
-      atomicOr(errors, seg_ok ? PL_ERR_QUEUE_OVERFLOW : PL_ERR_SEG_OVERFLOW);
-      return ~0u;
-    }
-    backoff(spins);   // logical mode: back-pressure (deadlock-free)
+    if (spins == 0) ++*stalls;
+    backoff(spins);
   }
 }
 
@@ -697,7 +695,7 @@ __device__ void run_node(Ctx& c, const Dna dna, int i, int gtid) {
   L.W_pub = -1; L.empties = 0;
   Rep R;
   R.m = 0; R.B = 0; R.c0 = 0; R.empties = 0;
-  uint64_t firings = 0, consumed = 0, produced = 0, spilled = 0, overruns = 0;
+  uint64_t firings = 0, consumed = 0, produced = 0, spilled = 0, overruns = 0, stalls = 0;
   int64_t active = 0, busy_ns = 0, lateness = 0, t_end = 0, max_fire = 0;
   uint64_t start_ns = 0;
   uint32_t pend_root = NO_ROOT;          // lane: physical terminal event awaiting its end time
@@ -716,7 +714,7 @@ __device__ void run_node(Ctx& c, const Dna dna, int i, int gtid) {
       T = d.T; n = d.n; head = (uint32_t)R.c0;
       if (leader) {
         if (rec & PL_REC_FIRINGS) G.log_idx[par] = atomicAdd(&c.sh->log_count, 1u);
-        G.out_loc[par] = nd.sink ? LOC_SMEM : reserve_out(nd, L, n * nd.umax, &c.sh->errors);
+        G.out_loc[par] = nd.sink ? LOC_SMEM : reserve_out(nd, L, n * nd.umax, &stalls);
         G.out_base[par] = L.out_tail;
         tc = clock64();
         ph[0] += (uint64_t)(tc - c0);
@@ -741,7 +739,7 @@ __device__ void run_node(Ctx& c, const Dna dna, int i, int gtid) {
         G.in_spill_end[par] = vld(&nd.Ein->spill_end);
         if (!d.done) {
           if (rec & PL_REC_FIRINGS) G.log_idx[par] = atomicAdd(&c.sh->log_count, 1u);
-          G.out_loc[par] = nd.sink ? LOC_SMEM : reserve_out(nd, L, d.n * nd.umax, &c.sh->errors);
+          G.out_loc[par] = nd.sink ? LOC_SMEM : reserve_out(nd, L, d.n * nd.umax, &stalls);
           G.out_base[par] = L.out_tail;
         } else {
           publish_W(nd, L, PL_INF64);
@@ -939,6 +937,7 @@ __device__ void run_node(Ctx& c, const Dna dna, int i, int gtid) {
     S.busy_ns[i] = busy_ns;
     S.spilled[i] = spilled;
     S.overruns[i] = overruns;
+    S.stalls[i] = stalls;
     S.lateness[i] = lateness;
     S.sched_cycles[i] = ph[0];
     S.max_fire_ns[i] = max_fire;
@@ -1222,6 +1221,7 @@ __device__ void run_monolithic(Ctx& c) {
     for (int i = 0; i < PL_MAX_STAGES; ++i) {
       S.firings[i] = firings[i]; S.empty[i] = 0; S.consumed[i] = consumed[i]; S.produced[i] = produced[i];
       S.active_ne[i] = active[i]; S.busy_ns[i] = i == 0 ? busy_ns : 0; S.spilled[i] = 0; S.overruns[i] = 0;
+      S.stalls[i] = 0;
       S.lateness[i] = 0; S.sched_cycles[i] = 0; S.max_fire_ns[i] = 0;
       for (int k = 0; k < 6; ++k) S.phase_cycles[i][k] = 0;
     }

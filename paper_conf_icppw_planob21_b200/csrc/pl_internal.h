@@ -40,6 +40,7 @@ struct CtaStats {
   int64_t  busy_ns[PL_MAX_STAGES];
   uint64_t spilled[PL_MAX_STAGES];
   uint64_t overruns[PL_MAX_STAGES];
+  uint64_t stalls[PL_MAX_STAGES];
   int64_t  lateness[PL_MAX_STAGES];
   uint64_t sched_cycles[PL_MAX_STAGES];
   int64_t  max_fire_ns[PL_MAX_STAGES];

@@ -566,6 +566,7 @@ pl_status pl_pipeline_stats(pl_pipeline* pl, pl_stats* out) {
       out->busy_ns[i] += s.busy_ns[i];
       out->spilled[i] += s.spilled[i];
       out->overruns[i] += s.overruns[i];
+      out->stalls[i] += s.stalls[i];
       out->max_lateness_ns[i] = std::max(out->max_lateness_ns[i], s.lateness[i]);
       out->sched_cycles[i] += s.sched_cycles[i];
       out->max_fire_ns[i] = std::max(out->max_fire_ns[i], s.max_fire_ns[i]);
