@@ -1242,8 +1242,12 @@ __global__ void __launch_bounds__(MAXT, 1) pl_exec_enforced(const __grid_constan
   __syncthreads();
   if (threadIdx.x == 0) sh.T0 = gtimer() + (p.clock == PL_CLOCK_GLOBALTIMER ? PL_T0_OFFSET_NS : 0);
   __syncthreads();
-  const int gi = threadIdx.x / p.v;
-  if (gi < p.N) run_node(c, c.dna, gi, threadIdx.x % p.v);
+  // warp w serves node w % N (local warp w / N): with N = 4 every warp of node i sits on
+  // SM sub-partition i, so each SMSP's instruction cache holds one node's code path
+  const int w = threadIdx.x >> 5;
+  const int gi = w % p.N;
+  const int gt = (w / p.N) * 32 + (threadIdx.x & 31);
+  if (w < p.N * (p.v >> 5)) run_node(c, c.dna, gi, gt);
   __syncthreads();
   cta_finish(c, sh, p);
 }
