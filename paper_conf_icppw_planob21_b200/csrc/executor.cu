@@ -866,7 +866,9 @@ __device__ void run_node(Ctx& c, const Dna dna, int i, int gtid) {
         else __stcg(nd.out_spill + (s & (nd.capg - 1)), val);
       }
     }
-    if (gtid < 32) bar_sync(bidB, v);                                  // B4: outputs written
+    // B4: outputs written.  Non-leader warps only arrive; node 7 (no spare barrier id) syncs
+    // fully, since arrivals for B4 and the next B1 must not meet on one barrier instance.
+    if (gtid < 32 || bidB == bidA) bar_sync(bidB, v);
     else bar_arrive(bidB, v);
     if (leader) {
       { const long long t2 = clock64(); ph[4] += (uint64_t)(t2 - tc); tc = t2; }

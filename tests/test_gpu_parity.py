@@ -91,3 +91,38 @@ def test_ragged_streams_dna():
     cfg = _dna(C.FIXED_WAIT, db_len=40_003, streams=6)
     wl = workload_for(cfg)
     compare(cfg, run_gpu(cfg, wl), run_oracle(cfg, wl))
+
+
+@pytest.mark.parametrize("policy", [C.FIXED_WAIT, C.THRESHOLD_SLACK, C.MONOLITHIC])
+@pytest.mark.parametrize("v", [32, 64, 256])
+def test_vector_widths_dna(policy, v):
+    """v = 32..256 lanes per node (one warp group each; v = 256 -> 1024 threads, N = 4)."""
+    cfg = _dna(policy, db_len=1 << 15, streams=3).replace(vector_width=v)
+    if policy == C.THRESHOLD_SLACK:
+        cfg = cfg.replace(wait_threshold=tuple(min(t, v) for t in cfg.wait_threshold))
+    wl = workload_for(cfg)
+    compare(cfg, run_gpu(cfg, wl), run_oracle(cfg, wl))
+
+
+@pytest.mark.parametrize("policy", [C.FIXED_WAIT, C.THRESHOLD_SLACK])
+def test_eight_node_gain_pipeline(policy):
+    """N = 8 random-gain nodes (the ABI maximum), v = 128 -> 1024 threads."""
+    st = [C.Stage(C.BERNOULLI, 0.8, 1), C.Stage(C.POISSON_CAPPED, 1.3, 4), C.Stage(C.BERNOULLI, 0.6, 1),
+          C.Stage(C.FIXED_GAIN, 2.0, 2), C.Stage(C.BERNOULLI, 0.5, 1), C.Stage(C.KEEP_EVERY, 3.0, 1),
+          C.Stage(C.POISSON_CAPPED, 0.9, 3), C.Stage(C.BERNOULLI, 0.7, 1)]
+    cfg = C.Config(name="n8", stages=st, service_time=(40, 55, 30, 45, 25, 35, 50, 20), vector_width=128,
+                   deadline=20_000, interarrival=3, b=(1,) * 8, wait_time=(300, 100, 50, 80, 40, 60, 90, 30),
+                   wait_threshold=(64, 32, 16, 16, 8, 8, 4, 4), policy=policy, n_streams=3, n_roots=3000, seed=5)
+    compare(cfg, run_gpu(cfg, None), run_oracle(cfg, None))
+
+
+@pytest.mark.parametrize("policy", [C.THRESHOLD_SLACK, C.MONOLITHIC])
+def test_physical_other_policies_replay(policy):
+    """THRESHOLD_SLACK and MONOLITHIC under the %globaltimer clock commit the logical schedule."""
+    cfg = _dna(policy, db_len=1 << 15, streams=3).replace(
+        clock=C.CLOCK_GLOBALTIMER, ns_per_unit=1.0, service_time=(20_000,) * 4, interarrival=400,
+        deadline=10**7, wait_threshold=(64, 32, 16, 8), block_size=1024)
+    wl = workload_for(cfg)
+    g = run_gpu(cfg, wl)
+    compare(cfg, g, run_oracle(cfg, wl))
+    assert (g["lat_ns"] > 0).all()

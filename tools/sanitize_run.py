@@ -1,0 +1,27 @@
+"""Small executor runs for compute-sanitizer (memcheck / racecheck / synccheck)."""
+import sys
+
+sys.path.insert(0, ".")
+from plgen import configs as C
+from plgen import dna as G
+from paper_conf_icppw_planob21_b200 import Pipeline
+
+# random-gain pipeline, all policies, forced spills
+for policy in (C.FIXED_WAIT, C.THRESHOLD_SLACK, C.MONOLITHIC):
+    cfg = C.c1(n_streams=2, n_roots=600, wait_time=(64, 90), wait_threshold=(32, 23), policy=policy, block_size=64)
+    pl = Pipeline(cfg, None, flags=7, queue_capacity=32 if policy != C.MONOLITHIC else 0)
+    pl.push(None, cfg.n_roots)
+    pl.drain()
+    print(policy, pl.stats()["firings"][:2], flush=True)
+    pl.close()
+# DNA pipeline, logical and physical, forced spill
+cfg = C.c2(n_streams=3, dna=dict(db_len=1 << 14, q_len=1024, n_planted=4), wait_time=(993, 2422, 965, 1628))
+wl = G.make_dna(cfg.seed, **cfg.dna)
+for clock in (0, 1):
+    c = cfg if clock == 0 else cfg.replace(clock=1, service_time=(4000,) * 4, interarrival=100, wait_time=(0,) * 4,
+                                           deadline=10**7)
+    pl = Pipeline(c, wl, flags=7, queue_capacity=64)
+    pl.push(wl.db, wl.db_len)
+    pl.drain()
+    print("dna clock", clock, pl.stats()["firings"], flush=True)
+    pl.close()
