@@ -199,6 +199,21 @@ pl_status pl_pipeline_push(pl_pipeline* pl, const void* items, uint64_t n);
  * The buffer must stay alive until the last launch using it has completed.      */
 pl_status pl_pipeline_bind_device(pl_pipeline* pl, const void* dev_items, uint64_t n);
 
+/* Use a caller-owned PINNED HOST buffer (cudaHostAlloc'd, or cudaHostRegister'ed with
+ * cudaHostRegisterMapped) of n packed bases as the whole DB, with no device copy: every CTA
+ * stages its DB window straight from host memory with TMA bulk copies (cp.async.bulk over
+ * PCIe/C2C) when the executor starts; reads outside the window go to host memory.
+ * PL_EINVAL if the buffer is not mapped.  It must stay valid until the run completes.    */
+pl_status pl_pipeline_bind_host(pl_pipeline* pl, const void* host_items, uint64_t n);
+
+/* Compact result of the last run, reduced on the device (one 48-byte D->H copy).        */
+typedef struct {
+  uint64_t roots, matches, miss_events;
+  int64_t  max_latency, max_latency_ns;
+  uint32_t errors, launches;
+} pl_summary;
+pl_status pl_pipeline_summary(pl_pipeline* pl, pl_summary* out);
+
 /* Enqueue one executor run over every item pushed so far on the bound stream and
  * return immediately (asynchronous).  Resets per-run outputs first.             */
 pl_status pl_pipeline_launch(pl_pipeline* pl);

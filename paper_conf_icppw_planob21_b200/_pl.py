@@ -53,6 +53,12 @@ class pl_firing(C.Structure):
                 ("pad", C.c_uint32)]
 
 
+class pl_summary(C.Structure):
+    _fields_ = [("roots", C.c_uint64), ("matches", C.c_uint64), ("miss_events", C.c_uint64),
+                ("max_latency", C.c_int64), ("max_latency_ns", C.c_int64), ("errors", C.c_uint32),
+                ("launches", C.c_uint32)]
+
+
 _A8 = C.c_uint64 * PL_MAX_STAGES
 _I8 = C.c_int64 * PL_MAX_STAGES
 
@@ -92,6 +98,8 @@ def _load():
         "pl_pipeline_set_stream": (C.c_int32, [P, P]),
         "pl_pipeline_push": (C.c_int32, [P, P, C.c_uint64]),
         "pl_pipeline_bind_device": (C.c_int32, [P, P, C.c_uint64]),
+        "pl_pipeline_bind_host": (C.c_int32, [P, P, C.c_uint64]),
+        "pl_pipeline_summary": (C.c_int32, [P, C.POINTER(pl_summary)]),
         "pl_pipeline_launch": (C.c_int32, [P]),
         "pl_pipeline_drain": (C.c_int32, [P]),
         "pl_pipeline_rewind": (C.c_int32, [P]),
@@ -121,7 +129,8 @@ EXPORTED = ("pl_pipeline_create", "pl_pipeline_set_stream", "pl_pipeline_push", 
             "pl_pipeline_launch", "pl_pipeline_drain", "pl_pipeline_rewind", "pl_pipeline_stats",
             "pl_pipeline_results", "pl_pipeline_latency", "pl_pipeline_trace", "pl_pipeline_firings",
             "pl_pipeline_params", "pl_pipeline_destroy", "pl_last_error", "pl_solve_enforced_waits",
-            "pl_solve_monolithic", "pl_version", "pl_stage_batch")
+            "pl_solve_monolithic", "pl_version", "pl_stage_batch", "pl_pipeline_bind_host",
+            "pl_pipeline_summary")
 
 
 class PlError(RuntimeError):

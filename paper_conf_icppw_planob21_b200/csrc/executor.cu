@@ -1068,6 +1068,13 @@ __device__ void cta_finish(Ctx& c, Shared& sh, const DevParams& p) {
     S.n_roots = (uint64_t)c.X;
     S.n_log = sh.log_count < p.log_cap ? sh.log_count : p.log_cap;
     S.errors = sh.errors;
+    if (p.summary) {                     // device-side reduction for pl_pipeline_summary
+      atomicAdd(p.summary + 0, (unsigned long long)c.X);
+      atomicAdd(p.summary + 1, (unsigned long long)sh.miss_events);
+      atomicMax(p.summary + 2, (unsigned long long)sh.max_lat);
+      atomicMax(p.summary + 3, (unsigned long long)sh.max_lat_ns);
+      atomicOr(p.summary + 4, (unsigned long long)sh.errors);
+    }
   }
 }
 

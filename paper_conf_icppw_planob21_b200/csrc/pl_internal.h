@@ -98,6 +98,7 @@ struct DevParams {
   pl_firing* flog;                      // [n_streams][log_cap]
   uint32_t log_cap;
   CtaStats* stats;                      // [n_streams]
+  unsigned long long* summary;          // [6]: roots, miss_events, max_lat, max_lat_ns, errors, -
   DevStage st[PL_MAX_STAGES];
 };
 

@@ -123,13 +123,16 @@ struct pl_pipeline {
   int device = 0;
   uint64_t h2d = 0, d2h = 0;  // bytes moved across the host boundary (cumulative)
   unsigned long long* d_scratch = nullptr;   // stage-batch counters
+  unsigned long long* d_summary = nullptr;   // device-reduced run summary
+  bool bound_host = false;
 };
 
 namespace {
 
 void free_all(pl_pipeline* pl) {
   void* ptrs[] = {pl->d_db, pl->d_qoff, pl->d_qpos, pl->d_qw, pl->d_spill, pl->d_mono, pl->d_lat, pl->d_lat_ns,
-                  pl->d_trace, pl->d_matches, pl->d_match_count, pl->d_flog, pl->d_stats, pl->d_scratch};
+                  pl->d_trace, pl->d_matches, pl->d_match_count, pl->d_flog, pl->d_stats, pl->d_scratch,
+                  pl->d_summary};
   for (void* p : ptrs)
     if (p) cudaFree(p);
 }
@@ -442,6 +445,8 @@ pl_status pl_pipeline_create(const pl_config* cfg, const pl_workload* wl, pl_pip
     return bail(fail(PL_ENOMEM, "output buffers"));
   cudaMemset(pl->d_match_count, 0, 8);
   cudaMemset(pl->d_stats, 0, S * sizeof(CtaStats));
+  if (cudaMalloc(&pl->d_summary, 8 * 8) != cudaSuccess) return bail(fail(PL_ENOMEM, "summary"));
+  cudaMemset(pl->d_summary, 0, 64);
   d.lat = pl->d_lat;
   d.lat_ns = cfg->clock == PL_CLOCK_GLOBALTIMER ? pl->d_lat_ns : nullptr;
   if (!(cfg->flags & PL_REC_LATENCY)) d.lat_ns = nullptr;
@@ -450,6 +455,7 @@ pl_status pl_pipeline_create(const pl_config* cfg, const pl_workload* wl, pl_pip
   d.match_count = pl->d_match_count;
   d.flog = pl->d_flog;
   d.stats = pl->d_stats;
+  d.summary = pl->d_summary;
   cudaError_t e1 = pl_kernel_attributes(200 * 1024);
   if (e1 != cudaSuccess) return bail(fail(PL_EDEVICE, "cudaFuncSetAttribute: %s", cudaGetErrorString(e1)));
   cudaError_t e = cudaDeviceSynchronize();
@@ -490,7 +496,45 @@ pl_status pl_pipeline_bind_device(pl_pipeline* pl, const void* dev_items, uint64
   if (!pl->dna) return fail(PL_EINVAL, "bind_device is for DNA pipelines");
   if (n > pl->db_len) return fail(PL_EINVAL, "bound DB longer than db_len");
   pl->d_db_bound = (const uint32_t*)dev_items;
+  pl->bound_host = false;
   pl->pushed = n;
+  return PL_OK;
+}
+
+pl_status pl_pipeline_bind_host(pl_pipeline* pl, const void* host_items, uint64_t n) {
+  if (!pl || !host_items) return fail(PL_EINVAL, "NULL argument");
+  if (!pl->dna) return fail(PL_EINVAL, "bind_host is for DNA pipelines");
+  if (n > pl->db_len) return fail(PL_EINVAL, "bound DB longer than db_len");
+  cudaSetDevice(pl->device);
+  void* dptr = nullptr;
+  cudaError_t e = cudaHostGetDevicePointer(&dptr, const_cast<void*>(host_items), 0);
+  if (e != cudaSuccess || !dptr) {
+    cudaGetLastError();
+    return fail(PL_EINVAL, "host buffer is not pinned+mapped (cudaHostAlloc / cudaHostRegisterMapped)");
+  }
+  pl->d_db_bound = (const uint32_t*)dptr;
+  pl->bound_host = true;
+  pl->pushed = n;
+  return PL_OK;
+}
+
+pl_status pl_pipeline_summary(pl_pipeline* pl, pl_summary* out) {
+  if (!pl || !out) return fail(PL_EINVAL, "NULL argument");
+  cudaSetDevice(pl->device);
+  unsigned long long h[6];
+  CUDA_TRY(cudaMemcpyAsync(h, pl->d_summary, 48, cudaMemcpyDeviceToHost, pl->stream));
+  unsigned long long mc = 0;
+  CUDA_TRY(cudaMemcpyAsync(&mc, pl->d_match_count, 8, cudaMemcpyDeviceToHost, pl->stream));
+  CUDA_TRY(cudaStreamSynchronize(pl->stream));
+  pl->in_flight = false;
+  pl->d2h += 56;
+  out->roots = h[0];
+  out->miss_events = h[1];
+  out->max_latency = (int64_t)h[2];
+  out->max_latency_ns = (int64_t)h[3];
+  out->errors = (uint32_t)h[4];
+  out->matches = std::min<uint64_t>(mc, pl->dp.match_cap);
+  out->launches = pl->launches;
   return PL_OK;
 }
 
@@ -510,6 +554,7 @@ pl_status pl_pipeline_launch(pl_pipeline* pl) {
   }
   if (d.total_roots > pl->roots_cap) return fail(PL_EINVAL, "more roots than allocated");
   CUDA_TRY(cudaMemsetAsync(pl->d_match_count, 0, 8, pl->stream));
+  CUDA_TRY(cudaMemsetAsync(pl->d_summary, 0, 64, pl->stream));
   CUDA_TRY(pl_launch(d, pl->cfg.n_streams, pl->block, pl->smem, pl->stream));
   pl->in_flight = true;
   pl->launches++;

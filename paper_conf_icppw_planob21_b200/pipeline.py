@@ -106,6 +106,15 @@ class Pipeline:
     def bind_device(self, dev_ptr, n):
         check(lib.pl_pipeline_bind_device(self.h, C.c_void_p(dev_ptr), int(n)), "pl_pipeline_bind_device")
 
+    def bind_host(self, host_ptr, n):
+        """pl_pipeline_bind_host: the DB stays in pinned host memory; CTAs stage it by TMA."""
+        check(lib.pl_pipeline_bind_host(self.h, C.c_void_p(host_ptr), int(n)), "pl_pipeline_bind_host")
+
+    def summary(self) -> dict:
+        s = _pl.pl_summary()
+        check(lib.pl_pipeline_summary(self.h, C.byref(s)), "pl_pipeline_summary")
+        return {k: getattr(s, k) for k, _ in s._fields_}
+
     def launch(self):
         check(lib.pl_pipeline_launch(self.h), "pl_pipeline_launch")
 

@@ -126,3 +126,24 @@ def test_physical_other_policies_replay(policy):
     g = run_gpu(cfg, wl)
     compare(cfg, g, run_oracle(cfg, wl))
     assert (g["lat_ns"] > 0).all()
+
+
+def test_bind_host_tma_matches_push():
+    """pl_pipeline_bind_host: CTAs stage the DB straight from pinned host memory by TMA;
+    results are identical to the pushed (H2D-copied) DB and to the oracle."""
+    import torch
+    from paper_conf_icppw_planob21_b200 import Pipeline
+    cfg = _dna(C.FIXED_WAIT, db_len=1 << 16, streams=5)
+    wl = workload_for(cfg)
+    host = torch.from_numpy(wl.db.view("int32")).pin_memory()
+    pl = Pipeline(cfg, wl, flags=7)
+    pl.bind_host(host.data_ptr(), wl.db_len)
+    pl.drain()
+    g = dict(stats=pl.stats(), matches=pl.results(), firings=pl.firings(), trace=pl.trace())
+    g["lat"], g["lat_ns"] = pl.latency()
+    summ = pl.summary()
+    pl.close()
+    o = run_oracle(cfg, wl)
+    compare(cfg, g, o)
+    assert summ["roots"] == g["stats"]["roots"] and summ["matches"] == len(o.matches)
+    assert summ["max_latency"] == max(o.lat) and summ["miss_events"] == g["stats"]["miss_events"]
