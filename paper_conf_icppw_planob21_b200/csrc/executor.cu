@@ -87,15 +87,14 @@ struct Dna {
     const int64_t w = s >> 4;
     return __funnelshift_r(qww(w), qww(w + 1), (uint32_t)(s & 15) * 2u);
   }
-  // key(db, p) = sum_{j<k} db[p+j] 4^(k-1-j)  (first base most significant; R-S0)
-  __device__ __forceinline__ uint32_t key(uint32_t p) const {
-    const uint32_t x = db16(p);
-    uint32_t key = 0;
-#pragma unroll
-    for (int j = 0; j < PL_MAX_K; ++j)
-      if (j < k) key = (key << 2) | ((x >> (2 * j)) & 3u);
-    return key;
+  // key(db, p) = sum_{j<k} db[p+j] 4^(k-1-j)  (first base most significant; R-S0):
+  // reverse the order of the 2-bit fields of the window (bit-reverse, then swap each pair)
+  __device__ __forceinline__ uint32_t kmer_of(uint32_t x) const {
+    const uint32_t r = __brev(x);
+    const uint32_t pr = ((r >> 1) & 0x55555555u) | ((r & 0x55555555u) << 1);
+    return pr >> (32 - 2 * k);
   }
+  __device__ __forceinline__ uint32_t key(uint32_t p) const { return kmer_of(db16(p)); }
   // Walk d = 1..limit away from the seed scoring +1/-3 (R-S2/R-S3); stop early on
   // X-drop (X > 0: score <= best - X).  Returns best (>= 0) and the smallest d
   // attaining it.  dir = +1: db[p+k-1+d] vs query[q+k-1+d]; dir = -1: db[p-d] vs query[q-d].
@@ -158,7 +157,7 @@ struct GroupCtl {           // broadcast from a node's leader to its lanes, doub
   uint32_t n[2], head[2], done[2], segh[2], st[2], log_idx[2];
   uint32_t in_spill_end[2]; // input edge: end seq of its last spilled segment
   uint32_t out_base[2], out_loc[2];
-  uint32_t wtot[2][8];
+  alignas(16) uint32_t wtot[2][8];
 };
 struct Shared {
   EdgeCtl e[PL_MAX_STAGES];
@@ -219,6 +218,7 @@ struct Node {
   uint32_t kind, max_out, cfix, umax;
   int32_t ip1, ip2;
   MDiv dtau, dP;
+  int64_t Pq, Pr;               // floor(P / tau0), P mod tau0
   __device__ __forceinline__ int64_t arrival(uint32_t root) const { return (int64_t)(root - lo) * tau; }
 };
 
@@ -257,6 +257,8 @@ __device__ __forceinline__ Node make_node(const Ctx& c, int i) {
   n.ip1 = s.ip[1]; n.ip2 = s.ip[2];
   n.dtau.m = p.tau_m; n.dtau.d = p.tau;
   n.dP.m = p.P_m[i]; n.dP.d = p.P[i];
+  n.Pq = fdiv(p.P[i], n.dtau);
+  n.Pr = p.P[i] - n.Pq * p.tau;
   return n;
 }
 
@@ -427,6 +429,8 @@ struct Rep {
   int64_t B;        // THRESHOLD_SLACK: busy until
   int64_t c0;       // roots consumed
   uint64_t empties;
+  int64_t qT, rT;   // FIXED_WAIT: floor(m P / tau0) and remainder, advanced without division
+  bool qvalid;
 };
 __device__ __forceinline__ Decision decide0(const Node& nd, Rep& r) {
   Decision d;
@@ -434,7 +438,7 @@ __device__ __forceinline__ Decision decide0(const Node& nd, Rep& r) {
   d.T = 0;
   d.n = 0;
   if (d.done) return d;
-  int64_t T;
+  int64_t T, q;
   if (nd.fixed) {
     T = r.m * nd.P;
     if (T < r.c0 * nd.tau) {             // empty firings until the next root has arrived
@@ -442,7 +446,14 @@ __device__ __forceinline__ Decision decide0(const Node& nd, Rep& r) {
       r.empties += (uint64_t)(m2 - r.m);
       r.m = m2;
       T = r.m * nd.P;
+      r.qvalid = false;
     }
+    if (!r.qvalid) {                     // floor(T / tau0), then advanced by P per firing
+      r.qT = fdiv(T, nd.dtau);
+      r.rT = T - r.qT * nd.tau;
+      r.qvalid = true;
+    }
+    q = r.qT;
   } else {
     const int64_t ah = r.c0 * nd.tau;
     const int64_t Tth = (r.c0 + nd.theta - 1 < nd.X) ? ah + (int64_t)(nd.theta - 1) * nd.tau : PL_INF64;
@@ -450,13 +461,24 @@ __device__ __forceinline__ Decision decide0(const Node& nd, Rep& r) {
     if (Tf < ah) Tf = ah;
     T = Tth < Tf ? Tth : Tf;
     if (T < r.B) T = r.B;
+    q = fdiv(T, nd.dtau);
   }
-  int64_t arrived = fdiv(T, nd.dtau) + 1;
+  int64_t arrived = q + 1;
   if (arrived > nd.X) arrived = nd.X;
   const int64_t avail = arrived - r.c0;
   d.T = T;
   d.n = (uint32_t)(avail < (int64_t)nd.v ? avail : nd.v);
   return d;
+}
+
+// FIXED_WAIT node 0 after a firing: T += P, so floor(T/tau0) += floor(P/tau0) (+1 on carry)
+__device__ __forceinline__ void advance0(const Node& nd, Rep& r) {
+  ++r.m;
+  if (r.qvalid) {
+    r.qT += nd.Pq;
+    r.rT += nd.Pr;
+    if (r.rT >= nd.tau) { r.rT -= nd.tau; ++r.qT; }
+  }
 }
 
 // Nodes i >= 1: the leader decides from the published queue state and watermark.
@@ -572,11 +594,20 @@ __device__ __forceinline__ uint32_t group_scan(uint32_t* wtot, uint32_t x, uint3
   }
   if (lane == 31) wtot[w] = inc;
   bar_sync(bid, v);                                                    // B2
+  // warp totals: one or two 16-byte shared loads (wtot is 16-byte aligned, 8 slots)
+  const uint4 a = *reinterpret_cast<const uint4*>(wtot);
+  uint32_t t[8] = {a.x, a.y, a.z, a.w, 0u, 0u, 0u, 0u};
+  if (v > 128) {
+    const uint4 b = *reinterpret_cast<const uint4*>(wtot + 4);
+    t[4] = b.x; t[5] = b.y; t[6] = b.z; t[7] = b.w;
+  }
+  const int nw = v >> 5;
   uint32_t pre = 0, tot = 0;
-  for (int k = 0; k < (v >> 5); ++k) {
-    const uint32_t t = wtot[k];
-    pre += (k < w) ? t : 0u;
-    tot += t;
+#pragma unroll
+  for (int k = 0; k < 8; ++k) {
+    const uint32_t tk = k < nw ? t[k] : 0u;
+    pre += (k < w) ? tk : 0u;
+    tot += tk;
   }
   *total = tot;
   return pre + inc - x;
@@ -613,11 +644,7 @@ __device__ __forceinline__ void stage_batch(const Node& nd, const Dna& dna, cons
 #pragma unroll
       for (int j = 0; j < K; ++j) {
         const uint32_t x = __funnelshift_r(dna.win[r[j]], dna.win[r[j] + 1], (e[j].x & 15u) * 2u);
-        uint32_t kk = 0;
-#pragma unroll
-        for (int b = 0; b < PL_MAX_K; ++b)
-          if (b < dna.k) kk = (kk << 2) | ((x >> (2 * b)) & 3u);
-        key[j] = kk;
+        key[j] = dna.kmer_of(x);
       }
     } else {
 #pragma unroll
@@ -694,7 +721,7 @@ __device__ void run_node(Ctx& c, const Dna dna, int i, int gtid) {
   L.m = 0; L.B = 0; L.c0 = 0; L.head = 0; L.segh = 0; L.out_tail = 0; L.out_segt = 0;
   L.W_pub = -1; L.empties = 0;
   Rep R;
-  R.m = 0; R.B = 0; R.c0 = 0; R.empties = 0;
+  R.m = 0; R.B = 0; R.c0 = 0; R.empties = 0; R.qT = 0; R.rT = 0; R.qvalid = false;
   uint64_t firings = 0, consumed = 0, produced = 0, spilled = 0, overruns = 0, stalls = 0;
   int64_t active = 0, busy_ns = 0, lateness = 0, t_end = 0, max_fire = 0;
   uint64_t start_ns = 0;
@@ -915,7 +942,7 @@ __device__ void run_node(Ctx& c, const Dna dna, int i, int gtid) {
     }
     if (n0) {                            // replicated node-0 state, identical in every lane
       R.c0 += n;
-      if (nd.fixed) ++R.m; else R.B = T + nd.t;
+      if (nd.fixed) advance0(nd, R); else R.B = T + nd.t;
     }
     par ^= 1;
   }
