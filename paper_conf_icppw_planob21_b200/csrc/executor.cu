@@ -1269,8 +1269,8 @@ __device__ void run_monolithic(Ctx& c) {
 
 // FIXED_WAIT / THRESHOLD_SLACK executor: grid = n_streams, block = N*32 threads (one warp
 // per node); up to 4 CTAs (streams) per SM when N <= 4.
-template <int MAXT>
-__global__ void __launch_bounds__(MAXT, 1) pl_exec_enforced(const __grid_constant__ DevParams p) {
+template <int MAXT, int MINB>
+__global__ void __launch_bounds__(MAXT, MINB) pl_exec_enforced(const __grid_constant__ DevParams p) {
   extern __shared__ __align__(16) unsigned char dsm[];
   __shared__ Shared sh;
   Ctx c;
@@ -1315,16 +1315,20 @@ cudaError_t pl_launch(const DevParams& p, unsigned grid, unsigned block, unsigne
     if (block <= 512) pl_exec_monolithic<512><<<grid, block, smem, st>>>(p);
     else pl_exec_monolithic<1024><<<grid, block, smem, st>>>(p);
   } else {
-    if (block <= 512) pl_exec_enforced<512><<<grid, block, smem, st>>>(p);
-    else pl_exec_enforced<1024><<<grid, block, smem, st>>>(p);
+    // two CTAs (streams) per SM when the grid asks for more streams than there are SMs and
+    // the CTA fits twice (<= 512 threads, 64 registers, smem)
+    if (block <= 512 && p.ctas_per_sm >= 2) pl_exec_enforced<512, 2><<<grid, block, smem, st>>>(p);
+    else if (block <= 512) pl_exec_enforced<512, 1><<<grid, block, smem, st>>>(p);
+    else pl_exec_enforced<1024, 1><<<grid, block, smem, st>>>(p);
   }
   return cudaGetLastError();
 }
 
 cudaError_t pl_kernel_attributes(unsigned max_smem) {
   cudaError_t e;
-  if ((e = cudaFuncSetAttribute(pl_exec_enforced<512>, cudaFuncAttributeMaxDynamicSharedMemorySize, max_smem))) return e;
-  if ((e = cudaFuncSetAttribute(pl_exec_enforced<1024>, cudaFuncAttributeMaxDynamicSharedMemorySize, max_smem))) return e;
+  if ((e = cudaFuncSetAttribute(pl_exec_enforced<512, 2>, cudaFuncAttributeMaxDynamicSharedMemorySize, max_smem))) return e;
+  if ((e = cudaFuncSetAttribute(pl_exec_enforced<512, 1>, cudaFuncAttributeMaxDynamicSharedMemorySize, max_smem))) return e;
+  if ((e = cudaFuncSetAttribute(pl_exec_enforced<1024, 1>, cudaFuncAttributeMaxDynamicSharedMemorySize, max_smem))) return e;
   if ((e = cudaFuncSetAttribute(pl_exec_monolithic<512>, cudaFuncAttributeMaxDynamicSharedMemorySize, max_smem))) return e;
   return cudaFuncSetAttribute(pl_exec_monolithic<1024>, cudaFuncAttributeMaxDynamicSharedMemorySize, max_smem);
 }

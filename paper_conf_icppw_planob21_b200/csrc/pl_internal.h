@@ -69,6 +69,7 @@ struct DevParams {
   uint64_t total_roots;                 // roots over all streams
   int32_t  n_streams;
   uint32_t flags;
+  int32_t  ctas_per_sm;                 // launch variant: 2 -> 64-register kernel, two streams per SM
   // DNA workload
   const uint32_t* db;                   // packed DB (device)
   uint64_t db_len;

@@ -11,6 +11,7 @@
 #include <cmath>
 #include <cstdarg>
 #include <cstdio>
+#include <cstdlib>
 #include <cstring>
 #include <new>
 #include <string>
@@ -425,6 +426,12 @@ pl_status pl_pipeline_create(const pl_config* cfg, const pl_workload* wl, pl_pip
   d.spill = pl->d_spill;
   d.mono_buf = pl->d_mono;
   pl->smem = pl_layout_enforced_host(d);
+  // one CTA (stream) per SM: the two-per-SM variant (64 registers) spills and measured no gain
+  // (tools/streams_scaling.py); it stays selectable through PL_CTAS_PER_SM=2
+  d.ctas_per_sm = 1;
+  if (const char* e = getenv("PL_CTAS_PER_SM"))
+    if (atoi(e) == 2 && pl->block <= 512 && 2 * (pl->smem + 4096) <= (uint32_t)prop.sharedMemPerMultiprocessor)
+      d.ctas_per_sm = 2;
   if (pl->smem > 200 * 1024) return bail(fail(PL_EINVAL, "smem layout %u B exceeds budget; lower queue_capacity", pl->smem));
   // ---- outputs
   const uint64_t R = std::max<uint64_t>(pl->roots_cap, 1);
