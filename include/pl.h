@@ -152,6 +152,8 @@ typedef struct {
   uint64_t spilled[PL_MAX_STAGES];         /* entries written to the HBM overflow ring */
   uint64_t overruns[PL_MAX_STAGES];        /* physical: firings longer than t_i        */
   uint64_t stalls[PL_MAX_STAGES];          /* firings that waited for room in the next queue */
+  uint32_t max_queue[PL_MAX_STAGES];       /* longest input queue seen at a firing decision (entries;
+                                              PAPER.md L133: "maximum size b_i v"), max over streams */
   int64_t  max_lateness_ns[PL_MAX_STAGES]; /* physical: max(actual - scheduled start)  */
   uint64_t sched_cycles[PL_MAX_STAGES];    /* clock64 cycles spent deciding firings    */
   int64_t  max_fire_ns[PL_MAX_STAGES];     /* physical: longest firing (start->publish) */
@@ -205,6 +207,11 @@ pl_status pl_pipeline_bind_device(pl_pipeline* pl, const void* dev_items, uint64
  * PCIe/C2C) when the executor starts; reads outside the window go to host memory.
  * PL_EINVAL if the buffer is not mapped.  It must stay valid until the run completes.    */
 pl_status pl_pipeline_bind_host(pl_pipeline* pl, const void* host_items, uint64_t n);
+
+/* Per-stream input-queue peaks of the last run: buf[s*N + i] = longest queue (entries) node i
+ * of stream s saw at a firing decision.  The data of the paper's b_i calibration (L133,
+ * L227-L230).  buf == NULL: *n = n_streams * N.                                          */
+pl_status pl_pipeline_queue_peaks(pl_pipeline* pl, uint32_t* buf, uint64_t cap, uint64_t* n);
 
 /* Compact result of the last run, reduced on the device (one 48-byte D->H copy).        */
 typedef struct {

@@ -67,6 +67,7 @@ class pl_stats(C.Structure):
     _fields_ = [("n_stages", C.c_uint32), ("n_streams", C.c_uint32), ("roots", C.c_uint64),
                 ("firings", _A8), ("empty_firings", _A8), ("consumed", _A8), ("produced", _A8),
                 ("active_window", _I8), ("busy_ns", _I8), ("spilled", _A8), ("overruns", _A8), ("stalls", _A8),
+                ("max_queue", C.c_uint32 * PL_MAX_STAGES),
                 ("max_lateness_ns", _I8), ("sched_cycles", _A8), ("max_fire_ns", _I8),
                 ("phase_cycles", (C.c_uint64 * 6) * PL_MAX_STAGES), ("matches", C.c_uint64),
                 ("miss_events", C.c_uint64), ("misses", C.c_uint64), ("max_latency", C.c_int64),
@@ -100,6 +101,7 @@ def _load():
         "pl_pipeline_bind_device": (C.c_int32, [P, P, C.c_uint64]),
         "pl_pipeline_bind_host": (C.c_int32, [P, P, C.c_uint64]),
         "pl_pipeline_summary": (C.c_int32, [P, C.POINTER(pl_summary)]),
+        "pl_pipeline_queue_peaks": (C.c_int32, [P, P, C.c_uint64, C.POINTER(C.c_uint64)]),
         "pl_pipeline_launch": (C.c_int32, [P]),
         "pl_pipeline_drain": (C.c_int32, [P]),
         "pl_pipeline_rewind": (C.c_int32, [P]),
@@ -130,7 +132,7 @@ EXPORTED = ("pl_pipeline_create", "pl_pipeline_set_stream", "pl_pipeline_push", 
             "pl_pipeline_results", "pl_pipeline_latency", "pl_pipeline_trace", "pl_pipeline_firings",
             "pl_pipeline_params", "pl_pipeline_destroy", "pl_last_error", "pl_solve_enforced_waits",
             "pl_solve_monolithic", "pl_version", "pl_stage_batch", "pl_pipeline_bind_host",
-            "pl_pipeline_summary")
+            "pl_pipeline_summary", "pl_pipeline_queue_peaks")
 
 
 class PlError(RuntimeError):

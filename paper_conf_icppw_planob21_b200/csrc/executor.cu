@@ -383,6 +383,7 @@ struct Decision {
   bool done;
   int64_t T;
   uint32_t n;
+  uint32_t qlen;    // input-queue length at the decision (all queued entries; L133's b_i v)
 };
 
 struct Leader {   // leader-private schedule state of one node
@@ -437,6 +438,7 @@ __device__ __forceinline__ Decision decide0(const Node& nd, Rep& r) {
   d.done = r.c0 >= nd.X;
   d.T = 0;
   d.n = 0;
+  d.qlen = 0;
   if (d.done) return d;
   int64_t T, q;
   if (nd.fixed) {
@@ -468,6 +470,7 @@ __device__ __forceinline__ Decision decide0(const Node& nd, Rep& r) {
   const int64_t avail = arrived - r.c0;
   d.T = T;
   d.n = (uint32_t)(avail < (int64_t)nd.v ? avail : nd.v);
+  d.qlen = (uint32_t)(avail < 0xffffffffll ? avail : 0xffffffffll);
   return d;
 }
 
@@ -485,7 +488,7 @@ __device__ __forceinline__ void advance0(const Node& nd, Rep& r) {
 __device__ Decision decide(const Node& nd, Leader& L) {
   const uint32_t v = (uint32_t)nd.v;
   Decision d;
-  d.done = false; d.T = 0; d.n = 0;
+  d.done = false; d.T = 0; d.n = 0; d.qlen = 0;
   int spins = 0;
   for (;;) {
     // node i >= 1: read the upstream watermark first, then the published segments
@@ -498,7 +501,7 @@ __device__ Decision decide(const Node& nd, Leader& L) {
       const int64_t T = L.m * nd.P;
       const uint32_t cnt = count_le(nd, L, st, T);
       if (cnt >= v || Wup > T) {
-        if (cnt > 0) { d.T = T; d.n = cnt < v ? cnt : v; return d; }
+        if (cnt > 0) { d.T = T; d.n = cnt < v ? cnt : v; d.qlen = tail_known - L.head; return d; }
         if (!any && Wup == PL_INF64) { d.done = true; return d; }
         const int64_t r = any ? nd.in_seg[L.segh & nd.segmask].ready : Wup;
         int64_t m2 = cdiv(r, nd.dP);
@@ -538,7 +541,7 @@ __device__ Decision decide(const Node& nd, Leader& L) {
     if (Tk < L.B) Tk = L.B;
     if (th_known || Tk < Wup) {
       const uint32_t cnt = count_le(nd, L, st, Tk);
-      if (Wup > Tk || cnt >= v) { d.T = Tk; d.n = cnt < v ? cnt : v; return d; }
+      if (Wup > Tk || cnt >= v) { d.T = Tk; d.n = cnt < v ? cnt : v; d.qlen = tail_known - L.head; return d; }
     }
     int64_t lb = Tk < Wup ? Tk : Wup;
     if (lb < L.B) lb = L.B;
@@ -724,6 +727,7 @@ __device__ void run_node(Ctx& c, const Dna dna, int i, int gtid) {
   R.m = 0; R.B = 0; R.c0 = 0; R.empties = 0; R.qT = 0; R.rT = 0; R.qvalid = false;
   uint64_t firings = 0, consumed = 0, produced = 0, spilled = 0, overruns = 0, stalls = 0;
   int64_t active = 0, busy_ns = 0, lateness = 0, t_end = 0, max_fire = 0;
+  uint32_t max_queue = 0;
   uint64_t start_ns = 0;
   uint32_t pend_root = NO_ROOT;          // lane: physical terminal event awaiting its end time
   uint64_t ph[6] = {0, 0, 0, 0, 0, 0};   // leader: per-phase clock64 cycles
@@ -739,6 +743,7 @@ __device__ void run_node(Ctx& c, const Dna dna, int i, int gtid) {
       const Decision d = decide0(nd, R);
       if (d.done) break;
       T = d.T; n = d.n; head = (uint32_t)R.c0;
+      if (d.qlen > max_queue) max_queue = d.qlen;
       if (leader) {
         if (rec & PL_REC_FIRINGS) G.log_idx[par] = atomicAdd(&c.sh->log_count, 1u);
         G.out_loc[par] = nd.sink ? LOC_SMEM : reserve_out(nd, L, n * nd.umax, &stalls);
@@ -756,6 +761,7 @@ __device__ void run_node(Ctx& c, const Dna dna, int i, int gtid) {
       if (leader) {
         const long long c0 = clock64();
         const Decision d = decide(nd, L);
+        if (d.qlen > max_queue) max_queue = d.qlen;
         G.done[par] = d.done ? 1u : 0u;
         G.T[par] = d.T;
         G.n[par] = d.n;
@@ -967,6 +973,7 @@ __device__ void run_node(Ctx& c, const Dna dna, int i, int gtid) {
     S.spilled[i] = spilled;
     S.overruns[i] = overruns;
     S.stalls[i] = stalls;
+    S.max_queue[i] = max_queue;
     S.lateness[i] = lateness;
     S.sched_cycles[i] = ph[0];
     S.max_fire_ns[i] = max_fire;
@@ -1257,7 +1264,7 @@ __device__ void run_monolithic(Ctx& c) {
     for (int i = 0; i < PL_MAX_STAGES; ++i) {
       S.firings[i] = firings[i]; S.empty[i] = 0; S.consumed[i] = consumed[i]; S.produced[i] = produced[i];
       S.active_ne[i] = active[i]; S.busy_ns[i] = i == 0 ? busy_ns : 0; S.spilled[i] = 0; S.overruns[i] = 0;
-      S.stalls[i] = 0;
+      S.stalls[i] = 0; S.max_queue[i] = 0;
       S.lateness[i] = 0; S.sched_cycles[i] = 0; S.max_fire_ns[i] = 0;
       for (int k = 0; k < 6; ++k) S.phase_cycles[i][k] = 0;
     }

@@ -41,6 +41,7 @@ struct CtaStats {
   uint64_t spilled[PL_MAX_STAGES];
   uint64_t overruns[PL_MAX_STAGES];
   uint64_t stalls[PL_MAX_STAGES];
+  uint32_t max_queue[PL_MAX_STAGES];
   int64_t  lateness[PL_MAX_STAGES];
   uint64_t sched_cycles[PL_MAX_STAGES];
   int64_t  max_fire_ns[PL_MAX_STAGES];

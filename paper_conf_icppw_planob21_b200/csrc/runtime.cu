@@ -525,6 +525,22 @@ pl_status pl_pipeline_bind_host(pl_pipeline* pl, const void* host_items, uint64_
   return PL_OK;
 }
 
+pl_status pl_pipeline_queue_peaks(pl_pipeline* pl, uint32_t* buf, uint64_t cap, uint64_t* n) {
+  if (!pl || !n) return fail(PL_EINVAL, "NULL argument");
+  const uint32_t S = pl->cfg.n_streams, N = pl->cfg.n_stages;
+  if (!buf) { *n = (uint64_t)S * N; return PL_OK; }
+  cudaSetDevice(pl->device);
+  CUDA_TRY(cudaStreamSynchronize(pl->stream));
+  std::vector<CtaStats> cs(S);
+  CUDA_TRY(cudaMemcpy(cs.data(), pl->d_stats, S * sizeof(CtaStats), cudaMemcpyDeviceToHost));
+  pl->d2h += S * sizeof(CtaStats);
+  uint64_t w = 0;
+  for (uint32_t s = 0; s < S; ++s)
+    for (uint32_t i = 0; i < N && w < cap; ++i) buf[w++] = cs[s].max_queue[i];
+  *n = w;
+  return PL_OK;
+}
+
 pl_status pl_pipeline_summary(pl_pipeline* pl, pl_summary* out) {
   if (!pl || !out) return fail(PL_EINVAL, "NULL argument");
   cudaSetDevice(pl->device);
@@ -619,6 +635,7 @@ pl_status pl_pipeline_stats(pl_pipeline* pl, pl_stats* out) {
       out->spilled[i] += s.spilled[i];
       out->overruns[i] += s.overruns[i];
       out->stalls[i] += s.stalls[i];
+      out->max_queue[i] = std::max(out->max_queue[i], s.max_queue[i]);
       out->max_lateness_ns[i] = std::max(out->max_lateness_ns[i], s.lateness[i]);
       out->sched_cycles[i] += s.sched_cycles[i];
       out->max_fire_ns[i] = std::max(out->max_fire_ns[i], s.max_fire_ns[i]);

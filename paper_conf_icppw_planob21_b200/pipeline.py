@@ -110,6 +110,14 @@ class Pipeline:
         """pl_pipeline_bind_host: the DB stays in pinned host memory; CTAs stage it by TMA."""
         check(lib.pl_pipeline_bind_host(self.h, C.c_void_p(host_ptr), int(n)), "pl_pipeline_bind_host")
 
+    def queue_peaks(self):
+        """pl_pipeline_queue_peaks -> uint32 array [n_streams, N]."""
+        n = C.c_uint64()
+        check(lib.pl_pipeline_queue_peaks(self.h, None, 0, C.byref(n)), "pl_pipeline_queue_peaks")
+        a = np.empty(n.value, dtype=np.uint32)
+        check(lib.pl_pipeline_queue_peaks(self.h, a.ctypes.data, n.value, C.byref(n)), "pl_pipeline_queue_peaks")
+        return a.reshape(-1, self.N)
+
     def summary(self) -> dict:
         s = _pl.pl_summary()
         check(lib.pl_pipeline_summary(self.h, C.byref(s)), "pl_pipeline_summary")

@@ -119,3 +119,52 @@ def monolithic_at(cfg, tau):
         return solve_monolithic(cfg.replace(interarrival=int(tau)))
     except RuntimeError:
         return None
+
+
+def calibrate_b(cfg, wl=None, db_dev=None, target=0.95, quantile=0.95, max_iter=10, log=None, stream=None):
+    """The paper's empirical b calibration, run on the device.
+
+    Start from b = 1 ("optimistic ... worst-case closely matches the average"), solve Fig. 1,
+    run all cfg.n_streams streams (independent seeds) in one launch, and accept once at least
+    `target` of them are miss-free.  Otherwise raise b_i to the `quantile` of the streams'
+    measured input-queue peaks divided by v -- L133 defines b_i v as the queue's maximum size
+    -- (or by one if that would not change b), re-solve and repeat.
+    Returns dict(b, w, T, miss_free, iterations, history)."""
+    import numpy as np
+    N, v = cfg.n_stages, cfg.vector_width
+    b = [1] * N
+    hist = []
+    for it in range(max_iter):
+        c = cfg.replace(b=tuple(b))
+        try:
+            w, th, T, Tc = solve_enforced_waits(c)
+        except RuntimeError:
+            return dict(b=tuple(b), w=None, T=None, miss_free=0.0, iterations=it, history=hist, infeasible=True)
+        c = c.replace(wait_time=tuple(w))
+        pl = Pipeline(c, wl, flags=1, stream=stream)
+        if wl is not None:
+            pl.bind_device(db_dev, wl.db_len)
+        else:
+            pl.push(None, c.n_roots)
+        pl.drain()
+        lat, lat_ns = pl.latency()
+        peaks = pl.queue_peaks()
+        pl.close()
+        L = lat_ns if c.clock == PHYS else lat
+        limit = c.deadline * (c.ns_per_unit if c.clock == PHYS else 1)
+        per = L[: (len(L) // c.n_streams) * c.n_streams].reshape(c.n_streams, -1)
+        mf = float(((per > limit).sum(axis=1) == 0).mean())
+        qb = [int(math.ceil(x / v)) for x in np.quantile(peaks, quantile, axis=0)]
+        rec = dict(iteration=it, b=tuple(b), T=T, miss_free=mf, queue_peak_q=[int(x) for x in
+                   np.quantile(peaks, quantile, axis=0)], b_from_queues=qb)
+        hist.append(rec)
+        if log:
+            log(rec)
+        if mf >= target:
+            return dict(b=tuple(b), w=tuple(w), T=T, miss_free=mf, iterations=it + 1, history=hist)
+        nb = [max(b[i], qb[i]) for i in range(N)]
+        if nb == b:   # queues already within b_i v: raise the node whose queue is closest to its bound
+            ratio = [peaks[:, i].max() / (b[i] * v) for i in range(N)]
+            nb[int(np.argmax(ratio))] += 1
+        b = nb
+    return dict(b=tuple(b), w=None, T=None, miss_free=hist[-1]["miss_free"], iterations=max_iter, history=hist)

@@ -51,3 +51,15 @@ def test_fig4_complementary_strengths():
     assert m - e >= 0.4
     e, m = both(100, 25_000)
     assert e - m >= 0.4
+
+
+@pytest.mark.parametrize("tau,D", [(10, 50_000), (50, 200_000)])
+def test_b_calibration_loop(tau, D):
+    """N1 / PAPER.md L227-L230: starting from b = 1, the on-device calibration (queue peaks
+    -> b_i, re-solve Fig. 1, 100 seeds per launch) reaches >= 95 % miss-free streams within a
+    few launches, with b no larger than the paper's conservative (1, 3, 9, 6)."""
+    from paper_conf_icppw_planob21_b200 import realtime
+    cfg = C.gain_model_blast(interarrival=tau, deadline=D, n_streams=S, n_roots=X, seed=21)
+    r = realtime.calibrate_b(cfg)
+    assert r["miss_free"] >= 0.95 and r["iterations"] <= 4
+    assert all(x <= y for x, y in zip(r["b"], C.PAPER_B))
