@@ -249,6 +249,7 @@ def main():
     clocks.start()
     ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(a.steps)]
     misses = 0
+    sched_misses = 0
     overruns = 0
     errors = 0
     roots = 0
@@ -259,7 +260,8 @@ def main():
         pl.launch()
         ev[k][1].record(stream)
         st = pl.stats()                                # syncs; outside the timed region
-        misses += st["miss_events"]
+        misses += st["miss_events_ns"]                 # measured on %globaltimer
+        sched_misses += st["miss_events"]              # the logical schedule's own
         overruns += sum(st["overruns"])
         errors |= st["errors"]
         roots += st["roots"]
@@ -271,12 +273,12 @@ def main():
         dist.barrier()
     st_last = allreduce_stats(dict(st, policy=0), device=dev)
     tt = torch.tensor([tot_ms], dtype=torch.float64, device=dev)
-    cnt = torch.tensor([roots, misses, overruns], dtype=torch.int64, device=dev)
+    cnt = torch.tensor([roots, misses, overruns, sched_misses], dtype=torch.int64, device=dev)
     if world > 1:
         dist.all_reduce(tt, op=dist.ReduceOp.MAX)
         dist.all_reduce(cnt, op=dist.ReduceOp.SUM)
     tot_ms = float(tt.item())
-    roots_all, misses_all, overruns_all = (int(x) for x in cnt.tolist())
+    roots_all, misses_all, overruns_all, sched_misses_all = (int(x) for x in cnt.tolist())
     value = roots_all / (tot_ms * 1e-3)
 
     # logical-clock throughput of the same executor (no real-time pacing)
@@ -344,7 +346,7 @@ def main():
             ple.launch()
             sm_ = ple.summary()
             e_roots += sm_["roots"]
-            e_miss += sm_["miss_events"]
+            e_miss += sm_["miss_events_ns"]
         e_dt = time.perf_counter() - t0
         s1 = ple.stats()
         s2 = ple.stats()                 # the size of one stats read, to exclude it
@@ -381,11 +383,16 @@ def main():
                        "budgets_ns": list(budgets), "w_ns": list(w), "gains": [round(g, 5) for g in gains],
                        "streams_per_gpu": a.streams, "l2": "flushed between timed steps (256 MiB memset)",
                        "parallelism": f"{a.streams} streams x {world} GPUs (independent; NCCL stats all-reduce)"},
-            "misses": misses_all, "overruns": overruns_all, "errors": errors,
+            "misses": misses_all, "schedule_misses": sched_misses_all, "overruns": overruns_all, "errors": errors,
             "sustained_items_per_s": world * a.streams * 1e9 / tau,
             "logical_items_per_s": logical_ips,
             "utilisation": {"enforced_model": st_last["active_fraction"], "enforced_fig1_T": T,
                             "enforced_hw_busy": st["hw_busy_fraction"], "monolithic": mono},
+            "per_firing": {f"node{i}": {"firings": st["firings"][i],
+                                        "scheduler_cycles": round(st["phase_cycles"][i][0] / max(1, st["firings"][i])),
+                                        "firing_cycles": round(sum(st["phase_cycles"][i][1:]) / max(1, st["firings"][i])),
+                                        "mean_fire_ns": round(st["busy_ns"][i] / max(1, st["firings"][i])),
+                                        "max_fire_ns": st["max_fire_ns"][i]} for i in range(st["n_stages"])},
             "clocks": clk,
             "e2e": e2e,
             "gpu_launches": a.steps,

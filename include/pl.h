@@ -162,7 +162,9 @@ typedef struct {
    * [3] records+reserve, [4] output writes, [5] publish                        */
   uint64_t phase_cycles[PL_MAX_STAGES][6];
   uint64_t matches;
-  uint64_t miss_events;                    /* terminal events with latency > D        */
+  uint64_t miss_events;                    /* terminal events with latency > D (schedule) */
+  uint64_t miss_events_ns;                 /* physical clock: terminal events whose MEASURED
+                                              latency exceeded D (always counted)          */
   uint64_t misses;                         /* distinct roots (needs PL_REC_LATENCY)    */
   int64_t  max_latency;                    /* model units (logical schedule)          */
   int64_t  max_latency_ns;                 /* physical: measured                       */
@@ -213,9 +215,9 @@ pl_status pl_pipeline_bind_host(pl_pipeline* pl, const void* host_items, uint64_
  * L227-L230).  buf == NULL: *n = n_streams * N.                                          */
 pl_status pl_pipeline_queue_peaks(pl_pipeline* pl, uint32_t* buf, uint64_t cap, uint64_t* n);
 
-/* Compact result of the last run, reduced on the device (one 48-byte D->H copy).        */
+/* Compact result of the last run, reduced on the device (one small D->H copy).         */
 typedef struct {
-  uint64_t roots, matches, miss_events;
+  uint64_t roots, matches, miss_events, miss_events_ns;
   int64_t  max_latency, max_latency_ns;
   uint32_t errors, launches;
 } pl_summary;

@@ -55,7 +55,7 @@ class pl_firing(C.Structure):
 
 class pl_summary(C.Structure):
     _fields_ = [("roots", C.c_uint64), ("matches", C.c_uint64), ("miss_events", C.c_uint64),
-                ("max_latency", C.c_int64), ("max_latency_ns", C.c_int64), ("errors", C.c_uint32),
+                ("miss_events_ns", C.c_uint64), ("max_latency", C.c_int64), ("max_latency_ns", C.c_int64), ("errors", C.c_uint32),
                 ("launches", C.c_uint32)]
 
 
@@ -70,7 +70,8 @@ class pl_stats(C.Structure):
                 ("max_queue", C.c_uint32 * PL_MAX_STAGES),
                 ("max_lateness_ns", _I8), ("sched_cycles", _A8), ("max_fire_ns", _I8),
                 ("phase_cycles", (C.c_uint64 * 6) * PL_MAX_STAGES), ("matches", C.c_uint64),
-                ("miss_events", C.c_uint64), ("misses", C.c_uint64), ("max_latency", C.c_int64),
+                ("miss_events", C.c_uint64), ("miss_events_ns", C.c_uint64), ("misses", C.c_uint64),
+                ("max_latency", C.c_int64),
                 ("max_latency_ns", C.c_int64), ("window", C.c_int64), ("t_end", C.c_int64),
                 ("active_fraction", C.c_double), ("active_fraction_nonempty", C.c_double),
                 ("hw_busy_fraction", C.c_double), ("wall_ns", C.c_int64), ("errors", C.c_uint32),

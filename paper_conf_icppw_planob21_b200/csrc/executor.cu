@@ -165,6 +165,7 @@ struct Shared {
   uint32_t max_lat;         // per-stream aggregates: 32-bit so the smem atomics are native
   uint32_t max_lat_ns;      // (64-bit smem atomicMax compiles to a CAS loop)
   uint32_t miss_events;
+  uint32_t miss_events_ns;  // physical: terminal items whose measured latency exceeded D
   uint32_t errors;
   uint32_t log_count;       // firing-log records reserved by all nodes of this stream
   uint64_t T0;
@@ -793,6 +794,7 @@ __device__ void run_node(Ctx& c, const Dna dna, int i, int gtid) {
         const int64_t l = (int64_t)G.end_ns[par ^ 1] - (int64_t)a_ns;
         if (rec & PL_REC_LATENCY) atomicMax((long long*)&p.lat_ns[pend_root], (long long)l);
         atomicMax(&c.sh->max_lat_ns, (uint32_t)(l > 0 ? (l < 0xffffffffll ? l : 0xffffffffll) : 0));
+        if ((double)l > (double)nd.D * nd.nspu) atomicAdd(&c.sh->miss_events_ns, 1u);
         pend_root = NO_ROOT;
       }
       if (G.done[par]) break;
@@ -824,6 +826,7 @@ __device__ void run_node(Ctx& c, const Dna dna, int i, int gtid) {
       const int64_t l = (int64_t)G.end_ns[par ^ 1] - (int64_t)a_ns;
       if (rec & PL_REC_LATENCY) atomicMax((long long*)&p.lat_ns[pend_root], (long long)l);
       atomicMax(&c.sh->max_lat_ns, (uint32_t)(l > 0 ? (l < 0xffffffffll ? l : 0xffffffffll) : 0));
+      if ((double)l > (double)nd.D * nd.nspu) atomicAdd(&c.sh->miss_events_ns, 1u);
       pend_root = NO_ROOT;
     }
     // --- release the input slots (every lane has loaded its entry: B2 passed)
@@ -960,6 +963,7 @@ __device__ void run_node(Ctx& c, const Dna dna, int i, int gtid) {
       const int64_t l = (int64_t)G.end_ns[par ^ 1] - (int64_t)a_ns;
       if (rec & PL_REC_LATENCY) atomicMax((long long*)&p.lat_ns[pend_root], (long long)l);
       atomicMax(&c.sh->max_lat_ns, (uint32_t)(l > 0 ? (l < 0xffffffffll ? l : 0xffffffffll) : 0));
+      if ((double)l > (double)nd.D * nd.nspu) atomicAdd(&c.sh->miss_events_ns, 1u);
     }
   }
   if (leader) {
@@ -1079,7 +1083,9 @@ __device__ void cta_setup(Ctx& c, Shared& sh, unsigned char* dsm, const DevParam
     EdgeCtl& E = sh.e[tid];
     E.head = 0; E.seg_head = 0; E.seg_tail = 0; E.tail = 0; E.W = -1; E.spill_end = 0; E.pad = 0;
   }
-  if (tid == 0) { sh.max_lat = 0; sh.max_lat_ns = 0; sh.miss_events = 0; sh.errors = 0; sh.log_count = 0; }
+  if (tid == 0) {
+    sh.max_lat = 0; sh.max_lat_ns = 0; sh.miss_events = 0; sh.miss_events_ns = 0; sh.errors = 0; sh.log_count = 0;
+  }
   // per-root records of this stream
   if (p.flags & PL_REC_LATENCY)
     for (uint64_t r = c.lo + tid; r < c.hi; r += nt) { p.lat[r] = -1; if (p.lat_ns) p.lat_ns[r] = -1; }
@@ -1096,6 +1102,7 @@ __device__ void cta_finish(Ctx& c, Shared& sh, const DevParams& p) {
   if (threadIdx.x == 0) {
     CtaStats& S = p.stats[blockIdx.x];
     S.miss_events = sh.miss_events;
+    S.miss_events_ns = sh.miss_events_ns;
     S.max_lat = (int64_t)sh.max_lat;
     S.max_lat_ns = (int64_t)sh.max_lat_ns;
     S.wall_ns = (int64_t)(gtimer() - sh.T0);
@@ -1108,6 +1115,7 @@ __device__ void cta_finish(Ctx& c, Shared& sh, const DevParams& p) {
       atomicMax(p.summary + 2, (unsigned long long)sh.max_lat);
       atomicMax(p.summary + 3, (unsigned long long)sh.max_lat_ns);
       atomicOr(p.summary + 4, (unsigned long long)sh.errors);
+      atomicAdd(p.summary + 5, (unsigned long long)sh.miss_events_ns);
     }
   }
 }
@@ -1202,6 +1210,7 @@ __device__ void run_monolithic(Ctx& c) {
               const int64_t ln = (int64_t)gtimer() - (int64_t)a_ns;
               if (rec & PL_REC_LATENCY) atomicMax((long long*)&p.lat_ns[e.x], (long long)ln);
               atomicMax(&c.sh->max_lat_ns, (uint32_t)(ln > 0 ? (ln < 0xffffffffll ? ln : 0xffffffffll) : 0));
+              if ((double)ln > (double)p.D * p.ns_per_unit) atomicAdd(&c.sh->miss_events_ns, 1u);
             }
           }
           if ((rec & PL_REC_FIRINGS) && (idx % (uint32_t)v == 0 || idx == ncur - 1 || idx % (uint32_t)v == (uint32_t)v - 1)) {

@@ -47,6 +47,7 @@ struct CtaStats {
   int64_t  max_fire_ns[PL_MAX_STAGES];
   uint64_t phase_cycles[PL_MAX_STAGES][6];
   uint64_t miss_events;
+  uint64_t miss_events_ns;              // physical: measured latency > D
   int64_t  max_lat;                     // model units
   int64_t  max_lat_ns;
   int64_t  t_end;                       // drain end (model units)

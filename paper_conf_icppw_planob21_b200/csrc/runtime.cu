@@ -553,6 +553,7 @@ pl_status pl_pipeline_summary(pl_pipeline* pl, pl_summary* out) {
   pl->d2h += 56;
   out->roots = h[0];
   out->miss_events = h[1];
+  out->miss_events_ns = h[5];
   out->max_latency = (int64_t)h[2];
   out->max_latency_ns = (int64_t)h[3];
   out->errors = (uint32_t)h[4];
@@ -648,6 +649,7 @@ pl_status pl_pipeline_stats(pl_pipeline* pl, pl_stats* out) {
       }
     }
     out->miss_events += s.miss_events;
+    out->miss_events_ns += s.miss_events_ns;
     out->max_latency = std::max(out->max_latency, s.max_lat);
     out->max_latency_ns = std::max(out->max_latency_ns, s.max_lat_ns);
     out->wall_ns = std::max(out->wall_ns, s.wall_ns);

@@ -82,9 +82,9 @@ def find_rate(cfg, wl, db_dev, tries=12, grow=1.15, stream=None, log=None, over=
         c = cfg.replace(interarrival=int(tau), wait_time=tuple(w), clock=PHYS)
         try:
             st = _run(c, db_dev, wl.db_len, wl, flags=1, stream=stream, over=over)
-            ok = st["misses"] == 0 and st["errors"] == 0
+            ok = st["misses"] == 0 and st["miss_events_ns"] == 0 and st["errors"] == 0
         except PlError:          # device-side overflow reported by drain
-            st, ok = {"misses": -1, "errors": -1, "overruns": [], "max_latency_ns": -1}, False
+            st, ok = {"misses": -1, "miss_events_ns": -1, "errors": -1, "overruns": [], "max_latency_ns": -1}, False
         if log:
             log(dict(tau=tau, w=w, T=T, misses=st["misses"], overruns=st["overruns"], errors=st["errors"],
                      max_latency_ns=st["max_latency_ns"]))

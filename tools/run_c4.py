@@ -12,6 +12,9 @@ from plgen import dna as G
 from paper_conf_icppw_planob21_b200 import Pipeline, realtime, solve_enforced_waits
 
 D = int(sys.argv[1]) if len(sys.argv) > 1 else 350_000
+import subprocess
+smi = subprocess.Popen(["nvidia-smi", "--query-gpu=clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active",
+                        "--format=csv,noheader", "-lms", "500"], stdout=open("gpurun_out/c4_clocks.csv", "w"))
 base = C.c4()
 t0 = time.time()
 wl = G.make_dna(base.seed, **base.dna)
@@ -62,3 +65,5 @@ try:
                       "active_fraction": st["active_fraction"], "hw_busy": st["hw_busy_fraction"]}), flush=True)
 except RuntimeError as ex:
     print(json.dumps({"physical": "failed", "why": str(ex)}), flush=True)
+
+smi.terminate()
