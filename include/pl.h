@@ -112,6 +112,11 @@ typedef struct {
   uint32_t spill_capacity;         /* HBM overflow entries per edge per stream (2^k; 0->dflt) */
   uint32_t firing_log_capacity;    /* records per stream when PL_REC_FIRINGS (0 -> dflt) */
   uint64_t match_capacity;         /* pl_match records (0 -> default)                   */
+  const int64_t* arrivals;         /* NULL: root r of a stream arrives at r*tau0 (L63).  Else
+                                      arrival time (units, from its stream's start) of every
+                                      root, non-decreasing within a stream, e.g. Poisson (L263);
+                                      copied at create; n_arrivals must equal the root count */
+  uint64_t n_arrivals;
 } pl_config;
 
 /* Workload of the DNA pipeline: the query is known up front; the database is the

@@ -103,14 +103,15 @@ def _overlap(s, e, lo, hi):
 
 
 def simulate_stream(cfg: C.Config, fns, lo: int, hi: int, wait_time=None, theta=None,
-                    block_size=None, check_invariants=False, node_order=None) -> StreamResult:
+                    block_size=None, check_invariants=False, node_order=None, arrivals=None) -> StreamResult:
     """Simulate one independent stream whose roots are the global ids [lo, hi).
 
-    Root r (global) arrives at a(r) = (r - lo) * tau0.  ``node_order`` permutes
-    the order in which nodes are visited inside phases 1 and 3 (pin P5).
+    Root r (global) arrives at a(r) = (r - lo) * tau0, or at arrivals[r - lo]
+    when an arrival-time array is given (non-decreasing; Poisson arrivals, L263).
+    ``node_order`` permutes the order in which nodes are visited inside phases 1 and 3 (pin P5).
     """
     if cfg.policy == C.MONOLITHIC:
-        return _simulate_monolithic(cfg, fns, lo, hi, block_size)
+        return _simulate_monolithic(cfg, fns, lo, hi, block_size, arrivals)
     N = cfg.n_stages
     t = list(cfg.service_time)
     v = cfg.vector_width
@@ -118,6 +119,7 @@ def simulate_stream(cfg: C.Config, fns, lo: int, hi: int, wait_time=None, theta=
     D = cfg.deadline
     X = hi - lo
     H = X * tau
+    arr = [r * tau for r in range(X)] if arrivals is None else [int(x) for x in arrivals]
     order = list(range(N)) if node_order is None else list(node_order)
     match_sink = cfg.stages[-1].kind == C.UNGAPPED_XDROP
     fixed = cfg.policy == C.FIXED_WAIT
@@ -145,7 +147,7 @@ def simulate_stream(cfg: C.Config, fns, lo: int, hi: int, wait_time=None, theta=
     active_H_ne = [0] * N
     T_end = 0
     next_root = 0
-    heap = [0]
+    heap = [0] + ([arr[0]] if X else [])
     last_T = None
     entered = [0] * N                            # for invariant checks (P4)
 
@@ -171,29 +173,29 @@ def simulate_stream(cfg: C.Config, fns, lo: int, hi: int, wait_time=None, theta=
                     trace[r * (N + 1) + N] += len(ch)
                     if match_sink:
                         matches.extend(ch)
-                    lat[r] = max(lat[r], T - r * tau)
+                    lat[r] = max(lat[r], T - arr[r])
                 elif ch:
                     Q[i + 1].extend(ch)
                     entered[i + 1] += len(ch)
                 else:
-                    lat[r] = max(lat[r], T - r * tau)
+                    lat[r] = max(lat[r], T - arr[r])
             if f[2]:
                 T_end = max(T_end, T)
         # ---- 2. arrivals
-        if next_root < X and next_root * tau == T:
-            while next_root < X and next_root * tau == T:
+        if next_root < X and arr[next_root] == T:
+            while next_root < X and arr[next_root] == T:
                 Q[0].append((lo + next_root, 0, None))
                 entered[0] += 1
                 next_root += 1
             if next_root < X:
-                push(next_root * tau)
+                push(arr[next_root])
         # ---- 3. starts
         for i in order:
             fire = False
             if fixed:
                 fire = next_start[i] == T
             elif inflight[i] is None and Q[i]:
-                a_head = (Q[i][0][0] - lo) * tau
+                a_head = arr[Q[i][0][0] - lo]
                 fire = len(Q[i]) >= th[i] or T >= a_head + D - R[i]
             if fire:
                 n = min(len(Q[i]), v)
@@ -216,7 +218,7 @@ def simulate_stream(cfg: C.Config, fns, lo: int, hi: int, wait_time=None, theta=
                     next_start[i] = T + P[i]
                     push(next_start[i])
             if not fixed and Q[i]:
-                fdl = (Q[i][0][0] - lo) * tau + D - R[i]
+                fdl = arr[Q[i][0][0] - lo] + D - R[i]
                 if fdl > T and last_force[i] != fdl:
                     last_force[i] = fdl
                     push(fdl)
@@ -248,7 +250,7 @@ def _check_conservation(N, entered, consumed, Q, produced, next_root, X, trace, 
     assert done <= next_root
 
 
-def _simulate_monolithic(cfg, fns, lo, hi, M):
+def _simulate_monolithic(cfg, fns, lo, hi, M, arrivals=None):
     """MONOLITHIC (§5; reading R-MONO)."""
     N = cfg.n_stages
     t = list(cfg.service_time)
@@ -257,6 +259,7 @@ def _simulate_monolithic(cfg, fns, lo, hi, M):
     X = hi - lo
     H = X * tau
     M = int(M if M is not None else cfg.block_size)
+    arr = [r * tau for r in range(X)] if arrivals is None else [int(x) for x in arrivals]
     lat = [-1] * X
     trace = [0] * (X * (N + 1))
     matches = []
@@ -270,7 +273,7 @@ def _simulate_monolithic(cfg, fns, lo, hi, M):
     T_end = 0
     for b0 in range(0, X, M):
         b1 = min(b0 + M, X)
-        ready = (b1 - 1) * tau                   # last root of the block has arrived
+        ready = arr[b1 - 1]                      # last root of the block has arrived
         T = max(ready, proc_free)
         cur = [(lo + r, 0, None) for r in range(b0, b1)]
         for i in range(N):
@@ -293,11 +296,11 @@ def _simulate_monolithic(cfg, fns, lo, hi, M):
                         trace[r * (N + 1) + N] += len(ch)
                         if cfg.stages[-1].kind == C.UNGAPPED_XDROP:
                             matches.extend(ch)
-                        lat[r] = max(lat[r], e_ - r * tau)
+                        lat[r] = max(lat[r], e_ - arr[r])
                     elif ch:
                         nxt.extend(ch)
                     else:
-                        lat[r] = max(lat[r], e_ - r * tau)
+                        lat[r] = max(lat[r], e_ - arr[r])
                 T_end = max(T_end, e_)
             cur = nxt
         proc_free = T
@@ -341,7 +344,7 @@ def stream_ranges(cfg: C.Config, n_roots_total: int):
     return [((s * n_roots_total) // S, ((s + 1) * n_roots_total) // S) for s in range(S)]
 
 
-def run(cfg: C.Config, workload=None, streams=None, **kw) -> Result:
+def run(cfg: C.Config, workload=None, streams=None, arrivals=None, **kw) -> Result:
     """Simulate every stream of ``cfg`` (or the subset ``streams``) and merge.
 
     DNA configs need ``workload`` (plgen.dna.DnaWorkload); roots are DB
@@ -357,7 +360,8 @@ def run(cfg: C.Config, workload=None, streams=None, **kw) -> Result:
     fns = make_stage_fns(cfg, ctx)
     rng = stream_ranges(cfg, total)
     idx = range(len(rng)) if streams is None else streams
-    res = [simulate_stream(cfg, fns, rng[s][0], rng[s][1], **kw) for s in idx]
+    res = [simulate_stream(cfg, fns, rng[s][0], rng[s][1],
+                           arrivals=None if arrivals is None else arrivals[rng[s][0]:rng[s][1]], **kw) for s in idx]
     lat, trace, matches = [], [], []
     for r in res:
         lat += r.lat

@@ -35,7 +35,7 @@ class pl_config(C.Structure):
                 ("n_roots", C.c_uint64), ("seed", C.c_uint64), ("device", C.c_int32),
                 ("ns_per_unit", C.c_double), ("flags", C.c_uint32), ("queue_capacity", C.c_uint32),
                 ("spill_capacity", C.c_uint32), ("firing_log_capacity", C.c_uint32),
-                ("match_capacity", C.c_uint64)]
+                ("match_capacity", C.c_uint64), ("arrivals", C.POINTER(C.c_int64)), ("n_arrivals", C.c_uint64)]
 
 
 class pl_workload(C.Structure):

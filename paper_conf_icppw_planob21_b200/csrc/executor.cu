@@ -181,7 +181,9 @@ struct Ctx {
   int64_t X, H;
 };
 
-__device__ __forceinline__ int64_t arrival(const Ctx& c, uint32_t root) { return (int64_t)(root - c.lo) * c.p->tau; }
+__device__ __forceinline__ int64_t arrival(const Ctx& c, uint32_t root) {
+  return c.p->arr ? __ldg(c.p->arr + root) : (int64_t)(root - c.lo) * c.p->tau;
+}
 
 // floor(a / d) for 0 <= a < 2^63 by a host-precomputed reciprocal m = floor((2^64-1)/d):
 // umulhi(a, m) is floor(a/d) or one less, fixed by one compare (no 64-bit division).
@@ -220,7 +222,10 @@ struct Node {
   int32_t ip1, ip2;
   MDiv dtau, dP;
   int64_t Pq, Pr;               // floor(P / tau0), P mod tau0
-  __device__ __forceinline__ int64_t arrival(uint32_t root) const { return (int64_t)(root - lo) * tau; }
+  const int64_t* arr;           // per-root arrival times (NULL: fixed rate, L63)
+  __device__ __forceinline__ int64_t arrival(uint32_t root) const {
+    return arr ? __ldg(arr + root) : (int64_t)(root - lo) * tau;
+  }
 };
 
 __host__ __device__ inline uint32_t layout_enforced(const DevParams& p, SmemLayout* L);
@@ -260,6 +265,7 @@ __device__ __forceinline__ Node make_node(const Ctx& c, int i) {
   n.dP.m = p.P_m[i]; n.dP.d = p.P[i];
   n.Pq = fdiv(p.P[i], n.dtau);
   n.Pr = p.P[i] - n.Pq * p.tau;
+  n.arr = p.arr;
   return n;
 }
 
@@ -441,6 +447,29 @@ __device__ __forceinline__ Decision decide0(const Node& nd, Rep& r) {
   d.n = 0;
   d.qlen = 0;
   if (d.done) return d;
+  if (nd.arr) {   // arrival times given as data: the lanes test their own item (sorted -> a prefix)
+    const int64_t* A = nd.arr + nd.lo;
+    const int64_t ah = __ldg(A + r.c0);
+    int64_t T;
+    if (nd.fixed) {
+      T = r.m * nd.P;
+      if (T < ah) {
+        const int64_t m2 = cdiv(ah, nd.dP);
+        r.empties += (uint64_t)(m2 - r.m);
+        r.m = m2;
+        T = r.m * nd.P;
+      }
+    } else {
+      const int64_t Tth = (r.c0 + nd.theta - 1 < nd.X) ? __ldg(A + r.c0 + nd.theta - 1) : PL_INF64;
+      int64_t Tf = ah + nd.D - nd.R;
+      if (Tf < ah) Tf = ah;
+      T = Tth < Tf ? Tth : Tf;
+      if (T < r.B) T = r.B;
+    }
+    d.T = T;
+    d.n = (uint32_t)nd.v;                // upper bound; the exact count comes out of the scan
+    return d;
+  }
   int64_t T, q;
   if (nd.fixed) {
     T = r.m * nd.P;
@@ -738,7 +767,7 @@ __device__ void run_node(Ctx& c, const Dna dna, int i, int gtid) {
 
   for (;;) {
     int64_t T;
-    uint32_t n, head;
+    uint32_t n, head;                    // n: items consumed (node 0 with arrival data: from the scan)
     if (n0) {
       const long long c0 = leader ? clock64() : 0;
       const Decision d = decide0(nd, R);
@@ -800,7 +829,10 @@ __device__ void run_node(Ctx& c, const Dna dna, int i, int gtid) {
       if (G.done[par]) break;
       T = G.T[par]; n = G.n[par]; head = G.head[par];
     }
-    const bool act = (uint32_t)gtid < n;
+    const bool arrmode = n0 && nd.arr != nullptr;
+    const bool act = arrmode ? ((uint32_t)gtid < n && R.c0 + gtid < nd.X &&
+                                __ldg(nd.arr + nd.lo + R.c0 + gtid) <= T)
+                             : (uint32_t)gtid < n;
     uint2 e[1];
     const bool acts[1] = {act};
     LaneOut o[1];
@@ -819,7 +851,16 @@ __device__ void run_node(Ctx& c, const Dna dna, int i, int gtid) {
       default: stage_batch<1, PL_UNGAPPED_WINDOW>(nd, dna, p, e, acts, o); break;   // S2 / S3
     }
     uint32_t total;
-    const uint32_t off = group_scan(G.wtot[par], o[0].c, &total, gtid, v, bidA, nd.umax <= 1);   // B2
+    uint32_t off;
+    if (arrmode) {   // count the arrived items in the same scan: (items << 16) | outputs
+      uint32_t packed;
+      const uint32_t ex = group_scan(G.wtot[par], ((act ? 1u : 0u) << 16) | o[0].c, &packed, gtid, v, bidA, false);
+      off = ex & 0xffffu;
+      total = packed & 0xffffu;
+      n = packed >> 16;
+    } else {
+      off = group_scan(G.wtot[par], o[0].c, &total, gtid, v, bidA, nd.umax <= 1);                 // B2
+    }
     if (leader) { const long long t2 = clock64(); ph[2] += (uint64_t)(t2 - tc); tc = t2; }
     if (n0 && pend_root != NO_ROOT) {    // node 0: the previous publish time arrives through B2
       const uint64_t a_ns = T0 + (uint64_t)((double)nd.arrival(pend_root) * nd.nspu);
@@ -1164,7 +1205,7 @@ __device__ void run_monolithic(Ctx& c) {
   const int64_t M = p.M;
   for (int64_t b0 = 0; b0 < c.X; b0 += M) {
     const int64_t b1 = (b0 + M < c.X) ? b0 + M : c.X;
-    const int64_t ready = (b1 - 1) * p.tau;
+    const int64_t ready = arrival(c, (uint32_t)(c.lo + b1 - 1));
     int64_t T = ready > proc_free ? ready : proc_free;
     if (phys) {
       if (tid == 0) {

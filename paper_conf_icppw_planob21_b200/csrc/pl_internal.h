@@ -101,7 +101,8 @@ struct DevParams {
   pl_firing* flog;                      // [n_streams][log_cap]
   uint32_t log_cap;
   CtaStats* stats;                      // [n_streams]
-  unsigned long long* summary;          // [6]: roots, miss_events, max_lat, max_lat_ns, errors, -
+  unsigned long long* summary;          // [6]: roots, miss_events, max_lat, max_lat_ns, errors, miss_ns
+  const int64_t* arr;                   // per-root arrival times (NULL: r * tau0)
   DevStage st[PL_MAX_STAGES];
 };
 

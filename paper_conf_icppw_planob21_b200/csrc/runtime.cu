@@ -125,6 +125,7 @@ struct pl_pipeline {
   uint64_t h2d = 0, d2h = 0;  // bytes moved across the host boundary (cumulative)
   unsigned long long* d_scratch = nullptr;   // stage-batch counters
   unsigned long long* d_summary = nullptr;   // device-reduced run summary
+  int64_t* d_arr = nullptr;                  // per-root arrival times (optional)
   bool bound_host = false;
 };
 
@@ -133,7 +134,7 @@ namespace {
 void free_all(pl_pipeline* pl) {
   void* ptrs[] = {pl->d_db, pl->d_qoff, pl->d_qpos, pl->d_qw, pl->d_spill, pl->d_mono, pl->d_lat, pl->d_lat_ns,
                   pl->d_trace, pl->d_matches, pl->d_match_count, pl->d_flog, pl->d_stats, pl->d_scratch,
-                  pl->d_summary};
+                  pl->d_summary, pl->d_arr};
   for (void* p : ptrs)
     if (p) cudaFree(p);
 }
@@ -463,6 +464,22 @@ pl_status pl_pipeline_create(const pl_config* cfg, const pl_workload* wl, pl_pip
   d.flog = pl->d_flog;
   d.stats = pl->d_stats;
   d.summary = pl->d_summary;
+  if (cfg->arrivals) {   // arrival process given as data (Poisson, L263): per root, per stream
+    if (cfg->n_arrivals != pl->roots_cap)
+      return bail(fail(PL_EINVAL, "n_arrivals %llu != root count %llu", (unsigned long long)cfg->n_arrivals,
+                       (unsigned long long)pl->roots_cap));
+    const uint64_t R = pl->roots_cap;
+    for (uint32_t s = 0; s < S; ++s) {
+      const uint64_t lo = R * s / S, hi = R * (s + 1) / S;
+      for (uint64_t r = lo; r < hi; ++r)
+        if (cfg->arrivals[r] < 0 || (r > lo && cfg->arrivals[r] < cfg->arrivals[r - 1]))
+          return bail(fail(PL_EINVAL, "arrivals must be >= 0 and non-decreasing within a stream"));
+    }
+    if (cudaMalloc(&pl->d_arr, R * 8) != cudaSuccess) return bail(fail(PL_ENOMEM, "arrival times"));
+    cudaMemcpy(pl->d_arr, cfg->arrivals, R * 8, cudaMemcpyHostToDevice);
+    pl->h2d += R * 8;
+  }
+  d.arr = pl->d_arr;
   cudaError_t e1 = pl_kernel_attributes(200 * 1024);
   if (e1 != cudaSuccess) return bail(fail(PL_EDEVICE, "cudaFuncSetAttribute: %s", cudaGetErrorString(e1)));
   cudaError_t e = cudaDeviceSynchronize();
@@ -577,6 +594,9 @@ pl_status pl_pipeline_launch(pl_pipeline* pl) {
     d.total_roots = pl->pushed * pl->cfg.n_streams;
   }
   if (d.total_roots > pl->roots_cap) return fail(PL_EINVAL, "more roots than allocated");
+  if (pl->d_arr && d.total_roots != pl->roots_cap)
+    return fail(PL_EINVAL, "arrival times were given for %llu roots; push the whole stream",
+                (unsigned long long)pl->roots_cap);
   CUDA_TRY(cudaMemsetAsync(pl->d_match_count, 0, 8, pl->stream));
   CUDA_TRY(cudaMemsetAsync(pl->d_summary, 0, 64, pl->stream));
   CUDA_TRY(pl_launch(d, pl->cfg.n_streams, pl->block, pl->smem, pl->stream));

@@ -71,9 +71,14 @@ def make_config(cfg, flags=0, device=0, n_streams=None, **over):
 class Pipeline:
     """pl_pipeline_* on one handle.  Raises ``PlError`` on every non-OK status."""
 
-    def __init__(self, cfg, workload=None, flags=0, device=0, stream=None, **over):
+    def __init__(self, cfg, workload=None, flags=0, device=0, stream=None, arrivals=None, **over):
         self.cfg = cfg
         self._c, self._keep = make_config(cfg, flags=flags, device=device, **over)
+        if arrivals is not None:   # per-root arrival times (pl_config.arrivals; copied at create)
+            arr = np.ascontiguousarray(arrivals, dtype=np.int64)
+            self._keep.append(arr)
+            self._c.arrivals = arr.ctypes.data_as(C.POINTER(C.c_int64))
+            self._c.n_arrivals = arr.shape[0]
         wl = None
         if workload is not None:
             q = np.ascontiguousarray(workload.query, dtype=np.uint32)

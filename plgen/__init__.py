@@ -10,7 +10,8 @@ read:
 * ``gaintab``  — the per-stage random-gain thresholds of the paper's gain model
                  (§6.1): the *distribution tables* the method
                  draws from, passed to both sides as input.
+* ``arrivals`` — random arrival times (Poisson) as an input array.
 * ``configs``  — the named configurations of BASELINE.json (c1..c5) and the
                  timing parameters of PAPER.md Table 1 (L218–L225).
 """
-from . import dna, gaintab, configs  # noqa: F401
+from . import arrivals, dna, gaintab, configs  # noqa: F401

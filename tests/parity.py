@@ -14,9 +14,9 @@ def workload_for(cfg):
     return G.make_dna(cfg.seed, **cfg.dna)
 
 
-def run_gpu(cfg, wl, flags=7, **over):
+def run_gpu(cfg, wl, flags=7, arrivals=None, **over):
     from paper_conf_icppw_planob21_b200 import Pipeline
-    pl = Pipeline(cfg, wl, flags=flags, **over)
+    pl = Pipeline(cfg, wl, flags=flags, arrivals=arrivals, **over)
     if wl is not None:
         pl.push(wl.db, wl.db_len)
     else:
@@ -34,9 +34,9 @@ def run_gpu(cfg, wl, flags=7, **over):
     return out
 
 
-def run_oracle(cfg, wl, streams=None):
+def run_oracle(cfg, wl, streams=None, arrivals=None):
     from oracle import des
-    return des.run(cfg, wl, streams=streams)
+    return des.run(cfg, wl, streams=streams, arrivals=arrivals)
 
 
 def oracle_firings(res, stream_ids=None):

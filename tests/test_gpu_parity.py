@@ -147,3 +147,23 @@ def test_bind_host_tma_matches_push():
     compare(cfg, g, o)
     assert summ["roots"] == g["stats"]["roots"] and summ["matches"] == len(o.matches)
     assert summ["max_latency"] == max(o.lat) and summ["miss_events"] == g["stats"]["miss_events"]
+
+
+@pytest.mark.parametrize("policy", [C.FIXED_WAIT, C.THRESHOLD_SLACK, C.MONOLITHIC])
+def test_poisson_arrivals_gain_model(policy):
+    """N2: Poisson arrivals given as per-root arrival times."""
+    from plgen import arrivals as A
+    cfg = _c1(policy, n_streams=4, n_roots=3000)
+    arr = A.poisson(9, A.stream_sizes(cfg.n_roots * cfg.n_streams, cfg.n_streams), cfg.interarrival)
+    g = run_gpu(cfg, None, arrivals=arr)
+    compare(cfg, g, run_oracle(cfg, None, arrivals=arr))
+
+
+@pytest.mark.parametrize("policy", [C.FIXED_WAIT, C.THRESHOLD_SLACK, C.MONOLITHIC])
+def test_poisson_arrivals_dna(policy):
+    from plgen import arrivals as A
+    cfg = _dna(policy, db_len=1 << 15, streams=3)
+    wl = workload_for(cfg)
+    arr = A.poisson(3, A.stream_sizes(wl.db_len - 6 + 1, cfg.n_streams), cfg.interarrival)
+    g = run_gpu(cfg, wl, arrivals=arr)
+    compare(cfg, g, run_oracle(cfg, wl, arrivals=arr))

@@ -256,3 +256,78 @@ def test_monolithic_hand_example():
     assert r.lat == [6, 2, 9, 11]
     assert [(i, s, n) for (i, s, n, _, _) in r.firings] == [(0, 1, 2), (1, 3, 1), (0, 6, 2), (1, 8, 2), (1, 11, 1)]
     assert r.T_end == 14
+
+
+# ------------------------------------------------------------- arrival-time inputs (N2)
+
+def test_explicit_fixed_rate_arrivals_match_default():
+    """arrivals[r] = r * tau0 passed as data reproduces the built-in fixed-rate run exactly."""
+    for policy in (C.FIXED_WAIT, C.THRESHOLD_SLACK, C.MONOLITHIC):
+        cfg = gm_cfg(3, (5, 9, 4), (7, 3, 11), 4, 2, 300, seed=4, policy=policy, theta=(3, 2, 4), D=120)
+        cfg = cfg.replace(block_size=16)
+        a = des.run(cfg)
+        b = des.run(cfg, arrivals=[r * 2 for r in range(300)])
+        assert (a.lat, a.trace, a.streams[0].firings) == (b.lat, b.trace, b.streams[0].firings)
+
+
+def _enum_with_arrivals(N, t, v, arr, fns, horizon):
+    """Every fire/wait schedule for arbitrary (sorted) arrival times; time-stepped, written
+    separately from oracle.des."""
+    X = len(arr)
+    out = {}
+
+    def rec(T, Q, busy, lat, arrived, log):
+        Q = [list(q) for q in Q]
+        busy = list(busy)
+        lat = list(lat)
+        for i in range(N):
+            if busy[i] and busy[i][0] == T:
+                for e in busy[i][1]:
+                    ch = fns[i](e)
+                    if i < N - 1 and ch:
+                        Q[i + 1] += ch
+                    else:
+                        lat[e[0]] = max(lat[e[0]], T - arr[e[0]])
+                busy[i] = None
+        while arrived < X and arr[arrived] == T:
+            Q[0].append((arrived, 0, None))
+            arrived += 1
+        if arrived == X and not any(Q) and not any(busy):
+            out[tuple(log)] = tuple(lat)
+            return
+        if T > horizon:
+            return
+        cand = [i for i in range(N) if busy[i] is None and Q[i]]
+        for k in range(len(cand) + 1):
+            for fire in itertools.combinations(cand, k):
+                Q2 = [list(q) for q in Q]
+                b2 = list(busy)
+                lg = list(log)
+                for i in fire:
+                    n = min(len(Q2[i]), v)
+                    b2[i] = (T + t[i], Q2[i][:n])
+                    Q2[i] = Q2[i][n:]
+                    lg.append((i, T, n))
+                rec(T + 1, Q2, b2, lat, arrived, lg)
+
+    rec(0, [[] for _ in range(N)], [None] * N, [-1] * X, 0, [])
+    return out
+
+
+@pytest.mark.parametrize("arr", [(0, 0, 3, 4), (0, 2, 2, 7), (0, 1, 5, 5)])
+def test_p6_enumeration_with_arrival_times(arr):
+    """P6 with irregular (Poisson-like, simultaneous) arrivals: the DES schedule of each
+    policy is one of the enumerated schedules, with identical latencies."""
+    N, t, v = 2, (2, 3), 2
+    fns = _toy_fns()
+    allsched = _enum_with_arrivals(N, t, v, list(arr), fns, horizon=arr[-1] + 16)
+    for policy, prm in ((C.FIXED_WAIT, (0, 0)), (C.FIXED_WAIT, (1, 2)), (C.THRESHOLD_SLACK, (2, 1)),
+                        (C.THRESHOLD_SLACK, (1, 2))):
+        cfg = C.Config(name="p6a", stages=[C.Stage(C.KEEP_EVERY, 1), C.Stage(C.KEEP_EVERY, 1)],
+                       service_time=t, vector_width=v, deadline=12, interarrival=2, b=(1, 1),
+                       wait_time=prm if policy == C.FIXED_WAIT else None,
+                       wait_threshold=prm if policy == C.THRESHOLD_SLACK else None, policy=policy, n_roots=4)
+        r = des.simulate_stream(cfg, fns, 0, 4, arrivals=list(arr))
+        log = tuple((i, s, n) for (i, s, n, _, _) in r.firings)
+        assert log in allsched, (policy, prm, log)
+        assert allsched[log] == tuple(r.lat)
