@@ -41,7 +41,6 @@ __device__ __forceinline__ T vld(const T* p) { return *(const volatile T*)p; }
 template <class T>
 __device__ __forceinline__ void vst(T* p, T v) { *(volatile T*)p = v; }
 
-__device__ __forceinline__ int64_t ceil_div64(int64_t a, int64_t b) { return a <= 0 ? 0 : (a + b - 1) / b; }
 
 // ------------------------------------------------------------- counter-based RNG
 // SplitMix64 finaliser; h = mix(seed ^ stage*GAMMA ^ root*M1 ^ lineage)  (DESIGN.md R-RNG)
@@ -292,6 +291,34 @@ struct LaneOut {
   uint32_t q_start, len;
 };
 
+// S2 / S3 for one entry.
+__device__ __forceinline__ LaneOut stage_count_ext(const Node& nd, const Dna& dna, uint2 e) {
+  LaneOut o;
+  o.c = 0; o.a = 0; o.score = 0; o.q_start = 0; o.len = 0;
+  const uint32_t q = e.y & 0xffffu;
+  if (nd.kind == PL_UNGAPPED_WINDOW) {
+    const int64_t W = nd.ip1;
+    int d;
+    const int64_t ll = dna.left_limit(e.x, q), rl = dna.right_limit(e.x, q);
+    const int bl = dna.extend(e.x, q, -1, ll < W ? ll : W, 0, &d);
+    const int br = dna.extend(e.x, q, +1, rl < W ? rl : W, 0, &d);
+    o.c = (dna.k + bl + br >= nd.ip2) ? 1u : 0u;
+  } else {
+    int dl, dr;
+    const int bl = dna.extend(e.x, q, -1, dna.left_limit(e.x, q), nd.ip1, &dl);
+    const int br = dna.extend(e.x, q, +1, dna.right_limit(e.x, q), nd.ip1, &dr);
+    const int score = dna.k + bl + br;
+    if (score >= nd.ip2) {
+      o.c = 1;
+      o.score = score;
+      o.a = e.x - dl;
+      o.q_start = q - dl;
+      o.len = dna.k + dl + dr;
+    }
+  }
+  return o;
+}
+
 __device__ __forceinline__ LaneOut stage_count(const Node& nd, const Dna& dna, const DevParams& p, uint2 e) {
   LaneOut o;
   o.c = 0; o.a = 0; o.score = 0; o.q_start = 0; o.len = 0;
@@ -318,59 +345,8 @@ __device__ __forceinline__ LaneOut stage_count(const Node& nd, const Dna& dna, c
       o.c = cnt < nd.max_out ? cnt : nd.max_out;
       break;
     }
-    case PL_UNGAPPED_WINDOW: {
-      const uint32_t q = e.y & 0xffffu;
-      const int64_t W = nd.ip1;
-      int d;
-      const int64_t ll = dna.left_limit(e.x, q), rl = dna.right_limit(e.x, q);
-      const int bl = dna.extend(e.x, q, -1, ll < W ? ll : W, 0, &d);
-      const int br = dna.extend(e.x, q, +1, rl < W ? rl : W, 0, &d);
-      o.c = (dna.k + bl + br >= nd.ip2) ? 1u : 0u;
-      break;
-    }
-    case PL_UNGAPPED_XDROP: {
-      const uint32_t q = e.y & 0xffffu;
-      int dl, dr;
-      const int bl = dna.extend(e.x, q, -1, dna.left_limit(e.x, q), nd.ip1, &dl);
-      const int br = dna.extend(e.x, q, +1, dna.right_limit(e.x, q), nd.ip1, &dr);
-      const int score = dna.k + bl + br;
-      if (score >= nd.ip2) {
-        o.c = 1;
-        o.score = score;
-        o.a = e.x - dl;
-        o.q_start = q - dl;
-        o.len = dna.k + dl + dr;
-      }
-      break;
-    }
-  }
-  return o;
-}
-
-// S2 / S3 for one entry.
-__device__ __forceinline__ LaneOut stage_count_ext(const Node& nd, const Dna& dna, uint2 e) {
-  LaneOut o;
-  o.c = 0; o.a = 0; o.score = 0; o.q_start = 0; o.len = 0;
-  const uint32_t q = e.y & 0xffffu;
-  if (nd.kind == PL_UNGAPPED_WINDOW) {
-    const int64_t W = nd.ip1;
-    int d;
-    const int64_t ll = dna.left_limit(e.x, q), rl = dna.right_limit(e.x, q);
-    const int bl = dna.extend(e.x, q, -1, ll < W ? ll : W, 0, &d);
-    const int br = dna.extend(e.x, q, +1, rl < W ? rl : W, 0, &d);
-    o.c = (dna.k + bl + br >= nd.ip2) ? 1u : 0u;
-  } else {
-    int dl, dr;
-    const int bl = dna.extend(e.x, q, -1, dna.left_limit(e.x, q), nd.ip1, &dl);
-    const int br = dna.extend(e.x, q, +1, dna.right_limit(e.x, q), nd.ip1, &dr);
-    const int score = dna.k + bl + br;
-    if (score >= nd.ip2) {
-      o.c = 1;
-      o.score = score;
-      o.a = e.x - dl;
-      o.q_start = q - dl;
-      o.len = dna.k + dl + dr;
-    }
+    case PL_UNGAPPED_WINDOW:
+    case PL_UNGAPPED_XDROP: o = stage_count_ext(nd, dna, e); break;
   }
   return o;
 }
@@ -1201,7 +1177,7 @@ __device__ void run_monolithic(Ctx& c) {
   uint64_t firings[PL_MAX_STAGES], consumed[PL_MAX_STAGES], produced[PL_MAX_STAGES];
   int64_t active[PL_MAX_STAGES];
   for (int i = 0; i < PL_MAX_STAGES; ++i) { firings[i] = consumed[i] = produced[i] = 0; active[i] = 0; }
-  int64_t proc_free = 0, t_end = 0, busy_ns = 0, lateness = 0;
+  int64_t proc_free = 0, t_end = 0, busy_ns = 0;
   const int64_t M = p.M;
   for (int64_t b0 = 0; b0 < c.X; b0 += M) {
     const int64_t b1 = (b0 + M < c.X) ? b0 + M : c.X;
@@ -1306,7 +1282,6 @@ __device__ void run_monolithic(Ctx& c) {
     if (phys && tid == 0) {
       const uint64_t en = gtimer();
       busy_ns += (int64_t)(en - sh_start_ns);
-      (void)lateness;
     }
   }
   if (tid == 0) {

@@ -11,7 +11,7 @@
 // (block value sqrt(sum c / (lambda sum a))), which is then clipped to the
 // order-compatible bounds [max_{j>=i} G_j t_j, v tau0].  lambda is found by
 // bisection on the (monotone) deadline slack.  The integer answer (reading A17)
-// is the best feasible point of a chain-aware neighbourhood search, ties broken
+// is the best feasible point of a chain-aware branch-and-bound search, ties broken
 // towards the lexicographically smallest w.
 // Fig. 2: exhaustive search over M while b M tau0 + S Tbar(M) <= D.
 #include <cmath>
@@ -117,21 +117,30 @@ int solve_fig1(int N, const int64_t* t, const double* g, const uint32_t* b, uint
   }
   for (int i = 0; i < N; ++i) Pc[i] = Q[i] / G[i];
   *Tc = objective(N, t, Pc);
-  // integer search (reading A17): depth-first over stages; stage i tries the
-  // floor/ceil neighbourhood of the continuous P_i and the two largest integers
-  // allowed by the chain bound g_{i-1} P_i <= P_{i-1} of the chosen predecessor.
+  // integer search (reading A17): branch and bound, depth-first over stages.  Stage i tries
+  // floor(P_i) - R .. floor(P_i) + R + 1 around the continuous optimum and the R+1 largest
+  // integers allowed by the chain bound g_{i-1} P_i <= P_{i-1} of the chosen predecessor;
+  // branches that cannot meet the deadline or beat the incumbent objective are cut.
+  const int RW = 8;
   int64_t bestP[PL_MAX_STAGES], P[PL_MAX_STAGES];
   bool found = false;
   double best = 0;
-  double Pd[PL_MAX_STAGES];
   int64_t bsum_suffix_min[PL_MAX_STAGES + 1];
+  double obj_suffix_lb[PL_MAX_STAGES + 1];
   bsum_suffix_min[N] = 0;
+  obj_suffix_lb[N] = 0;
   for (int i = N - 1; i >= 0; --i) bsum_suffix_min[i] = bsum_suffix_min[i + 1] + (int64_t)b[i] * t[i];
-  struct Frame { int64_t cand[8]; int nc, k; int64_t bsum; };
+  for (int i = N - 1; i >= 0; --i) {
+    // P_i <= (D - sum_{j != i} b_j t_j) / b_i bounds t_i / P_i from below
+    const double ub = (double)(D - (bsum_suffix_min[0] - (int64_t)b[i] * t[i])) / (double)b[i];
+    obj_suffix_lb[i] = obj_suffix_lb[i + 1] + (ub > 0 ? (double)t[i] / ub : 0.0);
+  }
+  const int MAXC = 4 * RW + 4;
+  struct Frame { int64_t cand[4 * 8 + 4]; int nc, k; int64_t bsum; double obj; };
   Frame fr[PL_MAX_STAGES];
-  auto fill = [&](int i, int64_t prevP, int64_t bsum) {
+  auto fill = [&](int i, int64_t prevP, int64_t bsum, double obj) {
     Frame& f = fr[i];
-    f.nc = 0; f.k = 0; f.bsum = bsum;
+    f.nc = 0; f.k = 0; f.bsum = bsum; f.obj = obj;
     int64_t ub;
     if (i == 0) {
       ub = (int64_t)std::floor((double)v * (double)tau);
@@ -141,9 +150,12 @@ int solve_fig1(int N, const int64_t* t, const double* g, const uint32_t* b, uint
       while ((double)(ub + 1) * g[i - 1] <= (double)prevP) ++ub;
     }
     const int64_t fl = (int64_t)std::floor(Pc[i]);
-    const int64_t c8[6] = {ub, ub - 1, fl + 1, fl, fl - 1, fl + 2};
-    for (int j = 0; j < 6; ++j) {
-      const int64_t x = c8[j];
+    int64_t c[4 * 8 + 4];
+    int nc = 0;
+    for (int d = 0; d <= RW; ++d) c[nc++] = ub - d;
+    for (int d = -RW; d <= RW + 1; ++d) c[nc++] = fl + d;
+    for (int j = 0; j < nc && f.nc < MAXC; ++j) {
+      const int64_t x = c[j];
       if (x < t[i] || x > ub) continue;
       if (bsum + (int64_t)b[i] * x + bsum_suffix_min[i + 1] > D) continue;
       bool dup = false;
@@ -152,18 +164,21 @@ int solve_fig1(int N, const int64_t* t, const double* g, const uint32_t* b, uint
     }
   };
   int depth = 0;
-  fill(0, 0, 0);
+  fill(0, 0, 0, 0.0);
   while (depth >= 0) {
     Frame& f = fr[depth];
     if (f.k >= f.nc) { --depth; continue; }
     P[depth] = f.cand[f.k++];
     const int64_t bs = f.bsum + (int64_t)b[depth] * P[depth];
+    const double ob = f.obj + (double)t[depth] / (double)P[depth];
+    if (found && (ob + obj_suffix_lb[depth + 1]) / N > best * (1 + 1e-12)) continue;
     if (depth + 1 < N) {
-      fill(depth + 1, P[depth], bs);
+      fill(depth + 1, P[depth], bs, ob);
       ++depth;
       continue;
     }
     if (!feasible(N, t, g, b, v, tau, D, P)) continue;
+    double Pd[PL_MAX_STAGES];
     for (int i = 0; i < N; ++i) Pd[i] = (double)P[i];
     const double T = objective(N, t, Pd);
     bool better = !found || T < best;

@@ -107,3 +107,34 @@ def test_solver_fig2_matches_oracle(tau, D):
     M, T = solve_monolithic(C.gain_model_blast(interarrival=tau, deadline=D))
     Mo, To = SV.fig2_exhaustive(C.TABLE1_T, C.TABLE1_G, 128, tau, D)
     assert (M, T) == (Mo, To)
+
+
+def _random_fig1_problem(rnd):
+    N = rnd.randint(1, 3)
+    t = tuple(rnd.randint(1, 9) for _ in range(N))
+    g = tuple(round(rnd.uniform(0.2, 2.5), 3) for _ in range(N - 1))
+    b = tuple(rnd.randint(1, 3) for _ in range(N))
+    v = rnd.choice([2, 4, 8])
+    tau = rnd.randint(1, 6)
+    D = rnd.randint(sum(x * y for x, y in zip(t, b)), 4 * sum(x * y for x, y in zip(t, b)) + 40)
+    return t, g, b, v, tau, D
+
+
+@pytest.mark.parametrize("seed", range(40))
+def test_solver_fig1_random_vs_bruteforce(seed):
+    """Property: on random small problems the C++ Fig. 1 solver returns exactly the integer
+    optimum of the oracle's brute-force enumeration (or both report infeasible)."""
+    import random
+    from paper_conf_icppw_planob21_b200 import PlError, solve_enforced_waits
+    t, g, b, v, tau, D = _random_fig1_problem(random.Random(seed))
+    cfg = C.Config(name="r", stages=[C.Stage(C.BERNOULLI, 0.5, 1)] * len(t), service_time=t, vector_width=32,
+                   deadline=D, interarrival=tau, b=b, gain=g)
+    cfg.vector_width = v
+    Pi, Ti = SV.fig1_bruteforce_int(t, g, b, v, tau, D)
+    try:
+        w, th, T, Tc = solve_enforced_waits(cfg)
+    except PlError:
+        assert Pi is None
+        return
+    assert Pi is not None
+    assert abs(T - Ti) < 1e-12, (t, g, b, v, tau, D, [w[i] + t[i] for i in range(len(t))], Pi)
