@@ -287,6 +287,11 @@ pl_status pl_solve_monolithic(const pl_config* cfg, uint32_t* M_out, double* T_o
 pl_status pl_stage_batch(pl_pipeline* pl, uint32_t stage, const void* in_dev, uint64_t n, uint64_t first_root,
                          void* out_dev, uint64_t cap, uint64_t* n_out, uint64_t* max_vec_cycles);
 
+/* Measurement utility (SURVEY §8(f) N3 co-runner experiment; not part of the method): launch
+ * n_ctas CTAs of 128 threads of a compute-bound FMA kernel (iters rounds, 8 chains/thread) on
+ * `stream`; `sink` is a device float[n_ctas] that is (almost) never written.  0 or PL_EDEVICE. */
+int pl_corunner_launch(void* stream, uint32_t n_ctas, uint64_t iters, float* sink);
+
 /* Library build identity (for logs): "plgpu <version> sm_100a".                  */
 const char* pl_version(void);
 

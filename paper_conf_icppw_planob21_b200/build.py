@@ -17,7 +17,7 @@ LIB = os.path.join(HERE, "libplgpu.so")
 NVCC = os.environ.get("NVCC", "nvcc")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 FLAGS = ["-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC,-O2", f"-I{ROOT}/include", f"-I{CSRC}"]
-SOURCES = ["executor.cu", "runtime.cu", "solver.cpp"]
+SOURCES = ["executor.cu", "runtime.cu", "solver.cpp", "corunner.cu"]
 
 
 def _stale() -> bool:
