@@ -326,6 +326,37 @@ def main():
         mono["common_rate"] = {"tau0_ns": tau_m, "monolithic": run_policy(2, tau_m, Mm[0]),
                                "enforced": run_policy(0, tau_m), "fig2_objective": Mm[1]}
 
+    # the north_star's threshold / deadline-slack rule (THRESHOLD_SLACK, theta_i from Fig. 1;
+    # the slack reserve R_i gets a guard of the largest budget for real-time lateness)
+    thr = None
+    try:
+        cfg_t = cfg.replace(slack_guard=int(max(budgets)))
+        tau_t, w_t, th_t, T_t, _ = realtime.find_rate(cfg_t, wl, db_ptr, stream=stream, policy=1)
+        plt = Pipeline(cfg_t.replace(interarrival=tau_t, wait_threshold=tuple(th_t), policy=1), wl, flags=0,
+                       stream=stream)
+        plt.bind_device(db_ptr, wl.db_len)
+        plt.launch()
+        plt.summary()
+        x0, x1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        tms, troots, tmiss = 0.0, 0, 0
+        for _ in range(a.steps):
+            flush.zero_()
+            x0.record(stream)
+            plt.launch()
+            x1.record(stream)
+            sm_t = plt.summary()
+            tms += x0.elapsed_time(x1)
+            troots += sm_t["roots"]
+            tmiss += sm_t["miss_events_ns"]
+        stt = plt.stats()
+        plt.close()
+        thr = {"tau0_ns": tau_t, "theta": list(th_t), "slack_guard_ns": int(max(budgets)),
+               "value": troots / (tms * 1e-3), "ms_per_step": tms / a.steps, "misses": tmiss,
+               "sustained_items_per_s": a.streams * 1e9 / tau_t, "active_fraction": stt["active_fraction"],
+               "max_latency_ns": stt["max_latency_ns"]}
+    except RuntimeError as ex:
+        thr = {"failed": str(ex)}
+
     # e2e through the C-ABI with host buffers: the DB stays in pinned host memory and every
     # CTA stages its window from it by TMA (pl_pipeline_bind_host); the step's result is the
     # device-reduced summary (one 56-byte D->H read).  Host wall clock, synchronised.
@@ -386,6 +417,7 @@ def main():
             "misses": misses_all, "schedule_misses": sched_misses_all, "overruns": overruns_all, "errors": errors,
             "sustained_items_per_s": world * a.streams * 1e9 / tau,
             "logical_items_per_s": logical_ips,
+            "threshold_slack": thr,
             "utilisation": {"enforced_model": st_last["active_fraction"], "enforced_fig1_T": T,
                             "enforced_hw_busy": st["hw_busy_fraction"], "monolithic": mono},
             "per_firing": {f"node{i}": {"firings": st["firings"][i],

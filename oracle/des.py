@@ -66,7 +66,8 @@ def gains_G(g):
 
 
 def reserve(t, i):
-    """R_i = t_i + 2 * sum_{j>i} t_j (THRESHOLD_SLACK slack reserve)."""
+    """R_i = t_i + 2 * sum_{j>i} t_j (THRESHOLD_SLACK slack reserve; the config's
+    slack_guard is added on top, DESIGN.md R-THRESH)."""
     return t[i] + 2 * sum(t[i + 1:])
 
 
@@ -129,7 +130,7 @@ def simulate_stream(cfg: C.Config, fns, lo: int, hi: int, wait_time=None, theta=
         next_start = [0] * N                     # phase 0 for every node (R-PHASE)
     else:
         th = list(theta if theta is not None else cfg.wait_threshold)
-        R = [reserve(t, i) for i in range(N)]
+        R = [reserve(t, i) + getattr(cfg, "slack_guard", 0) for i in range(N)]
         last_force = [None] * N
 
     Q = [deque() for _ in range(N)]              # entries (root, lin, q)

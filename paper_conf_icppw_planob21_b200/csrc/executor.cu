@@ -547,7 +547,13 @@ __device__ Decision decide(const Node& nd, Leader& L) {
     if (Tk < L.B) Tk = L.B;
     if (th_known || Tk < Wup) {
       const uint32_t cnt = count_le(nd, L, st, Tk);
-      if (Wup > Tk || cnt >= v) { d.T = Tk; d.n = cnt < v ? cnt : v; d.qlen = tail_known - L.head; return d; }
+      if (Wup > Tk || cnt >= v) {
+        d.T = Tk; d.n = cnt < v ? cnt : v; d.qlen = tail_known - L.head;
+        // committed: nothing leaves this node before Tk + t_i.  Publish it now -- a physical
+        // firing may be paced far into the future (slack) and downstream must not wait for it.
+        publish_W(nd, L, Tk + nd.t);
+        return d;
+      }
     }
     int64_t lb = Tk < Wup ? Tk : Wup;
     if (lb < L.B) lb = L.B;
@@ -751,6 +757,7 @@ __device__ void run_node(Ctx& c, const Dna dna, int i, int gtid) {
       T = d.T; n = d.n; head = (uint32_t)R.c0;
       if (d.qlen > max_queue) max_queue = d.qlen;
       if (leader) {
+        publish_W(nd, L, T + nd.t);      // committed: nothing leaves node 0 before T + t_0
         if (rec & PL_REC_FIRINGS) G.log_idx[par] = atomicAdd(&c.sh->log_count, 1u);
         G.out_loc[par] = nd.sink ? LOC_SMEM : reserve_out(nd, L, n * nd.umax, &stalls);
         G.out_base[par] = L.out_tail;

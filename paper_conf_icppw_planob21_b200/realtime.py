@@ -66,8 +66,9 @@ def min_feasible_tau(cfg, lo=1, hi=1 << 20):
     return lo
 
 
-def find_rate(cfg, wl, db_dev, tries=12, grow=1.15, stream=None, log=None, over=None):
-    """Smallest tau0 (ns) at which a physical FIXED_WAIT run has zero deadline misses and
+def find_rate(cfg, wl, db_dev, tries=12, grow=1.15, stream=None, log=None, over=None, policy=0):
+    """Smallest tau0 (ns) at which a physical run (FIXED_WAIT, or THRESHOLD_SLACK with the
+    Fig. 1-derived thresholds when policy=1) has zero deadline misses and
     no queue overflow (budget overruns are counted and reported, not fatal: they delay
     firings, and any delay that matters shows up as a miss).  Starts at the smallest tau0
     for which Fig. 1 is feasible, grows by `grow` until a run is clean, then bisects between
@@ -79,7 +80,8 @@ def find_rate(cfg, wl, db_dev, tries=12, grow=1.15, stream=None, log=None, over=
         if sol is None:
             return None
         w, th, T = sol
-        c = cfg.replace(interarrival=int(tau), wait_time=tuple(w), clock=PHYS)
+        c = cfg.replace(interarrival=int(tau), wait_time=tuple(w), wait_threshold=tuple(th), clock=PHYS,
+                        policy=policy)
         try:
             st = _run(c, db_dev, wl.db_len, wl, flags=1, stream=stream, over=over)
             ok = st["misses"] == 0 and st["miss_events_ns"] == 0 and st["errors"] == 0

@@ -58,6 +58,7 @@ class Config:
     n_roots: int = 0             # gain model: roots per stream; DNA: derived from db_len
     seed: int = 0
     ns_per_unit: float = 1.0
+    slack_guard: int = 0         # THRESHOLD_SLACK: extra reserve added to R_i (physical lateness guard)
     # DNA workload recipe (plgen.dna.make_dna kwargs); None for gain-model pipelines
     dna: Optional[dict] = None
 

@@ -104,6 +104,13 @@ def test_vector_widths_dna(policy, v):
     compare(cfg, run_gpu(cfg, wl), run_oracle(cfg, wl))
 
 
+def test_threshold_slack_guard():
+    """THRESHOLD_SLACK with a slack guard added to every R_i (both sides)."""
+    cfg = _dna(C.THRESHOLD_SLACK, db_len=1 << 15, streams=3).replace(slack_guard=7000)
+    wl = workload_for(cfg)
+    compare(cfg, run_gpu(cfg, wl), run_oracle(cfg, wl))
+
+
 @pytest.mark.parametrize("policy", [C.FIXED_WAIT, C.THRESHOLD_SLACK])
 def test_eight_node_gain_pipeline(policy):
     """N = 8 random-gain nodes (the ABI maximum), v = 128 -> 1024 threads."""
