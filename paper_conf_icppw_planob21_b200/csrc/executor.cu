@@ -40,6 +40,10 @@ template <class T>
 __device__ __forceinline__ T vld(const T* p) { return *(const volatile T*)p; }
 template <class T>
 __device__ __forceinline__ void vst(T* p, T v) { *(volatile T*)p = v; }
+// CTA-scope acquire-release fence between the data and the flag of the SPSC queues (pure
+// message passing, so no sequentially consistent fence is needed): MEMBAR.ALL.CTA in SASS,
+// where __threadfence_block() emits the costlier MEMBAR.SC.CTA.
+__device__ __forceinline__ void fence_cta() { asm volatile("fence.acq_rel.cta;" ::: "memory"); }
 
 
 // ------------------------------------------------------------- counter-based RNG
@@ -157,10 +161,18 @@ struct GroupCtl {           // broadcast from a node's leader to its lanes, doub
   uint32_t in_spill_end[2]; // input edge: end seq of its last spilled segment
   uint32_t out_base[2], out_loc[2];
   alignas(16) uint32_t wtot[2][8];
+  alignas(16) uint32_t rmin[8];   // per warp: smallest terminal root of the current firing
+};
+struct NodeAcc {            // leader-only per-node accumulators: in smem, updated by fire-and-forget
+  unsigned long long firings, consumed, produced, spilled, overruns, stalls, active, busy_ns;  // atomics,
+  unsigned long long ph[6];  // so that they take no registers in the node loop
+  long long t_end;
+  uint32_t max_queue, lateness, max_fire, lmax, lmax_ns, nmiss, nmiss_ns, pad;
 };
 struct Shared {
   EdgeCtl e[PL_MAX_STAGES];
   GroupCtl g[PL_MAX_STAGES];
+  NodeAcc acc[PL_MAX_STAGES];
   uint32_t max_lat;         // per-stream aggregates: 32-bit so the smem atomics are native
   uint32_t max_lat_ns;      // (64-bit smem atomicMax compiles to a CAS loop)
   uint32_t miss_events;
@@ -205,7 +217,7 @@ struct Node {
   int64_t t, P, R, D, tau, X, H;
   uint32_t theta;
   uint64_t lo;
-  double nspu;
+  double nspu, D_ns;            // D in ns (physical deadline test)
   uint32_t segmask, capg;
   EdgeCtl* Ein;                 // input edge (i > 0)
   const uint2* in_ent;
@@ -222,6 +234,7 @@ struct Node {
   MDiv dtau, dP;
   int64_t Pq, Pr;               // floor(P / tau0), P mod tau0
   const int64_t* arr;           // per-root arrival times (NULL: fixed rate, L63)
+  uint32_t* troot;              // smem [v]: the current firing's terminal root per lane (or NO_ROOT)
   __device__ __forceinline__ int64_t arrival(uint32_t root) const {
     return arr ? __ldg(arr + root) : (int64_t)(root - lo) * tau;
   }
@@ -242,6 +255,7 @@ __device__ __forceinline__ Node make_node(const Ctx& c, int i) {
   n.theta = p.theta[i];
   n.lo = c.lo;
   n.nspu = p.ns_per_unit;
+  n.D_ns = (double)p.D * p.ns_per_unit;
   n.segmask = p.segcap - 1;
   n.capg = p.cap_g;
   n.Ein = &c.sh->e[i];
@@ -265,6 +279,7 @@ __device__ __forceinline__ Node make_node(const Ctx& c, int i) {
   n.Pq = fdiv(p.P[i], n.dtau);
   n.Pr = p.P[i] - n.Pq * p.tau;
   n.arr = p.arr;
+  n.troot = (uint32_t*)(c.dsm + Lo.off_troot) + (uint32_t)i * (uint32_t)p.v;
   return n;
 }
 
@@ -383,7 +398,7 @@ __device__ __forceinline__ void publish_W(const Node& nd, Leader& L, int64_t w) 
   if (nd.sink) return;
   if (w > L.W_pub) {
     L.W_pub = w;
-    __threadfence_block();
+    fence_cta();
     vst(&nd.Eout->W, w);
   }
 }
@@ -499,7 +514,7 @@ __device__ Decision decide(const Node& nd, Leader& L) {
   for (;;) {
     // node i >= 1: read the upstream watermark first, then the published segments
     const int64_t Wup = vld(&nd.Ein->W);
-    __threadfence_block();
+    fence_cta();
     const uint32_t st = vld(&nd.Ein->seg_tail);
     const uint32_t tail_known = (st != L.segh) ? nd.in_seg[(st - 1) & nd.segmask].end : L.head;
     const bool any = tail_known != L.head;
@@ -530,7 +545,7 @@ __device__ Decision decide(const Node& nd, Leader& L) {
       continue;
     }
     const Seg& hs = nd.in_seg[L.segh & nd.segmask];
-    __threadfence_block();
+    fence_cta();
     const uint2 he = load_entry(nd, L.head, L.segh, st, vld(&nd.Ein->spill_end));
     int64_t Tf = nd.arrival(he.x) + nd.D - nd.R;
     if (Tf < hs.ready) Tf = hs.ready;
@@ -566,7 +581,7 @@ __device__ Decision decide(const Node& nd, Leader& L) {
 // stage runs so that no extra barrier is needed).  Returns the location.  A full queue
 // back-pressures the producer in both clock modes (deadlock-free):
 // in physical mode the wait shows up as lateness and, if it matters, as deadline misses.
-__device__ uint32_t reserve_out(const Node& nd, Leader& L, uint32_t worst, uint64_t* stalls) {
+__device__ uint32_t reserve_out(const Node& nd, Leader& L, uint32_t worst, unsigned long long* stalls) {
   int spins = 0;
   for (;;) {
     const uint32_t h = vld(&nd.Eout->head), sh = vld(&nd.Eout->seg_head);
@@ -574,7 +589,7 @@ __device__ uint32_t reserve_out(const Node& nd, Leader& L, uint32_t worst, uint6
     const uint32_t need = L.out_tail + worst - h;
     if (seg_ok && need <= nd.out_cap) return LOC_SMEM;
     if (seg_ok && need <= nd.capg) return LOC_SPILL;
-    if (spins == 0) ++*stalls;
+    if (spins == 0) atomicAdd(stalls, 1ull);
     backoff(spins);
   }
 }
@@ -708,6 +723,16 @@ __device__ __forceinline__ uint2 stage_output_k(const Node& nd, const Dna& dna, 
   else return e;
 }
 
+// Physical-clock latency of a terminal item of the previous firing (its end time is that
+// firing's publish time), per root: parity runs (PL_REC_LATENCY) only.  The per-stream
+// maximum and the deadline misses are evaluated by the leader (run_node, "bookkeeping").
+__device__ __forceinline__ void record_lat_ns(const Node& nd, const Ctx& c, uint64_t T0, uint64_t end_ns,
+                                              uint32_t& pend_root) {
+  const uint64_t a_ns = T0 + (uint64_t)((double)nd.arrival(pend_root) * nd.nspu);
+  atomicMax((long long*)&c.p->lat_ns[pend_root], (long long)((int64_t)end_ns - (int64_t)a_ns));
+  pend_root = NO_ROOT;
+}
+
 // ------------------------------------------------------------------- node loop
 // One warp group of v threads per node, one item per lane.  Measured faster on B200 than
 // one warp with v/32 items per lane: the group's warps run the per-item latency chains in
@@ -718,6 +743,8 @@ __device__ __forceinline__ uint2 stage_output_k(const Node& nd, const Dna& dna, 
 // segment and its watermark.  Node 0 skips B1: its arrivals are fully known, so every lane
 // evaluates the decision itself and the leader's reservation reaches the lanes through
 // B2.  Broadcast slots are double-buffered by firing parity.
+// REC: per-item records compiled in (parity / tracing runs); the bench kernel has none.
+template <bool REC>
 __device__ void run_node(Ctx& c, const Dna dna, int i, int gtid) {
   const DevParams& p = *c.p;
   const Node nd = make_node(c, i);
@@ -728,8 +755,9 @@ __device__ void run_node(Ctx& c, const Dna dna, int i, int gtid) {
   const int bidB = (i < 7) ? 9 + i : bidA;       // barrier ids 9..15 for the output barrier
   GroupCtl& G = c.sh->g[i];
   const uint32_t stream = blockIdx.x;
-  const uint32_t rec = p.flags;
+  const uint32_t rec = REC ? p.flags : (p.flags & PL_FIXED_SERVICE);
   const uint64_t T0 = c.sh->T0;
+  NodeAcc& A = c.sh->acc[i];
   const uint32_t lt_mask = (1u << (gtid & 31)) - 1u;
 
   Leader L;
@@ -737,15 +765,18 @@ __device__ void run_node(Ctx& c, const Dna dna, int i, int gtid) {
   L.W_pub = -1; L.empties = 0;
   Rep R;
   R.m = 0; R.B = 0; R.c0 = 0; R.empties = 0; R.qT = 0; R.rT = 0; R.qvalid = false;
-  uint64_t firings = 0, consumed = 0, produced = 0, spilled = 0, overruns = 0, stalls = 0;
-  int64_t active = 0, busy_ns = 0, lateness = 0, t_end = 0, max_fire = 0;
-  uint32_t max_queue = 0;
+  auto clamp32 = [](int64_t x) { return (uint32_t)(x > 0 ? (x < 0xffffffffll ? x : 0xffffffffll) : 0); };
   uint64_t start_ns = 0;
-  uint32_t pend_root = NO_ROOT;          // lane: physical terminal event awaiting its end time
-  uint64_t ph[6] = {0, 0, 0, 0, 0, 0};   // leader: per-phase clock64 cycles
+  uint32_t pend_root = NO_ROOT;          // lane: physical terminal event awaiting its end time (REC)
   long long tc = 0;
   int par = 0;
-  if (leader) { G.end_ns[0] = 0; G.end_ns[1] = 0; }
+  if (leader) {
+    G.end_ns[0] = 0; G.end_ns[1] = 0;
+    A.firings = A.consumed = A.produced = A.spilled = A.overruns = A.stalls = A.active = A.busy_ns = 0;
+    for (int k = 0; k < 6; ++k) A.ph[k] = 0;
+    A.t_end = 0;
+    A.max_queue = A.lateness = A.max_fire = A.lmax = A.lmax_ns = A.nmiss = A.nmiss_ns = 0;
+  }
 
   for (;;) {
     int64_t T;
@@ -755,60 +786,62 @@ __device__ void run_node(Ctx& c, const Dna dna, int i, int gtid) {
       const Decision d = decide0(nd, R);
       if (d.done) break;
       T = d.T; n = d.n; head = (uint32_t)R.c0;
-      if (d.qlen > max_queue) max_queue = d.qlen;
       if (leader) {
+        atomicMax(&A.max_queue, d.qlen);
         publish_W(nd, L, T + nd.t);      // committed: nothing leaves node 0 before T + t_0
         if (rec & PL_REC_FIRINGS) G.log_idx[par] = atomicAdd(&c.sh->log_count, 1u);
-        G.out_loc[par] = nd.sink ? LOC_SMEM : reserve_out(nd, L, n * nd.umax, &stalls);
+        G.out_loc[par] = nd.sink ? LOC_SMEM : reserve_out(nd, L, n * nd.umax, &A.stalls);
         G.out_base[par] = L.out_tail;
         tc = clock64();
-        ph[0] += (uint64_t)(tc - c0);
+        atomicAdd(&A.ph[0], (unsigned long long)(tc - c0));
       }
-      if (nd.phys && (gtid & 31) == 0) {   // every warp paces itself against %globaltimer
+      if (nd.phys && (p.variant & 1u)) {  // the leader paces, one barrier releases the lanes
+        if (leader) {
+          int64_t late;
+          pace(T0, nd.nspu, T, &start_ns, &late);
+          atomicMax(&A.lateness, clamp32(late));
+        }
+        bar_sync(bidA, v);
+        if (leader) tc = clock64();
+      } else if (nd.phys && (gtid & 31) == 0) {   // every warp paces itself against %globaltimer
         uint64_t s_ns; int64_t late;
         pace(T0, nd.nspu, T, &s_ns, &late);
-        if (leader) { start_ns = s_ns; if (late > lateness) lateness = late; tc = clock64(); }
+        if (leader) { start_ns = s_ns; atomicMax(&A.lateness, clamp32(late)); tc = clock64(); }
       }
       __syncwarp();
     } else {
       if (leader) {
         const long long c0 = clock64();
         const Decision d = decide(nd, L);
-        if (d.qlen > max_queue) max_queue = d.qlen;
+        atomicMax(&A.max_queue, d.qlen);
         G.done[par] = d.done ? 1u : 0u;
         G.T[par] = d.T;
         G.n[par] = d.n;
         G.head[par] = L.head;
         G.segh[par] = L.segh;
         G.st[par] = vld(&nd.Ein->seg_tail);
-        __threadfence_block();
+        fence_cta();
         G.in_spill_end[par] = vld(&nd.Ein->spill_end);
         if (!d.done) {
           if (rec & PL_REC_FIRINGS) G.log_idx[par] = atomicAdd(&c.sh->log_count, 1u);
-          G.out_loc[par] = nd.sink ? LOC_SMEM : reserve_out(nd, L, d.n * nd.umax, &stalls);
+          G.out_loc[par] = nd.sink ? LOC_SMEM : reserve_out(nd, L, d.n * nd.umax, &A.stalls);
           G.out_base[par] = L.out_tail;
         } else {
           publish_W(nd, L, PL_INF64);
         }
         tc = clock64();
-        ph[0] += (uint64_t)(tc - c0);
+        atomicAdd(&A.ph[0], (unsigned long long)(tc - c0));
         if (!d.done && nd.phys) {
           int64_t late;
           pace(T0, nd.nspu, d.T, &start_ns, &late);
-          if (late > lateness) lateness = late;
+          atomicMax(&A.lateness, clamp32(late));
           tc = clock64();
         }
       }
       bar_sync(bidA, v);                                               // B1: decision
-      if (leader) { const long long t2 = clock64(); ph[1] += (uint64_t)(t2 - tc); tc = t2; }
-      if (pend_root != NO_ROOT) {        // deferred physical latency of the previous firing
-        const uint64_t a_ns = T0 + (uint64_t)((double)nd.arrival(pend_root) * nd.nspu);
-        const int64_t l = (int64_t)G.end_ns[par ^ 1] - (int64_t)a_ns;
-        if (rec & PL_REC_LATENCY) atomicMax((long long*)&p.lat_ns[pend_root], (long long)l);
-        atomicMax(&c.sh->max_lat_ns, (uint32_t)(l > 0 ? (l < 0xffffffffll ? l : 0xffffffffll) : 0));
-        if ((double)l > (double)nd.D * nd.nspu) atomicAdd(&c.sh->miss_events_ns, 1u);
-        pend_root = NO_ROOT;
-      }
+      if (leader) { const long long t2 = clock64(); atomicAdd(&A.ph[1], (unsigned long long)(t2 - tc)); tc = t2; }
+      if (REC && pend_root != NO_ROOT)   // deferred physical latency of the previous firing
+        record_lat_ns(nd, c, T0, G.end_ns[par ^ 1], pend_root);
       if (G.done[par]) break;
       T = G.T[par]; n = G.n[par]; head = G.head[par];
     }
@@ -824,14 +857,17 @@ __device__ void run_node(Ctx& c, const Dna dna, int i, int gtid) {
       if (n0) e[0] = make_uint2((uint32_t)(nd.lo + head + ld), 0u);
       else e[0] = load_entry(nd, head + ld, G.segh[par], G.st[par], G.in_spill_end[par]);
     }
-    switch (nd.kind) {   // warp-uniform dispatch to the stage body
-      case PL_SEED_LOOKUP: stage_batch<1, PL_SEED_LOOKUP>(nd, dna, p, e, acts, o); break;
-      case PL_HIT_ENUM: stage_batch<1, PL_HIT_ENUM>(nd, dna, p, e, acts, o); break;
-      case PL_BERNOULLI: stage_batch<1, PL_BERNOULLI>(nd, dna, p, e, acts, o); break;
-      case PL_FIXED_GAIN: stage_batch<1, PL_FIXED_GAIN>(nd, dna, p, e, acts, o); break;
-      case PL_KEEP_EVERY: stage_batch<1, PL_KEEP_EVERY>(nd, dna, p, e, acts, o); break;
-      case PL_POISSON_CAPPED: stage_batch<1, PL_POISSON_CAPPED>(nd, dna, p, e, acts, o); break;
-      default: stage_batch<1, PL_UNGAPPED_WINDOW>(nd, dna, p, e, acts, o); break;   // S2 / S3
+    {   // warp-uniform dispatch to the stage body: direct compare-and-branch chain (a switch
+        // compiles to an indirect BRX, measured ~200 cycles per dispatch)
+      const uint32_t kd = nd.kind;
+      if (kd == PL_SEED_LOOKUP) stage_batch<1, PL_SEED_LOOKUP>(nd, dna, p, e, acts, o);
+      else if (kd == PL_HIT_ENUM) stage_batch<1, PL_HIT_ENUM>(nd, dna, p, e, acts, o);
+      else if (kd == PL_UNGAPPED_WINDOW || kd == PL_UNGAPPED_XDROP)
+        stage_batch<1, PL_UNGAPPED_WINDOW>(nd, dna, p, e, acts, o);   // S2 / S3
+      else if (kd == PL_BERNOULLI) stage_batch<1, PL_BERNOULLI>(nd, dna, p, e, acts, o);
+      else if (kd == PL_FIXED_GAIN) stage_batch<1, PL_FIXED_GAIN>(nd, dna, p, e, acts, o);
+      else if (kd == PL_KEEP_EVERY) stage_batch<1, PL_KEEP_EVERY>(nd, dna, p, e, acts, o);
+      else stage_batch<1, PL_POISSON_CAPPED>(nd, dna, p, e, acts, o);
     }
     uint32_t total;
     uint32_t off;
@@ -844,21 +880,15 @@ __device__ void run_node(Ctx& c, const Dna dna, int i, int gtid) {
     } else {
       off = group_scan(G.wtot[par], o[0].c, &total, gtid, v, bidA, nd.umax <= 1);                 // B2
     }
-    if (leader) { const long long t2 = clock64(); ph[2] += (uint64_t)(t2 - tc); tc = t2; }
-    if (n0 && pend_root != NO_ROOT) {    // node 0: the previous publish time arrives through B2
-      const uint64_t a_ns = T0 + (uint64_t)((double)nd.arrival(pend_root) * nd.nspu);
-      const int64_t l = (int64_t)G.end_ns[par ^ 1] - (int64_t)a_ns;
-      if (rec & PL_REC_LATENCY) atomicMax((long long*)&p.lat_ns[pend_root], (long long)l);
-      atomicMax(&c.sh->max_lat_ns, (uint32_t)(l > 0 ? (l < 0xffffffffll ? l : 0xffffffffll) : 0));
-      if ((double)l > (double)nd.D * nd.nspu) atomicAdd(&c.sh->miss_events_ns, 1u);
-      pend_root = NO_ROOT;
-    }
+    if (leader) { const long long t2 = clock64(); atomicAdd(&A.ph[2], (unsigned long long)(t2 - tc)); tc = t2; }
+    if (REC && n0 && pend_root != NO_ROOT)   // node 0: the previous publish time came through B2
+      record_lat_ns(nd, c, T0, G.end_ns[par ^ 1], pend_root);
     // --- release the input slots (every lane has loaded its entry: B2 passed)
     if (leader && !n0) {
       L.head = head + n;
       const uint32_t st = G.st[par];
       while (L.segh != st && (int32_t)(nd.in_seg[L.segh & nd.segmask].end - L.head) <= 0) ++L.segh;
-      __threadfence_block();
+      fence_cta();
       vst(&nd.Ein->head, L.head);
       vst(&nd.Ein->seg_head, L.segh);
     }
@@ -866,13 +896,15 @@ __device__ void run_node(Ctx& c, const Dna dna, int i, int gtid) {
     const uint2 ei = e[0];
     const LaneOut oi = o[0];
     const bool term = act && (nd.sink || oi.c == 0);
-    const int64_t lat = T + nd.t - nd.arrival(ei.x);
-    if (rec) {                            // optional per-item records (parity / tracing runs)
+    if (REC && (rec & 7u)) {              // optional per-item records (parity / tracing runs)
       if (act && (rec & PL_REC_TRACE)) {
         atomicAdd(&p.trace[(uint64_t)ei.x * (N + 1) + i], 1u);
         if (nd.sink && oi.c) atomicAdd(&p.trace[(uint64_t)ei.x * (N + 1) + N], oi.c);
       }
-      if (term && (rec & PL_REC_LATENCY)) atomicMax((long long*)&p.lat[ei.x], (long long)lat);
+      if (term && (rec & PL_REC_LATENCY)) {
+        atomicMax((long long*)&p.lat[ei.x], (long long)(T + nd.t - nd.arrival(ei.x)));
+        if (nd.phys) pend_root = ei.x;
+      }
       if (act && (rec & PL_REC_FIRINGS) && (gtid == 0 || (uint32_t)gtid == n - 1)) {
         const uint32_t li = G.log_idx[par];
         if (li < p.log_cap) {
@@ -884,15 +916,14 @@ __device__ void run_node(Ctx& c, const Dna dna, int i, int gtid) {
         }
       }
     }
-    if (term && nd.phys) pend_root = ei.x;
-    {   // per-stream max latency / deadline misses: one smem atomic per warp
-      const uint32_t l32 = term ? (uint32_t)(lat > 0 ? (lat < 0xffffffffll ? lat : 0xffffffffll) : 0) : 0u;
-      const uint32_t lmax = __reduce_max_sync(0xffffffffu, l32);
-      const uint32_t missb = __ballot_sync(0xffffffffu, term && lat > nd.D);
-      if ((gtid & 31) == 0) {
-        if (lmax) atomicMax(&c.sh->max_lat, lmax);
-        if (missb) atomicAdd(&c.sh->miss_events, (uint32_t)__popc(missb));
-      }
+    {   // latency bookkeeping, off the firing's path: arrivals are non-decreasing in root order
+        // (L63, or sorted arrival data), so the firing's largest latency is that of its smallest
+        // terminal root.  The lanes leave their terminal roots in smem; the leader evaluates
+        // them after the publish (and counts misses root by root only when one exceeds D).
+      const uint32_t tr = term ? ei.x : NO_ROOT;
+      nd.troot[gtid] = tr;
+      const uint32_t wmin = __reduce_min_sync(0xffffffffu, tr);
+      if ((gtid & 31) == 0) G.rmin[gtid >> 5] = wmin;
     }
     if (nd.sink && nd.kind == PL_UNGAPPED_XDROP) {   // matches: one global atomic per warp
       const bool hit = act && oi.c;
@@ -914,14 +945,17 @@ __device__ void run_node(Ctx& c, const Dna dna, int i, int gtid) {
         }
       }
     }
-    if (leader) { const long long t2 = clock64(); ph[3] += (uint64_t)(t2 - tc); tc = t2; }
+    if (leader) { const long long t2 = clock64(); atomicAdd(&A.ph[3], (unsigned long long)(t2 - tc)); tc = t2; }
     // --- compaction into the next queue (stable: lane order, then child order)
     const uint32_t out_loc = G.out_loc[par];
     if (!nd.sink && act && oi.c && out_loc != ~0u) {
       const uint32_t base = G.out_base[par] + off;
       for (uint32_t j = 0; j < oi.c; ++j) {
         const uint32_t s = base + j;
-        const uint2 val = stage_output(nd, dna, ei, oi, j);
+        const uint32_t kd = nd.kind;
+        const uint2 val = kd == PL_HIT_ENUM ? stage_output_k<PL_HIT_ENUM>(nd, dna, ei, oi, j)
+                        : kd == PL_FIXED_GAIN ? stage_output_k<PL_FIXED_GAIN>(nd, dna, ei, oi, j)
+                        : kd == PL_POISSON_CAPPED ? stage_output_k<PL_POISSON_CAPPED>(nd, dna, ei, oi, j) : ei;
         if (out_loc == LOC_SMEM) nd.out_ent[s & (nd.out_cap - 1)] = val;
         else __stcg(nd.out_spill + (s & (nd.capg - 1)), val);
       }
@@ -931,34 +965,35 @@ __device__ void run_node(Ctx& c, const Dna dna, int i, int gtid) {
     if (gtid < 32 || bidB == bidA) bar_sync(bidB, v);
     else bar_arrive(bidB, v);
     if (leader) {
-      { const long long t2 = clock64(); ph[4] += (uint64_t)(t2 - tc); tc = t2; }
+      { const long long t2 = clock64(); atomicAdd(&A.ph[4], (unsigned long long)(t2 - tc)); tc = t2; }
       if (nd.phys) {
         uint64_t en = gtimer();
-        const uint64_t due = T0 + (uint64_t)((double)(T + nd.t) * nd.nspu);
-        if ((double)(en - start_ns) > (double)nd.t * nd.nspu) ++overruns;   // work outlasted t_i
-        if ((int64_t)(en - start_ns) > max_fire) max_fire = (int64_t)(en - start_ns);
+        const uint64_t fire = en - start_ns;
+        if ((double)fire > (double)nd.t * nd.nspu) atomicAdd(&A.overruns, 1ull);   // work outlasted t_i
+        atomicMax(&A.max_fire, clamp32((int64_t)fire));
         if (rec & PL_FIXED_SERVICE) {   // hold the outputs until start + t_i (L69)
+          const uint64_t due = T0 + (uint64_t)((double)(T + nd.t) * nd.nspu);
           while (en < due) {
             __nanosleep(due - en > 256 ? 128 : 0);
             en = gtimer();
           }
         }
-        busy_ns += (int64_t)(en - start_ns);
+        atomicAdd(&A.busy_ns, (unsigned long long)(en - start_ns));
         G.end_ns[par] = en;
       }
-      ++firings;
-      consumed += n;
-      produced += total;
-      active += overlap(T, T + nd.t, 0, nd.H);
-      if (T + nd.t > t_end) t_end = T + nd.t;
+      atomicAdd(&A.firings, 1ull);
+      atomicAdd(&A.consumed, (unsigned long long)n);
+      atomicAdd(&A.produced, (unsigned long long)total);
+      atomicAdd(&A.active, (unsigned long long)overlap(T, T + nd.t, 0, nd.H));
+      A.t_end = T + nd.t;                // firing starts increase: the last one ends last
       if (!nd.sink && total > 0 && out_loc != ~0u) {
         Seg sg;
         sg.ready = T + nd.t;
         sg.end = L.out_tail + total;
         sg.loc = out_loc;
         nd.out_seg[L.out_segt & nd.segmask] = sg;
-        if (out_loc == LOC_SPILL) { vst(&nd.Eout->spill_end, sg.end); spilled += total; }
-        __threadfence_block();
+        if (out_loc == LOC_SPILL) { vst(&nd.Eout->spill_end, sg.end); atomicAdd(&A.spilled, (unsigned long long)total); }
+        fence_cta();
         ++L.out_segt;
         L.out_tail += total;
         vst(&nd.Eout->seg_tail, L.out_segt);
@@ -971,7 +1006,38 @@ __device__ void run_node(Ctx& c, const Dna dna, int i, int gtid) {
         L.B = T + nd.t;
         publish_W(nd, L, L.B + nd.t);
       }
-      ph[5] += (uint64_t)(clock64() - tc);
+      // bookkeeping of this firing's terminal items (after the publish; the lanes' troot /
+      // rmin stores were ordered before B4): the smallest root has the largest latency
+      uint32_t rmin = NO_ROOT;
+      for (int k = 0; k < (v >> 5); ++k) rmin = min(rmin, G.rmin[k]);
+      if (rmin != NO_ROOT) {
+        const int64_t lat = T + nd.t - nd.arrival(rmin);
+        atomicMax(&A.lmax, clamp32(lat));
+        if (lat > nd.D) {                // a miss in this firing: count the late items exactly
+          uint32_t m = 0;
+          for (int k = 0; k < v; ++k) {
+            const uint32_t r = nd.troot[k];
+            if (r != NO_ROOT && T + nd.t - nd.arrival(r) > nd.D) ++m;
+          }
+          atomicAdd(&A.nmiss, m);
+        }
+        if (nd.phys) {
+          const uint64_t en = G.end_ns[par];
+          const int64_t l = (int64_t)en - (int64_t)(T0 + (uint64_t)((double)nd.arrival(rmin) * nd.nspu));
+          atomicMax(&A.lmax_ns, clamp32(l));
+          if ((double)l > nd.D_ns) {
+            uint32_t m = 0;
+            for (int k = 0; k < v; ++k) {
+              const uint32_t r = nd.troot[k];
+              if (r == NO_ROOT) continue;
+              const int64_t lr = (int64_t)en - (int64_t)(T0 + (uint64_t)((double)nd.arrival(r) * nd.nspu));
+              if ((double)lr > nd.D_ns) ++m;
+            }
+            atomicAdd(&A.nmiss_ns, m);
+          }
+        }
+      }
+      atomicAdd(&A.ph[5], (unsigned long long)(clock64() - tc));
     }
     if (n0) {                            // replicated node-0 state, identical in every lane
       R.c0 += n;
@@ -982,31 +1048,29 @@ __device__ void run_node(Ctx& c, const Dna dna, int i, int gtid) {
   if (n0) {
     if (leader) publish_W(nd, L, PL_INF64);   // after the last segment was published
     bar_sync(bidA, v);                   // the last publish time is visible to every lane
-    if (pend_root != NO_ROOT) {
-      const uint64_t a_ns = T0 + (uint64_t)((double)nd.arrival(pend_root) * nd.nspu);
-      const int64_t l = (int64_t)G.end_ns[par ^ 1] - (int64_t)a_ns;
-      if (rec & PL_REC_LATENCY) atomicMax((long long*)&p.lat_ns[pend_root], (long long)l);
-      atomicMax(&c.sh->max_lat_ns, (uint32_t)(l > 0 ? (l < 0xffffffffll ? l : 0xffffffffll) : 0));
-      if ((double)l > (double)nd.D * nd.nspu) atomicAdd(&c.sh->miss_events_ns, 1u);
-    }
+    if (REC && pend_root != NO_ROOT) record_lat_ns(nd, c, T0, G.end_ns[par ^ 1], pend_root);
   }
   if (leader) {
+    if (A.lmax) atomicMax(&c.sh->max_lat, A.lmax);
+    if (A.lmax_ns) atomicMax(&c.sh->max_lat_ns, A.lmax_ns);
+    if (A.nmiss) atomicAdd(&c.sh->miss_events, A.nmiss);
+    if (A.nmiss_ns) atomicAdd(&c.sh->miss_events_ns, A.nmiss_ns);
     CtaStats& S = p.stats[stream];
-    S.firings[i] = firings;
+    S.firings[i] = A.firings;
     S.empty[i] = n0 ? R.empties : L.empties;
-    S.consumed[i] = consumed;
-    S.produced[i] = produced;
-    S.active_ne[i] = active;
-    S.busy_ns[i] = busy_ns;
-    S.spilled[i] = spilled;
-    S.overruns[i] = overruns;
-    S.stalls[i] = stalls;
-    S.max_queue[i] = max_queue;
-    S.lateness[i] = lateness;
-    S.sched_cycles[i] = ph[0];
-    S.max_fire_ns[i] = max_fire;
-    for (int k = 0; k < 6; ++k) S.phase_cycles[i][k] = ph[k];
-    atomicMax((long long*)&S.t_end, (long long)t_end);
+    S.consumed[i] = A.consumed;
+    S.produced[i] = A.produced;
+    S.active_ne[i] = (int64_t)A.active;
+    S.busy_ns[i] = (int64_t)A.busy_ns;
+    S.spilled[i] = A.spilled;
+    S.overruns[i] = A.overruns;
+    S.stalls[i] = A.stalls;
+    S.max_queue[i] = A.max_queue;
+    S.lateness[i] = (int64_t)A.lateness;
+    S.sched_cycles[i] = A.ph[0];
+    S.max_fire_ns[i] = (int64_t)A.max_fire;
+    for (int k = 0; k < 6; ++k) S.phase_cycles[i][k] = A.ph[k];
+    atomicMax((long long*)&S.t_end, (long long)A.t_end);
   }
 }
 
@@ -1019,6 +1083,8 @@ __host__ __device__ inline uint32_t layout_enforced(const DevParams& p, SmemLayo
     L->off_seg[i] = off;
     off += p.segcap * (uint32_t)sizeof(Seg);
   }
+  L->off_troot = off;
+  off += (uint32_t)p.N * (uint32_t)p.v * 4u;
   L->off_qoff = off;
   const bool dna = p.k > 0;
   off += dna ? (((1u << (2 * p.k)) + 1u) * 2u + 15u) & ~15u : 0u;
@@ -1308,7 +1374,7 @@ __device__ void run_monolithic(Ctx& c) {
 
 // FIXED_WAIT / THRESHOLD_SLACK executor: grid = n_streams, block = N*32 threads (one warp
 // per node); up to 4 CTAs (streams) per SM when N <= 4.
-template <int MAXT, int MINB>
+template <int MAXT, int MINB, bool REC>
 __global__ void __launch_bounds__(MAXT, MINB) pl_exec_enforced(const __grid_constant__ DevParams p) {
   extern __shared__ __align__(16) unsigned char dsm[];
   __shared__ Shared sh;
@@ -1320,9 +1386,10 @@ __global__ void __launch_bounds__(MAXT, MINB) pl_exec_enforced(const __grid_cons
   // warp w serves node w % N (local warp w / N): with N = 4 every warp of node i sits on
   // SM sub-partition i, so each SMSP's instruction cache holds one node's code path
   const int w = threadIdx.x >> 5;
-  const int gi = w % p.N;
-  const int gt = (w / p.N) * 32 + (threadIdx.x & 31);
-  if (w < p.N * (p.v >> 5)) run_node(c, c.dna, gi, gt);
+  const bool contig = p.variant & 2u;   // experiment: node i owns warps [i v/32, (i+1) v/32)
+  const int gi = contig ? w / (p.v >> 5) : w % p.N;
+  const int gt = (contig ? w % (p.v >> 5) : w / p.N) * 32 + (threadIdx.x & 31);
+  if (w < p.N * (p.v >> 5)) run_node<REC>(c, c.dna, gi, gt);
   __syncthreads();
   cta_finish(c, sh, p);
 }
@@ -1356,18 +1423,30 @@ cudaError_t pl_launch(const DevParams& p, unsigned grid, unsigned block, unsigne
   } else {
     // two CTAs (streams) per SM when the grid asks for more streams than there are SMs and
     // the CTA fits twice (<= 512 threads, 64 registers, smem)
-    if (block <= 512 && p.ctas_per_sm >= 2) pl_exec_enforced<512, 2><<<grid, block, smem, st>>>(p);
-    else if (block <= 512) pl_exec_enforced<512, 1><<<grid, block, smem, st>>>(p);
-    else pl_exec_enforced<1024, 1><<<grid, block, smem, st>>>(p);
+    // per-item records (parity / tracing) select the REC instantiation; the bench runs without
+    const bool rec = (p.flags & (PL_REC_LATENCY | PL_REC_TRACE | PL_REC_FIRINGS)) != 0;
+    if (block <= 512 && p.ctas_per_sm >= 2) {
+      if (rec) pl_exec_enforced<512, 2, true><<<grid, block, smem, st>>>(p);
+      else pl_exec_enforced<512, 2, false><<<grid, block, smem, st>>>(p);
+    } else if (block <= 512) {
+      if (rec) pl_exec_enforced<512, 1, true><<<grid, block, smem, st>>>(p);
+      else pl_exec_enforced<512, 1, false><<<grid, block, smem, st>>>(p);
+    } else {
+      if (rec) pl_exec_enforced<1024, 1, true><<<grid, block, smem, st>>>(p);
+      else pl_exec_enforced<1024, 1, false><<<grid, block, smem, st>>>(p);
+    }
   }
   return cudaGetLastError();
 }
 
 cudaError_t pl_kernel_attributes(unsigned max_smem) {
   cudaError_t e;
-  if ((e = cudaFuncSetAttribute(pl_exec_enforced<512, 2>, cudaFuncAttributeMaxDynamicSharedMemorySize, max_smem))) return e;
-  if ((e = cudaFuncSetAttribute(pl_exec_enforced<512, 1>, cudaFuncAttributeMaxDynamicSharedMemorySize, max_smem))) return e;
-  if ((e = cudaFuncSetAttribute(pl_exec_enforced<1024, 1>, cudaFuncAttributeMaxDynamicSharedMemorySize, max_smem))) return e;
+  if ((e = cudaFuncSetAttribute(pl_exec_enforced<512, 2, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, max_smem))) return e;
+  if ((e = cudaFuncSetAttribute(pl_exec_enforced<512, 2, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, max_smem))) return e;
+  if ((e = cudaFuncSetAttribute(pl_exec_enforced<512, 1, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, max_smem))) return e;
+  if ((e = cudaFuncSetAttribute(pl_exec_enforced<512, 1, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, max_smem))) return e;
+  if ((e = cudaFuncSetAttribute(pl_exec_enforced<1024, 1, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, max_smem))) return e;
+  if ((e = cudaFuncSetAttribute(pl_exec_enforced<1024, 1, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, max_smem))) return e;
   if ((e = cudaFuncSetAttribute(pl_exec_monolithic<512>, cudaFuncAttributeMaxDynamicSharedMemorySize, max_smem))) return e;
   return cudaFuncSetAttribute(pl_exec_monolithic<1024>, cudaFuncAttributeMaxDynamicSharedMemorySize, max_smem);
 }

@@ -72,6 +72,7 @@ struct DevParams {
   int32_t  n_streams;
   uint32_t flags;
   int32_t  ctas_per_sm;                 // launch variant: 2 -> 64-register kernel, two streams per SM
+  uint32_t variant;                     // experiment bits (PL_VARIANT): 1 leader-paced node 0, 2 contiguous warps
   // DNA workload
   const uint32_t* db;                   // packed DB (device)
   uint64_t db_len;
@@ -110,6 +111,7 @@ struct DevParams {
 struct SmemLayout {
   uint32_t off_ent[PL_MAX_STAGES];      // uint2 rings, edge into node i (i >= 1)
   uint32_t off_seg[PL_MAX_STAGES];
+  uint32_t off_troot;                   // [N][v] u32: terminal root per lane of the current firing
   uint32_t off_qoff, off_qpos, off_qw, off_win;
   uint32_t total;
 };

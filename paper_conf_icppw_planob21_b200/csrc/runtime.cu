@@ -430,6 +430,8 @@ pl_status pl_pipeline_create(const pl_config* cfg, const pl_workload* wl, pl_pip
   // one CTA (stream) per SM: the two-per-SM variant (64 registers) spills and measured no gain
   // (tools/streams_scaling.py); it stays selectable through PL_CTAS_PER_SM=2
   d.ctas_per_sm = 1;
+  d.variant = 0;
+  if (const char* e = getenv("PL_VARIANT")) d.variant = (uint32_t)atoi(e);
   if (const char* e = getenv("PL_CTAS_PER_SM"))
     if (atoi(e) == 2 && pl->block <= 512 && 2 * (pl->smem + 4096) <= (uint32_t)prop.sharedMemPerMultiprocessor)
       d.ctas_per_sm = 2;

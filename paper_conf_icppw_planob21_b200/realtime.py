@@ -33,14 +33,16 @@ def measure_gains(cfg, wl, db_dev, stream=None, over=None):
 
 
 def calibrate_budgets(cfg, wl, db_dev, margin=1.25, slack_ns=256, probe_t=20_000, probe_tau=100, stream=None,
-                      over=None):
+                      over=None, flags=0):
     """Service-time budgets t_i (ns): the longest measured firing of each node in a
     physical run with generous budgets, times `margin`, plus `slack_ns`.  The probe's
-    arrivals (probe_t / probe_tau > v per period) keep node 0's vectors full."""
+    arrivals (probe_t / probe_tau > v per period) keep node 0's vectors full.  `flags`
+    must match the runs the budgets are for: per-item records (PL_REC_*) select the
+    recording kernel, whose firings are longer."""
     N = cfg.n_stages
     probe = cfg.replace(clock=PHYS, service_time=(probe_t,) * N, wait_time=(0,) * N, interarrival=probe_tau,
                         deadline=10**12, policy=0, gain=None, ns_per_unit=1.0)
-    st = _run(probe, db_dev, wl.db_len, wl, stream=stream, over=over)
+    st = _run(probe, db_dev, wl.db_len, wl, flags=flags, stream=stream, over=over)
     return tuple(int(math.ceil(margin * st["max_fire_ns"][i])) + slack_ns for i in range(N)), st
 
 

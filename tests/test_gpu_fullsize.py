@@ -32,12 +32,13 @@ def test_c2_full_size_logical(c2wl, policy):
 
 @pytest.fixture(scope="module")
 def budgets(c2wl):
-    """B200 service-time budgets (ns) measured the way bench.py does (realtime.calibrate_budgets)."""
+    """B200 service-time budgets (ns) measured the way bench.py does (realtime.calibrate_budgets),
+    with the per-item records on (flags 7) since the tests below record latencies / traces."""
     import torch
     from paper_conf_icppw_planob21_b200 import realtime
     cfg, wl = c2wl
     db = torch.from_numpy(wl.db.view("int32")).cuda()
-    t, _ = realtime.calibrate_budgets(cfg, wl, db.data_ptr())
+    t, _ = realtime.calibrate_budgets(cfg, wl, db.data_ptr(), flags=7)
     torch.cuda.synchronize()
     return t
 
