@@ -69,6 +69,7 @@ struct Dna {
   uint64_t db_len;
   const uint32_t* win;     // smem copy of DB words [win_lo, win_lo + win_n)
   int64_t win_lo;
+  uint32_t win_lo32;        // (uint32_t)win_lo: window word index arithmetic in 32 bits
   uint32_t win_n;
   const uint32_t* qw;      // query words (smem), nqw valid words
   uint32_t nqw;
@@ -624,20 +625,15 @@ __device__ __forceinline__ uint32_t group_scan(uint32_t* wtot, uint32_t x, uint3
   }
   if (lane == 31) wtot[w] = inc;
   bar_sync(bid, v);                                                    // B2
-  // warp totals: one or two 16-byte shared loads (wtot is 16-byte aligned, 8 slots)
+  // warp totals: one or two 16-byte shared loads (wtot is 16-byte aligned, 8 slots; the
+  // slots of absent warps stay zero from run_node's initialisation)
   const uint4 a = *reinterpret_cast<const uint4*>(wtot);
-  uint32_t t[8] = {a.x, a.y, a.z, a.w, 0u, 0u, 0u, 0u};
+  uint32_t tot = (a.x + a.y) + (a.z + a.w);
+  uint32_t pre = (w > 0 ? a.x : 0u) + (w > 1 ? a.y : 0u) + (w > 2 ? a.z : 0u);
   if (v > 128) {
     const uint4 b = *reinterpret_cast<const uint4*>(wtot + 4);
-    t[4] = b.x; t[5] = b.y; t[6] = b.z; t[7] = b.w;
-  }
-  const int nw = v >> 5;
-  uint32_t pre = 0, tot = 0;
-#pragma unroll
-  for (int k = 0; k < 8; ++k) {
-    const uint32_t tk = k < nw ? t[k] : 0u;
-    pre += (k < w) ? tk : 0u;
-    tot += tk;
+    tot += (b.x + b.y) + (b.z + b.w);
+    pre += (w > 3 ? a.w : 0u) + (w > 4 ? b.x : 0u) + (w > 5 ? b.y : 0u) + (w > 6 ? b.z : 0u);
   }
   *total = tot;
   return pre + inc - x;
@@ -666,7 +662,7 @@ __device__ __forceinline__ void stage_batch(const Node& nd, const Dna& dna, cons
     bool inwin = true;
 #pragma unroll
     for (int j = 0; j < K; ++j) {
-      r[j] = (uint32_t)((int64_t)(e[j].x >> 4) - dna.win_lo);
+      r[j] = (e[j].x >> 4) - dna.win_lo32;
       inwin &= r[j] + 1u < dna.win_n;
     }
     uint32_t key[K];
@@ -744,6 +740,8 @@ __device__ __forceinline__ void record_lat_ns(const Node& nd, const Ctx& c, uint
 // evaluates the decision itself and the leader's reservation reaches the lanes through
 // B2.  Broadcast slots are double-buffered by firing parity.
 // REC: per-item records compiled in (parity / tracing runs); the bench kernel has none.
+// (A separate node-0 instantiation was measured: faster alone, 1.33x slower with all nodes
+// running -- the SM's instruction cache holds one ~76 KB node loop, not two.)
 template <bool REC>
 __device__ void run_node(Ctx& c, const Dna dna, int i, int gtid) {
   const DevParams& p = *c.p;
@@ -772,6 +770,7 @@ __device__ void run_node(Ctx& c, const Dna dna, int i, int gtid) {
   int par = 0;
   if (leader) {
     G.end_ns[0] = 0; G.end_ns[1] = 0;
+    for (int k = 0; k < 8; ++k) { G.wtot[0][k] = 0; G.wtot[1][k] = 0; }
     A.firings = A.consumed = A.produced = A.spilled = A.overruns = A.stalls = A.active = A.busy_ns = 0;
     for (int k = 0; k < 6; ++k) A.ph[k] = 0;
     A.t_end = 0;
@@ -880,6 +879,7 @@ __device__ void run_node(Ctx& c, const Dna dna, int i, int gtid) {
     } else {
       off = group_scan(G.wtot[par], o[0].c, &total, gtid, v, bidA, nd.umax <= 1);                 // B2
     }
+    const uint32_t out_loc = G.out_loc[par], out_base = G.out_base[par];   // leader's reservation (B2)
     if (leader) { const long long t2 = clock64(); atomicAdd(&A.ph[2], (unsigned long long)(t2 - tc)); tc = t2; }
     if (REC && n0 && pend_root != NO_ROOT)   // node 0: the previous publish time came through B2
       record_lat_ns(nd, c, T0, G.end_ns[par ^ 1], pend_root);
@@ -947,10 +947,12 @@ __device__ void run_node(Ctx& c, const Dna dna, int i, int gtid) {
     }
     if (leader) { const long long t2 = clock64(); atomicAdd(&A.ph[3], (unsigned long long)(t2 - tc)); tc = t2; }
     // --- compaction into the next queue (stable: lane order, then child order)
-    const uint32_t out_loc = G.out_loc[par];
     if (!nd.sink && act && oi.c && out_loc != ~0u) {
-      const uint32_t base = G.out_base[par] + off;
-      for (uint32_t j = 0; j < oi.c; ++j) {
+      const uint32_t base = out_base + off;
+      if (nd.umax <= 1 && nd.kind != PL_HIT_ENUM) {   // one output, the entry itself (S0, S2, Bernoulli, ...)
+        if (out_loc == LOC_SMEM) nd.out_ent[base & (nd.out_cap - 1)] = ei;
+        else __stcg(nd.out_spill + (base & (nd.capg - 1)), ei);
+      } else for (uint32_t j = 0; j < oi.c; ++j) {
         const uint32_t s = base + j;
         const uint32_t kd = nd.kind;
         const uint2 val = kd == PL_HIT_ENUM ? stage_output_k<PL_HIT_ENUM>(nd, dna, ei, oi, j)
@@ -1120,6 +1122,7 @@ __device__ void cta_setup(Ctx& c, Shared& sh, unsigned char* dsm, const DevParam
   c.dna.nqw = (uint32_t)(p.q_len + 15) / 16u;
   c.dna.win = (const uint32_t*)(dsm + Lo.off_win);
   c.dna.win_lo = 0;
+  c.dna.win_lo32 = 0;
   c.dna.win_n = 0;
   // DNA: the query index (offsets, positions, packed query) and this stream's DB window
   // (its roots plus the k-1 overlap and a halo for the extensions) are staged into smem
@@ -1140,6 +1143,7 @@ __device__ void cta_setup(Ctx& c, Shared& sh, unsigned char* dsm, const DevParam
       if (whi < wlo) whi = wlo;
     }
     c.dna.win_lo = wlo;
+    c.dna.win_lo32 = (uint32_t)wlo;
     c.dna.win_n = (uint32_t)(whi - wlo);
     uint32_t* win = (uint32_t*)(dsm + Lo.off_win);
     const bool win_tma = p.db_tma && c.dna.win_n;
@@ -1478,7 +1482,7 @@ __global__ void __launch_bounds__(MAXT, 1) pl_stage_batch_kernel(const __grid_co
   c.dna.qpos = (const uint16_t*)(dsm + Lo.off_qpos);
   c.dna.qw = (const uint32_t*)(dsm + Lo.off_qw);
   c.dna.nqw = (uint32_t)(p.q_len + 15) / 16u;
-  c.dna.win = nullptr; c.dna.win_lo = 0; c.dna.win_n = 0;
+  c.dna.win = nullptr; c.dna.win_lo = 0; c.dna.win_lo32 = 0; c.dna.win_n = 0;
   const uint32_t tid = threadIdx.x, v = blockDim.x;
   if (p.k > 0) {
     const uint32_t nko = (1u << (2 * p.k)) + 1u, nqp = (uint32_t)(p.q_len - p.k + 1);
