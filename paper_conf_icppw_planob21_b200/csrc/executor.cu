@@ -164,9 +164,16 @@ struct GroupCtl {           // broadcast from a node's leader to its lanes, doub
   alignas(16) uint32_t wtot[2][8];
   alignas(16) uint32_t rmin[8];   // per warp: smallest terminal root of the current firing
 };
-struct NodeAcc {            // leader-only per-node accumulators: in smem, updated by fire-and-forget
-  unsigned long long firings, consumed, produced, spilled, overruns, stalls, active, busy_ns;  // atomics,
-  unsigned long long ph[6];  // so that they take no registers in the node loop
+// Leader-only per-node accumulators, in smem so that they take no registers in the node loop.
+// 64-bit shared atomics compile to CAS spin loops (ATOMS.CAST.SPIN.64), so the single writer
+// stores per-firing 32-bit deltas (d[]) as it goes and folds everything into the 64-bit sums
+// with one vectorised read-modify-write per firing; maxima use native 32-bit ATOMS.MAX.
+enum { C_FIRINGS, C_CONSUMED, C_PRODUCED, C_ACTIVE, C_BUSY, C_OVERRUNS, C_SPILLED, C_STALLS, C_N };
+enum { D_PH0, D_PH1, D_PH2, D_PH3, D_STALL, D_N = 8 };
+struct NodeAcc {
+  alignas(16) unsigned long long cnt[C_N];
+  alignas(16) unsigned long long ph[6];
+  alignas(16) uint32_t d[D_N];
   long long t_end;
   uint32_t max_queue, lateness, max_fire, lmax, lmax_ns, nmiss, nmiss_ns, pad;
 };
@@ -218,7 +225,9 @@ struct Node {
   int64_t t, P, R, D, tau, X, H;
   uint32_t theta;
   uint64_t lo;
-  double nspu, D_ns;            // D in ns (physical deadline test)
+  double nspu;
+  bool ns1;                     // ns_per_unit == 1: unit -> ns conversions are the identity
+  int64_t t_ns, D_ns;           // floor(t_i ns_per_unit), floor(D ns_per_unit): integer tests x > t_i nspu
   uint32_t segmask, capg;
   EdgeCtl* Ein;                 // input edge (i > 0)
   const uint2* in_ent;
@@ -243,6 +252,11 @@ struct Node {
 
 __host__ __device__ inline uint32_t layout_enforced(const DevParams& p, SmemLayout* L);
 
+// logical time units -> ns of %globaltimer (physical clock)
+__device__ __forceinline__ uint64_t units_ns(const Node& nd, int64_t t) {
+  return nd.ns1 ? (uint64_t)t : (uint64_t)((double)t * nd.nspu);
+}
+
 __device__ __forceinline__ Node make_node(const Ctx& c, int i) {
   const DevParams& p = *c.p;
   SmemLayout Lo;
@@ -256,7 +270,9 @@ __device__ __forceinline__ Node make_node(const Ctx& c, int i) {
   n.theta = p.theta[i];
   n.lo = c.lo;
   n.nspu = p.ns_per_unit;
-  n.D_ns = (double)p.D * p.ns_per_unit;
+  n.ns1 = p.ns_per_unit == 1.0;
+  n.t_ns = (int64_t)((double)p.t[i] * p.ns_per_unit);
+  n.D_ns = (int64_t)((double)p.D * p.ns_per_unit);
   n.segmask = p.segcap - 1;
   n.capg = p.cap_g;
   n.Ein = &c.sh->e[i];
@@ -582,7 +598,7 @@ __device__ Decision decide(const Node& nd, Leader& L) {
 // stage runs so that no extra barrier is needed).  Returns the location.  A full queue
 // back-pressures the producer in both clock modes (deadlock-free):
 // in physical mode the wait shows up as lateness and, if it matters, as deadline misses.
-__device__ uint32_t reserve_out(const Node& nd, Leader& L, uint32_t worst, unsigned long long* stalls) {
+__device__ uint32_t reserve_out(const Node& nd, Leader& L, uint32_t worst, uint32_t* stalled) {
   int spins = 0;
   for (;;) {
     const uint32_t h = vld(&nd.Eout->head), sh = vld(&nd.Eout->seg_head);
@@ -590,13 +606,12 @@ __device__ uint32_t reserve_out(const Node& nd, Leader& L, uint32_t worst, unsig
     const uint32_t need = L.out_tail + worst - h;
     if (seg_ok && need <= nd.out_cap) return LOC_SMEM;
     if (seg_ok && need <= nd.capg) return LOC_SPILL;
-    if (spins == 0) atomicAdd(stalls, 1ull);
+    *stalled = 1u;
     backoff(spins);
   }
 }
 
-__device__ __forceinline__ void pace(uint64_t T0, double nspu, int64_t T, uint64_t* start_ns, int64_t* late) {
-  const uint64_t target = T0 + (uint64_t)((double)T * nspu);
+__device__ __forceinline__ void pace(uint64_t target, uint64_t* start_ns, int64_t* late) {
   uint64_t now = gtimer();
   while (now < target) {   // __nanosleep rounds up to powers of two: sleep at most ~rem/4
     const uint64_t rem = target - now;
@@ -724,7 +739,7 @@ __device__ __forceinline__ uint2 stage_output_k(const Node& nd, const Dna& dna, 
 // maximum and the deadline misses are evaluated by the leader (run_node, "bookkeeping").
 __device__ __forceinline__ void record_lat_ns(const Node& nd, const Ctx& c, uint64_t T0, uint64_t end_ns,
                                               uint32_t& pend_root) {
-  const uint64_t a_ns = T0 + (uint64_t)((double)nd.arrival(pend_root) * nd.nspu);
+  const uint64_t a_ns = T0 + units_ns(nd, nd.arrival(pend_root));
   atomicMax((long long*)&c.p->lat_ns[pend_root], (long long)((int64_t)end_ns - (int64_t)a_ns));
   pend_root = NO_ROOT;
 }
@@ -771,8 +786,10 @@ __device__ void run_node(Ctx& c, const Dna dna, int i, int gtid) {
   if (leader) {
     G.end_ns[0] = 0; G.end_ns[1] = 0;
     for (int k = 0; k < 8; ++k) { G.wtot[0][k] = 0; G.wtot[1][k] = 0; }
-    A.firings = A.consumed = A.produced = A.spilled = A.overruns = A.stalls = A.active = A.busy_ns = 0;
+    for (int k = 0; k < C_N; ++k) A.cnt[k] = 0;
     for (int k = 0; k < 6; ++k) A.ph[k] = 0;
+    for (int k = 0; k < D_N; ++k) A.d[k] = 0;
+    for (int k = 0; k < 8; ++k) G.rmin[k] = NO_ROOT;   // slots of absent warps stay NO_ROOT
     A.t_end = 0;
     A.max_queue = A.lateness = A.max_fire = A.lmax = A.lmax_ns = A.nmiss = A.nmiss_ns = 0;
   }
@@ -789,22 +806,23 @@ __device__ void run_node(Ctx& c, const Dna dna, int i, int gtid) {
         atomicMax(&A.max_queue, d.qlen);
         publish_W(nd, L, T + nd.t);      // committed: nothing leaves node 0 before T + t_0
         if (rec & PL_REC_FIRINGS) G.log_idx[par] = atomicAdd(&c.sh->log_count, 1u);
-        G.out_loc[par] = nd.sink ? LOC_SMEM : reserve_out(nd, L, n * nd.umax, &A.stalls);
+        A.d[D_STALL] = 0;
+        G.out_loc[par] = nd.sink ? LOC_SMEM : reserve_out(nd, L, n * nd.umax, &A.d[D_STALL]);
         G.out_base[par] = L.out_tail;
         tc = clock64();
-        atomicAdd(&A.ph[0], (unsigned long long)(tc - c0));
+        A.d[D_PH0] = (uint32_t)(tc - c0);
       }
       if (nd.phys && (p.variant & 1u)) {  // the leader paces, one barrier releases the lanes
         if (leader) {
           int64_t late;
-          pace(T0, nd.nspu, T, &start_ns, &late);
+          pace(T0 + units_ns(nd, T), &start_ns, &late);
           atomicMax(&A.lateness, clamp32(late));
         }
         bar_sync(bidA, v);
         if (leader) tc = clock64();
       } else if (nd.phys && (gtid & 31) == 0) {   // every warp paces itself against %globaltimer
         uint64_t s_ns; int64_t late;
-        pace(T0, nd.nspu, T, &s_ns, &late);
+        pace(T0 + units_ns(nd, T), &s_ns, &late);
         if (leader) { start_ns = s_ns; atomicMax(&A.lateness, clamp32(late)); tc = clock64(); }
       }
       __syncwarp();
@@ -823,22 +841,23 @@ __device__ void run_node(Ctx& c, const Dna dna, int i, int gtid) {
         G.in_spill_end[par] = vld(&nd.Ein->spill_end);
         if (!d.done) {
           if (rec & PL_REC_FIRINGS) G.log_idx[par] = atomicAdd(&c.sh->log_count, 1u);
-          G.out_loc[par] = nd.sink ? LOC_SMEM : reserve_out(nd, L, d.n * nd.umax, &A.stalls);
+          A.d[D_STALL] = 0;
+          G.out_loc[par] = nd.sink ? LOC_SMEM : reserve_out(nd, L, d.n * nd.umax, &A.d[D_STALL]);
           G.out_base[par] = L.out_tail;
         } else {
           publish_W(nd, L, PL_INF64);
         }
         tc = clock64();
-        atomicAdd(&A.ph[0], (unsigned long long)(tc - c0));
+        A.d[D_PH0] = (uint32_t)(tc - c0);
         if (!d.done && nd.phys) {
           int64_t late;
-          pace(T0, nd.nspu, d.T, &start_ns, &late);
+          pace(T0 + units_ns(nd, d.T), &start_ns, &late);
           atomicMax(&A.lateness, clamp32(late));
           tc = clock64();
         }
       }
       bar_sync(bidA, v);                                               // B1: decision
-      if (leader) { const long long t2 = clock64(); atomicAdd(&A.ph[1], (unsigned long long)(t2 - tc)); tc = t2; }
+      if (leader) { const long long t2 = clock64(); A.d[D_PH1] = (uint32_t)(t2 - tc); tc = t2; }
       if (REC && pend_root != NO_ROOT)   // deferred physical latency of the previous firing
         record_lat_ns(nd, c, T0, G.end_ns[par ^ 1], pend_root);
       if (G.done[par]) break;
@@ -880,7 +899,7 @@ __device__ void run_node(Ctx& c, const Dna dna, int i, int gtid) {
       off = group_scan(G.wtot[par], o[0].c, &total, gtid, v, bidA, nd.umax <= 1);                 // B2
     }
     const uint32_t out_loc = G.out_loc[par], out_base = G.out_base[par];   // leader's reservation (B2)
-    if (leader) { const long long t2 = clock64(); atomicAdd(&A.ph[2], (unsigned long long)(t2 - tc)); tc = t2; }
+    if (leader) { const long long t2 = clock64(); A.d[D_PH2] = (uint32_t)(t2 - tc); tc = t2; }
     if (REC && n0 && pend_root != NO_ROOT)   // node 0: the previous publish time came through B2
       record_lat_ns(nd, c, T0, G.end_ns[par ^ 1], pend_root);
     // --- release the input slots (every lane has loaded its entry: B2 passed)
@@ -945,7 +964,7 @@ __device__ void run_node(Ctx& c, const Dna dna, int i, int gtid) {
         }
       }
     }
-    if (leader) { const long long t2 = clock64(); atomicAdd(&A.ph[3], (unsigned long long)(t2 - tc)); tc = t2; }
+    if (leader) { const long long t2 = clock64(); A.d[D_PH3] = (uint32_t)(t2 - tc); tc = t2; }
     // --- compaction into the next queue (stable: lane order, then child order)
     if (!nd.sink && act && oi.c && out_loc != ~0u) {
       const uint32_t base = out_base + off;
@@ -967,34 +986,30 @@ __device__ void run_node(Ctx& c, const Dna dna, int i, int gtid) {
     if (gtid < 32 || bidB == bidA) bar_sync(bidB, v);
     else bar_arrive(bidB, v);
     if (leader) {
-      { const long long t2 = clock64(); atomicAdd(&A.ph[4], (unsigned long long)(t2 - tc)); tc = t2; }
+      long long t4 = clock64();
+      const uint32_t ph4 = (uint32_t)(t4 - tc);
+      uint64_t en = 0, fire = 0;
       if (nd.phys) {
-        uint64_t en = gtimer();
-        const uint64_t fire = en - start_ns;
-        if ((double)fire > (double)nd.t * nd.nspu) atomicAdd(&A.overruns, 1ull);   // work outlasted t_i
+        en = gtimer();
+        fire = en - start_ns;
         atomicMax(&A.max_fire, clamp32((int64_t)fire));
         if (rec & PL_FIXED_SERVICE) {   // hold the outputs until start + t_i (L69)
-          const uint64_t due = T0 + (uint64_t)((double)(T + nd.t) * nd.nspu);
+          const uint64_t due = T0 + units_ns(nd, T + nd.t);
           while (en < due) {
             __nanosleep(due - en > 256 ? 128 : 0);
             en = gtimer();
           }
         }
-        atomicAdd(&A.busy_ns, (unsigned long long)(en - start_ns));
         G.end_ns[par] = en;
       }
-      atomicAdd(&A.firings, 1ull);
-      atomicAdd(&A.consumed, (unsigned long long)n);
-      atomicAdd(&A.produced, (unsigned long long)total);
-      atomicAdd(&A.active, (unsigned long long)overlap(T, T + nd.t, 0, nd.H));
-      A.t_end = T + nd.t;                // firing starts increase: the last one ends last
+      // publish: the segment (outputs ready at T + t_i), then the watermark
       if (!nd.sink && total > 0 && out_loc != ~0u) {
         Seg sg;
         sg.ready = T + nd.t;
         sg.end = L.out_tail + total;
         sg.loc = out_loc;
         nd.out_seg[L.out_segt & nd.segmask] = sg;
-        if (out_loc == LOC_SPILL) { vst(&nd.Eout->spill_end, sg.end); atomicAdd(&A.spilled, (unsigned long long)total); }
+        if (out_loc == LOC_SPILL) vst(&nd.Eout->spill_end, sg.end);
         fence_cta();
         ++L.out_segt;
         L.out_tail += total;
@@ -1008,12 +1023,21 @@ __device__ void run_node(Ctx& c, const Dna dna, int i, int gtid) {
         L.B = T + nd.t;
         publish_W(nd, L, L.B + nd.t);
       }
-      // bookkeeping of this firing's terminal items (after the publish; the lanes' troot /
-      // rmin stores were ordered before B4): the smallest root has the largest latency
-      uint32_t rmin = NO_ROOT;
-      for (int k = 0; k < (v >> 5); ++k) rmin = min(rmin, G.rmin[k]);
+      A.t_end = T + nd.t;                // firing starts increase: the last one ends last
+      // bookkeeping of this firing's terminal items (the lanes' troot / rmin stores were
+      // ordered before B4): the smallest root has the largest latency
+      uint32_t rmin;
+      {
+        const uint4 a = *reinterpret_cast<const uint4*>(G.rmin);
+        rmin = min(min(a.x, a.y), min(a.z, a.w));
+        if (v > 128) {
+          const uint4 b = *reinterpret_cast<const uint4*>(G.rmin + 4);
+          rmin = min(rmin, min(min(b.x, b.y), min(b.z, b.w)));
+        }
+      }
       if (rmin != NO_ROOT) {
-        const int64_t lat = T + nd.t - nd.arrival(rmin);
+        const int64_t ar = nd.arrival(rmin);
+        const int64_t lat = T + nd.t - ar;
         atomicMax(&A.lmax, clamp32(lat));
         if (lat > nd.D) {                // a miss in this firing: count the late items exactly
           uint32_t m = 0;
@@ -1024,22 +1048,37 @@ __device__ void run_node(Ctx& c, const Dna dna, int i, int gtid) {
           atomicAdd(&A.nmiss, m);
         }
         if (nd.phys) {
-          const uint64_t en = G.end_ns[par];
-          const int64_t l = (int64_t)en - (int64_t)(T0 + (uint64_t)((double)nd.arrival(rmin) * nd.nspu));
+          const int64_t l = (int64_t)en - (int64_t)(T0 + units_ns(nd, ar));
           atomicMax(&A.lmax_ns, clamp32(l));
-          if ((double)l > nd.D_ns) {
+          if (l > nd.D_ns) {
             uint32_t m = 0;
             for (int k = 0; k < v; ++k) {
               const uint32_t r = nd.troot[k];
-              if (r == NO_ROOT) continue;
-              const int64_t lr = (int64_t)en - (int64_t)(T0 + (uint64_t)((double)nd.arrival(r) * nd.nspu));
-              if ((double)lr > nd.D_ns) ++m;
+              if (r != NO_ROOT && (int64_t)en - (int64_t)(T0 + units_ns(nd, nd.arrival(r))) > nd.D_ns) ++m;
             }
             atomicAdd(&A.nmiss_ns, m);
           }
         }
       }
-      atomicAdd(&A.ph[5], (unsigned long long)(clock64() - tc));
+      {   // fold this firing into the 64-bit sums: one vectorised read-modify-write
+        ulonglong2* Cp = reinterpret_cast<ulonglong2*>(A.cnt);
+        ulonglong2* Pp = reinterpret_cast<ulonglong2*>(A.ph);
+        ulonglong2 c0 = Cp[0], c1 = Cp[1], c2 = Cp[2], c3 = Cp[3], p0 = Pp[0], p1 = Pp[1], p2 = Pp[2];
+        const uint4 dd = *reinterpret_cast<const uint4*>(A.d);
+        const uint32_t stl = A.d[D_STALL];
+        c0.x += 1ull;
+        c0.y += n;
+        c1.x += total;
+        c1.y += (unsigned long long)overlap(T, T + nd.t, 0, nd.H);
+        c2.x += nd.phys ? (en - start_ns) : 0ull;
+        c2.y += (nd.phys && (int64_t)fire > nd.t_ns) ? 1ull : 0ull;   // work outlasted t_i
+        c3.x += (!nd.sink && out_loc == LOC_SPILL) ? (unsigned long long)total : 0ull;
+        c3.y += stl;
+        p0.x += dd.x; p0.y += dd.y; p1.x += dd.z; p1.y += dd.w;
+        p2.x += ph4;
+        p2.y += (uint64_t)(clock64() - t4);
+        Cp[0] = c0; Cp[1] = c1; Cp[2] = c2; Cp[3] = c3; Pp[0] = p0; Pp[1] = p1; Pp[2] = p2;
+      }
     }
     if (n0) {                            // replicated node-0 state, identical in every lane
       R.c0 += n;
@@ -1058,15 +1097,15 @@ __device__ void run_node(Ctx& c, const Dna dna, int i, int gtid) {
     if (A.nmiss) atomicAdd(&c.sh->miss_events, A.nmiss);
     if (A.nmiss_ns) atomicAdd(&c.sh->miss_events_ns, A.nmiss_ns);
     CtaStats& S = p.stats[stream];
-    S.firings[i] = A.firings;
+    S.firings[i] = A.cnt[C_FIRINGS];
     S.empty[i] = n0 ? R.empties : L.empties;
-    S.consumed[i] = A.consumed;
-    S.produced[i] = A.produced;
-    S.active_ne[i] = (int64_t)A.active;
-    S.busy_ns[i] = (int64_t)A.busy_ns;
-    S.spilled[i] = A.spilled;
-    S.overruns[i] = A.overruns;
-    S.stalls[i] = A.stalls;
+    S.consumed[i] = A.cnt[C_CONSUMED];
+    S.produced[i] = A.cnt[C_PRODUCED];
+    S.active_ne[i] = (int64_t)A.cnt[C_ACTIVE];
+    S.busy_ns[i] = (int64_t)A.cnt[C_BUSY];
+    S.spilled[i] = A.cnt[C_SPILLED];
+    S.overruns[i] = A.cnt[C_OVERRUNS];
+    S.stalls[i] = A.cnt[C_STALLS];
     S.max_queue[i] = A.max_queue;
     S.lateness[i] = (int64_t)A.lateness;
     S.sched_cycles[i] = A.ph[0];
@@ -1263,7 +1302,7 @@ __device__ void run_monolithic(Ctx& c) {
     if (phys) {
       if (tid == 0) {
         uint64_t s_ns; int64_t late;
-        pace(c.sh->T0, p.ns_per_unit, ready, &s_ns, &late);   // the block is complete in real time
+        pace(c.sh->T0 + (uint64_t)((double)ready * p.ns_per_unit), &s_ns, &late);   // the block is complete in real time
         sh_start_ns = s_ns;
       }
       __syncthreads();

@@ -37,6 +37,7 @@ for tau in (150, 25):
         r[f"node{i}"]["mean_fire_ns"] = round(st["busy_ns"][i] / f)
         r[f"node{i}"]["max_fire_ns"] = st["max_fire_ns"][i]
         r[f"node{i}"]["firings"] = st["firings"][i]
+        r[f"node{i}"]["loop"] = sum(st["phase_cycles"][i][k] for k in range(6)) // f
     out[f"tau{tau}"] = r
 print(json.dumps(out), flush=True)
 '''
