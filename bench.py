@@ -53,6 +53,8 @@ def parse():
     ap.add_argument("--cpu-sample-streams", type=int, default=148)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--drain", default="eager", choices=["eager", "periodic"],
+                    help="end of stream: R-DRAIN work-conserving drain (PL_EAGER_DRAIN) or the periodic rule")
     return ap.parse_args()
 
 
@@ -226,7 +228,7 @@ def main():
         budgets = tuple(int(x) for x in t.tolist())
     log({"gains": gains, "budgets_ns": budgets, "cal_max_fire_ns": cal["max_fire_ns"]})
     cfg = base.replace(clock=1, ns_per_unit=1.0, service_time=budgets, gain=gains, deadline=a.deadline_ns,
-                       b=C.PAPER_B)
+                       b=C.PAPER_B, eager_drain=a.drain == "eager")
     # 2./3. the fastest miss-free rate
     tau, w, th, T, st_ok = realtime.find_rate(cfg, wl, db_ptr, stream=stream, log=log)
     if world > 1:
@@ -280,6 +282,31 @@ def main():
     tot_ms = float(tt.item())
     roots_all, misses_all, overruns_all, sched_misses_all = (int(x) for x in cnt.tolist())
     value = roots_all / (tot_ms * 1e-3)
+
+    # the other end-of-stream rule at the same rate and waits (the paper's periodic schedule
+    # runs to the drain; R-DRAIN switches every node to work-conserving at the last arrival)
+    other = None
+    try:
+        plo = Pipeline(run_cfg.replace(eager_drain=a.drain != "eager"), wl, flags=0, stream=stream)
+        plo.bind_device(db_ptr, wl.db_len)
+        plo.launch()
+        plo.summary()
+        o0, o1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        oms, oroots, omiss = 0.0, 0, 0
+        for _ in range(a.steps):
+            flush.zero_()
+            o0.record(stream)
+            plo.launch()
+            o1.record(stream)
+            so = plo.summary()
+            oms += o0.elapsed_time(o1)
+            oroots += so["roots"]
+            omiss += so["miss_events_ns"]
+        plo.close()
+        other = {"drain": "periodic" if a.drain == "eager" else "eager", "value": oroots / (oms * 1e-3),
+                 "ms_per_step": oms / a.steps, "misses": omiss, "max_latency_ns": so["max_latency_ns"]}
+    except RuntimeError as ex:
+        other = {"failed": str(ex)}
 
     # logical-clock throughput of the same executor (no real-time pacing)
     lc = logical_cfg(base)
@@ -410,6 +437,8 @@ def main():
             "warmup": a.warmup, "ms_per_step": tot_ms / a.steps, "higher_is_better": True, "scaling": "weak",
             "vs_baseline": None, "dtype": "int32", "data": "synthetic",
             "config": {"workload": WORKLOAD, "policy": "FIXED_WAIT", "clock": "globaltimer (1 unit = 1 ns)",
+                       "drain": ("eager (R-DRAIN: every node work-conserving once the stream's last root "
+                                 "has arrived; PL_EAGER_DRAIN)" if a.drain == "eager" else "periodic (paper rule)"),
                        "deadline_ns": a.deadline_ns, "tau0_ns": tau, "b": list(C.PAPER_B),
                        "budgets_ns": list(budgets), "w_ns": list(w), "gains": [round(g, 5) for g in gains],
                        "streams_per_gpu": a.streams, "l2": "flushed between timed steps (256 MiB memset)",
@@ -418,11 +447,13 @@ def main():
             "sustained_items_per_s": world * a.streams * 1e9 / tau,
             "logical_items_per_s": logical_ips,
             "threshold_slack": thr,
+            "other_drain": other,
             "utilisation": {"enforced_model": st_last["active_fraction"], "enforced_fig1_T": T,
                             "enforced_hw_busy": st["hw_busy_fraction"], "monolithic": mono},
             "per_firing": {f"node{i}": {"firings": st["firings"][i],
                                         "scheduler_cycles": round(st["phase_cycles"][i][0] / max(1, st["firings"][i])),
-                                        "firing_cycles": round(sum(st["phase_cycles"][i][1:]) / max(1, st["firings"][i])),
+                                        "firing_cycles": round(sum(st["phase_cycles"][i][1:5]) / max(1, st["firings"][i])),
+                                        "publish_cycles": round(st["phase_cycles"][i][5] / max(1, st["firings"][i])),
                                         "mean_fire_ns": round(st["busy_ns"][i] / max(1, st["firings"][i])),
                                         "max_fire_ns": st["max_fire_ns"][i]} for i in range(st["n_stages"])},
             "clocks": clk,

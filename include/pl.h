@@ -76,6 +76,12 @@ enum pl_clock { PL_CLOCK_LOGICAL = 0, PL_CLOCK_GLOBALTIMER = 1 };
 #define PL_REC_FIRINGS  4u     /* per-stream log of non-empty firings                    */
 #define PL_FIXED_SERVICE 8u    /* physical clock: publish a firing's outputs at start + t_i,
                                   the paper's fixed service time (L69), not as soon as done */
+#define PL_EAGER_DRAIN  16u    /* end of stream (reading R-DRAIN): at times T >= A_last, the
+                                  stream's last arrival, every node fires whenever it is idle
+                                  and its queue is non-empty (FIXED_WAIT's time-triggered
+                                  starts at T >= A_last are dropped).  The paper models an
+                                  unbounded stream (L63) and is silent on its end; without
+                                  this flag the periodic / threshold rules run to the drain. */
 
 typedef struct {
   uint32_t kind;           /* enum pl_stage_kind                                        */

@@ -19,10 +19,16 @@ At each event time T, in this order (reading R-ORDER):
        THRESHOLD_SLACK — an idle node fires when |Q_i| >= theta_i or when
                          |Q_i| > 0 and T >= a(head) + D - R_i (north_star rule,
                          SURVEY A25), taking min(|Q_i|, v);
+     With ``cfg.eager_drain`` (reading R-DRAIN): at every event time
+     T >= A_last (the stream's last arrival) both policies give way to a
+     work-conserving drain -- an idle node with a non-empty queue fires at T,
+     taking min(|Q_i|, v); FIXED_WAIT's time-triggered starts at T >= A_last are
+     dropped.  Before A_last nothing changes.
   4. stop once every root has arrived, every queue is empty and no firing
      with inputs is in flight (FIXED_WAIT also keeps generating its
      time-triggered firings until every node's next start is >= H = X*tau0, so
-     that the window [0, H) is fully charged, R-WINDOW).
+     that the window [0, H) is fully charged, R-WINDOW; with eager_drain there
+     are none at T >= A_last).
 MONOLITHIC (L157, L184; R-MONO) is simulated by its own loop: blocks of M
 consecutive arrivals, ready at their last arrival, served FIFO by one
 processor; for each block node i fires ceil(n_i/v) times back to back.
@@ -124,6 +130,8 @@ def simulate_stream(cfg: C.Config, fns, lo: int, hi: int, wait_time=None, theta=
     order = list(range(N)) if node_order is None else list(node_order)
     match_sink = cfg.stages[-1].kind == C.UNGAPPED_XDROP
     fixed = cfg.policy == C.FIXED_WAIT
+    eager = bool(getattr(cfg, "eager_drain", False))
+    A_last = arr[X - 1] if X else 0              # R-DRAIN: the drain starts at the last arrival
     if fixed:
         w = list(wait_time if wait_time is not None else cfg.wait_time)
         P = [t[i] + w[i] for i in range(N)]
@@ -193,7 +201,9 @@ def simulate_stream(cfg: C.Config, fns, lo: int, hi: int, wait_time=None, theta=
         # ---- 3. starts
         for i in order:
             fire = False
-            if fixed:
+            if eager and T >= A_last:                # R-DRAIN: work-conserving after the last arrival
+                fire = inflight[i] is None and bool(Q[i])
+            elif fixed:
                 fire = next_start[i] == T
             elif inflight[i] is None and Q[i]:
                 a_head = arr[Q[i][0][0] - lo]
@@ -215,9 +225,11 @@ def simulate_stream(cfg: C.Config, fns, lo: int, hi: int, wait_time=None, theta=
                     firings.append((i, T, n, ents[0][0], ents[-1][0]))
                 else:
                     n_empty[i] += 1
-                if fixed:
+                if fixed and not (eager and T + P[i] >= A_last):
                     next_start[i] = T + P[i]
                     push(next_start[i])
+                elif fixed:
+                    next_start[i] = 1 << 62          # no time-triggered starts at or after A_last
             if not fixed and Q[i]:
                 fdl = arr[Q[i][0][0] - lo] + D - R[i]
                 if fdl > T and last_force[i] != fdl:

@@ -168,7 +168,7 @@ struct GroupCtl {           // broadcast from a node's leader to its lanes, doub
 // 64-bit shared atomics compile to CAS spin loops (ATOMS.CAST.SPIN.64), so the single writer
 // stores per-firing 32-bit deltas (d[]) as it goes and folds everything into the 64-bit sums
 // with one vectorised read-modify-write per firing; maxima use native 32-bit ATOMS.MAX.
-enum { C_FIRINGS, C_CONSUMED, C_PRODUCED, C_ACTIVE, C_BUSY, C_OVERRUNS, C_SPILLED, C_STALLS, C_N };
+enum { C_FIRINGS, C_CONSUMED, C_PRODUCED, C_ACTIVE, C_BUSY, C_OVERRUNS, C_SPILLED, C_STALLS, C_ACTIVE_E, C_PAD, C_N };
 enum { D_PH0, D_PH1, D_PH2, D_PH3, D_STALL, D_N = 8 };
 struct NodeAcc {
   alignas(16) unsigned long long cnt[C_N];
@@ -244,6 +244,10 @@ struct Node {
   MDiv dtau, dP;
   int64_t Pq, Pr;               // floor(P / tau0), P mod tau0
   const int64_t* arr;           // per-root arrival times (NULL: fixed rate, L63)
+  bool eager;                   // PL_EAGER_DRAIN (R-DRAIN): work-conserving at T >= A_last
+  int64_t A_last;               // the stream's last arrival
+  int64_t Mcap, B_per;          // FIXED_WAIT + eager: time-triggered slots m < Mcap (m P < A_last);
+                                // the last of them ends at B_per
   uint32_t* troot;              // smem [v]: the current firing's terminal root per lane (or NO_ROOT)
   __device__ __forceinline__ int64_t arrival(uint32_t root) const {
     return arr ? __ldg(arr + root) : (int64_t)(root - lo) * tau;
@@ -296,6 +300,10 @@ __device__ __forceinline__ Node make_node(const Ctx& c, int i) {
   n.Pq = fdiv(p.P[i], n.dtau);
   n.Pr = p.P[i] - n.Pq * p.tau;
   n.arr = p.arr;
+  n.eager = (p.flags & PL_EAGER_DRAIN) != 0u;
+  n.A_last = c.X > 0 ? n.arrival((uint32_t)(c.hi - 1)) : 0;
+  n.Mcap = (n.eager && n.fixed) ? cdiv(n.A_last, n.dP) : 0;
+  n.B_per = n.Mcap > 0 ? (n.Mcap - 1) * n.P + n.t : 0;
   n.troot = (uint32_t*)(c.dsm + Lo.off_troot) + (uint32_t)i * (uint32_t)p.v;
   return n;
 }
@@ -463,16 +471,19 @@ __device__ __forceinline__ Decision decide0(const Node& nd, Rep& r) {
       T = r.m * nd.P;
       if (T < ah) {
         const int64_t m2 = cdiv(ah, nd.dP);
-        r.empties += (uint64_t)(m2 - r.m);
+        const int64_t me = nd.eager ? min(m2, nd.Mcap) : m2;   // R-DRAIN: no slots at or after A_last
+        if (me > r.m) r.empties += (uint64_t)(me - r.m);
         r.m = m2;
         T = r.m * nd.P;
       }
+      if (nd.eager && r.m >= nd.Mcap) T = max(max(nd.B_per, r.B), nd.A_last);
     } else {
       const int64_t Tth = (r.c0 + nd.theta - 1 < nd.X) ? __ldg(A + r.c0 + nd.theta - 1) : PL_INF64;
       int64_t Tf = ah + nd.D - nd.R;
       if (Tf < ah) Tf = ah;
       T = Tth < Tf ? Tth : Tf;
       if (T < r.B) T = r.B;
+      if (nd.eager) T = min(T, max(r.B, nd.A_last));
     }
     d.T = T;
     d.n = (uint32_t)nd.v;                // upper bound; the exact count comes out of the scan
@@ -483,17 +494,23 @@ __device__ __forceinline__ Decision decide0(const Node& nd, Rep& r) {
     T = r.m * nd.P;
     if (T < r.c0 * nd.tau) {             // empty firings until the next root has arrived
       const int64_t m2 = cdiv(r.c0 * nd.tau, nd.dP);
-      r.empties += (uint64_t)(m2 - r.m);
+      const int64_t me = nd.eager ? min(m2, nd.Mcap) : m2;   // R-DRAIN: no slots at or after A_last
+      if (me > r.m) r.empties += (uint64_t)(me - r.m);
       r.m = m2;
       T = r.m * nd.P;
       r.qvalid = false;
     }
-    if (!r.qvalid) {                     // floor(T / tau0), then advanced by P per firing
-      r.qT = fdiv(T, nd.dtau);
-      r.rT = T - r.qT * nd.tau;
-      r.qvalid = true;
+    if (nd.eager && r.m >= nd.Mcap) {    // R-DRAIN: every root has arrived; fire when idle
+      T = max(max(nd.B_per, r.B), nd.A_last);
+      q = nd.X - 1;
+    } else {
+      if (!r.qvalid) {                   // floor(T / tau0), then advanced by P per firing
+        r.qT = fdiv(T, nd.dtau);
+        r.rT = T - r.qT * nd.tau;
+        r.qvalid = true;
+      }
+      q = r.qT;
     }
-    q = r.qT;
   } else {
     const int64_t ah = r.c0 * nd.tau;
     const int64_t Tth = (r.c0 + nd.theta - 1 < nd.X) ? ah + (int64_t)(nd.theta - 1) * nd.tau : PL_INF64;
@@ -501,6 +518,7 @@ __device__ __forceinline__ Decision decide0(const Node& nd, Rep& r) {
     if (Tf < ah) Tf = ah;
     T = Tth < Tf ? Tth : Tf;
     if (T < r.B) T = r.B;
+    if (nd.eager) T = min(T, max(r.B, nd.A_last));
     q = fdiv(T, nd.dtau);
   }
   int64_t arrived = q + 1;
@@ -536,6 +554,21 @@ __device__ Decision decide(const Node& nd, Leader& L) {
     const uint32_t tail_known = (st != L.segh) ? nd.in_seg[(st - 1) & nd.segmask].end : L.head;
     const bool any = tail_known != L.head;
     if (nd.fixed) {
+      if (nd.eager && L.m >= nd.Mcap) {  // R-DRAIN: work-conserving from A_last on
+        const int64_t B = max(max(nd.B_per, L.B), nd.A_last);
+        if (!any) {
+          if (Wup == PL_INF64) { d.done = true; return d; }
+          publish_W(nd, L, max(B, Wup) + nd.t);
+          backoff(spins);
+          continue;
+        }
+        const int64_t Te = max(B, nd.in_seg[L.segh & nd.segmask].ready);
+        const uint32_t cnt = count_le(nd, L, st, Te);
+        publish_W(nd, L, Te + nd.t);     // the firing starts at Te; only its size is pending
+        if (Wup > Te || cnt >= v) { d.T = Te; d.n = cnt < v ? cnt : v; d.qlen = tail_known - L.head; return d; }
+        backoff(spins);
+        continue;
+      }
       const int64_t T = L.m * nd.P;
       const uint32_t cnt = count_le(nd, L, st, T);
       if (cnt >= v || Wup > T) {
@@ -544,9 +577,10 @@ __device__ Decision decide(const Node& nd, Leader& L) {
         const int64_t r = any ? nd.in_seg[L.segh & nd.segmask].ready : Wup;
         int64_t m2 = cdiv(r, nd.dP);
         if (m2 < L.m + 1) m2 = L.m + 1;
-        L.empties += (uint64_t)(m2 - L.m);
+        const int64_t me = nd.eager ? min(m2, nd.Mcap) : m2;   // R-DRAIN: no slots at or after A_last
+        if (me > L.m) L.empties += (uint64_t)(me - L.m);
         L.m = m2;
-        publish_W(nd, L, L.m * nd.P + nd.t);
+        publish_W(nd, L, (nd.eager && L.m >= nd.Mcap ? max(max(nd.B_per, L.B), nd.A_last) : L.m * nd.P) + nd.t);
         spins = 0;
         continue;
       }
@@ -577,6 +611,7 @@ __device__ Decision decide(const Node& nd, Leader& L) {
     }
     int64_t Tk = Tth < Tf ? Tth : Tf;
     if (Tk < L.B) Tk = L.B;
+    if (nd.eager) Tk = min(Tk, max(max(L.B, nd.A_last), hs.ready));   // R-DRAIN
     if (th_known || Tk < Wup) {
       const uint32_t cnt = count_le(nd, L, st, Tk);
       if (Wup > Tk || cnt >= v) {
@@ -1018,7 +1053,11 @@ __device__ void run_node(Ctx& c, const Dna dna, int i, int gtid) {
       }
       if (nd.fixed) {
         ++L.m;
-        publish_W(nd, L, (n0 ? R.m + 1 : L.m) * nd.P + nd.t);
+        const bool ef = nd.eager && T >= nd.A_last;   // an R-DRAIN firing: busy until T + t_i
+        if (ef) L.B = T + nd.t;
+        const int64_t mn = n0 ? R.m + 1 : L.m;
+        const int64_t Bn = ef ? T + nd.t : (n0 ? R.B : L.B);
+        publish_W(nd, L, (nd.eager && mn >= nd.Mcap ? max(max(nd.B_per, Bn), nd.A_last) : mn * nd.P) + nd.t);
       } else {
         L.B = T + nd.t;
         publish_W(nd, L, L.B + nd.t);
@@ -1063,13 +1102,15 @@ __device__ void run_node(Ctx& c, const Dna dna, int i, int gtid) {
       {   // fold this firing into the 64-bit sums: one vectorised read-modify-write
         ulonglong2* Cp = reinterpret_cast<ulonglong2*>(A.cnt);
         ulonglong2* Pp = reinterpret_cast<ulonglong2*>(A.ph);
-        ulonglong2 c0 = Cp[0], c1 = Cp[1], c2 = Cp[2], c3 = Cp[3], p0 = Pp[0], p1 = Pp[1], p2 = Pp[2];
+        ulonglong2 c0 = Cp[0], c1 = Cp[1], c2 = Cp[2], c3 = Cp[3], c4 = Cp[4], p0 = Pp[0], p1 = Pp[1], p2 = Pp[2];
         const uint4 dd = *reinterpret_cast<const uint4*>(A.d);
         const uint32_t stl = A.d[D_STALL];
         c0.x += 1ull;
         c0.y += n;
         c1.x += total;
-        c1.y += (unsigned long long)overlap(T, T + nd.t, 0, nd.H);
+        const unsigned long long ov = (unsigned long long)overlap(T, T + nd.t, 0, nd.H);
+        c1.y += ov;
+        c4.x += (nd.eager && T >= nd.A_last) ? ov : 0ull;   // R-DRAIN firings (FIXED_WAIT window)
         c2.x += nd.phys ? (en - start_ns) : 0ull;
         c2.y += (nd.phys && (int64_t)fire > nd.t_ns) ? 1ull : 0ull;   // work outlasted t_i
         c3.x += (!nd.sink && out_loc == LOC_SPILL) ? (unsigned long long)total : 0ull;
@@ -1077,12 +1118,17 @@ __device__ void run_node(Ctx& c, const Dna dna, int i, int gtid) {
         p0.x += dd.x; p0.y += dd.y; p1.x += dd.z; p1.y += dd.w;
         p2.x += ph4;
         p2.y += (uint64_t)(clock64() - t4);
-        Cp[0] = c0; Cp[1] = c1; Cp[2] = c2; Cp[3] = c3; Pp[0] = p0; Pp[1] = p1; Pp[2] = p2;
+        Cp[0] = c0; Cp[1] = c1; Cp[2] = c2; Cp[3] = c3; Cp[4] = c4; Pp[0] = p0; Pp[1] = p1; Pp[2] = p2;
       }
     }
     if (n0) {                            // replicated node-0 state, identical in every lane
       R.c0 += n;
-      if (nd.fixed) advance0(nd, R); else R.B = T + nd.t;
+      if (nd.fixed) {
+        advance0(nd, R);
+        if (nd.eager && T >= nd.A_last) R.B = T + nd.t;   // R-DRAIN: busy until
+      } else {
+        R.B = T + nd.t;
+      }
     }
     par ^= 1;
   }
@@ -1102,6 +1148,15 @@ __device__ void run_node(Ctx& c, const Dna dna, int i, int gtid) {
     S.consumed[i] = A.cnt[C_CONSUMED];
     S.produced[i] = A.cnt[C_PRODUCED];
     S.active_ne[i] = (int64_t)A.cnt[C_ACTIVE];
+    if (nd.fixed) {   // every time-triggered firing m P_i < H is charged, empty or not (L97, R-WINDOW);
+                      // with R-DRAIN only the slots m P_i < A_last, plus the drain firings
+      const int64_t H = nd.H, P = nd.P, t = nd.t;
+      const int64_t K = nd.eager ? min(H / P, nd.Mcap - 1) : H / P;
+      S.active_win[i] = K < 0 ? 0 : K * t + min(t, H - K * P);
+      if (nd.eager) S.active_win[i] += (int64_t)A.cnt[C_ACTIVE_E];
+    } else {
+      S.active_win[i] = (int64_t)A.cnt[C_ACTIVE];
+    }
     S.busy_ns[i] = (int64_t)A.cnt[C_BUSY];
     S.spilled[i] = A.cnt[C_SPILLED];
     S.overruns[i] = A.cnt[C_OVERRUNS];
@@ -1404,7 +1459,8 @@ __device__ void run_monolithic(Ctx& c) {
     CtaStats& S = p.stats[stream];
     for (int i = 0; i < PL_MAX_STAGES; ++i) {
       S.firings[i] = firings[i]; S.empty[i] = 0; S.consumed[i] = consumed[i]; S.produced[i] = produced[i];
-      S.active_ne[i] = active[i]; S.busy_ns[i] = i == 0 ? busy_ns : 0; S.spilled[i] = 0; S.overruns[i] = 0;
+      S.active_ne[i] = active[i]; S.active_win[i] = active[i]; S.busy_ns[i] = i == 0 ? busy_ns : 0;
+      S.spilled[i] = 0; S.overruns[i] = 0;
       S.stalls[i] = 0; S.max_queue[i] = 0;
       S.lateness[i] = 0; S.sched_cycles[i] = 0; S.max_fire_ns[i] = 0;
       for (int k = 0; k < 6; ++k) S.phase_cycles[i][k] = 0;

@@ -37,6 +37,7 @@ struct CtaStats {
   uint64_t consumed[PL_MAX_STAGES];
   uint64_t produced[PL_MAX_STAGES];
   int64_t  active_ne[PL_MAX_STAGES];    // sum |[s,s+t_i) ∩ [0,H)| over non-empty firings
+  int64_t  active_win[PL_MAX_STAGES];   // the charged active time over [0,H) (R-WINDOW; R-DRAIN)
   int64_t  busy_ns[PL_MAX_STAGES];
   uint64_t spilled[PL_MAX_STAGES];
   uint64_t overruns[PL_MAX_STAGES];

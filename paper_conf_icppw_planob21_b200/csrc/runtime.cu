@@ -663,12 +663,7 @@ pl_status pl_pipeline_stats(pl_pipeline* pl, pl_stats* out) {
       out->sched_cycles[i] += s.sched_cycles[i];
       out->max_fire_ns[i] = std::max(out->max_fire_ns[i], s.max_fire_ns[i]);
       for (int k = 0; k < 6; ++k) out->phase_cycles[i][k] += s.phase_cycles[i][k];
-      if (pl->cfg.policy == PL_FIXED_WAIT) {   // every firing m*P_i < H is charged (L97, R-WINDOW)
-        const int64_t P = pl->dp.P[i], t = pl->t[i];
-        out->active_window[i] += (H / P) * t + std::min(t, H % P);
-      } else {
-        out->active_window[i] += s.active_ne[i];
-      }
+      out->active_window[i] += s.active_win[i];   // computed per node by the executor
     }
     out->miss_events += s.miss_events;
     out->miss_events_ns += s.miss_events_ns;

@@ -62,7 +62,7 @@ def make_config(cfg, flags=0, device=0, n_streams=None, **over):
     c.seed = int(cfg.seed)
     c.device = int(device)
     c.ns_per_unit = float(getattr(cfg, "ns_per_unit", 1.0))
-    c.flags = int(flags)
+    c.flags = int(flags) | (_pl.PL_EAGER_DRAIN if getattr(cfg, "eager_drain", False) else 0)
     for k, v in over.items():
         setattr(c, k, v)
     return c, keep

@@ -59,6 +59,7 @@ class Config:
     seed: int = 0
     ns_per_unit: float = 1.0
     slack_guard: int = 0         # THRESHOLD_SLACK: extra reserve added to R_i (physical lateness guard)
+    eager_drain: bool = False    # R-DRAIN: work-conserving firing once the stream's last root has arrived
     # DNA workload recipe (plgen.dna.make_dna kwargs); None for gain-model pipelines
     dna: Optional[dict] = None
 

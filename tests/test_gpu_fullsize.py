@@ -30,6 +30,16 @@ def test_c2_full_size_logical(c2wl, policy):
     compare(cfg, g, o)
 
 
+@pytest.mark.parametrize("policy", [C.FIXED_WAIT, C.THRESHOLD_SLACK])
+def test_c2_full_size_eager_drain(c2wl, policy):
+    """R-DRAIN at full size (the bench's end-of-stream rule)."""
+    cfg, wl = c2wl
+    cfg = cfg.replace(wait_time=W_PAPER, wait_threshold=(128, 127, 99, 10), policy=policy, eager_drain=True)
+    g = run_gpu(cfg, wl)
+    o = run_oracle_parallel(cfg, wl)
+    compare(cfg, g, o)
+
+
 @pytest.fixture(scope="module")
 def budgets(c2wl):
     """B200 service-time budgets (ns) measured the way bench.py does (realtime.calibrate_budgets),

@@ -174,3 +174,70 @@ def test_poisson_arrivals_dna(policy):
     arr = A.poisson(3, A.stream_sizes(wl.db_len - 6 + 1, cfg.n_streams), cfg.interarrival)
     g = run_gpu(cfg, wl, arrivals=arr)
     compare(cfg, g, run_oracle(cfg, wl, arrivals=arr))
+
+
+# ---------------------------------------------------------------- end of stream (R-DRAIN)
+
+@pytest.mark.parametrize("policy", [C.FIXED_WAIT, C.THRESHOLD_SLACK])
+@pytest.mark.parametrize("streams,X", [(1, 5000), (3, 3001), (7, 777)])
+def test_eager_drain_gain_model(policy, streams, X):
+    cfg = _c1(policy, n_streams=streams, n_roots=X).replace(eager_drain=True)
+    compare(cfg, run_gpu(cfg, None), run_oracle(cfg, None))
+
+
+@pytest.mark.parametrize("policy", [C.FIXED_WAIT, C.THRESHOLD_SLACK])
+def test_eager_drain_blast_gain_model(policy):
+    tau, D = 10, 50_000
+    cfg = C.gain_model_blast(interarrival=tau, deadline=D, n_streams=4, n_roots=6000, seed=3, eager_drain=True)
+    Pc, _ = SV.fig1_continuous(C.TABLE1_T, C.TABLE1_G, C.PAPER_B, 128, tau, D)
+    if policy == C.FIXED_WAIT:
+        cfg = cfg.replace(wait_time=tuple(int(Pc[i]) - C.TABLE1_T[i] for i in range(4)))
+    else:
+        cfg = cfg.replace(policy=policy, wait_threshold=tuple(SV.thresholds(C.TABLE1_G, [int(x) for x in Pc], tau, 128)))
+    compare(cfg, run_gpu(cfg, None), run_oracle(cfg, None))
+
+
+@pytest.mark.parametrize("policy", [C.FIXED_WAIT, C.THRESHOLD_SLACK])
+def test_eager_drain_dna(policy):
+    cfg = _dna(policy).replace(eager_drain=True)
+    wl = workload_for(cfg)
+    compare(cfg, run_gpu(cfg, wl), run_oracle(cfg, wl))
+
+
+@pytest.mark.parametrize("policy", [C.FIXED_WAIT, C.THRESHOLD_SLACK])
+def test_eager_drain_dna_forced_spill(policy):
+    cfg = _dna(policy, streams=3).replace(eager_drain=True)
+    wl = workload_for(cfg)
+    g = run_gpu(cfg, wl, queue_capacity=64)
+    assert sum(g["stats"]["spilled"]) > 0
+    compare(cfg, g, run_oracle(cfg, wl))
+
+
+@pytest.mark.parametrize("policy", [C.FIXED_WAIT, C.THRESHOLD_SLACK])
+def test_eager_drain_poisson(policy):
+    from plgen import arrivals as A
+    cfg = _c1(policy, n_streams=4, n_roots=3000).replace(eager_drain=True)
+    arr = A.poisson(11, A.stream_sizes(cfg.n_roots * cfg.n_streams, cfg.n_streams), cfg.interarrival)
+    compare(cfg, run_gpu(cfg, None, arrivals=arr), run_oracle(cfg, None, arrivals=arr))
+
+
+def test_eager_drain_eight_nodes():
+    st = [C.Stage(C.BERNOULLI, 0.8, 1), C.Stage(C.POISSON_CAPPED, 1.3, 4), C.Stage(C.BERNOULLI, 0.6, 1),
+          C.Stage(C.FIXED_GAIN, 2.0, 2), C.Stage(C.BERNOULLI, 0.5, 1), C.Stage(C.KEEP_EVERY, 3.0, 1),
+          C.Stage(C.POISSON_CAPPED, 0.9, 3), C.Stage(C.BERNOULLI, 0.7, 1)]
+    cfg = C.Config(name="n8e", stages=st, service_time=(40, 55, 30, 45, 25, 35, 50, 20), vector_width=128,
+                   deadline=20_000, interarrival=3, b=(1,) * 8, wait_time=(300, 100, 50, 80, 40, 60, 90, 30),
+                   n_streams=3, n_roots=3000, seed=5, eager_drain=True)
+    compare(cfg, run_gpu(cfg, None), run_oracle(cfg, None))
+
+
+@pytest.mark.parametrize("policy", [C.FIXED_WAIT, C.THRESHOLD_SLACK])
+def test_eager_drain_physical_replay(policy):
+    """Under %globaltimer the drain commits the logical schedule and shortens the run."""
+    cfg = _dna(policy, db_len=1 << 15, streams=3).replace(
+        clock=C.CLOCK_GLOBALTIMER, ns_per_unit=1.0, service_time=(20_000,) * 4, interarrival=400,
+        deadline=10**7, wait_time=(31_200, 60_000, 80_000, 100_000), wait_threshold=(64, 32, 16, 8), eager_drain=True)
+    wl = workload_for(cfg)
+    g = run_gpu(cfg, wl)
+    compare(cfg, g, run_oracle(cfg, wl))
+    assert (g["lat_ns"] > 0).all()

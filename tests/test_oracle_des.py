@@ -331,3 +331,99 @@ def test_p6_enumeration_with_arrival_times(arr):
         log = tuple((i, s, n) for (i, s, n, _, _) in r.firings)
         assert log in allsched, (policy, prm, log)
         assert allsched[log] == tuple(r.lat)
+
+
+# ------------------------------------------------------------- end of stream (R-DRAIN)
+
+@pytest.mark.parametrize("tau,P,t0,v,X", [(4, 128, 64, 32, 97), (3, 10, 7, 4, 23), (5, 5, 5, 1, 9), (2, 9, 1, 8, 40),
+                                          (3, 10, 7, 4, 1)])
+def test_drain_fixed_wait_single_node_closed_form(tau, P, t0, v, X):
+    """R-DRAIN on one FIXED_WAIT node (P <= v tau0): roots whose slot ceil(r tau/P) P precedes
+    A_last = (X-1) tau keep P2's latency; the rest leave in one drain firing at
+    s = max(A_last, end of the last slot before A_last)."""
+    assert P <= v * tau
+    cfg = C.Config(name="dr", stages=[C.Stage(C.KEEP_EVERY, 1.0, 1)], service_time=(t0,),
+                   vector_width=v, deadline=10**9, interarrival=tau, b=(1,), wait_time=(P - t0,),
+                   n_roots=X, eager_drain=True)
+    r = des.run(cfg)
+    A = (X - 1) * tau
+    M = -(-A // P)                                 # slots m P < A_last
+    s = max(A, (M - 1) * P + t0) if M else A
+    for rr in range(X):
+        slot = -(-rr * tau // P)
+        expect = slot * P - rr * tau + t0 if slot < M else s + t0 - rr * tau
+        assert r.lat[rr] == expect, (rr, r.lat[rr], expect)
+    assert r.streams[0].T_end == max(r.lat[rr] + rr * tau for rr in range(X))
+
+
+@pytest.mark.parametrize("tau,t0,v,X", [(4, 64, 32, 100), (3, 5, 4, 23), (1, 8, 8, 64), (2, 3, 4, 6)])
+def test_drain_threshold_single_node_closed_form(tau, t0, v, X):
+    """R-DRAIN on one THRESHOLD_SLACK node (theta = v, no slack force): full groups fire at
+    their v-th arrival; the last partial group at max(A_last, end of the last full group)."""
+    D = 10**6
+    assert t0 <= v * tau
+    cfg = C.Config(name="drt", stages=[C.Stage(C.KEEP_EVERY, 1.0, 1)], service_time=(t0,),
+                   vector_width=v, deadline=D, interarrival=tau, b=(1,), wait_threshold=(v,),
+                   policy=C.THRESHOLD_SLACK, n_roots=X, eager_drain=True)
+    r = des.run(cfg)
+    full = (X // v) * v
+    for rr in range(full):
+        assert r.lat[rr] == (v - 1 - rr % v) * tau + t0
+    s = max((X - 1) * tau, (full - 1) * tau + t0 if full else 0)
+    for rr in range(full, X):
+        assert r.lat[rr] == s + t0 - rr * tau
+
+
+@pytest.mark.parametrize("policy", [C.FIXED_WAIT, C.THRESHOLD_SLACK])
+@pytest.mark.parametrize("seed", [0, 1, 2, 3])
+def test_drain_changes_nothing_before_last_arrival(policy, seed):
+    """R-DRAIN acts only at T >= A_last: every firing that starts earlier is identical, and
+    the invariants of P4 hold throughout."""
+    rnd = random.Random(seed)
+    N = rnd.randint(2, 4)
+    t = [rnd.randint(3, 30) for _ in range(N)]
+    cfg = gm_cfg(N, t, [rnd.randint(0, 50) for _ in range(N)], rnd.choice([4, 8]), rnd.randint(1, 6),
+                 rnd.randint(50, 300), seed=seed, policy=policy,
+                 theta=[rnd.randint(1, 4) for _ in range(N)], D=rnd.randint(100, 400))
+    a = des.run(cfg)
+    b = des.run(cfg.replace(eager_drain=True), check_invariants=True)
+    A = (cfg.n_roots - 1) * cfg.interarrival
+    fa = [f for f in a.streams[0].firings if f[1] < A]
+    fb = [f for f in b.streams[0].firings if f[1] < A]
+    assert fa == fb
+    assert b.matches == a.matches and b.trace == a.trace          # the data path does not depend on it
+    assert b.streams[0].T_end <= a.streams[0].T_end
+
+
+@pytest.mark.parametrize("X,tau", [(3, 1), (4, 2)])
+def test_drain_schedule_enumeration(X, tau):
+    """P6 for R-DRAIN: the DES schedule is one of the enumerated fire/wait schedules, and the
+    independent stepper driven by the rule written out here reproduces it exactly."""
+    N, t, v = 2, (2, 3), 2
+    fns = _toy_fns()
+    D = 12
+    A = (X - 1) * tau
+    allsched = _enumerate_all(N, t, v, tau, X, fns, horizon=X * tau + 14)
+    for policy in (C.FIXED_WAIT, C.THRESHOLD_SLACK):
+        params = ([(0, 0), (1, 0), (0, 2), (2, 1), (3, 3)] if policy == C.FIXED_WAIT
+                  else [(1, 1), (2, 1), (2, 2), (1, 2)])
+        for prm in params:
+            cfg = C.Config(name="p6d", stages=[C.Stage(C.KEEP_EVERY, 1), C.Stage(C.KEEP_EVERY, 1)],
+                           service_time=t, vector_width=v, deadline=D, interarrival=tau, b=(1, 1),
+                           wait_time=prm if policy == C.FIXED_WAIT else None,
+                           wait_threshold=prm if policy == C.THRESHOLD_SLACK else None,
+                           policy=policy, n_roots=X, eager_drain=True)
+            r = des.simulate_stream(cfg, fns, 0, X)
+            log = tuple((i, s, n) for (i, s, n, _, _) in r.firings)
+            assert log in allsched, (policy, prm, log)
+            assert allsched[log][0] == tuple(r.lat)
+            if policy == C.FIXED_WAIT:
+                P = [t[i] + prm[i] for i in range(N)]
+                rule = lambda T, Q, b: [i for i in range(N)
+                                        if (T < A and T % P[i] == 0) or (T >= A and b[i] is None and Q[i])]
+            else:
+                R = [t[0] + 2 * t[1], t[1]]
+                rule = lambda T, Q, b: [i for i in range(N) if b[i] is None and Q[i] and (
+                    len(Q[i]) >= prm[i] or T >= Q[i][0][0] * tau + D - R[i] or T >= A)]
+            lat2, log2 = _enum_step_semantics(N, t, v, tau, X, fns, rule)
+            assert lat2 == tuple(r.lat) and tuple(log2) == log, (policy, prm)
