@@ -53,6 +53,14 @@ def budgets(c2wl):
     return t
 
 
+def _tau_for(budgets, floor):
+    """A rate 1.5x above the Fig. 1 feasibility limit of the measured budgets (>= floor)."""
+    from paper_conf_icppw_planob21_b200 import realtime
+    probe = C.c2(n_streams=148).replace(clock=C.CLOCK_GLOBALTIMER, ns_per_unit=1.0, service_time=budgets,
+                                         deadline=350_000, gain=(0.2234, 1.1469, 0.07856))
+    return max(floor, int(1.5 * realtime.min_feasible_tau(probe)))
+
+
 def _phys_cfg(t, tau, D=350_000):
     from paper_conf_icppw_planob21_b200 import solve_enforced_waits
     cfg = C.c2(n_streams=148).replace(clock=C.CLOCK_GLOBALTIMER, ns_per_unit=1.0, service_time=t,
@@ -69,7 +77,7 @@ def test_physical_replays_logical_schedule(c2wl, budgets, fixed_service):
     latencies and busy time agree with the logical prediction within 5 %; publishing as
     soon as done (default) the prediction is an upper bound up to the measured lateness."""
     _, wl = c2wl
-    cfg = _phys_cfg(budgets, 40)
+    cfg = _phys_cfg(budgets, _tau_for(budgets, 40))
     g = run_gpu(cfg, wl, flags=7 | (8 if fixed_service else 0))
     o = run_oracle_parallel(cfg, wl)
     compare(cfg, g, o)
@@ -92,8 +100,10 @@ def test_physical_replays_logical_schedule(c2wl, budgets, fixed_service):
 
 
 def test_physical_zero_misses_at_bench_rate(c2wl, budgets):
+    """Zero measured misses at a rate 1.5x above the Fig. 1 feasibility limit of the budgets
+    (at least tau0 = 30 ns)."""
     _, wl = c2wl
-    cfg = _phys_cfg(budgets, 30)
+    cfg = _phys_cfg(budgets, _tau_for(budgets, 30))
     g = run_gpu(cfg, wl, flags=1)
     st = g["stats"]
     assert st["misses"] == 0 and st["errors"] == 0
