@@ -126,7 +126,7 @@ def monolithic_at(cfg, tau):
 
 
 def calibrate_b(cfg, wl=None, db_dev=None, target=0.95, quantile=0.95, max_iter=10, log=None, stream=None,
-                arrivals=None):
+                arrivals=None, over=None):
     """The paper's empirical b calibration, run on the device.
 
     Start from b = 1 ("optimistic ... worst-case closely matches the average"), solve Fig. 1,
@@ -146,7 +146,7 @@ def calibrate_b(cfg, wl=None, db_dev=None, target=0.95, quantile=0.95, max_iter=
         except RuntimeError:
             return dict(b=tuple(b), w=None, T=None, miss_free=0.0, iterations=it, history=hist, infeasible=True)
         c = c.replace(wait_time=tuple(w))
-        pl = Pipeline(c, wl, flags=1, stream=stream, arrivals=arrivals)
+        pl = Pipeline(c, wl, flags=1, stream=stream, arrivals=arrivals, **(over or {}))
         if wl is not None:
             pl.bind_device(db_dev, wl.db_len)
         else:
