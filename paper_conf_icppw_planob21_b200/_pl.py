@@ -91,7 +91,7 @@ class pl_stats(C.Structure):
 
 def _load():
     if not os.path.exists(LIB_PATH):
-        raise ImportError(f"{LIB_PATH} not built — run `python -m paper_conf_icppw_planob21_b200.build` "
+        raise ImportError(f"{LIB_PATH} not built — run `python paper_conf_icppw_planob21_b200/build.py` "
                           "(there is no CPU fallback)")
     lib = C.CDLL(LIB_PATH)
     P = C.c_void_p

@@ -9,6 +9,14 @@ if ROOT not in sys.path:
 
 
 def pytest_configure(config):
+    # The C-ABI library is a git-ignored build artefact: (re)build it in-tree when it is
+    # missing or older than its sources, so a fresh checkout tests the current code.
+    import importlib.util
+    spec = importlib.util.spec_from_file_location(
+        "_plgpu_build", os.path.join(ROOT, "paper_conf_icppw_planob21_b200", "build.py"))
+    mod = importlib.util.module_from_spec(spec)
+    spec.loader.exec_module(mod)
+    mod.build()
     config.addinivalue_line("markers", "gpu: needs a CUDA device (B200, sm_100a)")
     config.addinivalue_line("markers", "slow: statistical / long-running oracle pins")
 
