@@ -53,6 +53,9 @@ def parse():
     ap.add_argument("--cpu-sample-streams", type=int, default=148)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--budget-margin", type=float, default=1.25)
+    ap.add_argument("--budget-slack", type=int, default=256)
+    ap.add_argument("--refine", type=int, default=0, help="budget refinement rounds at the operating point")
     ap.add_argument("--drain", default="eager", choices=["eager", "periodic"],
                     help="end of stream: R-DRAIN work-conserving drain (PL_EAGER_DRAIN) or the periodic rule")
     return ap.parse_args()
@@ -221,7 +224,13 @@ def main():
 
     # 1. gains (logical run) and budgets (physical run)
     gains = realtime.measure_gains(base.replace(wait_time=(0,) * 4), wl, db_ptr, stream=stream)
-    budgets, cal = realtime.calibrate_budgets(base, wl, db_ptr, stream=stream)
+    budgets, cal = realtime.calibrate_budgets(base, wl, db_ptr, stream=stream, margin=a.budget_margin,
+                                              slack_ns=a.budget_slack)
+    if a.refine:
+        cfg_r = base.replace(clock=1, ns_per_unit=1.0, service_time=budgets, gain=gains, deadline=a.deadline_ns,
+                             b=C.PAPER_B, eager_drain=a.drain == "eager")
+        budgets, _ = realtime.refine_budgets(cfg_r, wl, db_ptr, budgets, margin=a.budget_margin,
+                                             slack_ns=a.budget_slack, rounds=a.refine, stream=stream, log=log)
     if world > 1:   # every rank runs the same schedule: max budgets / min gains are conservative
         t = torch.tensor(budgets, dtype=torch.int64, device=dev)
         dist.all_reduce(t, op=dist.ReduceOp.MAX)

@@ -168,6 +168,9 @@ typedef struct {
   int64_t  max_lateness_ns[PL_MAX_STAGES]; /* physical: max(actual - scheduled start)  */
   uint64_t sched_cycles[PL_MAX_STAGES];    /* clock64 cycles spent deciding firings    */
   int64_t  max_fire_ns[PL_MAX_STAGES];     /* physical: longest firing (start->publish) */
+  int64_t  max_loop_ns[PL_MAX_STAGES];     /* physical: longest cycle from a firing's start to the
+                                              node's next decision (not counting waits for upstream):
+                                              the real per-firing service time, incl. bookkeeping */
   /* leader-lane clock64 cycles per phase of a firing, summed over firings:
    * [0] decide (scheduler), [1] release barrier, [2] load+stage+scan,
    * [3] records+reserve, [4] output writes, [5] publish                        */

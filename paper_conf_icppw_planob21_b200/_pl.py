@@ -68,7 +68,7 @@ class pl_stats(C.Structure):
                 ("firings", _A8), ("empty_firings", _A8), ("consumed", _A8), ("produced", _A8),
                 ("active_window", _I8), ("busy_ns", _I8), ("spilled", _A8), ("overruns", _A8), ("stalls", _A8),
                 ("max_queue", C.c_uint32 * PL_MAX_STAGES),
-                ("max_lateness_ns", _I8), ("sched_cycles", _A8), ("max_fire_ns", _I8),
+                ("max_lateness_ns", _I8), ("sched_cycles", _A8), ("max_fire_ns", _I8), ("max_loop_ns", _I8),
                 ("phase_cycles", (C.c_uint64 * 6) * PL_MAX_STAGES), ("matches", C.c_uint64),
                 ("miss_events", C.c_uint64), ("miss_events_ns", C.c_uint64), ("misses", C.c_uint64),
                 ("max_latency", C.c_int64),

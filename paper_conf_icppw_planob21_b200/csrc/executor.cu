@@ -24,9 +24,6 @@ namespace {
 
 constexpr uint32_t LOC_SMEM = 0, LOC_SPILL = 1;
 constexpr uint32_t NO_ROOT = 0xffffffffu;
-// physical clock: a stream's time origin is set this far after its CTA starts, so that
-// every warp group is resident and warm before the first arrival (absorbs start-up lateness)
-constexpr uint64_t PL_T0_OFFSET_NS = 2048;
 
 __device__ __forceinline__ uint64_t gtimer() {
   uint64_t t;
@@ -71,6 +68,8 @@ struct Dna {
   int64_t win_lo;
   uint32_t win_lo32;        // (uint32_t)win_lo: window word index arithmetic in 32 bits
   uint32_t win_n;
+  bool nofast;             // experiment switch (PL_VARIANT & 16): always the checked walk
+  const uint8_t* s2tab;    // smem: max(0, max prefix score) of an 8-step walk by mismatch pattern
   const uint32_t* qw;      // query words (smem), nqw valid words
   uint32_t nqw;
   const uint16_t* qoff;    // smem
@@ -137,6 +136,116 @@ struct Dna {
     *dbest = db_;
     return best;
   }
+  // Fast form of extend() for both walks of one seed whose DB words all lie in the smem
+  // window (in_win): the left walk (ll steps), then the right walk (rl steps), in ONE loop,
+  // so that a warp iterates max over lanes of (left + right) 16-base steps rather than
+  // max(left) + max(right) (seeds on one planted diagonal split it at different points).
+  // 32-bit indices, no per-word range checks, one new DB word and one new query word per
+  // step (the shift is the same for every step of a walk).  The query copy in smem carries
+  // zero pad words on both sides (layout_enforced), so reads past either end are in bounds;
+  // bases past a walk's limit are masked as in extend().  Scoring and X-drop as extend().
+  __device__ __forceinline__ void extend2_win(uint32_t p, uint32_t q, uint32_t ll, uint32_t rl, int X, int* bl,
+                                              int* dl, int* br, int* dr) const {
+    // left walk: step d+1+e compares db[p-d-1-e] with query[q-d-1-e]; its first 16-base
+    // window is [p-16, p) = words (w, w+1), w = (p-16)>>4; later windows slide down a word
+    int32_t sd = (int32_t)p - 16, sq = (int32_t)q - 16;
+    const uint32_t* dw = win + ((sd >> 4) - (int32_t)win_lo32);    // next word to load
+    const uint32_t* qp = qw + (sq >> 4);
+    uint32_t shd = (uint32_t)(sd & 15) * 2u, shq = (uint32_t)(sq & 15) * 2u;
+    uint32_t dc = dw[1], qc = qp[1];                                  // carried word
+    int step = -1;
+    bool right = false;
+    uint32_t limit = ll, d = 0;
+    int score = 0, best = 0, db_ = 0;
+    for (;;) {
+      bool fin = d >= limit;
+      if (!fin) {
+        const uint32_t dn = *dw, qn = *qp;
+        dw += step;
+        qp += step;
+        const uint32_t x = right ? (__funnelshift_r(dc, dn, shd) ^ __funnelshift_r(qc, qn, shq))
+                                 : (__funnelshift_r(dn, dc, shd) ^ __funnelshift_r(qn, qc, shq));
+        dc = dn;
+        qc = qn;
+        uint32_t mm = (x | (x >> 1)) & 0x55555555u;   // bit 2e set <=> mismatch at step d+1+e
+        if (!right) mm = __brev(mm) >> 1;             // left: window position 15-e is step d+1+e
+        const uint32_t n = (limit - d) < 16u ? (limit - d) : 16u;
+        uint32_t mmv = mm & (n >= 16u ? 0xffffffffu : ((1u << (2u * n)) - 1u));
+        int last = 0;
+        while (mmv) {
+          const int e = (__ffs(mmv) - 1) >> 1;
+          mmv &= mmv - 1;
+          score += e - last;
+          if (score > best) { best = score; db_ = (int)d + e; }
+          score -= 3;
+          last = e + 1;
+          if (X > 0 && score <= best - X) { fin = true; break; }
+        }
+        if (!fin) {
+          score += (int)n - last;
+          if (score > best) { best = score; db_ = (int)(d + n); }
+          d += n;
+        }
+      }
+      if (fin) {
+        if (right) break;
+        *bl = best;
+        *dl = db_;
+        // right walk: step d+1+e compares db[p+k+d+e] with query[q+k+d+e]; first window
+        // [p+k, p+k+16) = words (w, w+1), w = (p+k)>>4; later windows slide up a word
+        right = true;
+        step = 1;
+        limit = rl;
+        d = 0;
+        score = best = db_ = 0;
+        sd = (int32_t)(p + (uint32_t)k);
+        sq = (int32_t)(q + (uint32_t)k);
+        dw = win + ((sd >> 4) - (int32_t)win_lo32);
+        qp = qw + (sq >> 4);
+        shd = (uint32_t)(sd & 15) * 2u;
+        shq = (uint32_t)(sq & 15) * 2u;
+        dc = *dw++;
+        qc = *qp++;
+      }
+    }
+    *br = best;
+    *dr = db_;
+  }
+  // 16 bases starting at s (s >= win_lo * 16, in the window) / at query position s >= -16
+  __device__ __forceinline__ uint32_t db16w(int32_t s) const {
+    const uint32_t* w = win + ((s >> 4) - (int32_t)win_lo32);
+    return __funnelshift_r(w[0], w[1], (uint32_t)(s & 15) * 2u);
+  }
+  __device__ __forceinline__ uint32_t q16w(int32_t s) const {
+    const uint32_t* w = qw + (s >> 4);
+    return __funnelshift_r(w[0], w[1], (uint32_t)(s & 15) * 2u);
+  }
+  // bits 0, 2, .., 14 of x -> bits 0..7
+  static __device__ __forceinline__ uint32_t even_bits8(uint32_t x) {
+    x &= 0x5555u;
+    x = (x | (x >> 1)) & 0x3333u;
+    x = (x | (x >> 2)) & 0x0f0fu;
+    return (x | (x >> 4)) & 0x00ffu;
+  }
+  // S2 for limits ll, rl <= 8 (R-S2): best_left + best_right of the two +1/-3 walks, each
+  // looked up in the 256-entry table of max(0, max prefix score) over its 8-step mismatch
+  // pattern (bit e: mismatch at step e+1).  Steps past a limit are marked as mismatches,
+  // which never raise a prefix maximum, so the table value is the walk's best.  Needs in_win.
+  __device__ __forceinline__ int s2_best8(uint32_t p, uint32_t q, uint32_t ll, uint32_t rl) const {
+    const uint32_t xr = db16w((int32_t)(p + (uint32_t)k)) ^ q16w((int32_t)(q + (uint32_t)k));
+    const uint32_t xl = db16w((int32_t)p - 16) ^ q16w((int32_t)q - 16);
+    const uint32_t mr = even_bits8(xr | (xr >> 1)) | ((0xffu << rl) & 0xffu);
+    const uint32_t ml = even_bits8(__brev((xl | (xl >> 1)) & 0x55555555u) >> 1) | ((0xffu << ll) & 0xffu);
+    return (int)s2tab[ml] + (int)s2tab[mr];
+  }
+  // Every DB word a walk of ll bases left of p and rl bases right of the seed may read
+  // (extend_win reads whole 16-base steps plus one word ahead) lies in the smem window.
+  __device__ __forceinline__ bool in_win(uint32_t p, uint32_t ll, uint32_t rl) const {
+    if (nofast) return false;
+    const int32_t lo = ((int32_t)p - (int32_t)ll - 32) >> 4;
+    const int32_t hi = (int32_t)((p + (uint32_t)k + rl + 32u) >> 4);
+    return lo >= (int32_t)win_lo32 && hi < (int32_t)(win_lo32 + win_n);
+  }
   __device__ __forceinline__ int64_t right_limit(uint32_t p, uint32_t q) const {
     const int64_t a = (int64_t)db_len - ((int64_t)p + k), b = (int64_t)q_len - ((int64_t)q + k);
     const int64_t m = a < b ? a : b;
@@ -175,7 +284,8 @@ struct NodeAcc {
   alignas(16) unsigned long long ph[6];
   alignas(16) uint32_t d[D_N];
   long long t_end;
-  uint32_t max_queue, lateness, max_fire, lmax, lmax_ns, nmiss, nmiss_ns, pad;
+  uint32_t max_queue, lateness, max_fire, lmax, lmax_ns, nmiss, nmiss_ns;
+  uint32_t max_loop;   // physical: longest firing-to-next-decision cycle (the node's real service time)
 };
 struct Shared {
   EdgeCtl e[PL_MAX_STAGES];
@@ -336,17 +446,28 @@ __device__ __forceinline__ LaneOut stage_count_ext(const Node& nd, const Dna& dn
   LaneOut o;
   o.c = 0; o.a = 0; o.score = 0; o.q_start = 0; o.len = 0;
   const uint32_t q = e.y & 0xffffu;
+  // both limits are <= q_len, so they fit 32 bits
+  uint32_t ll = (uint32_t)dna.left_limit(e.x, q), rl = (uint32_t)dna.right_limit(e.x, q);
   if (nd.kind == PL_UNGAPPED_WINDOW) {
-    const int64_t W = nd.ip1;
-    int d;
-    const int64_t ll = dna.left_limit(e.x, q), rl = dna.right_limit(e.x, q);
-    const int bl = dna.extend(e.x, q, -1, ll < W ? ll : W, 0, &d);
-    const int br = dna.extend(e.x, q, +1, rl < W ? rl : W, 0, &d);
+    const uint32_t W = (uint32_t)nd.ip1;
+    ll = ll < W ? ll : W;
+    rl = rl < W ? rl : W;
+  }
+  const int X = nd.kind == PL_UNGAPPED_WINDOW ? 0 : nd.ip1;
+  int dl, dr, bl, br;
+  if (nd.kind == PL_UNGAPPED_WINDOW && nd.ip1 <= 8 && dna.in_win(e.x, ll, rl)) {
+    o.c = (dna.k + dna.s2_best8(e.x, q, ll, rl) >= nd.ip2) ? 1u : 0u;
+    return o;
+  }
+  if (dna.in_win(e.x, ll, rl)) {
+    dna.extend2_win(e.x, q, ll, rl, X, &bl, &dl, &br, &dr);
+  } else {
+    bl = dna.extend(e.x, q, -1, ll, X, &dl);
+    br = dna.extend(e.x, q, +1, rl, X, &dr);
+  }
+  if (nd.kind == PL_UNGAPPED_WINDOW) {
     o.c = (dna.k + bl + br >= nd.ip2) ? 1u : 0u;
   } else {
-    int dl, dr;
-    const int bl = dna.extend(e.x, q, -1, dna.left_limit(e.x, q), nd.ip1, &dl);
-    const int br = dna.extend(e.x, q, +1, dna.right_limit(e.x, q), nd.ip1, &dr);
     const int score = dna.k + bl + br;
     if (score >= nd.ip2) {
       o.c = 1;
@@ -541,7 +662,7 @@ __device__ __forceinline__ void advance0(const Node& nd, Rep& r) {
 }
 
 // Nodes i >= 1: the leader decides from the published queue state and watermark.
-__device__ Decision decide(const Node& nd, Leader& L) {
+__device__ Decision decide(const Node& nd, Leader& L, bool& waited) {
   const uint32_t v = (uint32_t)nd.v;
   Decision d;
   d.done = false; d.T = 0; d.n = 0; d.qlen = 0;
@@ -559,14 +680,14 @@ __device__ Decision decide(const Node& nd, Leader& L) {
         if (!any) {
           if (Wup == PL_INF64) { d.done = true; return d; }
           publish_W(nd, L, max(B, Wup) + nd.t);
-          backoff(spins);
+          backoff(spins); waited = true;
           continue;
         }
         const int64_t Te = max(B, nd.in_seg[L.segh & nd.segmask].ready);
         const uint32_t cnt = count_le(nd, L, st, Te);
         publish_W(nd, L, Te + nd.t);     // the firing starts at Te; only its size is pending
         if (Wup > Te || cnt >= v) { d.T = Te; d.n = cnt < v ? cnt : v; d.qlen = tail_known - L.head; return d; }
-        backoff(spins);
+        backoff(spins); waited = true;
         continue;
       }
       const int64_t T = L.m * nd.P;
@@ -585,14 +706,14 @@ __device__ Decision decide(const Node& nd, Leader& L) {
         continue;
       }
       publish_W(nd, L, T + nd.t);
-      backoff(spins);
+      backoff(spins); waited = true;
       continue;
     }
     // THRESHOLD_SLACK
     if (!any) {
       if (Wup == PL_INF64) { d.done = true; return d; }
       publish_W(nd, L, (Wup > L.B ? Wup : L.B) + nd.t);
-      backoff(spins);
+      backoff(spins); waited = true;
       continue;
     }
     const Seg& hs = nd.in_seg[L.segh & nd.segmask];
@@ -625,7 +746,7 @@ __device__ Decision decide(const Node& nd, Leader& L) {
     int64_t lb = Tk < Wup ? Tk : Wup;
     if (lb < L.B) lb = L.B;
     publish_W(nd, L, lb + nd.t);
-    backoff(spins);
+    backoff(spins); waited = true;
   }
 }
 
@@ -646,8 +767,9 @@ __device__ uint32_t reserve_out(const Node& nd, Leader& L, uint32_t worst, uint3
   }
 }
 
-__device__ __forceinline__ void pace(uint64_t target, uint64_t* start_ns, int64_t* late) {
+__device__ __forceinline__ void pace(uint64_t target, uint64_t* start_ns, int64_t* late, uint64_t* entry_ns = nullptr) {
   uint64_t now = gtimer();
+  if (entry_ns) *entry_ns = now;
   while (now < target) {   // __nanosleep rounds up to powers of two: sleep at most ~rem/4
     const uint64_t rem = target - now;
     __nanosleep(rem > 4096 ? 1024 : (rem > 1024 ? 256 : (rem > 256 ? 64 : 0)));
@@ -826,7 +948,7 @@ __device__ void run_node(Ctx& c, const Dna dna, int i, int gtid) {
     for (int k = 0; k < D_N; ++k) A.d[k] = 0;
     for (int k = 0; k < 8; ++k) G.rmin[k] = NO_ROOT;   // slots of absent warps stay NO_ROOT
     A.t_end = 0;
-    A.max_queue = A.lateness = A.max_fire = A.lmax = A.lmax_ns = A.nmiss = A.nmiss_ns = 0;
+    A.max_queue = A.lateness = A.max_fire = A.lmax = A.lmax_ns = A.nmiss = A.nmiss_ns = A.max_loop = 0;
   }
 
   for (;;) {
@@ -850,21 +972,28 @@ __device__ void run_node(Ctx& c, const Dna dna, int i, int gtid) {
       if (nd.phys && (p.variant & 1u)) {  // the leader paces, one barrier releases the lanes
         if (leader) {
           int64_t late;
-          pace(T0 + units_ns(nd, T), &start_ns, &late);
+          uint64_t entry;
+          const uint64_t prev = start_ns;
+          pace(T0 + units_ns(nd, T), &start_ns, &late, &entry);
           atomicMax(&A.lateness, clamp32(late));
+          if (prev) atomicMax(&A.max_loop, clamp32((int64_t)(entry - prev)));
         }
         bar_sync(bidA, v);
         if (leader) tc = clock64();
       } else if (nd.phys && (gtid & 31) == 0) {   // every warp paces itself against %globaltimer
-        uint64_t s_ns; int64_t late;
-        pace(T0 + units_ns(nd, T), &s_ns, &late);
-        if (leader) { start_ns = s_ns; atomicMax(&A.lateness, clamp32(late)); tc = clock64(); }
+        uint64_t s_ns, entry; int64_t late;
+        pace(T0 + units_ns(nd, T), &s_ns, &late, &entry);
+        if (leader) {
+          if (start_ns) atomicMax(&A.max_loop, clamp32((int64_t)(entry - start_ns)));
+          start_ns = s_ns; atomicMax(&A.lateness, clamp32(late)); tc = clock64();
+        }
       }
       __syncwarp();
     } else {
       if (leader) {
         const long long c0 = clock64();
-        const Decision d = decide(nd, L);
+        bool waited = false;             // the decision waited for upstream (no service-time sample)
+        const Decision d = decide(nd, L, waited);
         atomicMax(&A.max_queue, d.qlen);
         G.done[par] = d.done ? 1u : 0u;
         G.T[par] = d.T;
@@ -886,8 +1015,11 @@ __device__ void run_node(Ctx& c, const Dna dna, int i, int gtid) {
         A.d[D_PH0] = (uint32_t)(tc - c0);
         if (!d.done && nd.phys) {
           int64_t late;
-          pace(T0 + units_ns(nd, d.T), &start_ns, &late);
+          uint64_t entry;
+          const uint64_t prev = start_ns;
+          pace(T0 + units_ns(nd, d.T), &start_ns, &late, &entry);
           atomicMax(&A.lateness, clamp32(late));
+          if (prev && !waited) atomicMax(&A.max_loop, clamp32((int64_t)(entry - prev)));
           tc = clock64();
         }
       }
@@ -1165,6 +1297,7 @@ __device__ void run_node(Ctx& c, const Dna dna, int i, int gtid) {
     S.lateness[i] = (int64_t)A.lateness;
     S.sched_cycles[i] = A.ph[0];
     S.max_fire_ns[i] = (int64_t)A.max_fire;
+    S.max_loop_ns[i] = (int64_t)A.max_loop;
     for (int k = 0; k < 6; ++k) S.phase_cycles[i][k] = A.ph[k];
     atomicMax((long long*)&S.t_end, (long long)A.t_end);
   }
@@ -1186,10 +1319,13 @@ __host__ __device__ inline uint32_t layout_enforced(const DevParams& p, SmemLayo
   off += dna ? (((1u << (2 * p.k)) + 1u) * 2u + 15u) & ~15u : 0u;
   L->off_qpos = off;
   off += dna ? (((uint32_t)(p.q_len - p.k + 1) * 2u) + 15u) & ~15u : 0u;
-  L->off_qw = off;
-  off += dna ? (((uint32_t)(p.q_len + 15) / 16u) * 4u + 15u) & ~15u : 0u;
+  // packed query with one 16-byte pad on each side (Dna::extend_win reads one word past an end)
+  L->off_qw = off + (dna ? 16u : 0u);
+  off += dna ? 32u + ((((uint32_t)(p.q_len + 15) / 16u) * 4u + 15u) & ~15u) : 0u;
   L->off_win = off;
   off += p.win_cap * 4u;
+  L->off_s2 = off;                // S2 table (Dna::s2_best8): 256 bytes
+  off += dna ? 256u : 0u;
   L->total = off;
   return off;
 }
@@ -1218,6 +1354,18 @@ __device__ void cta_setup(Ctx& c, Shared& sh, unsigned char* dsm, const DevParam
   c.dna.win_lo = 0;
   c.dna.win_lo32 = 0;
   c.dna.win_n = 0;
+  if (s == 0 && tid < 8 && p.summary_next) p.summary_next[tid] = 0ull;   // the next launch's summary slot
+  c.dna.nofast = (p.variant & 16u) != 0;
+  c.dna.s2tab = dsm + Lo.off_s2;
+  if (p.k > 0)   // S2 table: max(0, max prefix) of the 8-step +1/-3 walk, bit e = mismatch at step e+1
+    for (uint32_t m = tid; m < 256u; m += nt) {
+      int sc = 0, best = 0;
+      for (int e = 0; e < 8; ++e) {
+        sc += ((m >> e) & 1u) ? -3 : 1;
+        best = sc > best ? sc : best;
+      }
+      (dsm + Lo.off_s2)[m] = (unsigned char)best;
+    }
   // DNA: the query index (offsets, positions, packed query) and this stream's DB window
   // (its roots plus the k-1 overlap and a halo for the extensions) are staged into smem
   // by TMA bulk copies (cp.async.bulk, one mbarrier), falling back to plain loads for an
@@ -1260,6 +1408,10 @@ __device__ void cta_setup(Ctx& c, Shared& sh, unsigned char* dsm, const DevParam
       while (!done)
         asm volatile("{ .reg .pred q; mbarrier.try_wait.parity.shared::cta.b64 q, [%1], 0; selp.u32 %0, 1, 0, q; }"
                      : "=r"(done) : "r"(bar) : "memory");
+    }
+    if (tid < 8) {   // the query's pad words (outside the TMA destination)
+      uint32_t* qwp = (uint32_t*)(dsm + Lo.off_qw);
+      qwp[tid < 4 ? (int)tid - 4 : (int)(b_qw / 4u + tid - 4u)] = 0u;
     }
     if (!win_tma)
       for (uint32_t j = tid; j < c.dna.win_n; j += nt) {
@@ -1462,7 +1614,7 @@ __device__ void run_monolithic(Ctx& c) {
       S.active_ne[i] = active[i]; S.active_win[i] = active[i]; S.busy_ns[i] = i == 0 ? busy_ns : 0;
       S.spilled[i] = 0; S.overruns[i] = 0;
       S.stalls[i] = 0; S.max_queue[i] = 0;
-      S.lateness[i] = 0; S.sched_cycles[i] = 0; S.max_fire_ns[i] = 0;
+      S.lateness[i] = 0; S.sched_cycles[i] = 0; S.max_fire_ns[i] = 0; S.max_loop_ns[i] = 0;
       for (int k = 0; k < 6; ++k) S.phase_cycles[i][k] = 0;
     }
     S.t_end = t_end;
@@ -1480,7 +1632,7 @@ __global__ void __launch_bounds__(MAXT, MINB) pl_exec_enforced(const __grid_cons
   Ctx c;
   cta_setup(c, sh, dsm, p);
   __syncthreads();
-  if (threadIdx.x == 0) sh.T0 = gtimer() + (p.clock == PL_CLOCK_GLOBALTIMER ? PL_T0_OFFSET_NS : 0);
+  if (threadIdx.x == 0) sh.T0 = gtimer() + (p.clock == PL_CLOCK_GLOBALTIMER ? p.t0_offset_ns : 0u);
   __syncthreads();
   // warp w serves node w % N (local warp w / N): with N = 4 every warp of node i sits on
   // SM sub-partition i, so each SMSP's instruction cache holds one node's code path
@@ -1506,7 +1658,7 @@ __global__ void __launch_bounds__(MAXT, 1) pl_exec_monolithic(const __grid_const
   Ctx c;
   cta_setup(c, sh, dsm, p);
   __syncthreads();
-  if (threadIdx.x == 0) sh.T0 = gtimer() + (p.clock == PL_CLOCK_GLOBALTIMER ? PL_T0_OFFSET_NS : 0);
+  if (threadIdx.x == 0) sh.T0 = gtimer() + (p.clock == PL_CLOCK_GLOBALTIMER ? p.t0_offset_ns : 0u);
   __syncthreads();
   run_monolithic(c);
   __syncthreads();
@@ -1577,7 +1729,7 @@ __global__ void __launch_bounds__(MAXT, 1) pl_stage_batch_kernel(const __grid_co
   c.dna.qpos = (const uint16_t*)(dsm + Lo.off_qpos);
   c.dna.qw = (const uint32_t*)(dsm + Lo.off_qw);
   c.dna.nqw = (uint32_t)(p.q_len + 15) / 16u;
-  c.dna.win = nullptr; c.dna.win_lo = 0; c.dna.win_lo32 = 0; c.dna.win_n = 0;
+  c.dna.win = nullptr; c.dna.win_lo = 0; c.dna.win_lo32 = 0; c.dna.win_n = 0; c.dna.nofast = true; c.dna.s2tab = nullptr;
   const uint32_t tid = threadIdx.x, v = blockDim.x;
   if (p.k > 0) {
     const uint32_t nko = (1u << (2 * p.k)) + 1u, nqp = (uint32_t)(p.q_len - p.k + 1);
@@ -1587,6 +1739,7 @@ __global__ void __launch_bounds__(MAXT, 1) pl_stage_batch_kernel(const __grid_co
     for (uint32_t j = tid; j < nko; j += v) qo[j] = p.qoff[j];
     for (uint32_t j = tid; j < nqp; j += v) qp[j] = p.qpos[j];
     for (uint32_t j = tid; j < c.dna.nqw; j += v) qw[j] = p.qwords[j];
+    if (tid < 8) qw[tid < 4 ? (int)tid - 4 : (int)(c.dna.nqw + tid - 4u)] = 0u;   // pad words
   }
   if (tid == 0) { sh.errors = 0; }
   __syncthreads();

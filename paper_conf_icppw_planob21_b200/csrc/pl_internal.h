@@ -46,6 +46,7 @@ struct CtaStats {
   int64_t  lateness[PL_MAX_STAGES];
   uint64_t sched_cycles[PL_MAX_STAGES];
   int64_t  max_fire_ns[PL_MAX_STAGES];
+  int64_t  max_loop_ns[PL_MAX_STAGES];
   uint64_t phase_cycles[PL_MAX_STAGES][6];
   uint64_t miss_events;
   uint64_t miss_events_ns;              // physical: measured latency > D
@@ -103,7 +104,11 @@ struct DevParams {
   pl_firing* flog;                      // [n_streams][log_cap]
   uint32_t log_cap;
   CtaStats* stats;                      // [n_streams]
-  unsigned long long* summary;          // [6]: roots, miss_events, max_lat, max_lat_ns, errors, miss_ns
+  unsigned long long* summary;          // [8]: roots, miss_events, max_lat, max_lat_ns, errors, miss_ns,
+                                        //      match count (= match_count), pad
+  uint32_t t0_offset_ns;                // physical clock: stream time origin = CTA start + this
+  unsigned long long* summary_next;     // the other slot of the double buffer: zeroed by this launch
+                                        // (stream order: the previous launch that used it is done)
   const int64_t* arr;                   // per-root arrival times (NULL: r * tau0)
   DevStage st[PL_MAX_STAGES];
 };
@@ -113,7 +118,7 @@ struct SmemLayout {
   uint32_t off_ent[PL_MAX_STAGES];      // uint2 rings, edge into node i (i >= 1)
   uint32_t off_seg[PL_MAX_STAGES];
   uint32_t off_troot;                   // [N][v] u32: terminal root per lane of the current firing
-  uint32_t off_qoff, off_qpos, off_qw, off_win;
+  uint32_t off_qoff, off_qpos, off_qw, off_win, off_s2;
   uint32_t total;
 };
 

@@ -112,7 +112,8 @@ struct pl_pipeline {
   int64_t *d_lat = nullptr, *d_lat_ns = nullptr;
   uint32_t* d_trace = nullptr;
   pl_match* d_matches = nullptr;
-  unsigned long long* d_match_count = nullptr;
+  unsigned long long* d_match_count = nullptr;   // match count of the last launch (inside d_summary)
+  uint32_t slot = 0;                             // d_summary slot of the next launch
   pl_firing* d_flog = nullptr;
   CtaStats* d_stats = nullptr;
   uint64_t roots_cap = 0;   // per-root arrays sized for this many roots
@@ -133,7 +134,7 @@ namespace {
 
 void free_all(pl_pipeline* pl) {
   void* ptrs[] = {pl->d_db, pl->d_qoff, pl->d_qpos, pl->d_qw, pl->d_spill, pl->d_mono, pl->d_lat, pl->d_lat_ns,
-                  pl->d_trace, pl->d_matches, pl->d_match_count, pl->d_flog, pl->d_stats, pl->d_scratch,
+                  pl->d_trace, pl->d_matches, pl->d_flog, pl->d_stats, pl->d_scratch,
                   pl->d_summary, pl->d_arr};
   for (void* p : ptrs)
     if (p) cudaFree(p);
@@ -383,7 +384,9 @@ pl_status pl_pipeline_create(const pl_config* cfg, const pl_workload* wl, pl_pip
     // smem DB window per stream: its roots + k-1 overlap + halo on both sides (capped at 64 KB)
     const uint64_t R = wl->db_len >= (uint64_t)pl->k ? wl->db_len - pl->k + 1 : 0;
     const uint64_t per = (R + cfg->n_streams - 1) / cfg->n_streams;
-    d.win_halo = 512;
+    // halo: an extension walks at most q_len bases from its seed (Dna::right/left_limit), so
+    // with q_len + 48 every walk of an interior root stays in the window (Dna::extend_win)
+    d.win_halo = std::max<uint32_t>(512u, (uint32_t)wl->q_len + 48u);
     uint64_t words = (per + pl->k + 2 * d.win_halo) / 16 + 8;
     words = (words + 3) & ~3ull;
     d.win_cap = (uint32_t)std::min<uint64_t>(words, 16384);
@@ -432,6 +435,10 @@ pl_status pl_pipeline_create(const pl_config* cfg, const pl_workload* wl, pl_pip
   d.ctas_per_sm = 1;
   d.variant = 0;
   if (const char* e = getenv("PL_VARIANT")) d.variant = (uint32_t)atoi(e);
+  // physical clock: a stream's time origin is set this far after its CTA has staged its
+  // inputs, so that every warp group is resident before the first arrival
+  d.t0_offset_ns = 2048;
+  if (const char* e = getenv("PL_T0_OFFSET_NS")) d.t0_offset_ns = (uint32_t)atoi(e);
   if (const char* e = getenv("PL_CTAS_PER_SM"))
     if (atoi(e) == 2 && pl->block <= 512 && 2 * (pl->smem + 4096) <= (uint32_t)prop.sharedMemPerMultiprocessor)
       d.ctas_per_sm = 2;
@@ -451,21 +458,25 @@ pl_status pl_pipeline_create(const pl_config* cfg, const pl_workload* wl, pl_pip
   d.match_cap = cfg->match_capacity ? cfg->match_capacity : (1ull << 20);
   if (!pl->dna) d.match_cap = 1;
   if (cudaMalloc(&pl->d_matches, d.match_cap * sizeof(pl_match)) != cudaSuccess ||
-      cudaMalloc(&pl->d_match_count, 8) != cudaSuccess || cudaMalloc(&pl->d_stats, S * sizeof(CtaStats)) != cudaSuccess)
+      cudaMalloc(&pl->d_stats, S * sizeof(CtaStats)) != cudaSuccess)
     return bail(fail(PL_ENOMEM, "output buffers"));
-  cudaMemset(pl->d_match_count, 0, 8);
   cudaMemset(pl->d_stats, 0, S * sizeof(CtaStats));
-  if (cudaMalloc(&pl->d_summary, 8 * 8) != cudaSuccess) return bail(fail(PL_ENOMEM, "summary"));
-  cudaMemset(pl->d_summary, 0, 64);
+  // run summary + match count, double-buffered: launch k accumulates into slot k & 1 and
+  // zeroes the other slot for launch k+1, so a launch needs no host-side memset
+  if (cudaMalloc(&pl->d_summary, 2 * 8 * 8) != cudaSuccess) return bail(fail(PL_ENOMEM, "summary"));
+  cudaMemset(pl->d_summary, 0, 2 * 64);
+  pl->slot = 0;
+  pl->d_match_count = pl->d_summary + 6;
   d.lat = pl->d_lat;
   d.lat_ns = cfg->clock == PL_CLOCK_GLOBALTIMER ? pl->d_lat_ns : nullptr;
   if (!(cfg->flags & PL_REC_LATENCY)) d.lat_ns = nullptr;
   d.trace = pl->d_trace;
   d.matches = pl->d_matches;
-  d.match_count = pl->d_match_count;
+  d.match_count = pl->d_summary + 6;
   d.flog = pl->d_flog;
   d.stats = pl->d_stats;
   d.summary = pl->d_summary;
+  d.summary_next = pl->d_summary + 8;
   if (cfg->arrivals) {   // arrival process given as data (Poisson, L263): per root, per stream
     if (cfg->n_arrivals != pl->roots_cap)
       return bail(fail(PL_EINVAL, "n_arrivals %llu != root count %llu", (unsigned long long)cfg->n_arrivals,
@@ -563,11 +574,10 @@ pl_status pl_pipeline_queue_peaks(pl_pipeline* pl, uint32_t* buf, uint64_t cap, 
 pl_status pl_pipeline_summary(pl_pipeline* pl, pl_summary* out) {
   if (!pl || !out) return fail(PL_EINVAL, "NULL argument");
   cudaSetDevice(pl->device);
-  unsigned long long h[6];
-  CUDA_TRY(cudaMemcpyAsync(h, pl->d_summary, 48, cudaMemcpyDeviceToHost, pl->stream));
-  unsigned long long mc = 0;
-  CUDA_TRY(cudaMemcpyAsync(&mc, pl->d_match_count, 8, cudaMemcpyDeviceToHost, pl->stream));
+  unsigned long long h[7];
+  CUDA_TRY(cudaMemcpyAsync(h, pl->d_match_count - 6, 56, cudaMemcpyDeviceToHost, pl->stream));
   CUDA_TRY(cudaStreamSynchronize(pl->stream));
+  const unsigned long long mc = h[6];
   pl->in_flight = false;
   pl->d2h += 56;
   out->roots = h[0];
@@ -599,9 +609,12 @@ pl_status pl_pipeline_launch(pl_pipeline* pl) {
   if (pl->d_arr && d.total_roots != pl->roots_cap)
     return fail(PL_EINVAL, "arrival times were given for %llu roots; push the whole stream",
                 (unsigned long long)pl->roots_cap);
-  CUDA_TRY(cudaMemsetAsync(pl->d_match_count, 0, 8, pl->stream));
-  CUDA_TRY(cudaMemsetAsync(pl->d_summary, 0, 64, pl->stream));
+  d.summary = pl->d_summary + 8 * pl->slot;
+  d.match_count = d.summary + 6;
+  d.summary_next = pl->d_summary + 8 * (pl->slot ^ 1u);
   CUDA_TRY(pl_launch(d, pl->cfg.n_streams, pl->block, pl->smem, pl->stream));
+  pl->d_match_count = d.summary + 6;       // readers see the slot of the last launch
+  pl->slot ^= 1u;
   pl->in_flight = true;
   pl->launches++;
   return PL_OK;
@@ -662,6 +675,7 @@ pl_status pl_pipeline_stats(pl_pipeline* pl, pl_stats* out) {
       out->max_lateness_ns[i] = std::max(out->max_lateness_ns[i], s.lateness[i]);
       out->sched_cycles[i] += s.sched_cycles[i];
       out->max_fire_ns[i] = std::max(out->max_fire_ns[i], s.max_fire_ns[i]);
+      out->max_loop_ns[i] = std::max(out->max_loop_ns[i], s.max_loop_ns[i]);
       for (int k = 0; k < 6; ++k) out->phase_cycles[i][k] += s.phase_cycles[i][k];
       out->active_window[i] += s.active_win[i];   // computed per node by the executor
     }
@@ -796,6 +810,9 @@ pl_status pl_stage_batch(pl_pipeline* pl, uint32_t stage, const void* in_dev, ui
     d.total_roots = first_root + n;
   }
   d.win_cap = 0;
+  d.match_count = pl->d_match_count;
+  d.summary = nullptr;
+  d.summary_next = nullptr;
   if (!pl->d_scratch && cudaMalloc(&pl->d_scratch, 16) != cudaSuccess) return fail(PL_ENOMEM, "scratch");
   CUDA_TRY(cudaMemsetAsync(pl->d_scratch, 0, 16, pl->stream));
   if (stage == pl->cfg.n_stages - 1) CUDA_TRY(cudaMemsetAsync(pl->d_match_count, 0, 8, pl->stream));

@@ -9,7 +9,7 @@ from __future__ import annotations
 
 SUM_KEYS = ("roots", "firings", "empty_firings", "consumed", "produced", "active_window", "busy_ns",
             "spilled", "overruns", "matches", "miss_events", "misses", "window", "t_end")
-MAX_KEYS = ("max_lateness_ns", "max_fire_ns", "max_latency", "max_latency_ns", "wall_ns", "errors")
+MAX_KEYS = ("max_lateness_ns", "max_fire_ns", "max_loop_ns", "max_latency", "max_latency_ns", "wall_ns", "errors")
 
 
 def _flatten(st, keys):

@@ -46,6 +46,33 @@ def calibrate_budgets(cfg, wl, db_dev, margin=1.25, slack_ns=256, probe_t=20_000
     return tuple(int(math.ceil(margin * st["max_fire_ns"][i])) + slack_ns for i in range(N)), st
 
 
+def refine_budgets(cfg, wl, db_dev, budgets, margin=1.10, slack_ns=128, rounds=2, reps=3, flags=0, stream=None,
+                   over=None, log=None):
+    """Budgets re-measured at the operating point.  The probe of calibrate_budgets fires every
+    node with a full vector at the same instant, a contention pattern the solved schedule
+    rarely produces; here each round finds the miss-free rate for the current budgets
+    (find_rate), runs that schedule `reps` times with the kernel the budgets are for (`flags`)
+    and takes ceil(margin * longest firing) + slack_ns per node, never raising a budget.
+    Stops when no budget shrinks.  Returns (budgets, history)."""
+    hist = []
+    for _ in range(rounds):
+        c = cfg.replace(service_time=tuple(budgets))
+        tau, w, th, T, st = find_rate(c, wl, db_dev, stream=stream, over=over)
+        worst = [0] * cfg.n_stages
+        for _ in range(reps):
+            s2 = _run(c.replace(interarrival=tau, wait_time=tuple(w), clock=PHYS), db_dev, wl.db_len, wl,
+                      flags=flags, stream=stream, over=over)
+            worst = [max(a, b) for a, b in zip(worst, s2["max_fire_ns"])]
+        nb = tuple(min(b, int(math.ceil(margin * x)) + slack_ns) for b, x in zip(budgets, worst))
+        hist.append(dict(budgets=tuple(budgets), tau=tau, max_fire_ns=worst, next=nb))
+        if log:
+            log(hist[-1])
+        if nb == tuple(budgets):
+            break
+        budgets = nb
+    return tuple(budgets), hist
+
+
 def solve_at(cfg, tau):
     """Fig. 1 at inter-arrival tau (None if infeasible)."""
     try:

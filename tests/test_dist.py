@@ -23,7 +23,7 @@ def _stats(rank):
             "consumed": [100 + rank, 50], "produced": [50, 100], "active_window": [640 + rank, 480],
             "busy_ns": [1000 * (rank + 1), 0], "spilled": [0, rank], "overruns": [0, 0], "matches": rank,
             "miss_events": 0, "misses": 0, "window": 400 + 4 * rank, "t_end": 500,
-            "max_lateness_ns": [rank * 7, 3], "max_fire_ns": [100 - rank, 50 + rank], "max_latency": 400 + rank,
+            "max_lateness_ns": [rank * 7, 3], "max_fire_ns": [100 - rank, 50 + rank], "max_loop_ns": [9 + rank, 4], "max_latency": 400 + rank,
             "max_latency_ns": 1000 * rank, "wall_ns": 5 + rank, "errors": 0, "active_fraction": 0.0}
 
 
@@ -45,7 +45,7 @@ def test_allreduce_stats_gloo_two_ranks():
         a, b = out[0], out[1]
     assert a == b
     assert a["roots"] == 201 and a["firings"] == [21, 10] and a["empty_firings"] == [2, 1]
-    assert a["max_lateness_ns"] == [7, 3] and a["max_fire_ns"] == [100, 51]
+    assert a["max_lateness_ns"] == [7, 3] and a["max_fire_ns"] == [100, 51] and a["max_loop_ns"] == [10, 4]
     assert a["max_latency"] == 401 and a["wall_ns"] == 6 and a["matches"] == 1
     assert a["window"] == 804
     assert abs(a["active_fraction"] - (641 + 640 + 960) / (2 * 804)) < 1e-12
