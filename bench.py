@@ -53,9 +53,12 @@ def parse():
     ap.add_argument("--cpu-sample-streams", type=int, default=148)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
-    ap.add_argument("--budget-margin", type=float, default=1.25)
-    ap.add_argument("--budget-slack", type=int, default=256)
-    ap.add_argument("--refine", type=int, default=0, help="budget refinement rounds at the operating point")
+    ap.add_argument("--budget-margin", type=float, default=1.10,
+                    help="t_i = margin x longest measured firing + slack (SURVEY 8(d): x1.1)")
+    ap.add_argument("--budget-slack", type=int, default=128)
+    ap.add_argument("--refine", type=int, default=2, help="budget refinement rounds at the operating point")
+    ap.add_argument("--max-lateness-ns", type=int, default=5000,
+                    help="rate search: every firing must start within this of its schedule (sustainability)")
     ap.add_argument("--drain", default="eager", choices=["eager", "periodic"],
                     help="end of stream: R-DRAIN work-conserving drain (PL_EAGER_DRAIN) or the periodic rule")
     return ap.parse_args()
@@ -239,7 +242,8 @@ def main():
     cfg = base.replace(clock=1, ns_per_unit=1.0, service_time=budgets, gain=gains, deadline=a.deadline_ns,
                        b=C.PAPER_B, eager_drain=a.drain == "eager")
     # 2./3. the fastest miss-free rate
-    tau, w, th, T, st_ok = realtime.find_rate(cfg, wl, db_ptr, stream=stream, log=log)
+    tau, w, th, T, st_ok = realtime.find_rate(cfg, wl, db_ptr, stream=stream, log=log,
+                                              max_lateness_ns=a.max_lateness_ns)
     if world > 1:
         t = torch.tensor([tau], dtype=torch.int64, device=dev)
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
@@ -262,6 +266,7 @@ def main():
     misses = 0
     sched_misses = 0
     overruns = 0
+    lateness = 0
     errors = 0
     roots = 0
     torch.cuda.synchronize()
@@ -274,6 +279,7 @@ def main():
         misses += st["miss_events_ns"]                 # measured on %globaltimer
         sched_misses += st["miss_events"]              # the logical schedule's own
         overruns += sum(st["overruns"])
+        lateness = max(lateness, max(st["max_lateness_ns"]))
         errors |= st["errors"]
         roots += st["roots"]
     torch.cuda.synchronize()
@@ -453,6 +459,7 @@ def main():
                        "streams_per_gpu": a.streams, "l2": "flushed between timed steps (256 MiB memset)",
                        "parallelism": f"{a.streams} streams x {world} GPUs (independent; NCCL stats all-reduce)"},
             "misses": misses_all, "schedule_misses": sched_misses_all, "overruns": overruns_all, "errors": errors,
+            "max_lateness_ns": lateness,
             "sustained_items_per_s": world * a.streams * 1e9 / tau,
             "logical_items_per_s": logical_ips,
             "threshold_slack": thr,
@@ -464,7 +471,8 @@ def main():
                                         "firing_cycles": round(sum(st["phase_cycles"][i][1:5]) / max(1, st["firings"][i])),
                                         "publish_cycles": round(st["phase_cycles"][i][5] / max(1, st["firings"][i])),
                                         "mean_fire_ns": round(st["busy_ns"][i] / max(1, st["firings"][i])),
-                                        "max_fire_ns": st["max_fire_ns"][i]} for i in range(st["n_stages"])},
+                                        "max_fire_ns": st["max_fire_ns"][i],
+                                        "max_loop_ns": st["max_loop_ns"][i]} for i in range(st["n_stages"])},
             "clocks": clk,
             "e2e": e2e,
             "gpu_launches": a.steps,

@@ -282,7 +282,7 @@ enum { D_PH0, D_PH1, D_PH2, D_PH3, D_STALL, D_N = 8 };
 struct NodeAcc {
   alignas(16) unsigned long long cnt[C_N];
   alignas(16) unsigned long long ph[6];
-  alignas(16) uint32_t d[D_N];
+  alignas(16) uint32_t d[2][D_N];   // per-firing 32-bit deltas, double-buffered by firing parity
   long long t_end;
   uint32_t max_queue, lateness, max_fire, lmax, lmax_ns, nmiss, nmiss_ns;
   uint32_t max_loop;   // physical: longest firing-to-next-decision cycle (the node's real service time)
@@ -945,7 +945,7 @@ __device__ void run_node(Ctx& c, const Dna dna, int i, int gtid) {
     for (int k = 0; k < 8; ++k) { G.wtot[0][k] = 0; G.wtot[1][k] = 0; }
     for (int k = 0; k < C_N; ++k) A.cnt[k] = 0;
     for (int k = 0; k < 6; ++k) A.ph[k] = 0;
-    for (int k = 0; k < D_N; ++k) A.d[k] = 0;
+    for (int k = 0; k < D_N; ++k) { A.d[0][k] = 0; A.d[1][k] = 0; }
     for (int k = 0; k < 8; ++k) G.rmin[k] = NO_ROOT;   // slots of absent warps stay NO_ROOT
     A.t_end = 0;
     A.max_queue = A.lateness = A.max_fire = A.lmax = A.lmax_ns = A.nmiss = A.nmiss_ns = A.max_loop = 0;
@@ -963,11 +963,11 @@ __device__ void run_node(Ctx& c, const Dna dna, int i, int gtid) {
         atomicMax(&A.max_queue, d.qlen);
         publish_W(nd, L, T + nd.t);      // committed: nothing leaves node 0 before T + t_0
         if (rec & PL_REC_FIRINGS) G.log_idx[par] = atomicAdd(&c.sh->log_count, 1u);
-        A.d[D_STALL] = 0;
-        G.out_loc[par] = nd.sink ? LOC_SMEM : reserve_out(nd, L, n * nd.umax, &A.d[D_STALL]);
+        A.d[par][D_STALL] = 0;
+        G.out_loc[par] = nd.sink ? LOC_SMEM : reserve_out(nd, L, n * nd.umax, &A.d[par][D_STALL]);
         G.out_base[par] = L.out_tail;
         tc = clock64();
-        A.d[D_PH0] = (uint32_t)(tc - c0);
+        A.d[par][D_PH0] = (uint32_t)(tc - c0);
       }
       if (nd.phys && (p.variant & 1u)) {  // the leader paces, one barrier releases the lanes
         if (leader) {
@@ -1005,14 +1005,14 @@ __device__ void run_node(Ctx& c, const Dna dna, int i, int gtid) {
         G.in_spill_end[par] = vld(&nd.Ein->spill_end);
         if (!d.done) {
           if (rec & PL_REC_FIRINGS) G.log_idx[par] = atomicAdd(&c.sh->log_count, 1u);
-          A.d[D_STALL] = 0;
-          G.out_loc[par] = nd.sink ? LOC_SMEM : reserve_out(nd, L, d.n * nd.umax, &A.d[D_STALL]);
+          A.d[par][D_STALL] = 0;
+          G.out_loc[par] = nd.sink ? LOC_SMEM : reserve_out(nd, L, d.n * nd.umax, &A.d[par][D_STALL]);
           G.out_base[par] = L.out_tail;
         } else {
           publish_W(nd, L, PL_INF64);
         }
         tc = clock64();
-        A.d[D_PH0] = (uint32_t)(tc - c0);
+        A.d[par][D_PH0] = (uint32_t)(tc - c0);
         if (!d.done && nd.phys) {
           int64_t late;
           uint64_t entry;
@@ -1024,7 +1024,7 @@ __device__ void run_node(Ctx& c, const Dna dna, int i, int gtid) {
         }
       }
       bar_sync(bidA, v);                                               // B1: decision
-      if (leader) { const long long t2 = clock64(); A.d[D_PH1] = (uint32_t)(t2 - tc); tc = t2; }
+      if (leader) { const long long t2 = clock64(); A.d[par][D_PH1] = (uint32_t)(t2 - tc); tc = t2; }
       if (REC && pend_root != NO_ROOT)   // deferred physical latency of the previous firing
         record_lat_ns(nd, c, T0, G.end_ns[par ^ 1], pend_root);
       if (G.done[par]) break;
@@ -1066,7 +1066,7 @@ __device__ void run_node(Ctx& c, const Dna dna, int i, int gtid) {
       off = group_scan(G.wtot[par], o[0].c, &total, gtid, v, bidA, nd.umax <= 1);                 // B2
     }
     const uint32_t out_loc = G.out_loc[par], out_base = G.out_base[par];   // leader's reservation (B2)
-    if (leader) { const long long t2 = clock64(); A.d[D_PH2] = (uint32_t)(t2 - tc); tc = t2; }
+    if (leader) { const long long t2 = clock64(); A.d[par][D_PH2] = (uint32_t)(t2 - tc); tc = t2; }
     if (REC && n0 && pend_root != NO_ROOT)   // node 0: the previous publish time came through B2
       record_lat_ns(nd, c, T0, G.end_ns[par ^ 1], pend_root);
     // --- release the input slots (every lane has loaded its entry: B2 passed)
@@ -1131,7 +1131,7 @@ __device__ void run_node(Ctx& c, const Dna dna, int i, int gtid) {
         }
       }
     }
-    if (leader) { const long long t2 = clock64(); A.d[D_PH3] = (uint32_t)(t2 - tc); tc = t2; }
+    if (leader) { const long long t2 = clock64(); A.d[par][D_PH3] = (uint32_t)(t2 - tc); tc = t2; }
     // --- compaction into the next queue (stable: lane order, then child order)
     if (!nd.sink && act && oi.c && out_loc != ~0u) {
       const uint32_t base = out_base + off;
@@ -1148,11 +1148,12 @@ __device__ void run_node(Ctx& c, const Dna dna, int i, int gtid) {
         else __stcg(nd.out_spill + (s & (nd.capg - 1)), val);
       }
     }
-    // B4: outputs written.  Non-leader warps only arrive; node 7 (no spare barrier id) syncs
-    // fully, since arrivals for B4 and the next B1 must not meet on one barrier instance.
-    if (gtid < 32 || bidB == bidA) bar_sync(bidB, v);
+    // B4: outputs written.  The leader's warp and the accountant's warp sync, the others only
+    // arrive; node 7 (no spare barrier id) syncs fully, since arrivals for B4 and the next B1
+    // must not meet on one barrier instance.
+    if (gtid < 64 || bidB == bidA) bar_sync(bidB, v);
     else bar_arrive(bidB, v);
-    if (leader) {
+    if (leader) {   // publish (the critical path to the next firing), then the leader's own sums
       long long t4 = clock64();
       const uint32_t ph4 = (uint32_t)(t4 - tc);
       uint64_t en = 0, fire = 0;
@@ -1194,9 +1195,25 @@ __device__ void run_node(Ctx& c, const Dna dna, int i, int gtid) {
         L.B = T + nd.t;
         publish_W(nd, L, L.B + nd.t);
       }
+      {   // measured busy time, overruns, publish-phase cycles (the leader's slots of the sums)
+        ulonglong2* Cp = reinterpret_cast<ulonglong2*>(A.cnt);
+        ulonglong2* Pp = reinterpret_cast<ulonglong2*>(A.ph);
+        ulonglong2 c2 = Cp[2], p2 = Pp[2];
+        c2.x += nd.phys ? (en - start_ns) : 0ull;
+        c2.y += (nd.phys && (int64_t)fire > nd.t_ns) ? 1ull : 0ull;   // work outlasted t_i
+        p2.x += ph4;
+        p2.y += (uint64_t)(clock64() - t4);
+        Cp[2] = c2; Pp[2] = p2;
+      }
+    }
+    // The accountant (lane 0 of the node's second warp; the leader when v = 32) books the
+    // firing off the leader's path: the lanes' troot / rmin stores and the leader's phase
+    // deltas A.d[par] were ordered before B4, and the next writes of each come after this
+    // warp has reached the next firing's scan barrier (A.d is double-buffered by parity).
+    if (v > 32 ? gtid == 32 : leader) {
+      const uint64_t en = nd.phys ? gtimer() : 0ull;   // completion time of the terminal items
       A.t_end = T + nd.t;                // firing starts increase: the last one ends last
-      // bookkeeping of this firing's terminal items (the lanes' troot / rmin stores were
-      // ordered before B4): the smallest root has the largest latency
+      // the smallest terminal root has the largest latency
       uint32_t rmin;
       {
         const uint4 a = *reinterpret_cast<const uint4*>(G.rmin);
@@ -1234,23 +1251,19 @@ __device__ void run_node(Ctx& c, const Dna dna, int i, int gtid) {
       {   // fold this firing into the 64-bit sums: one vectorised read-modify-write
         ulonglong2* Cp = reinterpret_cast<ulonglong2*>(A.cnt);
         ulonglong2* Pp = reinterpret_cast<ulonglong2*>(A.ph);
-        ulonglong2 c0 = Cp[0], c1 = Cp[1], c2 = Cp[2], c3 = Cp[3], c4 = Cp[4], p0 = Pp[0], p1 = Pp[1], p2 = Pp[2];
-        const uint4 dd = *reinterpret_cast<const uint4*>(A.d);
-        const uint32_t stl = A.d[D_STALL];
+        ulonglong2 c0 = Cp[0], c1 = Cp[1], c3 = Cp[3], c4 = Cp[4], p0 = Pp[0], p1 = Pp[1];
+        const uint4 dd = *reinterpret_cast<const uint4*>(A.d[par]);
+        const uint32_t stl = A.d[par][D_STALL];
         c0.x += 1ull;
         c0.y += n;
         c1.x += total;
         const unsigned long long ov = (unsigned long long)overlap(T, T + nd.t, 0, nd.H);
         c1.y += ov;
         c4.x += (nd.eager && T >= nd.A_last) ? ov : 0ull;   // R-DRAIN firings (FIXED_WAIT window)
-        c2.x += nd.phys ? (en - start_ns) : 0ull;
-        c2.y += (nd.phys && (int64_t)fire > nd.t_ns) ? 1ull : 0ull;   // work outlasted t_i
         c3.x += (!nd.sink && out_loc == LOC_SPILL) ? (unsigned long long)total : 0ull;
         c3.y += stl;
         p0.x += dd.x; p0.y += dd.y; p1.x += dd.z; p1.y += dd.w;
-        p2.x += ph4;
-        p2.y += (uint64_t)(clock64() - t4);
-        Cp[0] = c0; Cp[1] = c1; Cp[2] = c2; Cp[3] = c3; Cp[4] = c4; Pp[0] = p0; Pp[1] = p1; Pp[2] = p2;
+        Cp[0] = c0; Cp[1] = c1; Cp[3] = c3; Cp[4] = c4; Pp[0] = p0; Pp[1] = p1;
       }
     }
     if (n0) {                            // replicated node-0 state, identical in every lane

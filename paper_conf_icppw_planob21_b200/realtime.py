@@ -95,13 +95,19 @@ def min_feasible_tau(cfg, lo=1, hi=1 << 20):
     return lo
 
 
-def find_rate(cfg, wl, db_dev, tries=12, grow=1.15, stream=None, log=None, over=None, policy=0):
+def find_rate(cfg, wl, db_dev, tries=12, grow=1.15, stream=None, log=None, over=None, policy=0,
+              max_lateness_ns=5000, flags=0):
     """Smallest tau0 (ns) at which a physical run (FIXED_WAIT, or THRESHOLD_SLACK with the
-    Fig. 1-derived thresholds when policy=1) has zero deadline misses and
-    no queue overflow (budget overruns are counted and reported, not fatal: they delay
-    firings, and any delay that matters shows up as a miss).  Starts at the smallest tau0
+    Fig. 1-derived thresholds when policy=1) has zero deadline misses, no queue overflow
+    and, unless max_lateness_ns is None, every firing starting within max_lateness_ns of its
+    scheduled time.  The lateness bound is the sustainability check: a node whose real
+    per-firing cycle (firing + publish + next decision, pl_stats.max_loop_ns) exceeds its
+    period falls further behind with every firing, which a finite stream can hide inside D
+    (budget overruns are counted and reported, not fatal).  Starts at the smallest tau0
     for which Fig. 1 is feasible, grows by `grow` until a run is clean, then bisects between
-    the last failing and the first clean tau0.  Returns (tau0, w, theta, T, stats)."""
+    the last failing and the first clean tau0.  The trial runs use the kernel selected by
+    `flags` (default: the record-free kernel that the bench times; misses are counted on the
+    device either way).  Returns (tau0, w, theta, T, stats)."""
     from ._pl import PlError
 
     def trial(tau):
@@ -112,13 +118,17 @@ def find_rate(cfg, wl, db_dev, tries=12, grow=1.15, stream=None, log=None, over=
         c = cfg.replace(interarrival=int(tau), wait_time=tuple(w), wait_threshold=tuple(th), clock=PHYS,
                         policy=policy)
         try:
-            st = _run(c, db_dev, wl.db_len, wl, flags=1, stream=stream, over=over)
-            ok = st["misses"] == 0 and st["miss_events_ns"] == 0 and st["errors"] == 0
+            st = _run(c, db_dev, wl.db_len, wl, flags=flags, stream=stream, over=over)
+            ok = (st["misses"] == 0 and st["miss_events"] == 0 and st["miss_events_ns"] == 0
+                  and st["errors"] == 0)
+            if max_lateness_ns is not None:
+                ok = ok and max(st["max_lateness_ns"]) <= max_lateness_ns
         except PlError:          # device-side overflow reported by drain
-            st, ok = {"misses": -1, "miss_events_ns": -1, "errors": -1, "overruns": [], "max_latency_ns": -1}, False
+            st, ok = {"misses": -1, "miss_events_ns": -1, "errors": -1, "overruns": [], "max_latency_ns": -1,
+                      "max_lateness_ns": []}, False
         if log:
             log(dict(tau=tau, w=w, T=T, misses=st["misses"], overruns=st["overruns"], errors=st["errors"],
-                     max_latency_ns=st["max_latency_ns"]))
+                     max_latency_ns=st["max_latency_ns"], max_lateness_ns=st["max_lateness_ns"]))
         return (int(tau), w, th, T, st) if ok else None
 
     tau = min_feasible_tau(cfg)
