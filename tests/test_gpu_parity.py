@@ -241,3 +241,58 @@ def test_eager_drain_physical_replay(policy):
     g = run_gpu(cfg, wl)
     compare(cfg, g, run_oracle(cfg, wl))
     assert (g["lat_ns"] > 0).all()
+
+
+def test_repeated_launches_summary_double_buffer():
+    """The run summary and match count are double-buffered on the device (each launch zeroes
+    the slot of the next one, so no per-launch memset): back-to-back launches without reads
+    in between, then reads after each launch, all give the oracle's counts and matches."""
+    from paper_conf_icppw_planob21_b200 import Pipeline
+    cfg = _dna(C.FIXED_WAIT, db_len=1 << 16, streams=5)
+    wl = workload_for(cfg)
+    o = run_oracle(cfg, wl)
+    pl = Pipeline(cfg, wl, flags=0)
+    pl.push(wl.db, wl.db_len)
+    for _ in range(3):                   # unread launches: each must start from a zero slot
+        pl.launch()
+    first = None
+    for k in range(4):
+        pl.launch()
+        s = pl.summary()
+        first = first or s
+        assert s["roots"] == sum(hi - lo for lo, hi in _ranges(cfg, wl)), k
+        assert s["matches"] == len(o.matches), k
+        assert s["max_latency"] == max(o.lat) and s["miss_events"] == first["miss_events"], k
+        assert pl.results() == [tuple(m) for m in o.matches], k
+    st = pl.stats()
+    pl.close()
+    assert st["launches"] == 7 and st["matches"] == len(o.matches)
+
+
+def _ranges(cfg, wl):
+    from oracle import des
+    k = cfg.stages[0].iparam[0]
+    return des.stream_ranges(cfg, wl.db_len - k + 1)
+
+
+def test_physical_loop_time_reported():
+    """pl_stats.max_loop_ns (a firing's start to the node's next decision: the real per-firing
+    service time incl. publish and bookkeeping) is measured in the physical clock, bounds
+    the firing time, and is zero in the logical clock."""
+    from paper_conf_icppw_planob21_b200 import Pipeline
+    cfg = _dna(C.FIXED_WAIT, db_len=1 << 16, streams=4)
+    wl = workload_for(cfg)
+    out = {}
+    for clock in (0, 1):
+        c = cfg.replace(clock=clock, ns_per_unit=1.0, service_time=(4000, 8000, 8000, 20000), interarrival=100,
+                        deadline=10 ** 7, wait_time=(100, 100, 100, 100))
+        pl = Pipeline(c, wl, flags=0)
+        pl.push(wl.db, wl.db_len)
+        pl.drain()
+        out[clock] = pl.stats()
+        pl.close()
+    assert all(x == 0 for x in out[0]["max_loop_ns"][:4])
+    ph = out[1]
+    # node 0 never waits for upstream, so every firing is a sample and the cycle contains it
+    assert ph["max_loop_ns"][0] >= ph["max_fire_ns"][0] > 0
+    assert all(x >= 0 for x in ph["max_loop_ns"][:4])

@@ -14,7 +14,9 @@ from paper_conf_icppw_planob21_b200 import Pipeline
 a = [int(x) for x in sys.argv[1:]] or [16, 1976, 3616, 3816, 16336, 72, 5549, 4174, 25088, 1]
 tau, t, w = a[0], tuple(a[1:5]), tuple(a[5:9])
 eager = bool(a[9]) if len(a) > 9 else True
-cfg = C.c2(n_streams=148).replace(clock=1, ns_per_unit=1.0, service_time=t, wait_time=w, interarrival=tau,
+import os
+dbl = int(os.environ.get("DB_LEN", str(1 << 20)))   # longer streams: does the lateness stay bounded?
+cfg = C.c2(n_streams=148, dna=dict(db_len=dbl, q_len=1024, n_planted=64 * dbl // (1 << 20))).replace(clock=1, ns_per_unit=1.0, service_time=t, wait_time=w, interarrival=tau,
                                    deadline=350_000, b=C.PAPER_B, eager_drain=eager)
 wl = G.make_dna(cfg.seed, **cfg.dna)
 db = torch.from_numpy(wl.db.view("int32")).cuda()
