@@ -9,7 +9,7 @@ import ctypes as C
 import os
 
 HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(HERE, "libplgpu.so")
+LIB_PATH = os.environ.get("PLGPU_LIB") or os.path.join(HERE, "libplgpu.so")   # PLGPU_LIB: an experiment build
 
 PL_MAX_STAGES = 8
 PL_MAX_U = 16
