@@ -161,6 +161,17 @@ class Pipeline:
         check(lib.pl_pipeline_results(self.h, buf, n.value, C.byref(n)), "pl_pipeline_results")
         return sorted((m.p, m.q, m.db_start, m.q_start, m.len, m.score) for m in buf[:n.value])
 
+    def results_array(self):
+        """The match records as an (n, 6) int64 array (p, q, db_start, q_start, len, score),
+        rows in lexicographic order (the order of results())."""
+        n = C.c_uint64()
+        check(lib.pl_pipeline_results(self.h, None, 0, C.byref(n)), "pl_pipeline_results")
+        buf = np.empty((max(1, n.value), 6), dtype=np.uint32)
+        check(lib.pl_pipeline_results(self.h, buf.ctypes.data, n.value, C.byref(n)), "pl_pipeline_results")
+        a = buf[:n.value].astype(np.int64)
+        a[:, 5] = buf[:n.value, 5].view(np.int32)
+        return a[np.lexsort(a.T[::-1])] if len(a) else a
+
     def latency(self):
         n = C.c_uint64()
         check(lib.pl_pipeline_latency(self.h, None, None, 0, C.byref(n)), "pl_pipeline_latency")
