@@ -340,33 +340,44 @@ def main():
     pll.close()
 
     # monolithic baseline (§5, Fig. 2): at the enforced rate, and at the fastest
-    # rate where both strategies are feasible (the paper's utilisation comparison, L236-L255)
+    # rate where both strategies are feasible (the paper's utilisation comparison, L236-L255).
+    # Run on streams of the paper's length (50,000 roots each, L230) built the c2 way: a c2
+    # stream holds only 7,085 roots, less than one Fig. 2 block at these rates, so its [0, H)
+    # window would credit the monolithic processor with at most one partial block.
+    ul_len = a.streams * 50_000 + base.stages[0].iparam[0] - 1
+    ucfg = cfg.replace(dna=dict(base.dna, db_len=ul_len, n_planted=base.dna["n_planted"] * ul_len // base.dna["db_len"]))
+    uwl = G.make_dna(ucfg.seed, **ucfg.dna)
+    udb = torch.from_numpy(uwl.db.view("int32")).to(dev)
+
     def run_policy(policy, tau_x, M=0):
-        c = cfg.replace(interarrival=int(tau_x), policy=policy, block_size=M)
+        c = ucfg.replace(interarrival=int(tau_x), policy=policy, block_size=M)
         if policy == 0:
-            sol = realtime.solve_at(cfg, tau_x)
+            sol = realtime.solve_at(ucfg, tau_x)
             if sol is None:
                 return None
             c = c.replace(wait_time=tuple(sol[0]))
-        pp = Pipeline(c, wl, flags=1, stream=stream)
-        pp.bind_device(db_ptr, wl.db_len)
+        pp = Pipeline(c, uwl, flags=0, stream=stream)
+        pp.bind_device(udb.data_ptr(), uwl.db_len)
         pp.drain()
         sx = pp.stats()
         pp.close()
         return {"tau0_ns": int(tau_x), "active_fraction": sx["active_fraction"],
-                "hw_busy_fraction": sx["hw_busy_fraction"], "misses": sx["misses"],
+                "active_fraction_nonempty": sx["active_fraction_nonempty"],
+                "hw_busy_fraction": sx["hw_busy_fraction"], "misses": sx["miss_events_ns"],
                 "max_latency_ns": sx["max_latency_ns"], **({"M": M} if policy == 2 else {})}
 
-    mono = {}
-    Mr = realtime.monolithic_at(cfg, tau)
+    mono = {"stream_roots": 50_000}
+    Mr = realtime.monolithic_at(ucfg, tau)
     mono["at_enforced_rate"] = run_policy(2, tau, Mr[0]) if Mr is not None else {"feasible": False}
     tau_m = tau
-    while realtime.monolithic_at(cfg, tau_m) is None and tau_m < 100 * tau:
+    while realtime.monolithic_at(ucfg, tau_m) is None and tau_m < 100 * tau:
         tau_m = int(math.ceil(tau_m * 1.05)) + 1
-    Mm = realtime.monolithic_at(cfg, tau_m)
-    if Mm is not None:
-        mono["common_rate"] = {"tau0_ns": tau_m, "monolithic": run_policy(2, tau_m, Mm[0]),
-                               "enforced": run_policy(0, tau_m), "fig2_objective": Mm[1]}
+    for key, tx in (("common_rate", tau_m), ("slow_rate", 4 * tau_m)):
+        Mm = realtime.monolithic_at(ucfg, tx)
+        if Mm is not None:
+            mono[key] = {"tau0_ns": tx, "monolithic": run_policy(2, tx, Mm[0]), "enforced": run_policy(0, tx),
+                         "fig2_objective": Mm[1], "fig1_objective": (realtime.solve_at(ucfg, tx) or (0, 0, None))[2]}
+    del udb
 
     # the north_star's threshold / deadline-slack rule (THRESHOLD_SLACK, theta_i from Fig. 1;
     # the slack reserve R_i gets a guard of the largest budget for real-time lateness)

@@ -549,9 +549,12 @@ __device__ __forceinline__ void publish_W(const Node& nd, Leader& L, int64_t w) 
   }
 }
 
-__device__ __forceinline__ void backoff(int& spins) {
-  if (spins < 4) { ++spins; return; }
-  __nanosleep(spins < 64 ? 32 : 256);
+// Poll backoff.  The logical clock polls hard (its schedule advances as fast as the nodes do);
+// on the physical clock the %globaltimer ticks every 32 ns and a poll costs issue slots that
+// a waiting node is supposed to yield, so it backs off faster.
+__device__ __forceinline__ void backoff(int& spins, bool phys = false) {
+  if (spins < (phys ? 2 : 4)) { ++spins; return; }
+  __nanosleep(phys ? (spins < 16 ? 64 : 256) : (spins < 64 ? 32 : 256));
   ++spins;
 }
 
@@ -662,12 +665,39 @@ __device__ __forceinline__ void advance0(const Node& nd, Rep& r) {
 }
 
 // Nodes i >= 1: the leader decides from the published queue state and watermark.
-__device__ Decision decide(const Node& nd, Leader& L, bool& waited) {
+// Sleep until %globaltimer reaches `target` (chunks of at most a quarter of the remaining
+// time, __nanosleep rounds up); returns whether it slept at all.
+__device__ __forceinline__ bool nap_until(uint64_t target) {
+  uint64_t now = gtimer();
+  if (now >= target) return false;
+  while (now < target) {
+    const uint64_t rem = target - now;
+    __nanosleep(rem > 16384 ? 4096 : (rem > 4096 ? 1024 : (rem > 1024 ? 256 : 64)));
+    now = gtimer();
+  }
+  return true;
+}
+
+// A FIXED_WAIT node cannot start firing m before T = m P_i, so on the physical clock it sleeps
+// until this far ahead of T before it polls its upstream (a waiting node then costs issue slots
+// only for the poll that decides the firing; yielded time is usable).
+constexpr uint64_t PL_NAP_LEAD_NS = 768;
+
+__device__ Decision decide(const Node& nd, Leader& L, bool& waited, uint64_t T0) {
   const uint32_t v = (uint32_t)nd.v;
   Decision d;
   d.done = false; d.T = 0; d.n = 0; d.qlen = 0;
   int spins = 0;
+  int64_t napped = -1;
   for (;;) {
+    if (nd.phys && nd.fixed && !(nd.eager && L.m >= nd.Mcap)) {
+      const int64_t Tn = L.m * nd.P;
+      if (Tn != napped) {
+        napped = Tn;
+        const uint64_t due = T0 + units_ns(nd, Tn);
+        if (due > T0 + PL_NAP_LEAD_NS && nap_until(due - PL_NAP_LEAD_NS)) waited = true;
+      }
+    }
     // node i >= 1: read the upstream watermark first, then the published segments
     const int64_t Wup = vld(&nd.Ein->W);
     fence_cta();
@@ -680,14 +710,14 @@ __device__ Decision decide(const Node& nd, Leader& L, bool& waited) {
         if (!any) {
           if (Wup == PL_INF64) { d.done = true; return d; }
           publish_W(nd, L, max(B, Wup) + nd.t);
-          backoff(spins); waited = true;
+          backoff(spins, nd.phys); waited = true;
           continue;
         }
         const int64_t Te = max(B, nd.in_seg[L.segh & nd.segmask].ready);
         const uint32_t cnt = count_le(nd, L, st, Te);
         publish_W(nd, L, Te + nd.t);     // the firing starts at Te; only its size is pending
         if (Wup > Te || cnt >= v) { d.T = Te; d.n = cnt < v ? cnt : v; d.qlen = tail_known - L.head; return d; }
-        backoff(spins); waited = true;
+        backoff(spins, nd.phys); waited = true;
         continue;
       }
       const int64_t T = L.m * nd.P;
@@ -706,14 +736,14 @@ __device__ Decision decide(const Node& nd, Leader& L, bool& waited) {
         continue;
       }
       publish_W(nd, L, T + nd.t);
-      backoff(spins); waited = true;
+      backoff(spins, nd.phys); waited = true;
       continue;
     }
     // THRESHOLD_SLACK
     if (!any) {
       if (Wup == PL_INF64) { d.done = true; return d; }
       publish_W(nd, L, (Wup > L.B ? Wup : L.B) + nd.t);
-      backoff(spins); waited = true;
+      backoff(spins, nd.phys); waited = true;
       continue;
     }
     const Seg& hs = nd.in_seg[L.segh & nd.segmask];
@@ -746,7 +776,7 @@ __device__ Decision decide(const Node& nd, Leader& L, bool& waited) {
     int64_t lb = Tk < Wup ? Tk : Wup;
     if (lb < L.B) lb = L.B;
     publish_W(nd, L, lb + nd.t);
-    backoff(spins); waited = true;
+    backoff(spins, nd.phys); waited = true;
   }
 }
 
@@ -993,7 +1023,7 @@ __device__ void run_node(Ctx& c, const Dna dna, int i, int gtid) {
       if (leader) {
         const long long c0 = clock64();
         bool waited = false;             // the decision waited for upstream (no service-time sample)
-        const Decision d = decide(nd, L, waited);
+        const Decision d = decide(nd, L, waited, T0);
         atomicMax(&A.max_queue, d.qlen);
         G.done[par] = d.done ? 1u : 0u;
         G.T[par] = d.T;
