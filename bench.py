@@ -490,6 +490,14 @@ def main():
             "roofline": {"bound": "hbm", "achieved": achieved, "peak": pk, "unit": "GB/s", "frac": achieved / pk,
                          "traffic": ncu_traffic(), "peak_source": pk_src,
                          "algorithmic_bytes_per_launch": bytes_per_launch},
+            # the bound that actually sets the rate: Fig. 1 stability (L125/L145) needs
+            # P_0 = t_0 + w_0 <= v tau0, so tau0 >= t_0 / v at node 0's calibrated budget
+            "rate_bound": {"bound": "node-0 service time (Fig. 1 stability: tau0 >= t_0/v)",
+                           "achieved": world * a.streams * 1e9 / tau,
+                           "peak": world * a.streams * cfg.vector_width * 1e9 / budgets[0],
+                           "unit": "items/s",
+                           "frac": (world * a.streams * 1e9 / tau) / (world * a.streams * cfg.vector_width * 1e9 / budgets[0]),
+                           "t0_ns": budgets[0], "v": cfg.vector_width},
             "cpu_baseline": cpu,
         }
         print(json.dumps(line), flush=True)
