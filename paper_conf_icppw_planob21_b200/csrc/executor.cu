@@ -18,6 +18,7 @@
 // lateness / overruns instead of silently changing it.
 #include <cuda_runtime.h>
 #include <stdint.h>
+#include <stdio.h>
 #include "pl_internal.h"
 
 namespace {
@@ -60,6 +61,13 @@ __device__ __forceinline__ uint64_t gain_hash(uint64_t seed, uint32_t stage, uin
 // The DB is read through a per-stream smem window (staged by a TMA bulk copy at
 // CTA start, cta_setup) with an __ldg fallback outside it.  Extensions compare 16
 // bases per step: XOR of two 2-bit-packed 32-bit windows gives a mismatch mask.
+#ifndef PL_S3_MSB
+#define PL_S3_MSB 1
+#endif
+#ifndef PL_S3_DEBUG
+#define PL_S3_DEBUG 0
+#endif
+
 struct Dna {
   const uint32_t* db;      // packed DB (global)
   uint32_t nwords;
@@ -167,15 +175,31 @@ struct Dna {
                                  : (__funnelshift_r(dn, dc, shd) ^ __funnelshift_r(qn, qc, shq));
         dc = dn;
         qc = qn;
+        const uint32_t n = (limit - d) < 16u ? (limit - d) : 16u;
+#if PL_S3_MSB
+        // step-ordered from the most significant bit: step d+1+e owns bit 31-2e or 30-2e, so
+        // the next mismatch is e = clz >> 1 (one FLO per mismatch, where __ffs is BREV + FLO
+        // on the per-mismatch dependency chain) and it is cleared with everything above it.
+        // Left: window position 15-e is step d+1+e, already MSB-first; right: one BREV per word.
+        uint32_t mm = (x | (x >> 1)) & 0x55555555u;
+        if (right) mm = __brev(mm);
+        uint32_t mmv = mm & (0xffffffffu << (32u - 2u * n));   // n >= 1: steps e < n
+        int last = 0;
+        while (mmv) {
+          const uint32_t c = __clz(mmv);
+          const int e = (int)(c >> 1);
+          mmv &= 0x7fffffffu >> c;
+          score += e - last;
+#else
         uint32_t mm = (x | (x >> 1)) & 0x55555555u;   // bit 2e set <=> mismatch at step d+1+e
         if (!right) mm = __brev(mm) >> 1;             // left: window position 15-e is step d+1+e
-        const uint32_t n = (limit - d) < 16u ? (limit - d) : 16u;
         uint32_t mmv = mm & (n >= 16u ? 0xffffffffu : ((1u << (2u * n)) - 1u));
         int last = 0;
         while (mmv) {
           const int e = (__ffs(mmv) - 1) >> 1;
           mmv &= mmv - 1;
           score += e - last;
+#endif
           if (score > best) { best = score; db_ = (int)d + e; }
           score -= 3;
           last = e + 1;
@@ -908,8 +932,21 @@ __device__ __forceinline__ void stage_batch(const Node& nd, const Dna& dna, cons
     }
   } else {   // S2 window filter / S3 x-drop: per item, one shared copy of the code
 #pragma unroll
-    for (int j = 0; j < K; ++j)
+    for (int j = 0; j < K; ++j) {
+#if PL_S3_DEBUG
+      const long long t0 = clock64();
+      const bool inw = act[j] && dna.in_win(e[j].x, 1000, 1000);
+#endif
       if (act[j]) o[j] = stage_count_ext(nd, dna, e[j]);
+#if PL_S3_DEBUG
+      const unsigned dt = (unsigned)(clock64() - t0);
+      const unsigned mx = __reduce_max_sync(0xffffffffu, dt);
+      const unsigned nin = __popc(__ballot_sync(0xffffffffu, inw));
+      const unsigned nact = __popc(__ballot_sync(0xffffffffu, act[j]));
+      if (nd.kind == PL_UNGAPPED_XDROP && blockIdx.x == 3 && (threadIdx.x & 31) == 0)
+        printf("S3 warp %d: max %u cycles, lane0 %u, active %u, in_win %u\n", threadIdx.x >> 5, mx, dt, nact, nin);
+#endif
+    }
   }
 }
 
