@@ -241,6 +241,20 @@ pl_status pl_pipeline_summary(pl_pipeline* pl, pl_summary* out);
  * return immediately (asynchronous).  Resets per-run outputs first.             */
 pl_status pl_pipeline_launch(pl_pipeline* pl);
 
+/* Pipelined stepping (a stream of runs, as a real-time deployment issues them): enqueue one
+ * run (as pl_pipeline_launch) followed by an asynchronous D->H copy of its pl_summary words
+ * into pinned host memory owned by the handle, then -- if an earlier pl_pipeline_step run
+ * exists -- block until THAT run has completed and return its summary in *prev
+ * (*has_prev = 1; prev->launches = its launch index).  The device executes run k while the
+ * host reads run k-1.  The first call returns *has_prev = 0.  The copy is ordered before the
+ * next launch on the stream, which reuses the run's device summary slot.  Errors: PL_EINVAL
+ * (NULL argument), PL_ENOMEM (pinned buffer), PL_EDEVICE (CUDA error).                    */
+pl_status pl_pipeline_step(pl_pipeline* pl, pl_summary* prev, int* has_prev);
+
+/* Block until the last pl_pipeline_step run has completed and return its summary in *last
+ * (*has_last = 0 if no step is outstanding); ends the step sequence.                      */
+pl_status pl_pipeline_step_finish(pl_pipeline* pl, pl_summary* last, int* has_last);
+
 /* Launch if nothing is in flight, then block until the run has completed; checks
  * device-side error flags (PL_EOVERFLOW) and CUDA errors (PL_EDEVICE).          */
 pl_status pl_pipeline_drain(pl_pipeline* pl);

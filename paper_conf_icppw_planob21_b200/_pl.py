@@ -102,6 +102,8 @@ def _load():
         "pl_pipeline_bind_device": (C.c_int32, [P, P, C.c_uint64]),
         "pl_pipeline_bind_host": (C.c_int32, [P, P, C.c_uint64]),
         "pl_pipeline_summary": (C.c_int32, [P, C.POINTER(pl_summary)]),
+        "pl_pipeline_step": (C.c_int32, [P, C.POINTER(pl_summary), C.POINTER(C.c_int)]),
+        "pl_pipeline_step_finish": (C.c_int32, [P, C.POINTER(pl_summary), C.POINTER(C.c_int)]),
         "pl_pipeline_queue_peaks": (C.c_int32, [P, P, C.c_uint64, C.POINTER(C.c_uint64)]),
         "pl_corunner_launch": (C.c_int, [P, C.c_uint32, C.c_uint64, P]),
         "pl_pipeline_launch": (C.c_int32, [P]),
@@ -134,7 +136,8 @@ EXPORTED = ("pl_pipeline_create", "pl_pipeline_set_stream", "pl_pipeline_push", 
             "pl_pipeline_results", "pl_pipeline_latency", "pl_pipeline_trace", "pl_pipeline_firings",
             "pl_pipeline_params", "pl_pipeline_destroy", "pl_last_error", "pl_solve_enforced_waits",
             "pl_solve_monolithic", "pl_version", "pl_stage_batch", "pl_pipeline_bind_host",
-            "pl_pipeline_summary", "pl_pipeline_queue_peaks", "pl_corunner_launch")
+            "pl_pipeline_summary", "pl_pipeline_queue_peaks", "pl_corunner_launch",
+            "pl_pipeline_step", "pl_pipeline_step_finish")
 
 
 class PlError(RuntimeError):

@@ -128,6 +128,11 @@ struct pl_pipeline {
   unsigned long long* d_summary = nullptr;   // device-reduced run summary
   int64_t* d_arr = nullptr;                  // per-root arrival times (optional)
   bool bound_host = false;
+  // pl_pipeline_step: two pinned summary buffers + completion events, by step parity
+  unsigned long long* h_step = nullptr;      // 2 x 7 words (cudaHostAlloc)
+  cudaEvent_t step_ev[2] = {nullptr, nullptr};
+  uint32_t step_launch[2] = {0, 0};          // launch index of the run in each buffer
+  uint64_t steps = 0;                        // pl_pipeline_step calls since the last finish
 };
 
 namespace {
@@ -138,6 +143,9 @@ void free_all(pl_pipeline* pl) {
                   pl->d_summary, pl->d_arr};
   for (void* p : ptrs)
     if (p) cudaFree(p);
+  if (pl->h_step) cudaFreeHost(pl->h_step);
+  for (cudaEvent_t& e : pl->step_ev)
+    if (e) cudaEventDestroy(e);
 }
 
 bool v_too_big(const pl_pipeline* pl) { return pl->cfg.vector_width > 256; }
@@ -571,23 +579,70 @@ pl_status pl_pipeline_queue_peaks(pl_pipeline* pl, uint32_t* buf, uint64_t cap, 
   return PL_OK;
 }
 
-pl_status pl_pipeline_summary(pl_pipeline* pl, pl_summary* out) {
-  if (!pl || !out) return fail(PL_EINVAL, "NULL argument");
-  cudaSetDevice(pl->device);
-  unsigned long long h[7];
-  CUDA_TRY(cudaMemcpyAsync(h, pl->d_match_count - 6, 56, cudaMemcpyDeviceToHost, pl->stream));
-  CUDA_TRY(cudaStreamSynchronize(pl->stream));
-  const unsigned long long mc = h[6];
-  pl->in_flight = false;
-  pl->d2h += 56;
+namespace {
+void decode_summary(const pl_pipeline* pl, const unsigned long long* h, uint32_t launch, pl_summary* out) {
   out->roots = h[0];
   out->miss_events = h[1];
   out->miss_events_ns = h[5];
   out->max_latency = (int64_t)h[2];
   out->max_latency_ns = (int64_t)h[3];
   out->errors = (uint32_t)h[4];
-  out->matches = std::min<uint64_t>(mc, pl->dp.match_cap);
-  out->launches = pl->launches;
+  out->matches = std::min<uint64_t>(h[6], pl->dp.match_cap);
+  out->launches = launch;
+}
+}  // namespace
+
+pl_status pl_pipeline_summary(pl_pipeline* pl, pl_summary* out) {
+  if (!pl || !out) return fail(PL_EINVAL, "NULL argument");
+  cudaSetDevice(pl->device);
+  unsigned long long h[7];
+  CUDA_TRY(cudaMemcpyAsync(h, pl->d_match_count - 6, 56, cudaMemcpyDeviceToHost, pl->stream));
+  CUDA_TRY(cudaStreamSynchronize(pl->stream));
+  pl->in_flight = false;
+  pl->d2h += 56;
+  decode_summary(pl, h, pl->launches, out);
+  return PL_OK;
+}
+
+
+pl_status pl_pipeline_step(pl_pipeline* pl, pl_summary* prev, int* has_prev) {
+  if (!pl || !prev || !has_prev) return fail(PL_EINVAL, "NULL argument");
+  cudaSetDevice(pl->device);
+  if (!pl->h_step) {
+    CUDA_TRY(cudaHostAlloc((void**)&pl->h_step, 2 * 7 * sizeof(unsigned long long), cudaHostAllocDefault));
+    for (cudaEvent_t& e : pl->step_ev) CUDA_TRY(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
+  }
+  const uint32_t b = (uint32_t)(pl->steps & 1u);
+  pl_status st = pl_pipeline_launch(pl);
+  if (st != PL_OK) return st;
+  // the run's summary slot is copied before the next launch (which zeroes it) can start
+  CUDA_TRY(cudaMemcpyAsync(pl->h_step + 7 * b, pl->d_match_count - 6, 56, cudaMemcpyDeviceToHost, pl->stream));
+  CUDA_TRY(cudaEventRecord(pl->step_ev[b], pl->stream));
+  pl->step_launch[b] = pl->launches;
+  pl->d2h += 56;
+  *has_prev = 0;
+  if (pl->steps > 0) {   // the previous step's run: wait for it only, the new one keeps running
+    const uint32_t pb = b ^ 1u;
+    CUDA_TRY(cudaEventSynchronize(pl->step_ev[pb]));
+    decode_summary(pl, pl->h_step + 7 * pb, pl->step_launch[pb], prev);
+    *has_prev = 1;
+  }
+  ++pl->steps;
+  return PL_OK;
+}
+
+pl_status pl_pipeline_step_finish(pl_pipeline* pl, pl_summary* last, int* has_last) {
+  if (!pl || !last || !has_last) return fail(PL_EINVAL, "NULL argument");
+  cudaSetDevice(pl->device);
+  *has_last = 0;
+  if (pl->steps > 0) {
+    const uint32_t b = (uint32_t)((pl->steps - 1) & 1u);
+    CUDA_TRY(cudaEventSynchronize(pl->step_ev[b]));
+    decode_summary(pl, pl->h_step + 7 * b, pl->step_launch[b], last);
+    *has_last = 1;
+  }
+  pl->steps = 0;
+  pl->in_flight = false;
   return PL_OK;
 }
 

@@ -131,6 +131,19 @@ class Pipeline:
     def launch(self):
         check(lib.pl_pipeline_launch(self.h), "pl_pipeline_launch")
 
+    def step(self):
+        """Pipelined run (pl_pipeline_step): launch the next run, return the PREVIOUS step's
+        summary (None on the first call) while the new run executes."""
+        s, has = _pl.pl_summary(), C.c_int()
+        check(lib.pl_pipeline_step(self.h, C.byref(s), C.byref(has)), "pl_pipeline_step")
+        return {k: getattr(s, k) for k, _ in s._fields_} if has.value else None
+
+    def step_finish(self):
+        """Summary of the last pl_pipeline_step run (None if none is outstanding)."""
+        s, has = _pl.pl_summary(), C.c_int()
+        check(lib.pl_pipeline_step_finish(self.h, C.byref(s), C.byref(has)), "pl_pipeline_step_finish")
+        return {k: getattr(s, k) for k, _ in s._fields_} if has.value else None
+
     def drain(self):
         check(lib.pl_pipeline_drain(self.h), "pl_pipeline_drain")
 

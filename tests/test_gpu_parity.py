@@ -296,3 +296,32 @@ def test_physical_loop_time_reported():
     # node 0 never waits for upstream, so every firing is a sample and the cycle contains it
     assert ph["max_loop_ns"][0] >= ph["max_fire_ns"][0] > 0
     assert all(x >= 0 for x in ph["max_loop_ns"][:4])
+
+
+def test_pipelined_steps_match_oracle():
+    """pl_pipeline_step: run k executes while the host reads run k-1's summary (pinned
+    buffers by step parity, copy ordered before the next launch reuses the device slot).
+    Every step's summary equals the oracle's counts, from the bound host DB (bind_host TMA)."""
+    import torch
+    from paper_conf_icppw_planob21_b200 import Pipeline
+    cfg = _dna(C.FIXED_WAIT, db_len=1 << 16, streams=5)
+    wl = workload_for(cfg)
+    o = run_oracle(cfg, wl)
+    roots = sum(hi - lo for lo, hi in _ranges(cfg, wl))
+    host = torch.from_numpy(wl.db.view("int32")).pin_memory()
+    pl = Pipeline(cfg, wl, flags=0)
+    pl.bind_host(host.data_ptr(), wl.db_len)
+    got = []
+    assert pl.step() is None             # first step: nothing to return yet
+    for _ in range(5):
+        got.append(pl.step())
+    got.append(pl.step_finish())
+    assert pl.step_finish() is None
+    assert [g["launches"] for g in got] == list(range(1, 7))
+    for g in got:
+        assert g["roots"] == roots and g["matches"] == len(o.matches)
+        assert g["max_latency"] == max(o.lat) and g["errors"] == 0
+    s = pl.summary()                     # the synchronous read agrees with the last step
+    assert s["roots"] == roots and s["matches"] == len(o.matches)
+    assert pl.results() == [tuple(m) for m in o.matches]
+    pl.close()
