@@ -1223,11 +1223,16 @@ __device__ void run_node(Ctx& c, const Dna dna, int i, int gtid) {
     if (leader) {   // publish (the critical path to the next firing), then the leader's own sums
       long long t4 = clock64();
       const uint32_t ph4 = (uint32_t)(t4 - tc);
+      // the leader's sums are loaded first and the statistics stored after the publish's
+      // fences: a fence waits for the thread's outstanding shared-memory operations, so an
+      // atomic or a read-modify-write ahead of it would sit on the critical path
+      ulonglong2* Cp = reinterpret_cast<ulonglong2*>(A.cnt);
+      ulonglong2* Pp = reinterpret_cast<ulonglong2*>(A.ph);
+      ulonglong2 c2 = Cp[2], p2 = Pp[2];
       uint64_t en = 0, fire = 0;
       if (nd.phys) {
         en = gtimer();
         fire = en - start_ns;
-        atomicMax(&A.max_fire, clamp32((int64_t)fire));
         if (rec & PL_FIXED_SERVICE) {   // hold the outputs until start + t_i (L69)
           const uint64_t due = T0 + units_ns(nd, T + nd.t);
           while (en < due) {
@@ -1235,7 +1240,6 @@ __device__ void run_node(Ctx& c, const Dna dna, int i, int gtid) {
             en = gtimer();
           }
         }
-        G.end_ns[par] = en;
       }
       // publish: the segment (outputs ready at T + t_i), then the watermark
       if (!nd.sink && total > 0 && out_loc != ~0u) {
@@ -1262,16 +1266,16 @@ __device__ void run_node(Ctx& c, const Dna dna, int i, int gtid) {
         L.B = T + nd.t;
         publish_W(nd, L, L.B + nd.t);
       }
-      {   // measured busy time, overruns, publish-phase cycles (the leader's slots of the sums)
-        ulonglong2* Cp = reinterpret_cast<ulonglong2*>(A.cnt);
-        ulonglong2* Pp = reinterpret_cast<ulonglong2*>(A.ph);
-        ulonglong2 c2 = Cp[2], p2 = Pp[2];
-        c2.x += nd.phys ? (en - start_ns) : 0ull;
-        c2.y += (nd.phys && (int64_t)fire > nd.t_ns) ? 1ull : 0ull;   // work outlasted t_i
-        p2.x += ph4;
-        p2.y += (uint64_t)(clock64() - t4);
-        Cp[2] = c2; Pp[2] = p2;
+      if (nd.phys) {
+        G.end_ns[par] = en;
+        atomicMax(&A.max_fire, clamp32((int64_t)fire));
       }
+      // measured busy time, overruns, publish-phase cycles (the leader's slots of the sums)
+      c2.x += nd.phys ? (en - start_ns) : 0ull;
+      c2.y += (nd.phys && (int64_t)fire > nd.t_ns) ? 1ull : 0ull;   // work outlasted t_i
+      p2.x += ph4;
+      p2.y += (uint64_t)(clock64() - t4);
+      Cp[2] = c2; Pp[2] = p2;
     }
     // The accountant (lane 0 of the node's second warp; the leader when v = 32) books the
     // firing off the leader's path: the lanes' troot / rmin stores and the leader's phase
