@@ -73,3 +73,31 @@ try:
          **timed(c2.replace(interarrival=tau, wait_time=tuple(w)))})
 except RuntimeError as ex:
     log({"result": "calibrated_b", "failed": str(ex)})
+
+# THRESHOLD_SLACK (the north_star rule; theta from Fig. 1, slack guard = the largest budget):
+# it fires on queue size or deadline slack, so it can absorb the repeat islands' bursts
+ct = cfg.replace(slack_guard=int(max(budgets)))
+try:
+    tau, w, th, T, st = realtime.find_rate(ct, wl, ptr, over=over, grow=1.6, tries=14, policy=1,
+                                           log=lambda d: log(dict(d, search="threshold_slack")))
+    log({"result": "threshold_slack", "D": D, "theta": list(th), "tau0": tau, "sustained": 148e9 / tau,
+         **timed(ct.replace(interarrival=tau, wait_threshold=tuple(th), policy=1))})
+except RuntimeError as ex:
+    log({"result": "threshold_slack", "failed": str(ex)})
+
+# MONOLITHIC (Fig. 2's block size M; no internal waiting): the fastest miss-free tau0
+tau = realtime.min_feasible_tau(cfg) or 1
+found = None
+for _ in range(16):
+    Mm = realtime.monolithic_at(cfg, tau)
+    if Mm is not None:
+        r = timed(cfg.replace(interarrival=tau, policy=2, block_size=Mm[0]))
+        log(dict(r, search="monolithic", tau0=tau, M=Mm[0]))
+        if r["misses_ns"] == 0 and r["errors"] == 0:
+            found = (tau, Mm[0], r)
+            break
+    tau = int(tau * 1.6) + 1
+if found:
+    log({"result": "monolithic", "D": D, "tau0": found[0], "M": found[1], "sustained": 148e9 / found[0], **found[2]})
+else:
+    log({"result": "monolithic", "failed": "no miss-free tau0 found"})
