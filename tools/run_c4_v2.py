@@ -3,7 +3,9 @@ Budgets from a full-vector probe (probe tau0 = 20 ns: node 0 always fires full v
 the repeat islands drive node 1 to full vectors with up to u = 16 outputs each), R-DRAIN end
 of stream, the fastest miss-free rate with the paper's b, then with b calibrated on the
 device from the streams' input-queue peaks (realtime.calibrate_b).
-argv: [deadline_ns]"""
+argv: [deadline_ns] [max_lateness_ns or "none"] (runs longer than ~1 s meet ~1.7 ms platform
+pauses, profiles/r01_globaltimer_pauses.txt, so long c4 runs need D well above that and no
+lateness bound)"""
 import json
 import sys
 import time
@@ -16,6 +18,7 @@ from plgen import dna as G
 from paper_conf_icppw_planob21_b200 import Pipeline, realtime
 
 D = int(sys.argv[1]) if len(sys.argv) > 1 else 1_000_000
+ML = None if len(sys.argv) > 2 and sys.argv[2] == "none" else (int(sys.argv[2]) if len(sys.argv) > 2 else 5000)
 log = lambda d: print(json.dumps(d), flush=True)
 base = C.c4()
 t0 = time.time()
@@ -53,7 +56,7 @@ def timed(c):
 
 for label, c in (("paper_b", cfg),):
     try:
-        tau, w, th, T, st = realtime.find_rate(c, wl, ptr, over=over, grow=1.6, tries=14,
+        tau, w, th, T, st = realtime.find_rate(c, wl, ptr, over=over, grow=1.6, tries=14, max_lateness_ns=ML,
                                                log=lambda d: log(dict(d, search=label)))
         log({"result": label, "D": D, "b": list(c.b), "tau0": tau, "w": list(w), "sustained": 148e9 / tau,
              **timed(c.replace(interarrival=tau, wait_time=tuple(w)))})
@@ -67,7 +70,7 @@ cb = realtime.calibrate_b(cfg.replace(interarrival=tau_c), wl, ptr, target=1.0, 
 log({"calibrated_b": list(cb["b"]), "miss_free": cb["miss_free"], "iterations": cb["iterations"]})
 c2 = cfg.replace(b=tuple(cb["b"]))
 try:
-    tau, w, th, T, st = realtime.find_rate(c2, wl, ptr, over=over, grow=1.6, tries=14,
+    tau, w, th, T, st = realtime.find_rate(c2, wl, ptr, over=over, grow=1.6, tries=14, max_lateness_ns=ML,
                                            log=lambda d: log(dict(d, search="calibrated_b")))
     log({"result": "calibrated_b", "D": D, "b": list(c2.b), "tau0": tau, "w": list(w), "sustained": 148e9 / tau,
          **timed(c2.replace(interarrival=tau, wait_time=tuple(w)))})
@@ -78,7 +81,7 @@ except RuntimeError as ex:
 # it fires on queue size or deadline slack, so it can absorb the repeat islands' bursts
 ct = cfg.replace(slack_guard=int(max(budgets)))
 try:
-    tau, w, th, T, st = realtime.find_rate(ct, wl, ptr, over=over, grow=1.6, tries=14, policy=1,
+    tau, w, th, T, st = realtime.find_rate(ct, wl, ptr, over=over, grow=1.6, tries=14, policy=1, max_lateness_ns=ML,
                                            log=lambda d: log(dict(d, search="threshold_slack")))
     log({"result": "threshold_slack", "D": D, "theta": list(th), "tau0": tau, "sustained": 148e9 / tau,
          **timed(ct.replace(interarrival=tau, wait_threshold=tuple(th), policy=1))})
