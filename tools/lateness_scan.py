@@ -18,7 +18,9 @@ dbl = int(sys.argv[7]) if len(sys.argv) > 7 else 1 << 20
 base = C.c2(n_streams=148, dna=dict(db_len=dbl, q_len=1024, n_planted=64 * dbl // (1 << 20)))
 wl = G.make_dna(base.seed, **base.dna)
 db = torch.from_numpy(wl.db.view("int32")).cuda()
-gains = realtime.measure_gains(base.replace(wait_time=(0,) * 4), wl, db.data_ptr())
+import os
+gains = (tuple(float(x) for x in os.environ["GAINS"].split(",")) if os.environ.get("GAINS")
+         else realtime.measure_gains(base.replace(wait_time=(0,) * 4), wl, db.data_ptr()))
 cfg = base.replace(clock=1, ns_per_unit=1.0, service_time=t, gain=gains, deadline=350_000, b=C.PAPER_B,
                    eager_drain=True)
 for tau in taus:
