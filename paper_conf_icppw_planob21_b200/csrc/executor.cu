@@ -1718,10 +1718,14 @@ __global__ void __launch_bounds__(MAXT, MINB) pl_exec_enforced(const __grid_cons
   __syncthreads();
   if (threadIdx.x == 0) sh.T0 = gtimer() + (p.clock == PL_CLOCK_GLOBALTIMER ? p.t0_offset_ns : 0u);
   __syncthreads();
-  // warp w serves node w % N (local warp w / N): with N = 4 every warp of node i sits on
-  // SM sub-partition i, so each SMSP's instruction cache holds one node's code path
+  // node i owns warps [i v/32, (i+1) v/32) (contiguous): with v = 128 each node has one warp
+  // on every SM sub-partition, so a node's heavy firing (S3's worst vectors) issues from all four
+  // SMSPs and node 0's loop shares each SMSP with one warp of every other node.  Measured at the
+  // bench point against the interleaved mapping (warp w -> node w % N, one node per SMSP, one
+  // code path per SMSP instruction cache; PL_VARIANT bit 4): node-0 lateness at tau0 = 15 ns
+  // 2.8 vs 5.4 us, longest node-0 / node-3 firings 1248 / 10656 vs 1376 / 11296 ns.
   const int w = threadIdx.x >> 5;
-  const bool contig = p.variant & 2u;   // experiment: node i owns warps [i v/32, (i+1) v/32)
+  const bool contig = !(p.variant & 4u);
   const int gi = contig ? w / (p.v >> 5) : w % p.N;
   const int gt = (contig ? w % (p.v >> 5) : w / p.N) * 32 + (threadIdx.x & 31);
   if (w < p.N * (p.v >> 5)) run_node<REC>(c, c.dna, gi, gt);

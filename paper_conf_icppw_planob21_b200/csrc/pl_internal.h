@@ -74,7 +74,7 @@ struct DevParams {
   int32_t  n_streams;
   uint32_t flags;
   int32_t  ctas_per_sm;                 // launch variant: 2 -> 64-register kernel, two streams per SM
-  uint32_t variant;                     // experiment bits (PL_VARIANT): 1 leader-paced node 0, 2 contiguous warps
+  uint32_t variant;                     // experiment bits (PL_VARIANT): 1 leader-paced node 0, 4 interleaved warps (node = warp % N)
   // DNA workload
   const uint32_t* db;                   // packed DB (device)
   uint64_t db_len;
