@@ -186,6 +186,9 @@ typedef struct {
   int64_t  t_end;                          /* sum over streams of the drain end time   */
   double   active_fraction;                /* PAPER.md L75 over [0,H)                  */
   double   active_fraction_nonempty;       /* same, charging non-empty firings only    */
+  double   active_fraction_drain;          /* the same ratio over [0, T_end], the drain included
+                                              (SURVEY §8(c) C-D "Outputs"): every firing started
+                                              before the stream's last completion, clipped to it */
   double   hw_busy_fraction;               /* physical: busy_ns / (N * wall)           */
   int64_t  wall_ns;                        /* max over streams of kernel-side runtime  */
   uint32_t errors;                         /* PL_EOVERFLOW bits etc.                   */
@@ -255,8 +258,10 @@ pl_status pl_pipeline_step(pl_pipeline* pl, pl_summary* prev, int* has_prev);
  * (*has_last = 0 if no step is outstanding); ends the step sequence.                      */
 pl_status pl_pipeline_step_finish(pl_pipeline* pl, pl_summary* last, int* has_last);
 
-/* Launch if nothing is in flight, then block until the run has completed; checks
- * device-side error flags (PL_EOVERFLOW) and CUDA errors (PL_EDEVICE).          */
+/* Block until the last launched run has completed -- launching one first if nothing was
+ * launched since the last push / bind / rewind -- and check its device-side error flags
+ * (PL_EOVERFLOW) and CUDA errors (PL_EDEVICE).  pl_pipeline_summary / step_finish do not
+ * consume the run: launch -> summary -> drain checks that same run.                      */
 pl_status pl_pipeline_drain(pl_pipeline* pl);
 
 /* Allow another push/launch cycle with the same pipeline (rewinds the stream).   */
@@ -309,11 +314,6 @@ pl_status pl_solve_monolithic(const pl_config* cfg, uint32_t* M_out, double* T_o
  * NULL) = longest per-vector clock64 duration.  Needs a pushed or bound DB for DNA.  */
 pl_status pl_stage_batch(pl_pipeline* pl, uint32_t stage, const void* in_dev, uint64_t n, uint64_t first_root,
                          void* out_dev, uint64_t cap, uint64_t* n_out, uint64_t* max_vec_cycles);
-
-/* Measurement utility (SURVEY §8(f) N3 co-runner experiment; not part of the method): launch
- * n_ctas CTAs of 128 threads of a compute-bound FMA kernel (iters rounds, 8 chains/thread) on
- * `stream`; `sink` is a device float[n_ctas] that is (almost) never written.  0 or PL_EDEVICE. */
-int pl_corunner_launch(void* stream, uint32_t n_ctas, uint64_t iters, float* sink);
 
 /* Library build identity (for logs): "plgpu <version> sm_100a".                  */
 const char* pl_version(void);

@@ -14,7 +14,9 @@ Modules:
   solver  — the optimisation problems of Fig. 1 (L139–L151) and Fig. 2 (L165–L180)
             by their definitions (integer brute force, exhaustive M) plus scipy
             SLSQP for the continuous Fig. 1 optimum
-  run     — CLI used for the CPU baseline timing
+  run     — CLI / timing harness of the DES over a bounded sample of a configuration's
+            streams (`python -m oracle.run --config c4 ...`), used by bench.py's cpu_baseline
+            and --impl reference legs
 
 Parity status per function is listed in DESIGN.md "Oracle pins".  Functions
 without an independent pin say "parity unpinned" in their docstring.

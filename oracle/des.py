@@ -61,6 +61,8 @@ class StreamResult:
     active_drain: list   # per node: sum |[s, s+t_i) ∩ [0, T_end)| over firings with s < T_end
     H: int
     T_end: int
+    max_queue: list = None   # per node: max |Q_i| at its firing decisions ("maximum
+                             # size b_i v"), counted before the firing takes its inputs
 
 
 def gains_G(g):
@@ -154,6 +156,7 @@ def simulate_stream(cfg: C.Config, fns, lo: int, hi: int, wait_time=None, theta=
     produced = [0] * N
     active_H = [0] * N
     active_H_ne = [0] * N
+    max_queue = [0] * N
     T_end = 0
     next_root = 0
     heap = [0] + ([arr[0]] if X else [])
@@ -209,6 +212,7 @@ def simulate_stream(cfg: C.Config, fns, lo: int, hi: int, wait_time=None, theta=
                 a_head = arr[Q[i][0][0] - lo]
                 fire = len(Q[i]) >= th[i] or T >= a_head + D - R[i]
             if fire:
+                max_queue[i] = max(max_queue[i], len(Q[i]))
                 n = min(len(Q[i]), v)
                 ents = [Q[i].popleft() for _ in range(n)]
                 for e in ents:
@@ -246,7 +250,7 @@ def simulate_stream(cfg: C.Config, fns, lo: int, hi: int, wait_time=None, theta=
     active_drain = [sum(_overlap(s, s + t[i], 0, T_end) for s in starts[i] if s < T_end)
                     for i in range(N)]
     return StreamResult(lo, hi, lat, trace, matches, firings, n_firings, n_empty, consumed,
-                        produced, active_H, active_H_ne, active_drain, H, T_end)
+                        produced, active_H, active_H_ne, active_drain, H, T_end, max_queue)
 
 
 def _check_conservation(N, entered, consumed, Q, produced, next_root, X, trace, lat):
@@ -320,7 +324,7 @@ def _simulate_monolithic(cfg, fns, lo, hi, M, arrivals=None):
     active_drain = [sum(_overlap(s, s + t[i], 0, T_end) for s in starts[i] if s < T_end)
                     for i in range(N)]
     return StreamResult(lo, hi, lat, trace, matches, firings, n_firings, [0] * N, consumed,
-                        produced, active_H, list(active_H), active_drain, H, T_end)
+                        produced, active_H, list(active_H), active_drain, H, T_end, [0] * N)
 
 
 # ------------------------------------------------------------------ drivers
@@ -332,6 +336,10 @@ class Result:
     trace: list
     matches: list
     N: int
+
+    def max_queue(self):
+        """Per node: the longest input queue over all streams at a firing decision."""
+        return [max((s.max_queue[i] for s in self.streams), default=0) for i in range(self.N)]
 
     def misses(self, D):
         return sum(1 for x in self.lat if x > D)
@@ -347,6 +355,10 @@ class Result:
         return acc / H if policy == C.MONOLITHIC else acc / (self.N * H)
 
     def active_fraction_drain(self, policy):
+        """The same ratio over [0, T_end] (the drain included; SURVEY §8(c) C-D "Outputs"):
+        every firing that starts before T_end, clipped to it, over N T_end (enforced) or
+        T_end (monolithic), summed over streams.  Pinned by test_oracle_des.py::
+        test_p1_drain_window_closed_form (FIXED_WAIT charges every slot m P_i < T_end)."""
         acc = sum(sum(s.active_drain) for s in self.streams)
         Te = sum(s.T_end for s in self.streams)
         return acc / Te if policy == C.MONOLITHIC else acc / (self.N * Te)

@@ -66,6 +66,34 @@ def fig1_bruteforce_int(t, g, b, v, tau, D):
     return list(best[1]), best[0][0]
 
 
+def fig1_exact_int_absorb(t, g, b, v, tau, D):
+    """Exact integer Fig. 1 optimum for N = 2 or 3 at moderate sizes.  For fixed P_1..P_{N-1}
+    the objective falls as P_0 grows, and P_0 is constrained only by
+    max(t_0, g_0 P_1) <= P_0 <= min(v tau0, (D - sum_{j>=1} b_j P_j) / b_0), so the best P_0 is
+    the top of that interval: enumerating every integer P_1..P_{N-1} (numpy grid) with that
+    P_0 is an exhaustive search.  Returns the optimal objective (or None if infeasible)."""
+    import numpy as np
+    N = len(t)
+    assert N in (2, 3)
+    ub = [(D - sum(b[j] * t[j] for j in range(N) if j != i)) // b[i] for i in range(N)]
+    axes = [np.arange(t[i], ub[i] + 1, dtype=np.int64) for i in range(1, N)]
+    if any(len(a) == 0 for a in axes):
+        return None
+    grid = np.meshgrid(*axes, indexing="ij")
+    P = [None] + [x.ravel() for x in grid]
+    rest = sum(b[j] * P[j] for j in range(1, N))
+    P0 = np.minimum((D - rest) // b[0], int(math.floor(v * tau)))
+    ok = (P0 >= t[0]) & (P[1] * g[0] <= P0)
+    if N == 3:
+        ok &= P[2] * g[1] <= P[1]
+    if not ok.any():
+        return None
+    T = t[0] / P0[ok].astype(float)
+    for j in range(1, N):
+        T = T + t[j] / P[j][ok].astype(float)
+    return float(T.min()) / N
+
+
 def fig1_continuous(t, g, b, v, tau, D, starts=8, seed=0):
     """Continuous Fig. 1 optimum by scipy SLSQP from several feasible-ish starts."""
     import numpy as np

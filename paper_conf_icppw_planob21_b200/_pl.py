@@ -74,6 +74,7 @@ class pl_stats(C.Structure):
                 ("max_latency", C.c_int64),
                 ("max_latency_ns", C.c_int64), ("window", C.c_int64), ("t_end", C.c_int64),
                 ("active_fraction", C.c_double), ("active_fraction_nonempty", C.c_double),
+                ("active_fraction_drain", C.c_double),
                 ("hw_busy_fraction", C.c_double), ("wall_ns", C.c_int64), ("errors", C.c_uint32),
                 ("launches", C.c_uint32), ("h2d_bytes", C.c_uint64), ("d2h_bytes", C.c_uint64)]
 
@@ -105,7 +106,6 @@ def _load():
         "pl_pipeline_step": (C.c_int32, [P, C.POINTER(pl_summary), C.POINTER(C.c_int)]),
         "pl_pipeline_step_finish": (C.c_int32, [P, C.POINTER(pl_summary), C.POINTER(C.c_int)]),
         "pl_pipeline_queue_peaks": (C.c_int32, [P, P, C.c_uint64, C.POINTER(C.c_uint64)]),
-        "pl_corunner_launch": (C.c_int, [P, C.c_uint32, C.c_uint64, P]),
         "pl_pipeline_launch": (C.c_int32, [P]),
         "pl_pipeline_drain": (C.c_int32, [P]),
         "pl_pipeline_rewind": (C.c_int32, [P]),
@@ -136,7 +136,7 @@ EXPORTED = ("pl_pipeline_create", "pl_pipeline_set_stream", "pl_pipeline_push", 
             "pl_pipeline_results", "pl_pipeline_latency", "pl_pipeline_trace", "pl_pipeline_firings",
             "pl_pipeline_params", "pl_pipeline_destroy", "pl_last_error", "pl_solve_enforced_waits",
             "pl_solve_monolithic", "pl_version", "pl_stage_batch", "pl_pipeline_bind_host",
-            "pl_pipeline_summary", "pl_pipeline_queue_peaks", "pl_corunner_launch",
+            "pl_pipeline_summary", "pl_pipeline_queue_peaks",
             "pl_pipeline_step", "pl_pipeline_step_finish")
 
 

@@ -17,7 +17,10 @@ LIB = os.path.join(HERE, "libplgpu.so")
 NVCC = os.environ.get("NVCC", "nvcc")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 FLAGS = ["-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC,-O2", f"-I{ROOT}/include", f"-I{CSRC}"]
-SOURCES = ["executor.cu", "runtime.cu", "solver.cpp", "corunner.cu"]
+SOURCES = ["executor.cu", "runtime.cu", "solver.cpp"]
+# measurement tool, not part of the product library (N3 co-runner experiment, tools/corunner.py)
+CORUNNER_SRC = os.path.join(ROOT, "tools", "corunner", "corunner.cu")
+CORUNNER_LIB = os.path.join(ROOT, "tools", "corunner", "libplcorunner.so")
 
 
 def _stale() -> bool:
@@ -52,6 +55,17 @@ def build(force: bool = False, verbose: bool = False) -> str:
         raise RuntimeError(f"link failed:\n{r.stderr}")
     os.replace(tmp, LIB)
     return LIB
+
+
+def build_corunner() -> str:
+    """The co-runner kernel of the N3 experiment as its own small library."""
+    if os.path.exists(CORUNNER_LIB) and os.path.getmtime(CORUNNER_LIB) > os.path.getmtime(CORUNNER_SRC):
+        return CORUNNER_LIB
+    cmd = [NVCC, *ARCH, "-O3", "-Xcompiler", "-fPIC", "-shared", CORUNNER_SRC, "-o", CORUNNER_LIB]
+    r = subprocess.run(cmd, capture_output=True, text=True)
+    if r.returncode != 0:
+        raise RuntimeError(f"nvcc failed for corunner.cu:\n{r.stderr}")
+    return CORUNNER_LIB
 
 
 if __name__ == "__main__":

@@ -286,7 +286,7 @@ struct EdgeCtl {            // queue INTO node i
   uint32_t tail;            // producer: one past last published entry
   int64_t  W;               // producer watermark
   uint32_t spill_end;       // producer: end seq of the last spilled segment
-  uint32_t pad;
+  uint32_t stalled;         // producer: waiting for room in this queue (reserve_out)
 };
 struct GroupCtl {           // broadcast from a node's leader to its lanes, double-buffered
   int64_t  T[2];            // by firing parity so that no barrier is needed between firings
@@ -301,7 +301,7 @@ struct GroupCtl {           // broadcast from a node's leader to its lanes, doub
 // 64-bit shared atomics compile to CAS spin loops (ATOMS.CAST.SPIN.64), so the single writer
 // stores per-firing 32-bit deltas (d[]) as it goes and folds everything into the 64-bit sums
 // with one vectorised read-modify-write per firing; maxima use native 32-bit ATOMS.MAX.
-enum { C_FIRINGS, C_CONSUMED, C_PRODUCED, C_ACTIVE, C_BUSY, C_OVERRUNS, C_SPILLED, C_STALLS, C_ACTIVE_E, C_PAD, C_N };
+enum { C_FIRINGS, C_CONSUMED, C_PRODUCED, C_ACTIVE, C_BUSY, C_OVERRUNS, C_SPILLED, C_STALLS, C_ACTIVE_E, C_DRAINF, C_N };
 enum { D_PH0, D_PH1, D_PH2, D_PH3, D_STALL, D_N = 8 };
 struct NodeAcc {
   alignas(16) unsigned long long cnt[C_N];
@@ -594,6 +594,18 @@ __device__ __forceinline__ uint32_t count_le(const Node& nd, const Leader& L, ui
   return end - L.head;
 }
 
+// number of PUBLISHED entries of the input edge with ready <= T, uncapped: the queue length
+// |Q_i| at a firing decision at T (PAPER.md L133's "maximum size b_i v").  Segments are
+// published in firing order, so their ready times are non-decreasing: binary search.
+__device__ __forceinline__ uint32_t count_all_le(const Node& nd, const Leader& L, uint32_t st, int64_t T) {
+  uint32_t lo = L.segh, hi = st;          // first segment with ready > T
+  while (lo != hi) {
+    const uint32_t mid = lo + ((hi - lo) >> 1);
+    if (nd.in_seg[mid & nd.segmask].ready <= T) lo = mid + 1; else hi = mid;
+  }
+  return lo == L.segh ? 0u : nd.in_seg[(lo - 1) & nd.segmask].end - L.head;
+}
+
 // Node 0: arrivals are fully known (root lo+r arrives at r*tau0), so every
 // lane evaluates the firing decision itself from replicated state (no broadcast barrier).
 struct Rep {
@@ -707,6 +719,13 @@ __device__ __forceinline__ bool nap_until(uint64_t target) {
 // only for the poll that decides the firing; yielded time is usable).
 constexpr uint64_t PL_NAP_LEAD_NS = 768;
 
+// A node may commit a firing at T before its upstream watermark passes T once v entries with
+// ready <= T are queued (the firing is full whatever else arrives).  On the logical clock it
+// does so only when the producer is stalled on this queue -- needed for deadlock freedom,
+// so that every other decision sees the complete queue at T and the
+// recorded queue peak is the DES's |Q_i| exactly; the physical clock always may.
+__device__ __forceinline__ bool early_ok(const Node& nd) { return nd.phys || vld(&nd.Ein->stalled) != 0u; }
+
 __device__ Decision decide(const Node& nd, Leader& L, bool& waited, uint64_t T0) {
   const uint32_t v = (uint32_t)nd.v;
   Decision d;
@@ -740,14 +759,16 @@ __device__ Decision decide(const Node& nd, Leader& L, bool& waited, uint64_t T0)
         const int64_t Te = max(B, nd.in_seg[L.segh & nd.segmask].ready);
         const uint32_t cnt = count_le(nd, L, st, Te);
         publish_W(nd, L, Te + nd.t);     // the firing starts at Te; only its size is pending
-        if (Wup > Te || cnt >= v) { d.T = Te; d.n = cnt < v ? cnt : v; d.qlen = tail_known - L.head; return d; }
+        if (Wup > Te || (cnt >= v && early_ok(nd))) {
+          d.T = Te; d.n = cnt < v ? cnt : v; d.qlen = count_all_le(nd, L, st, Te); return d;
+        }
         backoff(spins, nd.phys); waited = true;
         continue;
       }
       const int64_t T = L.m * nd.P;
       const uint32_t cnt = count_le(nd, L, st, T);
-      if (cnt >= v || Wup > T) {
-        if (cnt > 0) { d.T = T; d.n = cnt < v ? cnt : v; d.qlen = tail_known - L.head; return d; }
+      if (Wup > T || (cnt >= v && early_ok(nd))) {
+        if (cnt > 0) { d.T = T; d.n = cnt < v ? cnt : v; d.qlen = count_all_le(nd, L, st, T); return d; }
         if (!any && Wup == PL_INF64) { d.done = true; return d; }
         const int64_t r = any ? nd.in_seg[L.segh & nd.segmask].ready : Wup;
         int64_t m2 = cdiv(r, nd.dP);
@@ -789,8 +810,8 @@ __device__ Decision decide(const Node& nd, Leader& L, bool& waited, uint64_t T0)
     if (nd.eager) Tk = min(Tk, max(max(L.B, nd.A_last), hs.ready));   // R-DRAIN
     if (th_known || Tk < Wup) {
       const uint32_t cnt = count_le(nd, L, st, Tk);
-      if (Wup > Tk || cnt >= v) {
-        d.T = Tk; d.n = cnt < v ? cnt : v; d.qlen = tail_known - L.head;
+      if (Wup > Tk || (cnt >= v && early_ok(nd))) {
+        d.T = Tk; d.n = cnt < v ? cnt : v; d.qlen = count_all_le(nd, L, st, Tk);
         // committed: nothing leaves this node before Tk + t_i.  Publish it now -- a physical
         // firing may be paced far into the future (slack) and downstream must not wait for it.
         publish_W(nd, L, Tk + nd.t);
@@ -814,8 +835,9 @@ __device__ uint32_t reserve_out(const Node& nd, Leader& L, uint32_t worst, uint3
     const uint32_t h = vld(&nd.Eout->head), sh = vld(&nd.Eout->seg_head);
     const bool seg_ok = (L.out_segt - sh) <= nd.segmask;
     const uint32_t need = L.out_tail + worst - h;
-    if (seg_ok && need <= nd.out_cap) return LOC_SMEM;
-    if (seg_ok && need <= nd.capg) return LOC_SPILL;
+    if (seg_ok && need <= nd.out_cap) { if (*stalled) vst(&nd.Eout->stalled, 0u); return LOC_SMEM; }
+    if (seg_ok && need <= nd.capg) { if (*stalled) vst(&nd.Eout->stalled, 0u); return LOC_SPILL; }
+    if (!*stalled) vst(&nd.Eout->stalled, 1u);
     *stalled = 1u;
     backoff(spins);
   }
@@ -1027,7 +1049,16 @@ __device__ void run_node(Ctx& c, const Dna dna, int i, int gtid) {
       if (d.done) break;
       T = d.T; n = d.n; head = (uint32_t)R.c0;
       if (leader) {
-        atomicMax(&A.max_queue, d.qlen);
+        uint32_t ql = d.qlen;
+        if (nd.arr) {                    // arrival data: roots arrived by T (binary search), not yet consumed
+          int64_t a = R.c0, b = nd.X;    // first local root with arrival > T
+          while (a < b) {
+            const int64_t mid = (a + b) >> 1;
+            if (__ldg(nd.arr + nd.lo + mid) <= T) a = mid + 1; else b = mid;
+          }
+          ql = (uint32_t)(a - R.c0);
+        }
+        atomicMax(&A.max_queue, ql);
         publish_W(nd, L, T + nd.t);      // committed: nothing leaves node 0 before T + t_0
         if (rec & PL_REC_FIRINGS) G.log_idx[par] = atomicAdd(&c.sh->log_count, 1u);
         A.d[par][D_STALL] = 0;
@@ -1331,6 +1362,7 @@ __device__ void run_node(Ctx& c, const Dna dna, int i, int gtid) {
         const unsigned long long ov = (unsigned long long)overlap(T, T + nd.t, 0, nd.H);
         c1.y += ov;
         c4.x += (nd.eager && T >= nd.A_last) ? ov : 0ull;   // R-DRAIN firings (FIXED_WAIT window)
+        c4.y += (nd.eager && T >= nd.A_last) ? 1ull : 0ull;
         c3.x += (!nd.sink && out_loc == LOC_SPILL) ? (unsigned long long)total : 0ull;
         c3.y += stl;
         p0.x += dd.x; p0.y += dd.y; p1.x += dd.z; p1.y += dd.w;
@@ -1377,6 +1409,7 @@ __device__ void run_node(Ctx& c, const Dna dna, int i, int gtid) {
     S.spilled[i] = A.cnt[C_SPILLED];
     S.overruns[i] = A.cnt[C_OVERRUNS];
     S.stalls[i] = A.cnt[C_STALLS];
+    S.drain_firings[i] = A.cnt[C_DRAINF];
     S.max_queue[i] = A.max_queue;
     S.lateness[i] = (int64_t)A.lateness;
     S.sched_cycles[i] = A.ph[0];
@@ -1505,7 +1538,7 @@ __device__ void cta_setup(Ctx& c, Shared& sh, unsigned char* dsm, const DevParam
   }
   if (tid < PL_MAX_STAGES) {
     EdgeCtl& E = sh.e[tid];
-    E.head = 0; E.seg_head = 0; E.seg_tail = 0; E.tail = 0; E.W = -1; E.spill_end = 0; E.pad = 0;
+    E.head = 0; E.seg_head = 0; E.seg_tail = 0; E.tail = 0; E.W = -1; E.spill_end = 0; E.stalled = 0;
   }
   if (tid == 0) {
     sh.max_lat = 0; sh.max_lat_ns = 0; sh.miss_events = 0; sh.miss_events_ns = 0; sh.errors = 0; sh.log_count = 0;
@@ -1697,7 +1730,7 @@ __device__ void run_monolithic(Ctx& c) {
       S.firings[i] = firings[i]; S.empty[i] = 0; S.consumed[i] = consumed[i]; S.produced[i] = produced[i];
       S.active_ne[i] = active[i]; S.active_win[i] = active[i]; S.busy_ns[i] = i == 0 ? busy_ns : 0;
       S.spilled[i] = 0; S.overruns[i] = 0;
-      S.stalls[i] = 0; S.max_queue[i] = 0;
+      S.stalls[i] = 0; S.max_queue[i] = 0; S.drain_firings[i] = 0;
       S.lateness[i] = 0; S.sched_cycles[i] = 0; S.max_fire_ns[i] = 0; S.max_loop_ns[i] = 0;
       for (int k = 0; k < 6; ++k) S.phase_cycles[i][k] = 0;
     }

@@ -42,6 +42,7 @@ struct CtaStats {
   uint64_t spilled[PL_MAX_STAGES];
   uint64_t overruns[PL_MAX_STAGES];
   uint64_t stalls[PL_MAX_STAGES];
+  uint64_t drain_firings[PL_MAX_STAGES]; // R-DRAIN firings (at T >= A_last)
   uint32_t max_queue[PL_MAX_STAGES];
   int64_t  lateness[PL_MAX_STAGES];
   uint64_t sched_cycles[PL_MAX_STAGES];

@@ -73,6 +73,7 @@ uint64_t prob_to_u64(double p) {
   uint64_t mant = (uint64_t)std::ldexp(m, 53);   // exact 53-bit integer
   int sh = 64 + e - 53;                     // p 2^64 = mant 2^(64+e-53)
   if (sh >= 0) return sh >= 11 + 53 ? ~0ull : (mant << sh);
+  if (-sh >= 64) return 0;                  // p < 2^-64 (a shift >= 64 would be undefined)
   return mant >> (-sh);
 }
 
@@ -120,13 +121,15 @@ struct pl_pipeline {
   uint64_t db_alloc_words = 0;
   // host state
   uint64_t pushed = 0;      // DNA: bases; gain: roots per stream
-  bool in_flight = false, drained = false;
+  bool launched = false;    // a run was launched since create / the last rewind (drain does not relaunch it)
+  bool drained = false;
   uint32_t launches = 0;
   int device = 0;
   uint64_t h2d = 0, d2h = 0;  // bytes moved across the host boundary (cumulative)
   unsigned long long* d_scratch = nullptr;   // stage-batch counters
   unsigned long long* d_summary = nullptr;   // device-reduced run summary
   int64_t* d_arr = nullptr;                  // per-root arrival times (optional)
+  std::vector<int64_t> h_arr;                // host copy (drain-window accounting)
   bool bound_host = false;
   // pl_pipeline_step: two pinned summary buffers + completion events, by step parity
   unsigned long long* h_step = nullptr;      // 2 x 7 words (cudaHostAlloc)
@@ -498,6 +501,7 @@ pl_status pl_pipeline_create(const pl_config* cfg, const pl_workload* wl, pl_pip
     }
     if (cudaMalloc(&pl->d_arr, R * 8) != cudaSuccess) return bail(fail(PL_ENOMEM, "arrival times"));
     cudaMemcpy(pl->d_arr, cfg->arrivals, R * 8, cudaMemcpyHostToDevice);
+    pl->h_arr.assign(cfg->arrivals, cfg->arrivals + R);
     pl->h2d += R * 8;
   }
   d.arr = pl->d_arr;
@@ -543,6 +547,7 @@ pl_status pl_pipeline_bind_device(pl_pipeline* pl, const void* dev_items, uint64
   pl->d_db_bound = (const uint32_t*)dev_items;
   pl->bound_host = false;
   pl->pushed = n;
+  pl->launched = false;
   return PL_OK;
 }
 
@@ -560,6 +565,7 @@ pl_status pl_pipeline_bind_host(pl_pipeline* pl, const void* host_items, uint64_
   pl->d_db_bound = (const uint32_t*)dptr;
   pl->bound_host = true;
   pl->pushed = n;
+  pl->launched = false;
   return PL_OK;
 }
 
@@ -598,7 +604,6 @@ pl_status pl_pipeline_summary(pl_pipeline* pl, pl_summary* out) {
   unsigned long long h[7];
   CUDA_TRY(cudaMemcpyAsync(h, pl->d_match_count - 6, 56, cudaMemcpyDeviceToHost, pl->stream));
   CUDA_TRY(cudaStreamSynchronize(pl->stream));
-  pl->in_flight = false;
   pl->d2h += 56;
   decode_summary(pl, h, pl->launches, out);
   return PL_OK;
@@ -642,7 +647,6 @@ pl_status pl_pipeline_step_finish(pl_pipeline* pl, pl_summary* last, int* has_la
     *has_last = 1;
   }
   pl->steps = 0;
-  pl->in_flight = false;
   return PL_OK;
 }
 
@@ -670,19 +674,18 @@ pl_status pl_pipeline_launch(pl_pipeline* pl) {
   CUDA_TRY(pl_launch(d, pl->cfg.n_streams, pl->block, pl->smem, pl->stream));
   pl->d_match_count = d.summary + 6;       // readers see the slot of the last launch
   pl->slot ^= 1u;
-  pl->in_flight = true;
+  pl->launched = true;
   pl->launches++;
   return PL_OK;
 }
 
 pl_status pl_pipeline_drain(pl_pipeline* pl) {
   if (!pl) return fail(PL_EINVAL, "NULL pipeline");
-  if (!pl->in_flight) {
+  if (!pl->launched) {     // nothing launched since create / rewind: run the pushed stream now
     pl_status s = pl_pipeline_launch(pl);
     if (s != PL_OK) return s;
   }
   CUDA_TRY(cudaStreamSynchronize(pl->stream));
-  pl->in_flight = false;
   pl->drained = true;
   std::vector<CtaStats> cs(pl->cfg.n_streams);
   CUDA_TRY(cudaMemcpy(cs.data(), pl->d_stats, cs.size() * sizeof(CtaStats), cudaMemcpyDeviceToHost));
@@ -696,6 +699,7 @@ pl_status pl_pipeline_drain(pl_pipeline* pl) {
 pl_status pl_pipeline_rewind(pl_pipeline* pl) {
   if (!pl) return fail(PL_EINVAL, "NULL pipeline");
   pl->drained = false;
+  pl->launched = false;
   if (!pl->d_db_bound) pl->pushed = 0;
   return PL_OK;
 }
@@ -755,6 +759,40 @@ pl_status pl_pipeline_stats(pl_pipeline* pl, pl_stats* out) {
   const double denom = pl->cfg.policy == PL_MONOLITHIC ? (double)out->window : (double)N * (double)out->window;
   out->active_fraction = out->window ? act / denom : 0.0;
   out->active_fraction_nonempty = out->window ? act_ne / denom : 0.0;
+  {   // drain-inclusive ratio over [0, T_end] per stream (SURVEY §8(c) C-D "Outputs"):
+      // FIXED_WAIT charges every time-triggered slot m P_i < T_end clipped to T_end (L97; with
+      // R-DRAIN only the slots m P_i < A_last) plus the drain firings; every other firing of
+      // any policy ends by T_end and is charged t_i.
+    double acc = 0, te_sum = 0;
+    uint64_t r0 = 0;
+    for (const CtaStats& s : cs) {
+      const int64_t Te = s.t_end;
+      te_sum += (double)Te;
+      for (uint32_t i = 0; i < N; ++i) {
+        const int64_t t = pl->t[i];
+        if (pl->cfg.policy == PL_FIXED_WAIT) {
+          const int64_t P = pl->t[i] + pl->w[i];
+          int64_t K = Te > 0 ? (Te + P - 1) / P : 0;          // slots m P < T_end
+          if (pl->cfg.flags & PL_EAGER_DRAIN) {
+            const int64_t A_last = s.n_roots == 0 ? 0
+                : (pl->h_arr.empty() ? (int64_t)(s.n_roots - 1) * tau : pl->h_arr[r0 + s.n_roots - 1]);
+            K = std::min<int64_t>(K, (A_last + P - 1) / P);   // slots m P < A_last
+            acc += (double)s.drain_firings[i] * (double)t;
+          }
+          if (K > 0) {
+            const int64_t full = Te >= t ? std::min<int64_t>(K, (Te - t) / P + 1) : 0;   // m P + t <= T_end
+            acc += (double)full * (double)t;
+            for (int64_t m = full; m < K; ++m) acc += (double)std::min<int64_t>(t, Te - m * P);
+          }
+        } else {
+          acc += (double)s.firings[i] * (double)t;
+        }
+      }
+      r0 += s.n_roots;
+    }
+    const double dd = pl->cfg.policy == PL_MONOLITHIC ? te_sum : (double)N * te_sum;
+    out->active_fraction_drain = dd > 0 ? acc / dd : 0.0;
+  }
   if (out->wall_ns > 0) {
     const double procs = pl->cfg.policy == PL_MONOLITHIC ? 1.0 : (double)N;
     out->hw_busy_fraction = busy / (procs * (double)out->wall_ns * (double)S);

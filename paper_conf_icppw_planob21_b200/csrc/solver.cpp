@@ -11,8 +11,11 @@
 // (block value sqrt(sum c / (lambda sum a))), which is then clipped to the
 // order-compatible bounds [max_{j>=i} G_j t_j, v tau0].  lambda is found by
 // bisection on the (monotone) deadline slack.  The integer answer (reading A17)
-// is the best feasible point of a chain-aware branch-and-bound search, ties broken
-// towards the lexicographically smallest w.
+// is the best feasible point of two neighbourhood searches around the continuous
+// optimum -- a chain-aware depth-first search, and a slack-absorption pass that gives
+// one stage the largest value the others leave it -- ties broken towards the
+// lexicographically smallest w.  Not a proof of integer optimality: it is checked
+// against the oracle's exact search (tests/test_abi.py) where that search is exact.
 // Fig. 2: exhaustive search over M while b M tau0 + S Tbar(M) <= D.
 #include <cmath>
 #include <cstdint>
@@ -191,6 +194,59 @@ int solve_fig1(int N, const int64_t* t, const double* g, const uint32_t* b, uint
       found = true;
       best = T;
       std::memcpy(bestP, P, sizeof(int64_t) * N);
+    }
+  }
+  // Slack absorption.  Rounding the other stages down can free more deadline units than the
+  // window above reaches, so for every stage a (the one that absorbs the slack): enumerate the
+  // other stages over floor(P_j) - RA .. floor(P_j) + RA + 1 and give P_a the LARGEST value the
+  // constraints allow (t_a / P_a falls as P_a grows, so for fixed others that is optimal):
+  // P_a <= v tau0 (a = 0), P_a <= P_{a-1} / g_{a-1}, g_a P_{a+1} <= P_a, b_a P_a <= D - rest.
+  {
+    const int RA = N <= 4 ? 8 : (N <= 5 ? 4 : (N <= 6 ? 2 : 1));
+    const int span = 2 * RA + 2;
+    int64_t Q2[PL_MAX_STAGES];
+    for (int a = 0; a < N; ++a) {
+      int64_t combos = 1;
+      for (int j = 0; j < N - 1; ++j) combos *= span;
+      for (int64_t code = 0; code < combos; ++code) {
+        int64_t cc = code;
+        int64_t rest = 0;
+        bool ok = true;
+        for (int j = 0; j < N && ok; ++j) {
+          if (j == a) continue;
+          Q2[j] = (int64_t)std::floor(Pc[j]) - RA + (cc % span);
+          cc /= span;
+          if (Q2[j] < t[j]) ok = false;
+          rest += (int64_t)b[j] * Q2[j];
+        }
+        if (!ok) continue;
+        int64_t ub = (D - rest) / (int64_t)b[a];
+        if (D - rest < 0) continue;
+        if (a == 0) ub = std::min<int64_t>(ub, (int64_t)std::floor((double)v * (double)tau));
+        if (a > 0) {
+          int64_t c2 = (int64_t)std::floor((double)Q2[a - 1] / g[a - 1]);
+          while (c2 > 0 && (double)c2 * g[a - 1] > (double)Q2[a - 1]) --c2;
+          while ((double)(c2 + 1) * g[a - 1] <= (double)Q2[a - 1]) ++c2;
+          ub = std::min(ub, c2);
+        }
+        if (ub < t[a]) continue;
+        Q2[a] = ub;
+        if (!feasible(N, t, g, b, v, tau, D, Q2)) continue;
+        double Pd[PL_MAX_STAGES];
+        for (int i = 0; i < N; ++i) Pd[i] = (double)Q2[i];
+        const double T = objective(N, t, Pd);
+        bool better = !found || T < best;
+        if (found && T == best) {
+          better = false;
+          for (int i = 0; i < N; ++i)
+            if (Q2[i] != bestP[i]) { better = Q2[i] < bestP[i]; break; }
+        }
+        if (better) {
+          found = true;
+          best = T;
+          std::memcpy(bestP, Q2, sizeof(int64_t) * N);
+        }
+      }
     }
   }
   if (!found) return PL_EINFEASIBLE;

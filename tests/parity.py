@@ -73,6 +73,13 @@ def compare(cfg, g, o, check_firings=True):
     elif "lat" in g:       # physical: pl_stats.misses counts measured latencies; the schedule's are exact
         assert int((g["lat"] > cfg.deadline).sum()) == o.misses(cfg.deadline)
     assert abs(st["active_fraction"] - o.active_fraction(cfg.policy)) < 1e-12
+    # the vacation reading of L97 (non-empty firings only) and the drain-inclusive ratio
+    assert abs(st["active_fraction_nonempty"] - o.active_fraction(cfg.policy, nonempty=True)) < 1e-12
+    assert abs(st["active_fraction_drain"] - o.active_fraction_drain(cfg.policy)) < 1e-12
+    # queue peaks at firing decisions (L133's b_i v): exact on the logical clock, where a node
+    # commits before its upstream watermark passes T only when the producer is stalled
+    if cfg.policy != C.MONOLITHIC and cfg.clock == C.CLOCK_LOGICAL and sum(st["stalls"]) == 0:
+        assert st["max_queue"] == o.max_queue(), (st["max_queue"], o.max_queue())
 
 
 _WL = None

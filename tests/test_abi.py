@@ -138,3 +138,46 @@ def test_solver_fig1_random_vs_bruteforce(seed):
         return
     assert Pi is not None
     assert abs(T - Ti) < 1e-12, (t, g, b, v, tau, D, [w[i] + t[i] for i in range(len(t))], Pi)
+
+
+@pytest.mark.parametrize("seed", range(60))
+def test_solver_fig1_random_vs_exact_absorb(seed):
+    """Larger random problems (b_i up to 16, deadlines of thousands of units: the regime where
+    rounding the b_i > 1 stages down frees slack for another stage) against the oracle's exact
+    search (every P_1..P_{N-1}, P_0 at the top of its feasible interval)."""
+    import random
+    from paper_conf_icppw_planob21_b200 import PlError, solve_enforced_waits
+    rnd = random.Random(1000 + seed)
+    N = rnd.choice([2, 3])
+    t = tuple(rnd.randint(20, 300) for _ in range(N))
+    g = tuple(round(rnd.uniform(0.3, 2.0), 3) for _ in range(N - 1))
+    b = tuple(rnd.randint(1, 16) for _ in range(N))
+    v = rnd.choice([16, 32, 128])
+    tau = rnd.randint(2, 40)
+    base = sum(x * y for x, y in zip(t, b))
+    D = rnd.randint(base, min(3 * base, base + 2500 * min(b)))
+    cfg = C.Config(name="r", stages=[C.Stage(C.BERNOULLI, 0.5, 1)] * N, service_time=t, vector_width=32,
+                   deadline=D, interarrival=tau, b=b, gain=g)
+    cfg.vector_width = v
+    To = SV.fig1_exact_int_absorb(t, g, b, v, tau, D)
+    try:
+        w, th, T, Tc = solve_enforced_waits(cfg)
+    except PlError:
+        assert To is None
+        return
+    assert To is not None
+    assert abs(T - To) <= 1e-12 * To, (t, g, b, v, tau, D, [w[i] + t[i] for i in range(N)])
+
+
+def test_solver_fig1_advisor_case():
+    """The case the round-1 review found (t=(2124,1196,1743,2851), g=(.5,1,.5), b=(1,16,7,16),
+    v=256, tau0=56, D=103030): P_0 = 8654 is feasible and better than 8653."""
+    from paper_conf_icppw_planob21_b200 import solve_enforced_waits
+    t, g, b, v, tau, D = (2124, 1196, 1743, 2851), (0.5, 1.0, 0.5), (1, 16, 7, 16), 256, 56, 103030
+    cfg = C.Config(name="r", stages=[C.Stage(C.BERNOULLI, 0.5, 1)] * 4, service_time=t, vector_width=32,
+                   deadline=D, interarrival=tau, b=b, gain=g)
+    cfg.vector_width = v
+    w, th, T, Tc = solve_enforced_waits(cfg)
+    P = [w[i] + t[i] for i in range(4)]
+    assert SV.fig1_feasible(t, g, b, v, tau, D, P)
+    assert P[0] >= 8654, P

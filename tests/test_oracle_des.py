@@ -52,6 +52,33 @@ def test_p1_fixed_wait_active_closed_form(case):
     assert abs(T - lim) <= sum(t) / (N * H) + 1e-12
 
 
+@pytest.mark.parametrize("case", range(12))
+def test_p1_drain_window_closed_form(case):
+    """The drain-inclusive accounting (SURVEY §8(c) C-D "Outputs"): over [0, T_end] FIXED_WAIT
+    charges every slot m P_i < T_end, clipped -- floor(T_end/P) t + min(t, T_end mod P) per node
+    for ANY data (L97: empty firings are charged), and THRESHOLD_SLACK charges t_i per firing
+    (every firing ends by T_end, the last completion)."""
+    rnd = random.Random(100 + case)
+    N = rnd.randint(1, 4)
+    t = [rnd.randint(3, 40) for _ in range(N)]
+    w = [rnd.randint(0, 60) for _ in range(N)]
+    v = rnd.choice([2, 4, 8, 32])
+    tau = rnd.randint(1, 9)
+    X = rnd.randint(1, 400)
+    r = des.run(gm_cfg(N, t, w, v, tau, X, seed=case))
+    s = r.streams[0]
+    for i in range(N):
+        P = t[i] + w[i]
+        assert s.active_drain[i] == (s.T_end // P) * t[i] + min(t[i], s.T_end % P), i
+    th = [rnd.randint(1, v) for _ in range(N)]
+    r = des.run(gm_cfg(N, t, None, v, tau, X, seed=case, policy=C.THRESHOLD_SLACK, theta=th, D=10**4))
+    s = r.streams[0]
+    for i in range(N):
+        assert s.active_drain[i] == s.n_firings[i] * t[i], i
+    acc = sum(s.active_drain)
+    assert r.active_fraction_drain(C.THRESHOLD_SLACK) == acc / (N * s.T_end)
+
+
 @pytest.mark.parametrize("tau,P,t0,v", [(4, 128, 64, 32), (3, 10, 7, 4), (5, 5, 5, 1), (2, 9, 1, 8)])
 def test_p2_fixed_wait_single_node_latency(tau, P, t0, v):
     assert P <= v * tau
@@ -126,6 +153,7 @@ def _enum_step_semantics(N, t, v, tau, X, fns, decide):
     busy = [None] * N                   # (end, entries)
     lat = [-1] * X
     log = []
+    qmax = [0] * N                      # longest queue at a firing decision (L133)
     T = 0
     arrived = 0
     while True:
@@ -142,12 +170,14 @@ def _enum_step_semantics(N, t, v, tau, X, fns, decide):
             Q[0].append((arrived, 0, None))
             arrived += 1
         for i in decide(T, Q, busy):
+            qmax[i] = max(qmax[i], len(Q[i]))
             n = min(len(Q[i]), v)
             ents, Q[i] = Q[i][:n], Q[i][n:]
             busy[i] = (T + t[i], ents)
             if n:
                 log.append((i, T, n))
         if arrived == X and not any(Q) and not any(b and b[1] for b in busy):
+            _enum_step_semantics.qmax = qmax
             return tuple(lat), log
         T += 1
 
@@ -233,6 +263,8 @@ def test_p6_schedule_enumeration(X, tau):
             lat2, log2 = _enum_step_semantics(N, t, v, tau, X, fns,
                                               lambda T, Q, b: sorted(starts.get(T, ())))
             assert lat2 == tuple(r.lat) and tuple(log2) == log
+            # the queue peaks at firing decisions (L133's b_i v) of the same schedule
+            assert _enum_step_semantics.qmax == r.max_queue, (policy, prm)
             # clairvoyant optimum among deadline-meeting schedules is no worse
             ok = [a for (lt, a) in allsched.values() if max(lt) <= D]
             if max(r.lat) <= D:

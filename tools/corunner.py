@@ -1,5 +1,5 @@
 """N3 co-runner experiment: does the processor time that
-enforced waiting yields serve other work?  A compute-bound background kernel (pl_corunner_launch,
+enforced waiting yields serve other work?  A compute-bound background kernel (tools/corunner/corunner.cu,
 ~8 CTAs/SM) runs beside the physical-clock executor (c2, v = 64 so that the executor CTA leaves
 register room on its SM) under FIXED_WAIT and under MONOLITHIC at the same (tau0, D); we time
 the co-runner alone and beside each executor, and check the executor's deadline misses."""
@@ -12,7 +12,10 @@ import torch
 
 from plgen import configs as C
 from plgen import dna as G
-from paper_conf_icppw_planob21_b200 import Pipeline, lib, realtime
+from paper_conf_icppw_planob21_b200 import Pipeline, realtime
+from paper_conf_icppw_planob21_b200.build import build_corunner
+
+lib = ctypes.CDLL(build_corunner())      # the co-runner is a measurement tool, not in libplgpu.so
 
 D = 350_000
 base = C.c2(n_streams=148, vector_width=64)
