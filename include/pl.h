@@ -123,6 +123,11 @@ typedef struct {
                                       root, non-decreasing within a stream, e.g. Poisson (L263);
                                       copied at create; n_arrivals must equal the root count */
   uint64_t n_arrivals;
+  uint32_t window_words;           /* per-stream smem DB window: a ring of this many 32-bit words
+                                      (power of 2, >= 2 chunks; 0 -> default: the whole stream range
+                                      when it fits, else 16 chunks = 64 KB), refilled by TMA as the
+                                      stream advances (a1); reads outside it go to the bound DB     */
+  uint32_t window_chunk_words;     /* refill unit in words (power of 2, >= 4; 0 -> default 1024)    */
 } pl_config;
 
 /* Workload of the DNA pipeline: the query is known up front; the database is the
@@ -195,6 +200,7 @@ typedef struct {
   uint32_t launches;                       /* executor launches so far                 */
   uint64_t h2d_bytes;                      /* host->device bytes copied by this handle (cumulative) */
   uint64_t d2h_bytes;                      /* device->host bytes copied by this handle (cumulative) */
+  uint64_t window_refills;                 /* DB-window chunks TMA-loaded as the streams advanced (a1) */
 } pl_stats;
 
 typedef struct pl_pipeline pl_pipeline;

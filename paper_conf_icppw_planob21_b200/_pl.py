@@ -35,7 +35,8 @@ class pl_config(C.Structure):
                 ("n_roots", C.c_uint64), ("seed", C.c_uint64), ("device", C.c_int32),
                 ("ns_per_unit", C.c_double), ("flags", C.c_uint32), ("queue_capacity", C.c_uint32),
                 ("spill_capacity", C.c_uint32), ("firing_log_capacity", C.c_uint32),
-                ("match_capacity", C.c_uint64), ("arrivals", C.POINTER(C.c_int64)), ("n_arrivals", C.c_uint64)]
+                ("match_capacity", C.c_uint64), ("arrivals", C.POINTER(C.c_int64)), ("n_arrivals", C.c_uint64),
+                ("window_words", C.c_uint32), ("window_chunk_words", C.c_uint32)]
 
 
 class pl_workload(C.Structure):
@@ -76,7 +77,8 @@ class pl_stats(C.Structure):
                 ("active_fraction", C.c_double), ("active_fraction_nonempty", C.c_double),
                 ("active_fraction_drain", C.c_double),
                 ("hw_busy_fraction", C.c_double), ("wall_ns", C.c_int64), ("errors", C.c_uint32),
-                ("launches", C.c_uint32), ("h2d_bytes", C.c_uint64), ("d2h_bytes", C.c_uint64)]
+                ("launches", C.c_uint32), ("h2d_bytes", C.c_uint64), ("d2h_bytes", C.c_uint64),
+                ("window_refills", C.c_uint64)]
 
     def as_dict(self):
         N = self.n_stages

@@ -58,8 +58,10 @@ __device__ __forceinline__ uint64_t gain_hash(uint64_t seed, uint32_t stage, uin
 }
 
 // ------------------------------------------------------------------ DNA access
-// The DB is read through a per-stream smem window (staged by a TMA bulk copy at
-// CTA start, cta_setup) with an __ldg fallback outside it.  Extensions compare 16
+// The DB is read through a per-stream smem window with an __ldg fallback outside it.  The
+// window is a ring of win_cap words (word w at slot w & win_mask) refilled chunk by chunk by
+// TMA bulk copies as the stream advances (win_step); [win_lo,
+// win_lo + win_n) is this thread's snapshot of the words it holds.  Extensions compare 16
 // bases per step: XOR of two 2-bit-packed 32-bit windows gives a mismatch mask.
 #ifndef PL_S3_MSB
 #define PL_S3_MSB 1
@@ -72,10 +74,11 @@ struct Dna {
   const uint32_t* db;      // packed DB (global)
   uint32_t nwords;
   uint64_t db_len;
-  const uint32_t* win;     // smem copy of DB words [win_lo, win_lo + win_n)
+  const uint32_t* win;     // smem ring of DB words: word w at win[w & win_mask], valid for [win_lo, win_lo + win_n)
   int64_t win_lo;
   uint32_t win_lo32;        // (uint32_t)win_lo: window word index arithmetic in 32 bits
   uint32_t win_n;
+  uint32_t win_mask;
   bool nofast;             // experiment switch (PL_VARIANT & 16): always the checked walk
   const uint8_t* s2tab;    // smem: max(0, max prefix score) of an 8-step walk by mismatch pattern
   const uint32_t* qw;      // query words (smem), nqw valid words
@@ -85,7 +88,7 @@ struct Dna {
   int k, q_len;
   __device__ __forceinline__ uint32_t dbw(int64_t w) const {
     const uint64_t r = (uint64_t)(w - win_lo);
-    if (r < win_n) return win[r];
+    if (r < win_n) return win[(uint32_t)w & win_mask];
     return (w >= 0 && w < (int64_t)nwords) ? __ldg(db + w) : 0u;
   }
   __device__ __forceinline__ uint32_t qww(int64_t w) const { return (w >= 0 && w < (int64_t)nqw) ? qw[w] : 0u; }
@@ -157,10 +160,10 @@ struct Dna {
     // left walk: step d+1+e compares db[p-d-1-e] with query[q-d-1-e]; its first 16-base
     // window is [p-16, p) = words (w, w+1), w = (p-16)>>4; later windows slide down a word
     int32_t sd = (int32_t)p - 16, sq = (int32_t)q - 16;
-    const uint32_t* dw = win + ((sd >> 4) - (int32_t)win_lo32);    // next word to load
+    uint32_t dw = (uint32_t)(sd >> 4);                                // next DB word to load (ring index)
     const uint32_t* qp = qw + (sq >> 4);
     uint32_t shd = (uint32_t)(sd & 15) * 2u, shq = (uint32_t)(sq & 15) * 2u;
-    uint32_t dc = dw[1], qc = qp[1];                                  // carried word
+    uint32_t dc = win[(dw + 1u) & win_mask], qc = qp[1];              // carried word
     int step = -1;
     bool right = false;
     uint32_t limit = ll, d = 0;
@@ -168,8 +171,8 @@ struct Dna {
     for (;;) {
       bool fin = d >= limit;
       if (!fin) {
-        const uint32_t dn = *dw, qn = *qp;
-        dw += step;
+        const uint32_t dn = win[dw & win_mask], qn = *qp;
+        dw += (uint32_t)step;
         qp += step;
         const uint32_t x = right ? (__funnelshift_r(dc, dn, shd) ^ __funnelshift_r(qc, qn, shq))
                                  : (__funnelshift_r(dn, dc, shd) ^ __funnelshift_r(qn, qc, shq));
@@ -224,11 +227,11 @@ struct Dna {
         score = best = db_ = 0;
         sd = (int32_t)(p + (uint32_t)k);
         sq = (int32_t)(q + (uint32_t)k);
-        dw = win + ((sd >> 4) - (int32_t)win_lo32);
+        dw = (uint32_t)(sd >> 4);
         qp = qw + (sq >> 4);
         shd = (uint32_t)(sd & 15) * 2u;
         shq = (uint32_t)(sq & 15) * 2u;
-        dc = *dw++;
+        dc = win[dw++ & win_mask];
         qc = *qp++;
       }
     }
@@ -237,8 +240,8 @@ struct Dna {
   }
   // 16 bases starting at s (s >= win_lo * 16, in the window) / at query position s >= -16
   __device__ __forceinline__ uint32_t db16w(int32_t s) const {
-    const uint32_t* w = win + ((s >> 4) - (int32_t)win_lo32);
-    return __funnelshift_r(w[0], w[1], (uint32_t)(s & 15) * 2u);
+    const uint32_t w = (uint32_t)(s >> 4);
+    return __funnelshift_r(win[w & win_mask], win[(w + 1u) & win_mask], (uint32_t)(s & 15) * 2u);
   }
   __device__ __forceinline__ uint32_t q16w(int32_t s) const {
     const uint32_t* w = qw + (s >> 4);
@@ -311,6 +314,17 @@ struct NodeAcc {
   uint32_t max_queue, lateness, max_fire, lmax, lmax_ns, nmiss, nmiss_ns;
   uint32_t max_loop;   // physical: longest firing-to-next-decision cycle (the node's real service time)
 };
+// Sliding DB window (a1): the ring holds chunks of 2^win_lg words at absolute chunk indices;
+// chunk c lives at ring slots [c CH, (c+1) CH) & win_mask.  Owned by one thread at a time (node
+// 0's accountant lane, or thread 0 of the monolithic kernel); readers see [cov_lo, cov_hi).
+struct WinCtl {
+  uint32_t cov_lo, cov_hi;  // words valid in the ring (absolute word indices), read as one 8-byte pair
+  uint32_t wlo, whi;        // the stream's window range (words)
+  uint32_t c_next, c_end;   // next chunk to load; one past the stream's last chunk
+  uint32_t inflight, phase; // a refill is in flight on mbar_w; its completion parity
+  uint32_t loaded_hi;       // cov_hi once the in-flight refill has landed
+  uint32_t refills;         // chunks loaded after the initial staging
+};
 struct Shared {
   EdgeCtl e[PL_MAX_STAGES];
   GroupCtl g[PL_MAX_STAGES];
@@ -322,7 +336,15 @@ struct Shared {
   uint32_t errors;
   uint32_t log_count;       // firing-log records reserved by all nodes of this stream
   uint64_t T0;
-  alignas(8) uint64_t mbar; // TMA completion barrier for the DB window
+  alignas(8) uint64_t mbar; // TMA completion barrier for the initial staging
+  alignas(8) uint64_t mbar_w;   // TMA completion barrier of the window refills
+  alignas(8) WinCtl win;
+  // per node: a lower bound on every root the node will still read the DB for.  Queues are FIFO
+  // and every stage emits in input order, so each node's input sequence is sorted by root: the
+  // first root of its current firing bounds its whole future.  Monotone; an idle node with an
+  // empty queue inherits its upstream's bound (decide).  The window may drop a chunk only below
+  // (min_i bnd[i] - q_len - 48) / 16 words (win_step).
+  uint32_t bnd[PL_MAX_STAGES];
 };
 
 struct Ctx {
@@ -332,7 +354,81 @@ struct Ctx {
   Dna dna;
   uint64_t lo, hi;             // roots [lo, hi)
   int64_t X, H;
+  bool sliding;                // the stream's DB range exceeds the window ring: refills (win_step)
 };
+
+__device__ __forceinline__ uint32_t smem_addr(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
+__device__ __forceinline__ bool mbar_test(uint32_t bar, uint32_t parity) {
+  uint32_t done;
+  asm volatile("{ .reg .pred q; mbarrier.test_wait.parity.shared::cta.b64 q, [%1], %2; selp.u32 %0, 1, 0, q; }"
+               : "=r"(done) : "r"(bar), "r"(parity) : "memory");
+  return done != 0;
+}
+// one TMA bulk copy global -> smem completing on mbarrier `bar` (bytes: multiple of 16)
+__device__ __forceinline__ void tma_load(uint32_t dst, const void* src, uint32_t bytes, uint32_t bar) {
+  asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
+               ::"r"(dst), "l"(src), "r"(bytes), "r"(bar) : "memory");
+}
+
+// Readers' snapshot of the window's valid range, taken before a firing's DB reads.
+__device__ __forceinline__ void win_snap(Dna& dna, const Shared& sh) {
+  uint32_t lo, hi;
+  asm volatile("ld.volatile.shared.v2.u32 {%0, %1}, [%2];" : "=r"(lo), "=r"(hi) : "r"(smem_addr(&sh.win.cov_lo)));
+  asm volatile("fence.acq_rel.cta;" ::: "memory");
+  dna.win_lo = lo;
+  dna.win_lo32 = lo;
+  dna.win_n = hi - lo;
+}
+
+// One step of the sliding window, by its single owner thread: complete an in-flight refill
+// (publish cov_hi), then start the next one if the chunk it overwrites is no longer needed.
+// A root p reads DB words >= (p - q_len - 48) / 16 (extension walks reach q_len bases to the
+// left, plus whole 16-base steps), so chunk c may replace chunk c - K once every node's bound
+// is past that.  A reader's stale snapshot is harmless: it only reads words of its own roots,
+// which are >= min bnd and so never in a dropped chunk.  wait = block until the refill lands.
+// Returns whether it made progress.
+__device__ bool win_step(Shared& sh, const DevParams& p, unsigned char* ring, bool wait) {
+  WinCtl& W = sh.win;
+  const uint32_t bar = smem_addr(&sh.mbar_w);
+  bool prog = false;
+  if (W.inflight) {
+    if (!mbar_test(bar, W.phase)) {
+      if (!wait) return false;
+      while (!mbar_test(bar, W.phase)) {}
+    }
+    W.phase ^= 1u;
+    W.inflight = 0;
+    asm volatile("fence.acq_rel.cta;" ::: "memory");
+    *(volatile uint32_t*)&W.cov_hi = W.loaded_hi;
+    prog = true;
+  }
+  if (W.c_next >= W.c_end) return prog;
+  uint32_t m = 0xffffffffu;
+  for (int i = 0; i < p.N; ++i) m = min(m, *(volatile uint32_t*)&sh.bnd[i]);
+  const uint32_t need = (uint32_t)p.q_len + 48u;
+  const uint32_t floor_w = m > need ? (m - need) >> 4 : 0u;
+  const uint32_t c = W.c_next, K = p.win_cap >> p.win_lg;
+  const uint32_t lo_new = (c - K + 1u) << p.win_lg;
+  if (floor_w < lo_new) return prog;       // chunk c - K is still needed
+  *(volatile uint32_t*)&W.cov_lo = lo_new;  // drop chunk c - K (readers only narrow their snapshots)
+  // the generic-proxy reads of the dropped chunk are ordered before the async-proxy refill
+  asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+  const uint32_t a = max(c << p.win_lg, W.wlo), b = min((c + 1u) << p.win_lg, W.whi);
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(bar), "r"((b - a) * 4u) : "memory");
+  tma_load(smem_addr(ring + (a & (p.win_cap - 1u)) * 4u), p.db + a, (b - a) * 4u, bar);
+  W.inflight = 1;
+  W.loaded_hi = b;
+  W.c_next = c + 1u;
+  W.refills++;
+  if (wait) {
+    while (!mbar_test(bar, W.phase)) {}
+    W.phase ^= 1u;
+    W.inflight = 0;
+    asm volatile("fence.acq_rel.cta;" ::: "memory");
+    *(volatile uint32_t*)&W.cov_hi = b;
+  }
+  return true;
+}
 
 __device__ __forceinline__ int64_t arrival(const Ctx& c, uint32_t root) {
   return c.p->arr ? __ldg(c.p->arr + root) : (int64_t)(root - c.lo) * c.p->tau;
@@ -383,6 +479,8 @@ struct Node {
   int64_t Mcap, B_per;          // FIXED_WAIT + eager: time-triggered slots m < Mcap (m P < A_last);
                                 // the last of them ends at B_per
   uint32_t* troot;              // smem [v]: the current firing's terminal root per lane (or NO_ROOT)
+  uint32_t* bnd;                // smem: Shared::bnd (sliding window only)
+  bool sliding;
   __device__ __forceinline__ int64_t arrival(uint32_t root) const {
     return arr ? __ldg(arr + root) : (int64_t)(root - lo) * tau;
   }
@@ -439,6 +537,8 @@ __device__ __forceinline__ Node make_node(const Ctx& c, int i) {
   n.Mcap = (n.eager && n.fixed) ? cdiv(n.A_last, n.dP) : 0;
   n.B_per = n.Mcap > 0 ? (n.Mcap - 1) * n.P + n.t : 0;
   n.troot = (uint32_t*)(c.dsm + Lo.off_troot) + (uint32_t)i * (uint32_t)p.v;
+  n.bnd = c.sh->bnd;
+  n.sliding = c.sliding;
   return n;
 }
 
@@ -741,12 +841,15 @@ __device__ Decision decide(const Node& nd, Leader& L, bool& waited, uint64_t T0)
         if (due > T0 + PL_NAP_LEAD_NS && nap_until(due - PL_NAP_LEAD_NS)) waited = true;
       }
     }
-    // node i >= 1: read the upstream watermark first, then the published segments
+    // node i >= 1: read the upstream watermark (and window bound) first, then the published segments
     const int64_t Wup = vld(&nd.Ein->W);
+    const uint32_t bup = nd.sliding ? vld(&nd.bnd[nd.i - 1]) : 0u;
     fence_cta();
     const uint32_t st = vld(&nd.Ein->seg_tail);
     const uint32_t tail_known = (st != L.segh) ? nd.in_seg[(st - 1) & nd.segmask].end : L.head;
     const bool any = tail_known != L.head;
+    // an empty queue: everything this node will still read comes from upstream's future
+    if (nd.sliding && !any && bup > vld(&nd.bnd[nd.i])) vst(&nd.bnd[nd.i], bup);
     if (nd.fixed) {
       if (nd.eager && L.m >= nd.Mcap) {  // R-DRAIN: work-conserving from A_last on
         const int64_t B = max(max(nd.B_per, L.B), nd.A_last);
@@ -917,7 +1020,9 @@ __device__ __forceinline__ void stage_batch(const Node& nd, const Dna& dna, cons
     if (__all_sync(0xffffffffu, inwin)) {
 #pragma unroll
       for (int j = 0; j < K; ++j) {
-        const uint32_t x = __funnelshift_r(dna.win[r[j]], dna.win[r[j] + 1], (e[j].x & 15u) * 2u);
+        const uint32_t w = e[j].x >> 4;
+        const uint32_t x = __funnelshift_r(dna.win[w & dna.win_mask], dna.win[(w + 1u) & dna.win_mask],
+                                           (e[j].x & 15u) * 2u);
         key[j] = dna.kmer_of(x);
       }
     } else {
@@ -1004,7 +1109,7 @@ __device__ __forceinline__ void record_lat_ns(const Node& nd, const Ctx& c, uint
 // (A separate node-0 instantiation was measured: faster alone, 1.33x slower with all nodes
 // running -- the SM's instruction cache holds one ~76 KB node loop, not two.)
 template <bool REC>
-__device__ void run_node(Ctx& c, const Dna dna, int i, int gtid) {
+__device__ void run_node(Ctx& c, Dna dna, int i, int gtid) {
   const DevParams& p = *c.p;
   const Node nd = make_node(c, i);
   const int v = nd.v, N = nd.N;
@@ -1140,6 +1245,10 @@ __device__ void run_node(Ctx& c, const Dna dna, int i, int gtid) {
       if (n0) e[0] = make_uint2((uint32_t)(nd.lo + head + ld), 0u);
       else e[0] = load_entry(nd, head + ld, G.segh[par], G.st[par], G.in_spill_end[par]);
     }
+    if (nd.sliding) {                    // the window's current range, and this node's bound
+      win_snap(dna, *c.sh);
+      if (leader && act && !n0) vst(&nd.bnd[i], e[0].x);   // the firing's first (smallest) root
+    }
     {   // warp-uniform dispatch to the stage body: direct compare-and-branch chain (a switch
         // compiles to an indirect BRX, measured ~200 cycles per dispatch)
       const uint32_t kd = nd.kind;
@@ -1164,6 +1273,7 @@ __device__ void run_node(Ctx& c, const Dna dna, int i, int gtid) {
       off = group_scan(G.wtot[par], o[0].c, &total, gtid, v, bidA, nd.umax <= 1);                 // B2
     }
     const uint32_t out_loc = G.out_loc[par], out_base = G.out_base[par];   // leader's reservation (B2)
+    if (nd.sliding && n0 && leader) vst(&nd.bnd[0], (uint32_t)(nd.lo + head));   // every lane is past the last firing
     if (leader) { const long long t2 = clock64(); A.d[par][D_PH2] = (uint32_t)(t2 - tc); tc = t2; }
     if (REC && n0 && pend_root != NO_ROOT)   // node 0: the previous publish time came through B2
       record_lat_ns(nd, c, T0, G.end_ns[par ^ 1], pend_root);
@@ -1368,6 +1478,7 @@ __device__ void run_node(Ctx& c, const Dna dna, int i, int gtid) {
         p0.x += dd.x; p0.y += dd.y; p1.x += dd.z; p1.y += dd.w;
         Cp[0] = c0; Cp[1] = c1; Cp[3] = c3; Cp[4] = c4; Pp[0] = p0; Pp[1] = p1;
       }
+      if (n0 && nd.sliding) win_step(*c.sh, p, (unsigned char*)dna.win, false);   // slide the DB window
     }
     if (n0) {                            // replicated node-0 state, identical in every lane
       R.c0 += n;
@@ -1380,6 +1491,7 @@ __device__ void run_node(Ctx& c, const Dna dna, int i, int gtid) {
     }
     par ^= 1;
   }
+  if (nd.sliding && leader) vst(&nd.bnd[i], 0xffffffffu);   // reads nothing more
   if (n0) {
     if (leader) publish_W(nd, L, PL_INF64);   // after the last segment was published
     bar_sync(bidA, v);                   // the last publish time is visible to every lane
@@ -1471,6 +1583,8 @@ __device__ void cta_setup(Ctx& c, Shared& sh, unsigned char* dsm, const DevParam
   c.dna.win_lo = 0;
   c.dna.win_lo32 = 0;
   c.dna.win_n = 0;
+  c.dna.win_mask = p.win_cap ? p.win_cap - 1u : 0u;
+  c.sliding = false;
   if (s == 0 && tid < 8 && p.summary_next) p.summary_next[tid] = 0ull;   // the next launch's summary slot
   c.dna.nofast = (p.variant & 16u) != 0;
   c.dna.s2tab = dsm + Lo.off_s2;
@@ -1483,10 +1597,10 @@ __device__ void cta_setup(Ctx& c, Shared& sh, unsigned char* dsm, const DevParam
       }
       (dsm + Lo.off_s2)[m] = (unsigned char)best;
     }
-  // DNA: the query index (offsets, positions, packed query) and this stream's DB window
-  // (its roots plus the k-1 overlap and a halo for the extensions) are staged into smem
-  // by TMA bulk copies (cp.async.bulk, one mbarrier), falling back to plain loads for an
-  // unaligned caller-owned DB.
+  // DNA: the query index (offsets, positions, packed query) and the first chunks of this
+  // stream's DB window (its roots plus the k-1 overlap and a halo for the extensions) are
+  // staged into smem by TMA bulk copies (cp.async.bulk, one mbarrier), falling back to plain
+  // loads for an unaligned caller-owned DB.  A stream longer than the ring slides it (win_step).
   if (p.k > 0) {
     const uint32_t nko = (1u << (2 * p.k)) + 1u, nqp = (uint32_t)(p.q_len - p.k + 1);
     const uint32_t nqw = (uint32_t)(p.q_len + 15) / 16u;
@@ -1498,29 +1612,47 @@ __device__ void cta_setup(Ctx& c, Shared& sh, unsigned char* dsm, const DevParam
       wlo = wlo < 0 ? 0 : (wlo & ~3ll);
       whi = (whi + 3) & ~3ll;
       if (whi > (int64_t)p.db_alloc_words) whi = (int64_t)p.db_alloc_words & ~3ll;
-      if (whi - wlo > (int64_t)p.win_cap) whi = wlo + p.win_cap;
       if (whi < wlo) whi = wlo;
     }
+    const uint32_t lg = p.win_lg, K = p.win_cap >> lg;
+    const uint32_t c0 = (uint32_t)wlo >> lg;
+    const uint32_t c_end = whi > wlo ? (uint32_t)((whi - 1) >> lg) + 1u : c0;
+    // without TMA (unaligned DB) the window holds the first K chunks and never slides
+    const uint32_t c_init = min(c_end, c0 + K);
+    const uint32_t hi0 = whi > wlo ? min((uint32_t)whi, c_init << lg) : (uint32_t)wlo;
+    c.sliding = p.db_tma && c_end > c_init;
     c.dna.win_lo = wlo;
     c.dna.win_lo32 = (uint32_t)wlo;
-    c.dna.win_n = (uint32_t)(whi - wlo);
+    c.dna.win_n = hi0 - (uint32_t)wlo;
     uint32_t* win = (uint32_t*)(dsm + Lo.off_win);
     const bool win_tma = p.db_tma && c.dna.win_n;
     if (tid == 0) {
-      const uint32_t bar = (uint32_t)__cvta_generic_to_shared(&sh.mbar);
+      WinCtl& W = sh.win;
+      W.cov_lo = (uint32_t)wlo;
+      W.cov_hi = hi0;
+      W.wlo = (uint32_t)wlo;
+      W.whi = (uint32_t)whi;
+      W.c_next = c.sliding ? c_init : c_end;
+      W.c_end = c_end;
+      W.inflight = 0;
+      W.phase = 0;
+      W.loaded_hi = hi0;
+      W.refills = 0;
+      const uint32_t bar = smem_addr(&sh.mbar);
       const uint32_t bytes = b_qo + b_qp + b_qw + (win_tma ? c.dna.win_n * 4u : 0u);
       asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(bar));
+      asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(smem_addr(&sh.mbar_w)));
       asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
       asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(bar), "r"(bytes) : "memory");
-      const void* src[4] = {p.qoff, p.qpos, p.qwords, p.db + wlo};
-      const uint32_t off[4] = {Lo.off_qoff, Lo.off_qpos, Lo.off_qw, Lo.off_win};
-      const uint32_t len[4] = {b_qo, b_qp, b_qw, win_tma ? c.dna.win_n * 4u : 0u};
-      for (int j = 0; j < 4; ++j) {
-        if (!len[j]) continue;
-        const uint32_t dst = (uint32_t)__cvta_generic_to_shared(dsm + off[j]);
-        asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
-                     ::"r"(dst), "l"(src[j]), "r"(len[j]), "r"(bar) : "memory");
-      }
+      const void* src[3] = {p.qoff, p.qpos, p.qwords};
+      const uint32_t off[3] = {Lo.off_qoff, Lo.off_qpos, Lo.off_qw};
+      const uint32_t len[3] = {b_qo, b_qp, b_qw};
+      for (int j = 0; j < 3; ++j) tma_load(smem_addr(dsm + off[j]), src[j], len[j], bar);
+      if (win_tma)   // one copy per chunk: chunk c sits at ring slots (c CH) & mask, contiguous
+        for (uint32_t ch = c0; ch < c_init; ++ch) {
+          const uint32_t a = max(ch << lg, (uint32_t)wlo), b = min((ch + 1u) << lg, (uint32_t)whi);
+          tma_load(smem_addr(dsm + Lo.off_win + (a & (p.win_cap - 1u)) * 4u), p.db + a, (b - a) * 4u, bar);
+        }
       uint32_t done = 0;
       while (!done)
         asm volatile("{ .reg .pred q; mbarrier.try_wait.parity.shared::cta.b64 q, [%1], 0; selp.u32 %0, 1, 0, q; }"
@@ -1533,9 +1665,10 @@ __device__ void cta_setup(Ctx& c, Shared& sh, unsigned char* dsm, const DevParam
     if (!win_tma)
       for (uint32_t j = tid; j < c.dna.win_n; j += nt) {
         const int64_t w = wlo + j;
-        win[j] = w < (int64_t)p.db_words ? p.db[w] : 0u;
+        win[(uint32_t)w & (p.win_cap - 1u)] = w < (int64_t)p.db_words ? p.db[w] : 0u;
       }
   }
+  if (tid < PL_MAX_STAGES) sh.bnd[tid] = (uint32_t)c.lo;   // no node reads below its stream's first root
   if (tid < PL_MAX_STAGES) {
     EdgeCtl& E = sh.e[tid];
     E.head = 0; E.seg_head = 0; E.seg_tail = 0; E.tail = 0; E.W = -1; E.spill_end = 0; E.stalled = 0;
@@ -1566,6 +1699,7 @@ __device__ void cta_finish(Ctx& c, Shared& sh, const DevParams& p) {
     S.n_roots = (uint64_t)c.X;
     S.n_log = sh.log_count < p.log_cap ? sh.log_count : p.log_cap;
     S.errors = sh.errors;
+    S.win_refills = p.k > 0 ? sh.win.refills : 0u;
     if (p.summary) {                     // device-side reduction for pl_pipeline_summary
       atomicAdd(p.summary + 0, (unsigned long long)c.X);
       atomicAdd(p.summary + 1, (unsigned long long)sh.miss_events);
@@ -1619,8 +1753,19 @@ __device__ void run_monolithic(Ctx& c) {
   for (int i = 0; i < PL_MAX_STAGES; ++i) { firings[i] = consumed[i] = produced[i] = 0; active[i] = 0; }
   int64_t proc_free = 0, t_end = 0, busy_ns = 0;
   const int64_t M = p.M;
+  if (c.sliding && tid == 0)             // one processor: only node 0's bound (the block) matters
+    for (int i = 1; i < N; ++i) c.sh->bnd[i] = 0xffffffffu;
   for (int64_t b0 = 0; b0 < c.X; b0 += M) {
     const int64_t b1 = (b0 + M < c.X) ? b0 + M : c.X;
+    if (c.sliding) {                     // slide the DB window over the block (blocking refills)
+      if (tid == 0) {
+        vst(&c.sh->bnd[0], (uint32_t)(c.lo + b0));
+        const uint32_t need_hi = min(c.sh->win.whi, (uint32_t)(((c.lo + b1 + p.k + p.win_halo) >> 4) + 1));
+        while (vld(&c.sh->win.cov_hi) < need_hi && win_step(*c.sh, p, (unsigned char*)c.dna.win, true)) {}
+      }
+      __syncthreads();
+      win_snap(c.dna, *c.sh);
+    }
     const int64_t ready = arrival(c, (uint32_t)(c.lo + b1 - 1));
     int64_t T = ready > proc_free ? ready : proc_free;
     if (phys) {
@@ -1850,7 +1995,9 @@ __global__ void __launch_bounds__(MAXT, 1) pl_stage_batch_kernel(const __grid_co
   c.dna.qpos = (const uint16_t*)(dsm + Lo.off_qpos);
   c.dna.qw = (const uint32_t*)(dsm + Lo.off_qw);
   c.dna.nqw = (uint32_t)(p.q_len + 15) / 16u;
-  c.dna.win = nullptr; c.dna.win_lo = 0; c.dna.win_lo32 = 0; c.dna.win_n = 0; c.dna.nofast = true; c.dna.s2tab = nullptr;
+  c.dna.win = nullptr; c.dna.win_lo = 0; c.dna.win_lo32 = 0; c.dna.win_n = 0; c.dna.win_mask = 0;
+  c.dna.nofast = true; c.dna.s2tab = nullptr;
+  c.sliding = false;
   const uint32_t tid = threadIdx.x, v = blockDim.x;
   if (p.k > 0) {
     const uint32_t nko = (1u << (2 * p.k)) + 1u, nqp = (uint32_t)(p.q_len - p.k + 1);

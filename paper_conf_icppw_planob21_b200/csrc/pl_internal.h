@@ -58,6 +58,8 @@ struct CtaStats {
   uint64_t n_roots;
   uint32_t n_log;                       // firing-log records written
   uint32_t errors;
+  uint32_t win_refills;                 // DB-window chunks loaded after the initial staging
+  uint32_t pad_;
 };
 
 struct DevParams {
@@ -84,7 +86,8 @@ struct DevParams {
   const uint16_t* qoff;                 // [4^k + 1]
   const uint16_t* qpos;                 // [q_len - k + 1]
   const uint32_t* qwords;               // [ceil(q_len/16)]
-  uint32_t win_cap;                     // smem DB window capacity (words, multiple of 4; 0 = off)
+  uint32_t win_cap;                     // smem DB window: a ring of win_cap words (power of 2; 0 = off)
+  uint32_t win_lg;                      // log2 of the ring's chunk (words): the unit of a TMA refill
   uint32_t win_halo;                    // bases staged beyond the stream's roots on each side
   uint64_t db_alloc_words;              // readable words at db (>= db_words)
   uint32_t db_tma;                      // db is 16-byte aligned and padded: stage with cp.async.bulk

@@ -392,15 +392,28 @@ pl_status pl_pipeline_create(const pl_config* cfg, const pl_workload* wl, pl_pip
     if (cudaMalloc(&pl->d_db, dbw * 4) != cudaSuccess) return bail(fail(PL_ENOMEM, "DB allocation"));
     cudaMemset(pl->d_db, 0, dbw * 4);
     pl->db_alloc_words = dbw;
-    // smem DB window per stream: its roots + k-1 overlap + halo on both sides (capped at 64 KB)
+    // smem DB window per stream: its roots + k-1 overlap + halo on both sides, as a ring of
+    // chunks refilled by TMA as the stream advances (executor.cu win_step).  Default: the whole
+    // stream range when it fits in 16 chunks of 1024 words (64 KB), else a 64 KB sliding ring.
     const uint64_t R = wl->db_len >= (uint64_t)pl->k ? wl->db_len - pl->k + 1 : 0;
     const uint64_t per = (R + cfg->n_streams - 1) / cfg->n_streams;
     // halo: an extension walks at most q_len bases from its seed (Dna::right/left_limit), so
     // with q_len + 48 every walk of an interior root stays in the window (Dna::extend_win)
     d.win_halo = std::max<uint32_t>(512u, (uint32_t)wl->q_len + 48u);
+    const uint32_t CH = cfg->window_chunk_words ? cfg->window_chunk_words : 1024u;
+    if (!is_pow2(CH) || CH < 4) return bail(fail(PL_EINVAL, "window_chunk_words must be a power of 2 >= 4"));
     uint64_t words = (per + pl->k + 2 * d.win_halo) / 16 + 8;
     words = (words + 3) & ~3ull;
-    d.win_cap = (uint32_t)std::min<uint64_t>(words, 16384);
+    const uint64_t chunks = (words + CH - 1) / CH + 1;     // + 1: chunks sit at absolute boundaries
+    uint32_t cap = CH * next_pow2((uint32_t)std::min<uint64_t>(chunks, 16));
+    if (cfg->window_words) {
+      if (!is_pow2(cfg->window_words) || cfg->window_words < 2 * CH)
+        return bail(fail(PL_EINVAL, "window_words must be a power of 2 >= 2 * window_chunk_words"));
+      cap = cfg->window_words;
+    }
+    d.win_cap = cap;
+    d.win_lg = 0;
+    while ((1u << d.win_lg) < CH) ++d.win_lg;
     pl->roots_cap = wl->db_len >= (uint64_t)pl->k ? wl->db_len - pl->k + 1 : 0;
   } else {
     pl->roots_cap = cfg->n_roots * cfg->n_streams;
@@ -744,6 +757,7 @@ pl_status pl_pipeline_stats(pl_pipeline* pl, pl_stats* out) {
     out->max_latency_ns = std::max(out->max_latency_ns, s.max_lat_ns);
     out->wall_ns = std::max(out->wall_ns, s.wall_ns);
     out->errors |= s.errors;
+    out->window_refills += s.win_refills;
   }
   unsigned long long mc = 0;
   CUDA_TRY(cudaMemcpy(&mc, pl->d_match_count, 8, cudaMemcpyDeviceToHost));
