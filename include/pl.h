@@ -201,6 +201,11 @@ typedef struct {
   uint64_t h2d_bytes;                      /* host->device bytes copied by this handle (cumulative) */
   uint64_t d2h_bytes;                      /* device->host bytes copied by this handle (cumulative) */
   uint64_t window_refills;                 /* DB-window chunks TMA-loaded as the streams advanced (a1) */
+  /* physical clock: agreement of every terminal item's MEASURED latency with the logical-clock
+   * prediction T + t_i - a(r) (north_star "within 5 % relative"; DESIGN.md R-AGREE: a floor of
+   * 64 ns = two %globaltimer ticks; with PL_FIXED_SERVICE a firing completes at start + t_i)   */
+  uint64_t latency_outliers;               /* terminal items with |err| > 5 % of their latency + 64 ns */
+  double   latency_rel_err_max;            /* largest |err| / logical latency over terminal items      */
 } pl_stats;
 
 typedef struct pl_pipeline pl_pipeline;
@@ -233,6 +238,15 @@ pl_status pl_pipeline_bind_device(pl_pipeline* pl, const void* dev_items, uint64
  * PL_EINVAL if the buffer is not mapped.  It must stay valid until the run completes.    */
 pl_status pl_pipeline_bind_host(pl_pipeline* pl, const void* host_items, uint64_t n);
 
+/* Direct the match records (pl_match, the last DNA stage's output) of later runs into a
+ * caller-owned buffer of `cap` records: device memory, or PINNED+MAPPED host memory
+ * (cudaHostAlloc(..., cudaHostAllocMapped) / cudaHostRegisterMapped), into which the executor
+ * writes them over the host link as they are produced -- so a run's result needs no separate
+ * device->host copy.  The buffer must stay valid until the last run using it has completed;
+ * records beyond cap set PL_EOVERFLOW.  buf == NULL restores the handle's own device buffer.
+ * pl_pipeline_results reads whichever buffer the last run used.                             */
+pl_status pl_pipeline_bind_results(pl_pipeline* pl, void* buf, uint64_t cap);
+
 /* Per-stream input-queue peaks of the last run: buf[s*N + i] = longest queue (entries) node i
  * of stream s saw at a firing decision.  The data of the paper's b_i calibration (L133,
  * L227-L230).  buf == NULL: *n = n_streams * N.                                          */
@@ -243,6 +257,7 @@ typedef struct {
   uint64_t roots, matches, miss_events, miss_events_ns;
   int64_t  max_latency, max_latency_ns;
   uint32_t errors, launches;
+  uint64_t latency_outliers;       /* physical: items outside the 5 % latency band (pl_stats) */
 } pl_summary;
 pl_status pl_pipeline_summary(pl_pipeline* pl, pl_summary* out);
 

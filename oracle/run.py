@@ -28,11 +28,7 @@ _CTX = {}
 
 def _one(args):
     cfg, lo, hi = args
-    wl = _CTX.get("wl")
-    ctx = None
-    if wl is not None:
-        ctx = S.DnaContext(wl.db, wl.db_len, wl.query, wl.q_len, cfg.stages[0].iparam[0])
-    fns = des.make_stage_fns(cfg, ctx)
+    fns = des.make_stage_fns(cfg, _CTX.get("ctx"))   # the context is built once, before the fork
     r = des.simulate_stream(cfg, fns, lo, hi)
     return hi - lo, max(r.lat) if r.lat else 0
 
@@ -50,7 +46,10 @@ def sample_ranges(cfg, wl, n_streams, max_roots):
 def time_oracle(cfg, wl, n_streams, max_roots=0, procs=None):
     """Wall-clock the DES over the sample on ``procs`` host processes.
     Returns dict(value items/s, cores, seconds, roots, sample)."""
-    _CTX["wl"] = wl
+    if _CTX.get("wl") is not wl:
+        _CTX["wl"] = wl
+        _CTX["ctx"] = (S.DnaContext(wl.db, wl.db_len, wl.query, wl.q_len, cfg.stages[0].iparam[0])
+                       if wl is not None else None)
     ranges = sample_ranges(cfg, wl, n_streams, max_roots)
     cores = procs or len(os.sched_getaffinity(0))
     t0 = time.perf_counter()
@@ -74,7 +73,10 @@ def oracle_schedule(cfg, gains=None):
     Pc, _ = SV.fig1_continuous(cfg.service_time, g, cfg.b, cfg.vector_width, cfg.interarrival, cfg.deadline)
     if Pc is None:
         raise RuntimeError("Fig. 1 infeasible")
-    P = [max(cfg.service_time[i], math.floor(Pc[i])) for i in range(N)]
+    # floored, then repaired down the chain so that g_{i-1} P_i <= P_{i-1} holds in integers
+    P = [max(cfg.service_time[0], min(math.floor(Pc[0]), cfg.vector_width * cfg.interarrival))]
+    for i in range(1, N):
+        P.append(max(cfg.service_time[i], min(math.floor(Pc[i]), math.floor(P[i - 1] / g[i - 1]))))
     if not SV.fig1_feasible(cfg.service_time, g, cfg.b, cfg.vector_width, cfg.interarrival, cfg.deadline, P):
         raise RuntimeError("floored Fig. 1 point infeasible")
     w = tuple(P[i] - cfg.service_time[i] for i in range(N))

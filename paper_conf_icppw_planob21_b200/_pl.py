@@ -57,7 +57,7 @@ class pl_firing(C.Structure):
 class pl_summary(C.Structure):
     _fields_ = [("roots", C.c_uint64), ("matches", C.c_uint64), ("miss_events", C.c_uint64),
                 ("miss_events_ns", C.c_uint64), ("max_latency", C.c_int64), ("max_latency_ns", C.c_int64), ("errors", C.c_uint32),
-                ("launches", C.c_uint32)]
+                ("launches", C.c_uint32), ("latency_outliers", C.c_uint64)]
 
 
 _A8 = C.c_uint64 * PL_MAX_STAGES
@@ -78,7 +78,8 @@ class pl_stats(C.Structure):
                 ("active_fraction_drain", C.c_double),
                 ("hw_busy_fraction", C.c_double), ("wall_ns", C.c_int64), ("errors", C.c_uint32),
                 ("launches", C.c_uint32), ("h2d_bytes", C.c_uint64), ("d2h_bytes", C.c_uint64),
-                ("window_refills", C.c_uint64)]
+                ("window_refills", C.c_uint64), ("latency_outliers", C.c_uint64),
+                ("latency_rel_err_max", C.c_double)]
 
     def as_dict(self):
         N = self.n_stages
@@ -108,6 +109,7 @@ def _load():
         "pl_pipeline_step": (C.c_int32, [P, C.POINTER(pl_summary), C.POINTER(C.c_int)]),
         "pl_pipeline_step_finish": (C.c_int32, [P, C.POINTER(pl_summary), C.POINTER(C.c_int)]),
         "pl_pipeline_queue_peaks": (C.c_int32, [P, P, C.c_uint64, C.POINTER(C.c_uint64)]),
+        "pl_pipeline_bind_results": (C.c_int32, [P, P, C.c_uint64]),
         "pl_pipeline_launch": (C.c_int32, [P]),
         "pl_pipeline_drain": (C.c_int32, [P]),
         "pl_pipeline_rewind": (C.c_int32, [P]),
@@ -139,7 +141,7 @@ EXPORTED = ("pl_pipeline_create", "pl_pipeline_set_stream", "pl_pipeline_push", 
             "pl_pipeline_params", "pl_pipeline_destroy", "pl_last_error", "pl_solve_enforced_waits",
             "pl_solve_monolithic", "pl_version", "pl_stage_batch", "pl_pipeline_bind_host",
             "pl_pipeline_summary", "pl_pipeline_queue_peaks",
-            "pl_pipeline_step", "pl_pipeline_step_finish")
+            "pl_pipeline_step", "pl_pipeline_step_finish", "pl_pipeline_bind_results")
 
 
 class PlError(RuntimeError):

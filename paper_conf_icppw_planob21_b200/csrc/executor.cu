@@ -299,6 +299,7 @@ struct GroupCtl {           // broadcast from a node's leader to its lanes, doub
   uint32_t out_base[2], out_loc[2];
   alignas(16) uint32_t wtot[2][8];
   alignas(16) uint32_t rmin[8];   // per warp: smallest terminal root of the current firing
+  alignas(16) uint32_t rmax[8];   // per warp: largest terminal root + 1 (0: none; physical clock only)
 };
 // Leader-only per-node accumulators, in smem so that they take no registers in the node loop.
 // 64-bit shared atomics compile to CAS spin loops (ATOMS.CAST.SPIN.64), so the single writer
@@ -333,6 +334,8 @@ struct Shared {
   uint32_t max_lat_ns;      // (64-bit smem atomicMax compiles to a CAS loop)
   uint32_t miss_events;
   uint32_t miss_events_ns;  // physical: terminal items whose measured latency exceeded D
+  uint32_t agr_bad;         // physical: terminal items outside the 5 % band of their logical latency
+  uint32_t agr_ppm;         // physical: largest |measured - logical| / logical latency (ppm)
   uint32_t errors;
   uint32_t log_count;       // firing-log records reserved by all nodes of this stream
   uint64_t T0;
@@ -1140,7 +1143,7 @@ __device__ void run_node(Ctx& c, Dna dna, int i, int gtid) {
     for (int k = 0; k < C_N; ++k) A.cnt[k] = 0;
     for (int k = 0; k < 6; ++k) A.ph[k] = 0;
     for (int k = 0; k < D_N; ++k) { A.d[0][k] = 0; A.d[1][k] = 0; }
-    for (int k = 0; k < 8; ++k) G.rmin[k] = NO_ROOT;   // slots of absent warps stay NO_ROOT
+    for (int k = 0; k < 8; ++k) { G.rmin[k] = NO_ROOT; G.rmax[k] = 0u; }   // absent warps keep these
     A.t_end = 0;
     A.max_queue = A.lateness = A.max_fire = A.lmax = A.lmax_ns = A.nmiss = A.nmiss_ns = A.max_loop = 0;
   }
@@ -1318,6 +1321,10 @@ __device__ void run_node(Ctx& c, Dna dna, int i, int gtid) {
       nd.troot[gtid] = tr;
       const uint32_t wmin = __reduce_min_sync(0xffffffffu, tr);
       if ((gtid & 31) == 0) G.rmin[gtid >> 5] = wmin;
+      if (nd.phys) {                     // the latest-arriving terminal root: smallest logical latency
+        const uint32_t wmax = __reduce_max_sync(0xffffffffu, term ? ei.x + 1u : 0u);
+        if ((gtid & 31) == 0) G.rmax[gtid >> 5] = wmax;
+      }
     }
     if (nd.sink && nd.kind == PL_UNGAPPED_XDROP) {   // matches: one global atomic per warp
       const bool hit = act && oi.c;
@@ -1457,6 +1464,33 @@ __device__ void run_node(Ctx& c, Dna dna, int i, int gtid) {
               if (r != NO_ROOT && (int64_t)en - (int64_t)(T0 + units_ns(nd, nd.arrival(r))) > nd.D_ns) ++m;
             }
             atomicAdd(&A.nmiss_ns, m);
+          }
+          // north_star: every item's measured latency within 5 % of the logical-clock prediction
+          // T + t_i - a(r) (floor PL_AGREE_FLOOR_NS, DESIGN.md R-AGREE).  A firing's terminal items
+          // complete together, so the error is common to them -- with PL_FIXED_SERVICE the firing
+          // completes at max(publish, start + t_i), the paper's fixed service time (L69) -- and its
+          // relative size is largest for the latest-arriving terminal root.
+          uint32_t rx;
+          {
+            const uint4 a = *reinterpret_cast<const uint4*>(G.rmax);
+            rx = max(max(a.x, a.y), max(a.z, a.w));
+            if (v > 128) {
+              const uint4 b = *reinterpret_cast<const uint4*>(G.rmax + 4);
+              rx = max(rx, max(max(b.x, b.y), max(b.z, b.w)));
+            }
+          }
+          const int64_t due = (int64_t)(T0 + units_ns(nd, T + nd.t));
+          const int64_t comp = (rec & PL_FIXED_SERVICE) ? max((int64_t)en, due) : (int64_t)en;
+          const int64_t err = comp > due ? comp - due : due - comp;
+          const int64_t lsmall = (int64_t)units_ns(nd, T + nd.t - nd.arrival(rx - 1u));
+          atomicMax(&c.sh->agr_ppm, clamp32((int64_t)((float)err * 1e6f / (float)(lsmall > 0 ? lsmall : 1))));
+          if (err * 20 > lsmall + 20 * PL_AGREE_FLOOR_NS) {   // count the items outside the band exactly
+            uint32_t m = 0;
+            for (int k = 0; k < v; ++k) {
+              const uint32_t r = nd.troot[k];
+              if (r != NO_ROOT && err * 20 > (int64_t)units_ns(nd, T + nd.t - nd.arrival(r)) + 20 * PL_AGREE_FLOOR_NS) ++m;
+            }
+            atomicAdd(&c.sh->agr_bad, m);
           }
         }
       }
@@ -1675,6 +1709,7 @@ __device__ void cta_setup(Ctx& c, Shared& sh, unsigned char* dsm, const DevParam
   }
   if (tid == 0) {
     sh.max_lat = 0; sh.max_lat_ns = 0; sh.miss_events = 0; sh.miss_events_ns = 0; sh.errors = 0; sh.log_count = 0;
+    sh.agr_bad = 0; sh.agr_ppm = 0;
   }
   // per-root records of this stream
   if (p.flags & PL_REC_LATENCY)
@@ -1700,6 +1735,8 @@ __device__ void cta_finish(Ctx& c, Shared& sh, const DevParams& p) {
     S.n_log = sh.log_count < p.log_cap ? sh.log_count : p.log_cap;
     S.errors = sh.errors;
     S.win_refills = p.k > 0 ? sh.win.refills : 0u;
+    S.agr_bad = sh.agr_bad;
+    S.agr_ppm = sh.agr_ppm;
     if (p.summary) {                     // device-side reduction for pl_pipeline_summary
       atomicAdd(p.summary + 0, (unsigned long long)c.X);
       atomicAdd(p.summary + 1, (unsigned long long)sh.miss_events);
@@ -1707,6 +1744,7 @@ __device__ void cta_finish(Ctx& c, Shared& sh, const DevParams& p) {
       atomicMax(p.summary + 3, (unsigned long long)sh.max_lat_ns);
       atomicOr(p.summary + 4, (unsigned long long)sh.errors);
       atomicAdd(p.summary + 5, (unsigned long long)sh.miss_events_ns);
+      if (sh.agr_bad) atomicAdd(p.summary + 7, (unsigned long long)sh.agr_bad);
     }
   }
 }

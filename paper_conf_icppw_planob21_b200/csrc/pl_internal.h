@@ -7,6 +7,7 @@
 
 #define PL_INF64 0x7fffffffffffffffLL
 #define PL_MAX_K 7                      // query index 4^k u16 entries must fit in smem
+#define PL_AGREE_FLOOR_NS 64            // R-AGREE: |measured - logical latency| <= 5 % + this (2 timer ticks)
 
 // Error bits written by the device (pl_stats.errors).
 #define PL_ERR_QUEUE_OVERFLOW   1u      // spill ring full in physical mode
@@ -59,6 +60,8 @@ struct CtaStats {
   uint32_t n_log;                       // firing-log records written
   uint32_t errors;
   uint32_t win_refills;                 // DB-window chunks loaded after the initial staging
+  uint32_t agr_bad;                     // physical: terminal items outside the 5 % latency band (R-AGREE)
+  uint32_t agr_ppm;                     // physical: largest relative latency error (ppm)
   uint32_t pad_;
 };
 
@@ -109,7 +112,7 @@ struct DevParams {
   uint32_t log_cap;
   CtaStats* stats;                      // [n_streams]
   unsigned long long* summary;          // [8]: roots, miss_events, max_lat, max_lat_ns, errors, miss_ns,
-                                        //      match count (= match_count), pad
+                                        //      match count (= match_count), latency outliers (R-AGREE)
   uint32_t t0_offset_ns;                // physical clock: stream time origin = CTA start + this
   unsigned long long* summary_next;     // the other slot of the double buffer: zeroed by this launch
                                         // (stream order: the previous launch that used it is done)

@@ -113,6 +113,7 @@ struct pl_pipeline {
   int64_t *d_lat = nullptr, *d_lat_ns = nullptr;
   uint32_t* d_trace = nullptr;
   pl_match* d_matches = nullptr;
+  uint64_t own_match_cap = 0;
   unsigned long long* d_match_count = nullptr;   // match count of the last launch (inside d_summary)
   uint32_t slot = 0;                             // d_summary slot of the next launch
   pl_firing* d_flog = nullptr;
@@ -481,6 +482,7 @@ pl_status pl_pipeline_create(const pl_config* cfg, const pl_workload* wl, pl_pip
     return bail(fail(PL_ENOMEM, "firing log"));
   d.match_cap = cfg->match_capacity ? cfg->match_capacity : (1ull << 20);
   if (!pl->dna) d.match_cap = 1;
+  pl->own_match_cap = d.match_cap;
   if (cudaMalloc(&pl->d_matches, d.match_cap * sizeof(pl_match)) != cudaSuccess ||
       cudaMalloc(&pl->d_stats, S * sizeof(CtaStats)) != cudaSuccess)
     return bail(fail(PL_ENOMEM, "output buffers"));
@@ -582,6 +584,34 @@ pl_status pl_pipeline_bind_host(pl_pipeline* pl, const void* host_items, uint64_
   return PL_OK;
 }
 
+pl_status pl_pipeline_bind_results(pl_pipeline* pl, void* buf, uint64_t cap) {
+  if (!pl) return fail(PL_EINVAL, "NULL pipeline");
+  if (!buf) {
+    pl->dp.matches = pl->d_matches;
+    pl->dp.match_cap = pl->own_match_cap;
+    return PL_OK;
+  }
+  if (!cap) return fail(PL_EINVAL, "cap must be > 0");
+  cudaSetDevice(pl->device);
+  cudaPointerAttributes at;
+  if (cudaPointerGetAttributes(&at, buf) != cudaSuccess) {
+    cudaGetLastError();
+    return fail(PL_EINVAL, "results buffer is neither device memory nor registered host memory");
+  }
+  void* dptr = buf;
+  if (at.type == cudaMemoryTypeHost) {
+    if (cudaHostGetDevicePointer(&dptr, buf, 0) != cudaSuccess || !dptr) {
+      cudaGetLastError();
+      return fail(PL_EINVAL, "host results buffer is not mapped (cudaHostAllocMapped / cudaHostRegisterMapped)");
+    }
+  } else if (at.type != cudaMemoryTypeDevice && at.type != cudaMemoryTypeManaged) {
+    return fail(PL_EINVAL, "results buffer is neither device memory nor pinned host memory");
+  }
+  pl->dp.matches = (pl_match*)dptr;
+  pl->dp.match_cap = cap;
+  return PL_OK;
+}
+
 pl_status pl_pipeline_queue_peaks(pl_pipeline* pl, uint32_t* buf, uint64_t cap, uint64_t* n) {
   if (!pl || !n) return fail(PL_EINVAL, "NULL argument");
   const uint32_t S = pl->cfg.n_streams, N = pl->cfg.n_stages;
@@ -608,16 +638,17 @@ void decode_summary(const pl_pipeline* pl, const unsigned long long* h, uint32_t
   out->errors = (uint32_t)h[4];
   out->matches = std::min<uint64_t>(h[6], pl->dp.match_cap);
   out->launches = launch;
+  out->latency_outliers = h[7];
 }
 }  // namespace
 
 pl_status pl_pipeline_summary(pl_pipeline* pl, pl_summary* out) {
   if (!pl || !out) return fail(PL_EINVAL, "NULL argument");
   cudaSetDevice(pl->device);
-  unsigned long long h[7];
-  CUDA_TRY(cudaMemcpyAsync(h, pl->d_match_count - 6, 56, cudaMemcpyDeviceToHost, pl->stream));
+  unsigned long long h[8];
+  CUDA_TRY(cudaMemcpyAsync(h, pl->d_match_count - 6, 64, cudaMemcpyDeviceToHost, pl->stream));
   CUDA_TRY(cudaStreamSynchronize(pl->stream));
-  pl->d2h += 56;
+  pl->d2h += 64;
   decode_summary(pl, h, pl->launches, out);
   return PL_OK;
 }
@@ -627,22 +658,22 @@ pl_status pl_pipeline_step(pl_pipeline* pl, pl_summary* prev, int* has_prev) {
   if (!pl || !prev || !has_prev) return fail(PL_EINVAL, "NULL argument");
   cudaSetDevice(pl->device);
   if (!pl->h_step) {
-    CUDA_TRY(cudaHostAlloc((void**)&pl->h_step, 2 * 7 * sizeof(unsigned long long), cudaHostAllocDefault));
+    CUDA_TRY(cudaHostAlloc((void**)&pl->h_step, 2 * 8 * sizeof(unsigned long long), cudaHostAllocDefault));
     for (cudaEvent_t& e : pl->step_ev) CUDA_TRY(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
   }
   const uint32_t b = (uint32_t)(pl->steps & 1u);
   pl_status st = pl_pipeline_launch(pl);
   if (st != PL_OK) return st;
   // the run's summary slot is copied before the next launch (which zeroes it) can start
-  CUDA_TRY(cudaMemcpyAsync(pl->h_step + 7 * b, pl->d_match_count - 6, 56, cudaMemcpyDeviceToHost, pl->stream));
+  CUDA_TRY(cudaMemcpyAsync(pl->h_step + 8 * b, pl->d_match_count - 6, 64, cudaMemcpyDeviceToHost, pl->stream));
   CUDA_TRY(cudaEventRecord(pl->step_ev[b], pl->stream));
   pl->step_launch[b] = pl->launches;
-  pl->d2h += 56;
+  pl->d2h += 64;
   *has_prev = 0;
   if (pl->steps > 0) {   // the previous step's run: wait for it only, the new one keeps running
     const uint32_t pb = b ^ 1u;
     CUDA_TRY(cudaEventSynchronize(pl->step_ev[pb]));
-    decode_summary(pl, pl->h_step + 7 * pb, pl->step_launch[pb], prev);
+    decode_summary(pl, pl->h_step + 8 * pb, pl->step_launch[pb], prev);
     *has_prev = 1;
   }
   ++pl->steps;
@@ -656,7 +687,7 @@ pl_status pl_pipeline_step_finish(pl_pipeline* pl, pl_summary* last, int* has_la
   if (pl->steps > 0) {
     const uint32_t b = (uint32_t)((pl->steps - 1) & 1u);
     CUDA_TRY(cudaEventSynchronize(pl->step_ev[b]));
-    decode_summary(pl, pl->h_step + 7 * b, pl->step_launch[b], last);
+    decode_summary(pl, pl->h_step + 8 * b, pl->step_launch[b], last);
     *has_last = 1;
   }
   pl->steps = 0;
@@ -758,6 +789,8 @@ pl_status pl_pipeline_stats(pl_pipeline* pl, pl_stats* out) {
     out->wall_ns = std::max(out->wall_ns, s.wall_ns);
     out->errors |= s.errors;
     out->window_refills += s.win_refills;
+    out->latency_outliers += s.agr_bad;
+    out->latency_rel_err_max = std::max(out->latency_rel_err_max, (double)s.agr_ppm * 1e-6);
   }
   unsigned long long mc = 0;
   CUDA_TRY(cudaMemcpy(&mc, pl->d_match_count, 8, cudaMemcpyDeviceToHost));
@@ -841,7 +874,7 @@ pl_status pl_pipeline_results(pl_pipeline* pl, pl_match* buf, uint64_t cap, uint
   uint64_t cnt = std::min<uint64_t>(mc, pl->dp.match_cap);
   if (!buf) { *n = cnt; return PL_OK; }
   cnt = std::min(cnt, cap);
-  if (cnt) CUDA_TRY(cudaMemcpy(buf, pl->d_matches, cnt * sizeof(pl_match), cudaMemcpyDeviceToHost));
+  if (cnt) CUDA_TRY(cudaMemcpy(buf, pl->dp.matches, cnt * sizeof(pl_match), cudaMemcpyDefault));
   pl->d2h += 8 + cnt * sizeof(pl_match);
   *n = cnt;
   return PL_OK;

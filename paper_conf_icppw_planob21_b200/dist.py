@@ -8,8 +8,10 @@ NCCL on NVLink/NVSwitch (gloo on CPU for tests).
 from __future__ import annotations
 
 SUM_KEYS = ("roots", "firings", "empty_firings", "consumed", "produced", "active_window", "busy_ns",
-            "spilled", "overruns", "matches", "miss_events", "misses", "window", "t_end")
-MAX_KEYS = ("max_lateness_ns", "max_fire_ns", "max_loop_ns", "max_latency", "max_latency_ns", "wall_ns", "errors")
+            "spilled", "overruns", "stalls", "matches", "miss_events", "miss_events_ns", "misses", "window", "t_end",
+            "latency_outliers", "window_refills")
+MAX_KEYS = ("max_lateness_ns", "max_fire_ns", "max_loop_ns", "max_latency", "max_latency_ns", "wall_ns",
+            "max_queue")
 
 
 def _flatten(st, keys):
@@ -41,12 +43,18 @@ def allreduce_stats(st: dict, device=None) -> dict:
     import torch.distributed as dist
     if not (dist.is_available() and dist.is_initialized()) or dist.get_world_size() == 1:
         return st
-    s = torch.tensor(_flatten(st, SUM_KEYS), dtype=torch.int64, device=device)
-    m = torch.tensor(_flatten(st, MAX_KEYS), dtype=torch.int64, device=device)
+    sk = [k for k in SUM_KEYS if k in st]
+    mk = [k for k in MAX_KEYS if k in st]
+    s = torch.tensor(_flatten(st, sk), dtype=torch.int64, device=device)
+    # the maxima, then the error flags one bit per slot (a MAX of whole bitmasks would lose bits)
+    m = torch.tensor(_flatten(st, mk) + [(int(st.get("errors", 0)) >> b) & 1 for b in range(32)],
+                     dtype=torch.int64, device=device)
     dist.all_reduce(s, op=dist.ReduceOp.SUM)
     dist.all_reduce(m, op=dist.ReduceOp.MAX)
-    res = _unflatten(st, SUM_KEYS, s.tolist())
-    res = _unflatten(res, MAX_KEYS, m.tolist())
+    res = _unflatten(st, sk, s.tolist())
+    mv = m.tolist()
+    res = _unflatten(res, mk, mv[:len(mv) - 32])
+    res["errors"] = sum(int(x) << b for b, x in enumerate(mv[len(mv) - 32:]))
     N = st["n_stages"]
     mono = st.get("policy") == 2
     if res["window"]:

@@ -115,6 +115,11 @@ class Pipeline:
         """pl_pipeline_bind_host: the DB stays in pinned host memory; CTAs stage it by TMA."""
         check(lib.pl_pipeline_bind_host(self.h, C.c_void_p(host_ptr), int(n)), "pl_pipeline_bind_host")
 
+    def bind_results(self, ptr, cap):
+        """pl_pipeline_bind_results: later runs write their match records into `ptr` (device memory
+        or pinned+mapped host memory, `cap` records); ptr=None restores the handle's own buffer."""
+        check(lib.pl_pipeline_bind_results(self.h, C.c_void_p(ptr or 0), int(cap)), "pl_pipeline_bind_results")
+
     def queue_peaks(self):
         """pl_pipeline_queue_peaks -> uint32 array [n_streams, N]."""
         n = C.c_uint64()

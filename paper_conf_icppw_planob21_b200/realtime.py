@@ -47,7 +47,7 @@ def calibrate_budgets(cfg, wl, db_dev, margin=1.25, slack_ns=256, probe_t=20_000
 
 
 def refine_budgets(cfg, wl, db_dev, budgets, margin=1.10, slack_ns=128, rounds=2, reps=3, flags=0, stream=None,
-                   over=None, log=None):
+                   over=None, log=None, policy=0, max_lateness_ns=5000, solve_deadline=None, guard_extra=0):
     """Budgets re-measured at the operating point.  The probe of calibrate_budgets fires every
     node with a full vector at the same instant, a contention pattern the solved schedule
     rarely produces; here each round finds the miss-free rate for the current budgets
@@ -57,11 +57,15 @@ def refine_budgets(cfg, wl, db_dev, budgets, margin=1.10, slack_ns=128, rounds=2
     hist = []
     for _ in range(rounds):
         c = cfg.replace(service_time=tuple(budgets))
-        tau, w, th, T, st = find_rate(c, wl, db_dev, stream=stream, over=over)
+        if policy == 1:   # THRESHOLD_SLACK: the slack guard follows the budgets
+            c = c.replace(slack_guard=int(max(budgets)) + guard_extra)
+        tau, w, th, T, st = find_rate(c, wl, db_dev, stream=stream, over=over, policy=policy, flags=flags,
+                                      max_lateness_ns=max_lateness_ns, solve_deadline=solve_deadline,
+                                      grow=1.5)
         worst = [0] * cfg.n_stages
         for _ in range(reps):
-            s2 = _run(c.replace(interarrival=tau, wait_time=tuple(w), clock=PHYS), db_dev, wl.db_len, wl,
-                      flags=flags, stream=stream, over=over)
+            s2 = _run(c.replace(interarrival=tau, wait_time=tuple(w), wait_threshold=tuple(th), clock=PHYS,
+                                policy=policy), db_dev, wl.db_len, wl, flags=flags, stream=stream, over=over)
             worst = [max(a, b) for a, b in zip(worst, s2["max_fire_ns"])]
         nb = tuple(min(b, int(math.ceil(margin * x)) + slack_ns) for b, x in zip(budgets, worst))
         hist.append(dict(budgets=tuple(budgets), tau=tau, max_fire_ns=worst, next=nb))
@@ -96,7 +100,7 @@ def min_feasible_tau(cfg, lo=1, hi=1 << 20):
 
 
 def find_rate(cfg, wl, db_dev, tries=12, grow=1.15, stream=None, log=None, over=None, policy=0,
-              max_lateness_ns=5000, flags=0):
+              max_lateness_ns=5000, flags=0, solve_deadline=None):
     """Smallest tau0 (ns) at which a physical run (FIXED_WAIT, or THRESHOLD_SLACK with the
     Fig. 1-derived thresholds when policy=1) has zero deadline misses, no queue overflow
     and, unless max_lateness_ns is None, every firing starting within max_lateness_ns of its
@@ -107,11 +111,14 @@ def find_rate(cfg, wl, db_dev, tries=12, grow=1.15, stream=None, log=None, over=
     for which Fig. 1 is feasible, grows by `grow` until a run is clean, then bisects between
     the last failing and the first clean tau0.  The trial runs use the kernel selected by
     `flags` (default: the record-free kernel that the bench times; misses are counted on the
-    device either way).  Returns (tau0, w, theta, T, stats)."""
+    device either way).  `solve_deadline`: the deadline Fig. 1 is solved at (default cfg's D; a
+    platform-stall allowance is kept out of it, DESIGN.md R-STALL), while misses count against
+    cfg's D.  Returns (tau0, w, theta, T, stats)."""
     from ._pl import PlError
+    scfg = cfg if solve_deadline is None else cfg.replace(deadline=int(solve_deadline))
 
     def trial(tau):
-        sol = solve_at(cfg, tau)
+        sol = solve_at(scfg, tau)
         if sol is None:
             return None
         w, th, T = sol
@@ -131,7 +138,7 @@ def find_rate(cfg, wl, db_dev, tries=12, grow=1.15, stream=None, log=None, over=
                      max_latency_ns=st["max_latency_ns"], max_lateness_ns=st["max_lateness_ns"]))
         return (int(tau), w, th, T, st) if ok else None
 
-    tau = min_feasible_tau(cfg)
+    tau = min_feasible_tau(scfg)
     if tau is None:
         raise RuntimeError("Fig. 1 infeasible for every tau0 at this deadline")
     bad = tau - 1

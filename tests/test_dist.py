@@ -24,7 +24,8 @@ def _stats(rank):
             "busy_ns": [1000 * (rank + 1), 0], "spilled": [0, rank], "overruns": [0, 0], "matches": rank,
             "miss_events": 0, "misses": 0, "window": 400 + 4 * rank, "t_end": 500,
             "max_lateness_ns": [rank * 7, 3], "max_fire_ns": [100 - rank, 50 + rank], "max_loop_ns": [9 + rank, 4], "max_latency": 400 + rank,
-            "max_latency_ns": 1000 * rank, "wall_ns": 5 + rank, "errors": 0, "active_fraction": 0.0}
+            "max_latency_ns": 1000 * rank, "wall_ns": 5 + rank, "errors": 1 << rank, "active_fraction": 0.0,
+            "miss_events_ns": rank, "max_queue": [3 + rank, 9 - rank]}
 
 
 def _worker(rank, port, out):
@@ -50,6 +51,8 @@ def test_allreduce_stats_gloo_two_ranks():
     assert a["window"] == 804
     assert abs(a["active_fraction"] - (641 + 640 + 960) / (2 * 804)) < 1e-12
     assert a["n_ranks"] == 2
+    assert a["errors"] == 3                      # each rank's overflow bit survives the reduction
+    assert a["miss_events_ns"] == 1 and a["max_queue"] == [4, 9]
 
 
 def test_single_process_is_identity():

@@ -192,3 +192,17 @@ def test_table1_golden_matches_configs():
     g = tuple(float(r[2]) for r in rows[:3])
     b = tuple(int(x) for x in rows[4][1:])
     assert t == C.TABLE1_T and g == C.TABLE1_G and b == C.PAPER_B
+
+
+def test_unpack_bytes_matches_base():
+    """The vectorised unpack (the oracle's DB view) gives base() for every position, including
+    a ragged last word."""
+    import numpy as np
+    from plgen import dna as G
+    rng = np.random.default_rng(7)
+    for n in (1, 15, 16, 17, 1000, 4099):
+        codes = rng.integers(0, 4, size=n, dtype=np.uint8)
+        words = G.pack(codes)
+        ub = S.unpack_bytes(words, n)
+        assert len(ub) == n
+        assert list(ub) == [S.base(words, j) for j in range(n)] == list(codes)
