@@ -74,8 +74,12 @@ enum pl_clock { PL_CLOCK_LOGICAL = 0, PL_CLOCK_GLOBALTIMER = 1 };
 #define PL_REC_LATENCY  1u     /* lat[r]: per-root latency (model units; + ns if physical) */
 #define PL_REC_TRACE    2u     /* cnt[r][0..N]: per-root surviving-stage trace           */
 #define PL_REC_FIRINGS  4u     /* per-stream log of non-empty firings                    */
-#define PL_FIXED_SERVICE 8u    /* physical clock: publish a firing's outputs at start + t_i,
-                                  the paper's fixed service time (L69), not as soon as done */
+#define PL_FIXED_SERVICE 8u    /* physical clock, time-triggered delivery: a firing occupies its
+                                  node until start + t_i, the paper's fixed service time (L69),
+                                  and its terminal items complete then (or when the work is done,
+                                  if later: an overrun); without it they complete when done.  The
+                                  schedule is the same either way (a segment's items are ready at
+                                  start + t_i and consumed at logical times >= that).           */
 #define PL_EAGER_DRAIN  16u    /* end of stream (reading R-DRAIN): at times T >= A_last, the
                                   stream's last arrival, every node fires whenever it is idle
                                   and its queue is non-empty (FIXED_WAIT's time-triggered
@@ -204,7 +208,8 @@ typedef struct {
   /* physical clock: agreement of every terminal item's MEASURED latency with the logical-clock
    * prediction T + t_i - a(r) (north_star "within 5 % relative"; DESIGN.md R-AGREE: a floor of
    * 64 ns = two %globaltimer ticks; with PL_FIXED_SERVICE a firing completes at start + t_i)   */
-  uint64_t latency_outliers;               /* terminal items with |err| > 5 % of their latency + 64 ns */
+  uint64_t latency_outliers;               /* terminal items with |err| > 5 % of their latency + 64 ns
+                                              (counted with PL_FIXED_SERVICE only)                    */
   double   latency_rel_err_max;            /* largest |err| / logical latency over terminal items      */
 } pl_stats;
 

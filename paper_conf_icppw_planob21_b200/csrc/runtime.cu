@@ -406,7 +406,9 @@ pl_status pl_pipeline_create(const pl_config* cfg, const pl_workload* wl, pl_pip
     uint64_t words = (per + pl->k + 2 * d.win_halo) / 16 + 8;
     words = (words + 3) & ~3ull;
     const uint64_t chunks = (words + CH - 1) / CH + 1;     // + 1: chunks sit at absolute boundaries
-    uint32_t cap = CH * next_pow2((uint32_t)std::min<uint64_t>(chunks, 16));
+    // a sliding ring of 8 chunks (32 KB = 128 K bases) holds far more than a stream's in-flight
+    // roots plus the extension halo; the rest of the smem goes to the queues (below)
+    uint32_t cap = CH * (chunks <= 16 ? next_pow2((uint32_t)chunks) : 8u);
     if (cfg->window_words) {
       if (!is_pow2(cfg->window_words) || cfg->window_words < 2 * CH)
         return bail(fail(PL_EINVAL, "window_words must be a power of 2 >= 2 * window_chunk_words"));
@@ -455,6 +457,19 @@ pl_status pl_pipeline_create(const pl_config* cfg, const pl_workload* wl, pl_pip
   d.spill = pl->d_spill;
   d.mono_buf = pl->d_mono;
   pl->smem = pl_layout_enforced_host(d);
+  // Spare shared memory deepens the smem ring behind the largest amplifier (the edge whose
+  // producer has the largest u): a burst of u outputs per input -- or the backlog after a
+  // platform stall -- then stays on chip instead of spilling to the HBM ring.
+  if (!cfg->queue_capacity && cfg->policy != PL_MONOLITHIC && N > 1) {
+    uint32_t e = 1;
+    for (uint32_t i = 2; i < N; ++i)
+      if (pl->stages[i - 1].max_out > pl->stages[e - 1].max_out) e = i;
+    while (2 * d.cap_s[e] <= d.cap_g) {
+      d.cap_s[e] *= 2;
+      if (pl_layout_enforced_host(d) > 196 * 1024) { d.cap_s[e] /= 2; break; }
+    }
+    pl->smem = pl_layout_enforced_host(d);
+  }
   // one CTA (stream) per SM: the two-per-SM variant (64 registers) spills and measured no gain
   // (tools/streams_scaling.py); it stays selectable through PL_CTAS_PER_SM=2
   d.ctas_per_sm = 1;

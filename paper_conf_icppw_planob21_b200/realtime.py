@@ -33,27 +33,36 @@ def measure_gains(cfg, wl, db_dev, stream=None, over=None):
 
 
 def calibrate_budgets(cfg, wl, db_dev, margin=1.25, slack_ns=256, probe_t=20_000, probe_tau=100, stream=None,
-                      over=None, flags=0):
+                      over=None, flags=0, reps=2):
     """Service-time budgets t_i (ns): the longest measured firing of each node in a
     physical run with generous budgets, times `margin`, plus `slack_ns`.  The probe's
     arrivals (probe_t / probe_tau > v per period) keep node 0's vectors full.  `flags`
     must match the runs the budgets are for: per-item records (PL_REC_*) select the
-    recording kernel, whose firings are longer."""
+    recording kernel, whose firings are longer.  The probe runs `reps` times and each node
+    keeps the smallest of its per-run maxima: a one-off outlier (a cold first launch, a
+    platform stall inside a firing) does not set a budget."""
     N = cfg.n_stages
     probe = cfg.replace(clock=PHYS, service_time=(probe_t,) * N, wait_time=(0,) * N, interarrival=probe_tau,
                         deadline=10**12, policy=0, gain=None, ns_per_unit=1.0)
-    st = _run(probe, db_dev, wl.db_len, wl, flags=flags, stream=stream, over=over)
+    runs = [_run(probe, db_dev, wl.db_len, wl, flags=flags, stream=stream, over=over) for _ in range(max(1, reps))]
+    st = dict(runs[-1], max_fire_ns=[min(r["max_fire_ns"][i] for r in runs) for i in range(N)],
+              max_fire_ns_runs=[r["max_fire_ns"] for r in runs])
     return tuple(int(math.ceil(margin * st["max_fire_ns"][i])) + slack_ns for i in range(N)), st
 
 
 def refine_budgets(cfg, wl, db_dev, budgets, margin=1.10, slack_ns=128, rounds=2, reps=3, flags=0, stream=None,
-                   over=None, log=None, policy=0, max_lateness_ns=5000, solve_deadline=None, guard_extra=0):
+                   over=None, log=None, policy=0, max_lateness_ns=5000, solve_deadline=None, guard_extra=0,
+                   stall_ns=100_000):
     """Budgets re-measured at the operating point.  The probe of calibrate_budgets fires every
-    node with a full vector at the same instant, a contention pattern the solved schedule
-    rarely produces; here each round finds the miss-free rate for the current budgets
-    (find_rate), runs that schedule `reps` times with the kernel the budgets are for (`flags`)
-    and takes ceil(margin * longest firing) + slack_ns per node, never raising a budget.
-    Stops when no budget shrinks.  Returns (budgets, history)."""
+    node with a full vector at a period of its own; at the operating point a node can fire
+    back to back (THRESHOLD_SLACK in a burst), and then its real per-firing cost is the whole
+    loop -- the firing, its publish and the next decision (pl_stats.max_loop_ns) -- not the
+    firing alone.  Each round finds the miss-free rate for the current budgets (find_rate),
+    runs that schedule `reps` times with the kernel the budgets are for (`flags`) and sets
+    t_i = ceil(margin * max(longest firing, longest loop)) + slack_ns, raising or lowering it.
+    A per-run maximum above max(stall_ns, 10 t_i) is a platform stall inside a firing
+    (profiles/r02_pause_control.txt), not the work: that run's value is ignored for the node.
+    Stops when no budget moves by more than 2 %.  Returns (budgets, history)."""
     hist = []
     for _ in range(rounds):
         c = cfg.replace(service_time=tuple(budgets))
@@ -64,16 +73,25 @@ def refine_budgets(cfg, wl, db_dev, budgets, margin=1.10, slack_ns=128, rounds=2
                                       grow=1.5)
         worst = [0] * cfg.n_stages
         for _ in range(reps):
-            s2 = _run(c.replace(interarrival=tau, wait_time=tuple(w), wait_threshold=tuple(th), clock=PHYS,
-                                policy=policy), db_dev, wl.db_len, wl, flags=flags, stream=stream, over=over)
-            worst = [max(a, b) for a, b in zip(worst, s2["max_fire_ns"])]
-        nb = tuple(min(b, int(math.ceil(margin * x)) + slack_ns) for b, x in zip(budgets, worst))
-        hist.append(dict(budgets=tuple(budgets), tau=tau, max_fire_ns=worst, next=nb))
+            for _attempt in range(3):   # a run that met a platform stall measures the stall: repeat it
+                s2 = _run(c.replace(interarrival=tau, wait_time=tuple(w), wait_threshold=tuple(th), clock=PHYS,
+                                    policy=policy), db_dev, wl.db_len, wl, flags=flags, stream=stream, over=over)
+                if not stalled(s2):
+                    break
+            if stalled(s2):
+                continue
+            for i in range(cfg.n_stages):
+                x = max(s2["max_fire_ns"][i], s2["max_loop_ns"][i])
+                if x <= max(stall_ns, 10 * budgets[i]):
+                    worst[i] = max(worst[i], x)
+        nb = tuple(int(math.ceil(margin * x)) + slack_ns if x else b for b, x in zip(budgets, worst))
+        hist.append(dict(budgets=tuple(budgets), tau=tau, max_fire_or_loop_ns=worst, next=nb))
         if log:
             log(hist[-1])
-        if nb == tuple(budgets):
-            break
+        moved = any(abs(x - y) > 0.02 * y for x, y in zip(nb, budgets))
         budgets = nb
+        if not moved:
+            break
     return tuple(budgets), hist
 
 
@@ -99,8 +117,20 @@ def min_feasible_tau(cfg, lo=1, hi=1 << 20):
     return lo
 
 
+STALL_NS = 1_000_000   # every node at least this late in one run: a platform SM stall (R-STALL)
+
+
+def stalled(st) -> bool:
+    """Whether a physical run met a platform stall: the B200 stops every SM for ~1.6 ms every
+    few seconds (profiles/r02_pause_control.txt), so every node of the stream falls ~1.6 ms
+    behind its schedule at once; an overloaded node alone does not look like that."""
+    lat = st.get("max_lateness_ns") or [0]
+    return min(lat) >= STALL_NS
+
+
 def find_rate(cfg, wl, db_dev, tries=12, grow=1.15, stream=None, log=None, over=None, policy=0,
-              max_lateness_ns=5000, flags=0, solve_deadline=None):
+              max_lateness_ns=5000, flags=0, solve_deadline=None, max_outliers=None, start=None,
+              stall_retries=2):
     """Smallest tau0 (ns) at which a physical run (FIXED_WAIT, or THRESHOLD_SLACK with the
     Fig. 1-derived thresholds when policy=1) has zero deadline misses, no queue overflow
     and, unless max_lateness_ns is None, every firing starting within max_lateness_ns of its
@@ -113,7 +143,9 @@ def find_rate(cfg, wl, db_dev, tries=12, grow=1.15, stream=None, log=None, over=
     `flags` (default: the record-free kernel that the bench times; misses are counted on the
     device either way).  `solve_deadline`: the deadline Fig. 1 is solved at (default cfg's D; a
     platform-stall allowance is kept out of it, DESIGN.md R-STALL), while misses count against
-    cfg's D.  Returns (tau0, w, theta, T, stats)."""
+    cfg's D.  `start`: the first tau0 tried (default: the smallest Fig. 1-feasible one).  A
+    failing run that met a platform stall (stalled()) is repeated up to `stall_retries` times: it
+    says nothing about the rate.  Returns (tau0, w, theta, T, stats)."""
     from ._pl import PlError
     scfg = cfg if solve_deadline is None else cfg.replace(deadline=int(solve_deadline))
 
@@ -124,23 +156,31 @@ def find_rate(cfg, wl, db_dev, tries=12, grow=1.15, stream=None, log=None, over=
         w, th, T = sol
         c = cfg.replace(interarrival=int(tau), wait_time=tuple(w), wait_threshold=tuple(th), clock=PHYS,
                         policy=policy)
-        try:
-            st = _run(c, db_dev, wl.db_len, wl, flags=flags, stream=stream, over=over)
-            ok = (st["misses"] == 0 and st["miss_events"] == 0 and st["miss_events_ns"] == 0
-                  and st["errors"] == 0)
-            if max_lateness_ns is not None:
-                ok = ok and max(st["max_lateness_ns"]) <= max_lateness_ns
-        except PlError:          # device-side overflow reported by drain
-            st, ok = {"misses": -1, "miss_events_ns": -1, "errors": -1, "overruns": [], "max_latency_ns": -1,
-                      "max_lateness_ns": []}, False
+        for attempt in range(stall_retries + 1):
+            try:
+                st = _run(c, db_dev, wl.db_len, wl, flags=flags, stream=stream, over=over)
+                ok = (st["misses"] == 0 and st["miss_events"] == 0 and st["miss_events_ns"] == 0
+                      and st["errors"] == 0)
+                if max_lateness_ns is not None:
+                    ok = ok and max(st["max_lateness_ns"]) <= max_lateness_ns
+                if max_outliers is not None:   # north_star 5 % per-item agreement (R-AGREE)
+                    ok = ok and st["latency_outliers"] <= max_outliers
+            except PlError:          # device-side overflow reported by drain
+                st, ok = {"misses": -1, "miss_events_ns": -1, "errors": -1, "overruns": [], "max_latency_ns": -1,
+                          "max_lateness_ns": []}, False
+            if ok or not stalled(st):
+                break
         if log:
             log(dict(tau=tau, w=w, T=T, misses=st["misses"], overruns=st["overruns"], errors=st["errors"],
-                     max_latency_ns=st["max_latency_ns"], max_lateness_ns=st["max_lateness_ns"]))
+                     max_latency_ns=st["max_latency_ns"], max_lateness_ns=st["max_lateness_ns"],
+                     outliers=st.get("latency_outliers")))
         return (int(tau), w, th, T, st) if ok else None
 
     tau = min_feasible_tau(scfg)
     if tau is None:
         raise RuntimeError("Fig. 1 infeasible for every tau0 at this deadline")
+    if start is not None and start > tau:
+        tau = int(start)
     bad = tau - 1
     good = None
     for _ in range(tries):
