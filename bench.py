@@ -17,7 +17,8 @@ Procedure:
   2. the deadline D (c4: 3.5 ms) with a platform-stall allowance of 2.7 ms (reading R-STALL:
      the B200 stops every SM for ~1.6 ms every few seconds, profiles/r02_pause_control.txt, and
      the pipeline needs a few hundred us to catch up): THRESHOLD_SLACK reserves it in every R_i,
-     FIXED_WAIT / MONOLITHIC solve Fig. 1 / Fig. 2 at D - 2.7 ms;  b = (1, 3, 9, 6) (L230);
+     FIXED_WAIT / MONOLITHIC solve Fig. 1 / Fig. 2 at D - 2.7 ms (the schedulable deadline,
+     0.8 ms);  b = (1, 3, 9, 6) (L230);
   3. the headline policy is the north_star's THRESHOLD_SLACK rule; tau0 = the smallest
      inter-arrival whose physical run has zero deadline misses (measured), no overflow;
   4. the timed steps run with PL_FIXED_SERVICE (a firing's outputs appear at start + t_i, the
@@ -81,7 +82,7 @@ def parse():
     ap.add_argument("--refine", type=int, default=2, help="budget refinement rounds at the operating point")
     ap.add_argument("--confirm", type=int, default=3,
                     help="confirmation runs the operating point must pass (else +10 %% and retry)")
-    ap.add_argument("--headroom", type=float, default=1.3,
+    ap.add_argument("--headroom", type=float, default=1.15,
                     help="operating tau0 = headroom x the fastest stall-free miss-free tau0 (R-STALL: the "
                          "pipeline must catch up after a ~1.6 ms platform stall within D)")
     a = ap.parse_args()
@@ -263,8 +264,13 @@ def main():
 
     # 1. gains (logical run) and budgets (physical probe, refined at the operating point)
     gains = realtime.measure_gains(base.replace(wait_time=(0,) * 4), wl, db_ptr, stream=stream, over=over)
+    # c4: the probe overloads every node (budgets of 1 us at tau0 = 20 ns), so that all four
+    # fire back to back and share the SM -- the 1/N processor share at which PAPER.md L69 defines
+    # t_i (profiles/r02_c4_probe.txt: 1.3-2.4x the firing times of an isolated node).  A
+    # pipeline recovering from a platform stall runs exactly like that.
     budgets, cal = realtime.calibrate_budgets(base, wl, db_ptr, stream=stream, margin=a.budget_margin,
-                                              slack_ns=a.budget_slack, probe_tau=20 if c4 else 100, over=over)
+                                              slack_ns=a.budget_slack, probe_tau=20 if c4 else 100, over=over,
+                                              probe_t=1000 if c4 else 20_000)
     # misses count against D; the schedules are solved at D - SG (R-STALL) and THRESHOLD_SLACK
     # reserves SG in every R_i on top of the largest budget
     cfg0 = base.replace(clock=1, ns_per_unit=1.0, service_time=budgets, gain=gains, deadline=D,
@@ -275,7 +281,8 @@ def main():
             budgets, _ = realtime.refine_budgets(thr_cfg(budgets), wl, db_ptr, budgets, margin=a.budget_margin,
                                                  slack_ns=a.budget_slack, rounds=a.refine, stream=stream, log=log,
                                                  over=over, policy=1, max_lateness_ns=None, solve_deadline=D - SG,
-                                                 guard_extra=SG, flags=0)   # publish mode: the work's own duration
+                                                 guard_extra=SG, flags=0,   # publish mode: the work's own duration
+                                                 lower=not c4)
         except RuntimeError as ex:   # no operating point for the refinement: keep the probe's budgets
             log({"refine_budgets": "skipped", "error": str(ex)})
     if world > 1:   # every rank runs the same schedule: max budgets are conservative

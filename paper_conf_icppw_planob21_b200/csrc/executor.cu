@@ -483,6 +483,7 @@ struct Node {
                                 // the last of them ends at B_per
   uint32_t* troot;              // smem [v]: the current firing's terminal root per lane (or NO_ROOT)
   uint32_t* bnd;                // smem: Shared::bnd (sliding window only)
+  uint32_t nap_cap_ns;          // physical: longest poll nap of a waiting leader (t_i / 8, >= 256 ns)
   bool sliding;
   __device__ __forceinline__ int64_t arrival(uint32_t root) const {
     return arr ? __ldg(arr + root) : (int64_t)(root - lo) * tau;
@@ -541,6 +542,10 @@ __device__ __forceinline__ Node make_node(const Ctx& c, int i) {
   n.B_per = n.Mcap > 0 ? (n.Mcap - 1) * n.P + n.t : 0;
   n.troot = (uint32_t*)(c.dsm + Lo.off_troot) + (uint32_t)i * (uint32_t)p.v;
   n.bnd = c.sh->bnd;
+  {
+    const int64_t cap = n.t_ns / 8;
+    n.nap_cap_ns = (uint32_t)(cap < 256 ? 256 : (cap > 8192 ? 8192 : cap));
+  }
   n.sliding = c.sliding;
   return n;
 }
@@ -676,12 +681,22 @@ __device__ __forceinline__ void publish_W(const Node& nd, Leader& L, int64_t w) 
   }
 }
 
-// Poll backoff.  The logical clock polls hard (its schedule advances as fast as the nodes do);
-// on the physical clock the %globaltimer ticks every 32 ns and a poll costs issue slots that
-// a waiting node is supposed to yield, so it backs off faster.
-__device__ __forceinline__ void backoff(int& spins, bool phys = false) {
+// Poll backoff.  The logical clock polls hard (its schedule advances as fast as the nodes do).
+// On the physical clock a poll costs issue slots that a waiting node is supposed to yield
+// (PAPER.md L75/L85), so the nap doubles from 64 ns up to `cap_ns` -- an eighth of the node's
+// service time (Node::nap_cap_ns): reacting that much later to an upstream publish delays a
+// firing start by at most t_i / 8, which the time-triggered delivery (PL_FIXED_SERVICE) absorbs
+// while the work itself takes well under t_i.  Measured on c4 (ncu source page): the fixed
+// 256 ns nap made the waiting leaders' polls ~90 % of all instructions issued.
+__device__ __forceinline__ void backoff(int& spins, bool phys = false, uint32_t cap_ns = 256) {
   if (spins < (phys ? 2 : 4)) { ++spins; return; }
-  __nanosleep(phys ? (spins < 16 ? 64 : 256) : (spins < 64 ? 32 : 256));
+  if (phys) {
+    const int e = spins - 2 < 16 ? spins - 2 : 16;
+    const uint32_t ns = 64u << e;
+    __nanosleep(ns < cap_ns ? ns : cap_ns);
+  } else {
+    __nanosleep(spins < 64 ? 32 : 256);
+  }
   ++spins;
 }
 
@@ -809,9 +824,9 @@ __device__ __forceinline__ void advance0(const Node& nd, Rep& r) {
 __device__ __forceinline__ bool nap_until(uint64_t target) {
   uint64_t now = gtimer();
   if (now >= target) return false;
-  while (now < target) {
+  while (now < target) {   // __nanosleep may round up to ~2x: nap a quarter of the remaining time
     const uint64_t rem = target - now;
-    __nanosleep(rem > 16384 ? 4096 : (rem > 4096 ? 1024 : (rem > 1024 ? 256 : 64)));
+    __nanosleep(rem > 4096 ? (uint32_t)min(rem >> 2, (uint64_t)(1u << 20)) : (rem > 1024 ? 256u : 64u));
     now = gtimer();
   }
   return true;
@@ -859,7 +874,7 @@ __device__ Decision decide(const Node& nd, Leader& L, bool& waited, uint64_t T0)
         if (!any) {
           if (Wup == PL_INF64) { d.done = true; return d; }
           publish_W(nd, L, max(B, Wup) + nd.t);
-          backoff(spins, nd.phys); waited = true;
+          backoff(spins, nd.phys, nd.nap_cap_ns); waited = true;
           continue;
         }
         const int64_t Te = max(B, nd.in_seg[L.segh & nd.segmask].ready);
@@ -868,7 +883,7 @@ __device__ Decision decide(const Node& nd, Leader& L, bool& waited, uint64_t T0)
         if (Wup > Te || (cnt >= v && early_ok(nd))) {
           d.T = Te; d.n = cnt < v ? cnt : v; d.qlen = count_all_le(nd, L, st, Te); return d;
         }
-        backoff(spins, nd.phys); waited = true;
+        backoff(spins, nd.phys, nd.nap_cap_ns); waited = true;
         continue;
       }
       const int64_t T = L.m * nd.P;
@@ -887,14 +902,14 @@ __device__ Decision decide(const Node& nd, Leader& L, bool& waited, uint64_t T0)
         continue;
       }
       publish_W(nd, L, T + nd.t);
-      backoff(spins, nd.phys); waited = true;
+      backoff(spins, nd.phys, nd.nap_cap_ns); waited = true;
       continue;
     }
     // THRESHOLD_SLACK
     if (!any) {
       if (Wup == PL_INF64) { d.done = true; return d; }
       publish_W(nd, L, (Wup > L.B ? Wup : L.B) + nd.t);
-      backoff(spins, nd.phys); waited = true;
+      backoff(spins, nd.phys, nd.nap_cap_ns); waited = true;
       continue;
     }
     const Seg& hs = nd.in_seg[L.segh & nd.segmask];
@@ -927,7 +942,7 @@ __device__ Decision decide(const Node& nd, Leader& L, bool& waited, uint64_t T0)
     int64_t lb = Tk < Wup ? Tk : Wup;
     if (lb < L.B) lb = L.B;
     publish_W(nd, L, lb + nd.t);
-    backoff(spins, nd.phys); waited = true;
+    backoff(spins, nd.phys, nd.nap_cap_ns); waited = true;
   }
 }
 
@@ -954,7 +969,7 @@ __device__ __forceinline__ void pace(uint64_t target, uint64_t* start_ns, int64_
   if (entry_ns) *entry_ns = now;
   while (now < target) {   // __nanosleep rounds up to powers of two: sleep at most ~rem/4
     const uint64_t rem = target - now;
-    __nanosleep(rem > 4096 ? 1024 : (rem > 1024 ? 256 : (rem > 256 ? 64 : 0)));
+    __nanosleep(rem > 4096 ? (uint32_t)min(rem >> 2, (uint64_t)(1u << 20)) : (rem > 1024 ? 256u : (rem > 256 ? 64u : 0u)));
     now = gtimer();
   }
   *start_ns = now;

@@ -52,14 +52,15 @@ def calibrate_budgets(cfg, wl, db_dev, margin=1.25, slack_ns=256, probe_t=20_000
 
 def refine_budgets(cfg, wl, db_dev, budgets, margin=1.10, slack_ns=128, rounds=2, reps=3, flags=0, stream=None,
                    over=None, log=None, policy=0, max_lateness_ns=5000, solve_deadline=None, guard_extra=0,
-                   stall_ns=100_000):
+                   stall_ns=100_000, lower=True):
     """Budgets re-measured at the operating point.  The probe of calibrate_budgets fires every
     node with a full vector at a period of its own; at the operating point a node can fire
     back to back (THRESHOLD_SLACK in a burst), and then its real per-firing cost is the whole
     loop -- the firing, its publish and the next decision (pl_stats.max_loop_ns) -- not the
     firing alone.  Each round finds the miss-free rate for the current budgets (find_rate),
     runs that schedule `reps` times with the kernel the budgets are for (`flags`) and sets
-    t_i = ceil(margin * max(longest firing, longest loop)) + slack_ns, raising or lowering it.
+    t_i = ceil(margin * max(longest firing, longest loop)) + slack_ns, raising it -- and lowering
+    it too unless lower=False.
     A per-run maximum above max(stall_ns, 10 t_i) is a platform stall inside a firing
     (profiles/r02_pause_control.txt), not the work: that run's value is ignored for the node.
     Stops when no budget moves by more than 2 %.  Returns (budgets, history)."""
@@ -85,6 +86,8 @@ def refine_budgets(cfg, wl, db_dev, budgets, margin=1.10, slack_ns=128, rounds=2
                 if x <= max(stall_ns, 10 * budgets[i]):
                     worst[i] = max(worst[i], x)
         nb = tuple(int(math.ceil(margin * x)) + slack_ns if x else b for b, x in zip(budgets, worst))
+        if not lower:    # keep the probe's budgets as a floor (e.g. measured at a 1/N share, L69)
+            nb = tuple(max(x, y) for x, y in zip(nb, budgets))
         hist.append(dict(budgets=tuple(budgets), tau=tau, max_fire_or_loop_ns=worst, next=nb))
         if log:
             log(hist[-1])
