@@ -82,12 +82,18 @@ def parse():
     ap.add_argument("--refine", type=int, default=2, help="budget refinement rounds at the operating point")
     ap.add_argument("--confirm", type=int, default=3,
                     help="confirmation runs the operating point must pass (else +10 %% and retry)")
-    ap.add_argument("--headroom", type=float, default=1.15,
+    ap.add_argument("--inject-period-ms", type=float, default=None,
+                    help="rate searches inject a platform-length stall every this many ms "
+                         "(pl_pipeline_inject_stalls; default: c4 100, c2 off)")
+    ap.add_argument("--inject-ms", type=float, default=1.8, help="length of an injected stall (R-STALL: ~1.6 ms)")
+    ap.add_argument("--headroom", type=float, default=1.0,
                     help="operating tau0 = headroom x the fastest stall-free miss-free tau0 (R-STALL: the "
                          "pipeline must catch up after a ~1.6 ms platform stall within D)")
     a = ap.parse_args()
     if a.deadline_ns is None:
         a.deadline_ns = 3_500_000 if a.workload == "c4" else 350_000
+    if a.inject_period_ms is None:
+        a.inject_period_ms = 100.0 if a.workload == "c4" else 0.0
     if a.stall_guard_ns is None:
         a.stall_guard_ns = 2_700_000 if a.workload == "c4" else 0
     return a
@@ -294,9 +300,11 @@ def main():
     cfg = thr_cfg(budgets)
 
     # 2./3. the fastest miss-free rate of the headline policy (THRESHOLD_SLACK; Fig. 1 thetas)
+    inject = (int(a.inject_period_ms * 1e6), int(a.inject_ms * 1e6)) if a.inject_period_ms > 0 else None
     tau, w, th, T, st_ok = realtime.find_rate(cfg, wl, db_ptr, stream=stream, log=log, policy=1, over=over,
                                               max_lateness_ns=None, grow=1.5 if c4 else 1.15, tries=16,
-                                              flags=PL_FIXED_SERVICE, solve_deadline=D - SG, max_outliers=0)
+                                              flags=PL_FIXED_SERVICE, solve_deadline=D - SG, max_outliers=0,
+                                              inject=inject)
     # the operating point: headroom over the edge the search found on stall-free runs, so that
     # the pipeline catches up after a platform stall within D (R-STALL); confirmed by --confirm
     # runs with zero measured misses whether or not they meet a stall, and zero latency
@@ -386,9 +394,11 @@ def main():
     # 4. beside it: FIXED_WAIT (the paper's rule) and MONOLITHIC (the no-wait baseline, Fig. 2)
     side = {}
 
-    def run_once(c, flags=PL_FIXED_SERVICE):
+    def run_once(c, flags=PL_FIXED_SERVICE, inj=None):
         pp = Pipeline(c, wl, flags=flags, stream=stream, **over)
         pp.bind_device(db_ptr, wl.db_len)
+        if inj:
+            pp.inject_stalls(*inj)
         e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         e0.record(stream)
         pp.launch()
@@ -407,7 +417,7 @@ def main():
             tf, wf, thf, Tf, _ = realtime.find_rate(fcfg, wl, db_ptr, stream=stream, over=over, grow=1.5,
                                                     tries=5 if c4 else 12, max_lateness_ns=None,
                                                     flags=PL_FIXED_SERVICE, solve_deadline=D - SG,
-                                                    start=tau if c4 else None)
+                                                    start=tau if c4 else None, inject=inject)
             side["fixed_wait"] = dict(run_once(fcfg.replace(interarrival=tf, wait_time=tuple(wf))),
                                       w_ns=list(wf), fig1_T=Tf)
         except RuntimeError as ex:
@@ -418,7 +428,7 @@ def main():
         for _ in range(20):
             Mm = realtime.monolithic_at(msolve, tm)
             if Mm is not None:
-                r = run_once(mcfg.replace(interarrival=tm, block_size=Mm[0]), flags=0)
+                r = run_once(mcfg.replace(interarrival=tm, block_size=Mm[0]), flags=0, inj=inject)
                 if r["misses"] == 0 and r["errors"] == 0:
                     found = dict(r, M=Mm[0], fig2_objective=Mm[1])
                     break
@@ -512,9 +522,15 @@ def main():
             "config": {"workload": WORKLOADS[a.workload], "policy": "THRESHOLD_SLACK (north_star rule; Fig. 1 thetas)",
                        "clock": "globaltimer (1 unit = 1 ns)", "service": "PL_FIXED_SERVICE (outputs at start + t_i, L69)",
                        "deadline_ns": D, "stall_guard_ns": SG, "tau0_ns": tau, "theta": list(th),
-                       "rate_criterion": (f"{a.headroom} x the fastest tau0 with zero measured misses and zero latency "
-                                          f"outliers on stall-free runs ({tau_edge} ns); then {a.confirm} confirmation "
-                                          f"runs with zero misses (tries: {confirm_log})"),
+                       "rate_criterion": ((f"{a.headroom} x the fastest tau0 with zero measured misses across "
+                                           f"{a.inject_ms} ms stalls injected every {a.inject_period_ms} ms "
+                                           f"(pl_pipeline_inject_stalls; R-STALL) ({tau_edge} ns)") if inject else
+                                          (f"{a.headroom} x the fastest tau0 with zero measured misses and zero latency "
+                                           f"outliers on stall-free runs ({tau_edge} ns)")) +
+                                          f"; then {a.confirm} confirmation runs without injection: zero misses, and "
+                                          f"zero latency outliers in those without a platform stall (tries: {confirm_log})",
+                       "stall_injection_in_rate_search": ({"period_ms": a.inject_period_ms, "len_ms": a.inject_ms}
+                                                          if inject else None),
                        "tau0_edge_ns": tau_edge, "edge_items_per_s": world * a.streams * 1e9 / tau_edge,
                        "b": list(C.PAPER_B), "budgets_ns": list(budgets), "gains": [round(g, 5) for g in gains],
                        "drain": "eager (R-DRAIN)" if not c4 else "periodic (paper rule)",

@@ -211,6 +211,8 @@ typedef struct {
   uint64_t latency_outliers;               /* terminal items with |err| > 5 % of their latency + 64 ns
                                               (counted with PL_FIXED_SERVICE only)                    */
   double   latency_rel_err_max;            /* largest |err| / logical latency over terminal items      */
+  uint64_t ingest_waits;                   /* live ingest: node-0 firings / blocks that waited for words */
+  int64_t  max_ingest_wait_ns;             /* live ingest: the longest such wait                        */
 } pl_stats;
 
 typedef struct pl_pipeline pl_pipeline;
@@ -265,6 +267,50 @@ typedef struct {
   uint64_t latency_outliers;       /* physical: items outside the 5 % latency band (pl_stats) */
 } pl_summary;
 pl_status pl_pipeline_summary(pl_pipeline* pl, pl_summary* out);
+
+/* ---- Live ingest (§2.1: "a stream of items, of unbounded length", arriving at
+ * rate rho0; SURVEY §8(b) push(stream, items, n); a1).  The DB is delivered WHILE one persistent
+ * run executes, through per-stream rings in device memory:
+ *   pl_pipeline_live_start(pl, R)   launches the run (on the bound stream) with a ring of R words
+ *                                   per stream (power of 2; 0 -> max(4 x the smem window, 64 K));
+ *   pl_pipeline_stream_words(pl,s)  the DB words stream s needs: [word_lo, word_hi) -- its roots
+ *                                   plus the k-1 overlap and a q_len halo on each side (the reach
+ *                                   of an extension walk, reading R-S3), 2-bit packed as in pl.h;
+ *   pl_pipeline_push_stream(pl, s, words, n, nonblocking)
+ *   pl_pipeline_push_all(pl, words[S], n[S], nonblocking)
+ *                                   append the next n words of stream s (of every stream), in
+ *                                   order; the library zero-pads each stream's last word;
+ *   pl_pipeline_drain(pl)           after the last words of every stream: waits for the run.
+ * Each push copies its words into a pinned host mirror of the ring (so `words` may be reused as
+ * soon as the call returns), enqueues their copy to the device ring on a handle-owned
+ * non-blocking copy stream, and then the stream's doorbell (its delivered-word count, in device
+ * memory) behind them in the same copy stream.  On the device, node 0 takes a root only once every word its descendants can
+ * read has been delivered, and the window slides by TMA from the ring as words arrive: the
+ * logical schedule stays the oracle's (root r arrives at r tau0 from the run's start, L63), and
+ * a late delivery appears as node-0 lateness, measured latency and pl_stats.ingest_waits.  Ring
+ * slots are reused once the device publishes (to mapped host memory) that no node reads below
+ * them: memory stays bounded however long the stream.  A push that finds its ring full blocks
+ * until room appears (PL_EAGAIN after 10 s without room), or with nonblocking != 0 returns
+ * PL_EAGAIN at once, having taken nothing.  Errors: PL_EINVAL (not DNA, arrival array given,
+ * n_streams above the resident-CTA count, bad ring size, a push past the stream's range),
+ * PL_ESTATE (push without a live run; launch / pl_pipeline_push during one; drain before every
+ * word was pushed), PL_ENOMEM, PL_EDEVICE.  A stream without delivery for 20 s proceeds on
+ * stale ring contents and sets error bit 16 (PL_EOVERFLOW at drain).                         */
+pl_status pl_pipeline_live_start(pl_pipeline* pl, uint32_t ring_words);
+pl_status pl_pipeline_stream_words(const pl_pipeline* pl, uint32_t stream, uint64_t* word_lo, uint64_t* word_hi);
+pl_status pl_pipeline_push_stream(pl_pipeline* pl, uint32_t stream, const uint32_t* words, uint64_t n,
+                                  int nonblocking);
+pl_status pl_pipeline_push_all(pl_pipeline* pl, const uint32_t* const* words, const uint64_t* n, int nonblocking);
+
+/* Fault injection for measurement (DESIGN.md R-STALL).  The B200 platform stops
+ * every SM for ~1.6 ms every few seconds (profiles/r02_pause_control.txt); with len_ns > 0 every
+ * node of every stream of later physical-clock runs stops at its next firing start inside the
+ * windows [T0 + j period_ns, T0 + j period_ns + len_ns), j >= 1, until the window ends -- the
+ * same event on demand, so that a rate search can require zero deadline misses across it.  The
+ * logical schedule (and so every parity output) is unchanged; only lateness and measured
+ * latencies move.  len_ns = 0 turns it off.  PL_EINVAL: len_ns < 0, period_ns <= len_ns, or a
+ * logical-clock pipeline.                                                                    */
+pl_status pl_pipeline_inject_stalls(pl_pipeline* pl, int64_t period_ns, int64_t len_ns);
 
 /* Enqueue one executor run over every item pushed so far on the bound stream and
  * return immediately (asynchronous).  Resets per-run outputs first.             */

@@ -79,7 +79,8 @@ class pl_stats(C.Structure):
                 ("hw_busy_fraction", C.c_double), ("wall_ns", C.c_int64), ("errors", C.c_uint32),
                 ("launches", C.c_uint32), ("h2d_bytes", C.c_uint64), ("d2h_bytes", C.c_uint64),
                 ("window_refills", C.c_uint64), ("latency_outliers", C.c_uint64),
-                ("latency_rel_err_max", C.c_double)]
+                ("latency_rel_err_max", C.c_double), ("ingest_waits", C.c_uint64),
+                ("max_ingest_wait_ns", C.c_int64)]
 
     def as_dict(self):
         N = self.n_stages
@@ -111,6 +112,11 @@ def _load():
         "pl_pipeline_queue_peaks": (C.c_int32, [P, P, C.c_uint64, C.POINTER(C.c_uint64)]),
         "pl_pipeline_bind_results": (C.c_int32, [P, P, C.c_uint64]),
         "pl_pipeline_launch": (C.c_int32, [P]),
+        "pl_pipeline_inject_stalls": (C.c_int32, [P, C.c_int64, C.c_int64]),
+        "pl_pipeline_live_start": (C.c_int32, [P, C.c_uint32]),
+        "pl_pipeline_stream_words": (C.c_int32, [P, C.c_uint32, C.POINTER(C.c_uint64), C.POINTER(C.c_uint64)]),
+        "pl_pipeline_push_stream": (C.c_int32, [P, C.c_uint32, P, C.c_uint64, C.c_int]),
+        "pl_pipeline_push_all": (C.c_int32, [P, P, P, C.c_int]),
         "pl_pipeline_drain": (C.c_int32, [P]),
         "pl_pipeline_rewind": (C.c_int32, [P]),
         "pl_pipeline_stats": (C.c_int32, [P, C.POINTER(pl_stats)]),
@@ -141,7 +147,9 @@ EXPORTED = ("pl_pipeline_create", "pl_pipeline_set_stream", "pl_pipeline_push", 
             "pl_pipeline_params", "pl_pipeline_destroy", "pl_last_error", "pl_solve_enforced_waits",
             "pl_solve_monolithic", "pl_version", "pl_stage_batch", "pl_pipeline_bind_host",
             "pl_pipeline_summary", "pl_pipeline_queue_peaks",
-            "pl_pipeline_step", "pl_pipeline_step_finish", "pl_pipeline_bind_results")
+            "pl_pipeline_step", "pl_pipeline_step_finish", "pl_pipeline_bind_results",
+            "pl_pipeline_inject_stalls", "pl_pipeline_live_start", "pl_pipeline_stream_words",
+            "pl_pipeline_push_stream", "pl_pipeline_push_all")
 
 
 class PlError(RuntimeError):

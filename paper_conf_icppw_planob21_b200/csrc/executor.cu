@@ -71,7 +71,9 @@ __device__ __forceinline__ uint64_t gain_hash(uint64_t seed, uint32_t stage, uin
 #endif
 
 struct Dna {
-  const uint32_t* db;      // packed DB (global)
+  const uint32_t* db;      // packed DB (global); live ingest: this stream's device ring (word w at db[w & dbmask])
+  uint32_t dbmask;         // ~0u, or the live ring's size - 1: then L2-only loads (__ldcg) -- the copy
+                           // engine rewrites the ring's slots and L1 is not coherent with it
   uint32_t nwords;
   uint64_t db_len;
   const uint32_t* win;     // smem ring of DB words: word w at win[w & win_mask], valid for [win_lo, win_lo + win_n)
@@ -89,7 +91,8 @@ struct Dna {
   __device__ __forceinline__ uint32_t dbw(int64_t w) const {
     const uint64_t r = (uint64_t)(w - win_lo);
     if (r < win_n) return win[(uint32_t)w & win_mask];
-    return (w >= 0 && w < (int64_t)nwords) ? __ldg(db + w) : 0u;
+    if (!(w >= 0 && w < (int64_t)nwords)) return 0u;
+    return dbmask == 0xffffffffu ? __ldg(db + w) : __ldcg(db + ((uint32_t)w & dbmask));
   }
   __device__ __forceinline__ uint32_t qww(int64_t w) const { return (w >= 0 && w < (int64_t)nqw) ? qw[w] : 0u; }
   // bases s..s+15 (base s in bits 0-1); s may be negative (out-of-range bases read as 0)
@@ -325,6 +328,14 @@ struct WinCtl {
   uint32_t inflight, phase; // a refill is in flight on mbar_w; its completion parity
   uint32_t loaded_hi;       // cov_hi once the in-flight refill has landed
   uint32_t refills;         // chunks loaded after the initial staging
+  uint32_t c_first;         // first chunk of the stream (chunks < c_first + K need no drop)
+  uint32_t a_next;          // next word to load (a chunk loads in pieces as live ingest delivers it)
+  uint32_t front;           // live: words [wlo, front) of the stream have been delivered (doorbell cache)
+  uint32_t pub;             // live: the last consumed watermark published to the host
+  uint32_t src_mask;        // source word index mask (~0u, or the live ring's size - 1)
+  const uint32_t* src;      // refill source: the DB, or this stream's live ring
+  const uint32_t* front_ptr;   // live: this stream's doorbell (device memory, written by the copy stream)
+  uint32_t* consumed_ptr;      // live: this stream's consumed watermark (mapped pinned host memory)
 };
 struct Shared {
   EdgeCtl e[PL_MAX_STAGES];
@@ -337,6 +348,8 @@ struct Shared {
   uint32_t agr_bad;         // physical: terminal items outside the 5 % band of their logical latency
   uint32_t agr_ppm;         // physical: largest |measured - logical| / logical latency (ppm)
   uint32_t errors;
+  uint32_t ingest_waits;    // live ingest: node-0 firings (or monolithic blocks) that waited for delivery
+  uint32_t ingest_max_ns;   // live ingest: the longest such wait
   uint32_t log_count;       // firing-log records reserved by all nodes of this stream
   uint64_t T0;
   alignas(8) uint64_t mbar; // TMA completion barrier for the initial staging
@@ -383,14 +396,37 @@ __device__ __forceinline__ void win_snap(Dna& dna, const Shared& sh) {
   dna.win_n = hi - lo;
 }
 
+__device__ __forceinline__ uint32_t ld_acquire_gpu(const uint32_t* a) {
+  uint32_t v;
+  asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(a) : "memory");
+  return v;
+}
+__device__ __forceinline__ void st_release_sys(uint32_t* a, uint32_t v) {
+  asm volatile("st.release.sys.global.u32 [%0], %1;" ::"l"(a), "r"(v) : "memory");
+}
+// Live ingest: the stream's delivered-word frontier, refreshed from its doorbell when `need`
+// lies beyond the cached value.  The copy stream writes the doorbell (cuStreamWriteValue32,
+// with its default system-scope fence) after the words' copy, so the acquire load orders every
+// later read of those words -- generic (__ldcg) and, after the proxy fence, TMA -- behind it.
+__device__ __forceinline__ uint32_t live_front(WinCtl& W, uint32_t need) {
+  uint32_t f = vld(&W.front);
+  if (f >= need) return f;
+  const uint32_t g = ld_acquire_gpu(W.front_ptr);
+  if (g > f) { atomicMax(&W.front, g); f = g; }
+  asm volatile("fence.proxy.async.global;" ::: "memory");
+  return f;
+}
+
 // One step of the sliding window, by its single owner thread: complete an in-flight refill
 // (publish cov_hi), then start the next one if the chunk it overwrites is no longer needed.
 // A root p reads DB words >= (p - q_len - 48) / 16 (extension walks reach q_len bases to the
 // left, plus whole 16-base steps), so chunk c may replace chunk c - K once every node's bound
 // is past that.  A reader's stale snapshot is harmless: it only reads words of its own roots,
 // which are >= min bnd and so never in a dropped chunk.  wait = block until the refill lands.
-// Returns whether it made progress.
-__device__ bool win_step(Shared& sh, const DevParams& p, unsigned char* ring, bool wait) {
+// Live ingest: a chunk loads in 16-byte-aligned pieces as its words are delivered, and the
+// consumed watermark min(floor, a_next) -- nothing below it is read or staged again -- goes to
+// the host, which may then overwrite those ring slots.  Returns whether it made progress.
+__device__ __noinline__ bool win_step(Shared& sh, const DevParams& p, unsigned char* ring, bool wait) {
   WinCtl& W = sh.win;
   const uint32_t bar = smem_addr(&sh.mbar_w);
   bool prog = false;
@@ -411,24 +447,42 @@ __device__ bool win_step(Shared& sh, const DevParams& p, unsigned char* ring, bo
   const uint32_t need = (uint32_t)p.q_len + 48u;
   const uint32_t floor_w = m > need ? (m - need) >> 4 : 0u;
   const uint32_t c = W.c_next, K = p.win_cap >> p.win_lg;
+  if (p.live) {
+    const uint32_t fl = min(floor_w, W.a_next);
+    if (fl >= W.pub + 64u) { W.pub = fl; st_release_sys(W.consumed_ptr, fl); }
+  }
+  const uint32_t b = min((c + 1u) << p.win_lg, W.whi);
+  const bool drop = W.a_next == max(c << p.win_lg, W.wlo) && c >= W.c_first + K;   // first piece of chunk c
   const uint32_t lo_new = (c - K + 1u) << p.win_lg;
-  if (floor_w < lo_new) return prog;       // chunk c - K is still needed
-  *(volatile uint32_t*)&W.cov_lo = lo_new;  // drop chunk c - K (readers only narrow their snapshots)
-  // the generic-proxy reads of the dropped chunk are ordered before the async-proxy refill
-  asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
-  const uint32_t a = max(c << p.win_lg, W.wlo), b = min((c + 1u) << p.win_lg, W.whi);
-  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(bar), "r"((b - a) * 4u) : "memory");
-  tma_load(smem_addr(ring + (a & (p.win_cap - 1u)) * 4u), p.db + a, (b - a) * 4u, bar);
+  if (drop && floor_w < lo_new) return prog;       // chunk c - K is still needed
+  uint32_t e = b;
+  if (p.live) {
+    e = min(b, live_front(W, b) & ~3u);            // TMA moves whole 16-byte units
+    if (e <= W.a_next) return prog;
+  }
+  if (drop) {
+    *(volatile uint32_t*)&W.cov_lo = lo_new;  // drop chunk c - K (readers only narrow their snapshots)
+    // the generic-proxy reads of the dropped chunk are ordered before the async-proxy refill
+    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+  }
+  const uint32_t a = W.a_next;
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(bar), "r"((e - a) * 4u) : "memory");
+  tma_load(smem_addr(ring + (a & (p.win_cap - 1u)) * 4u), W.src + (a & W.src_mask), (e - a) * 4u, bar);
   W.inflight = 1;
-  W.loaded_hi = b;
-  W.c_next = c + 1u;
-  W.refills++;
+  W.loaded_hi = e;
+  if (e == b) {
+    W.c_next = c + 1u;
+    W.a_next = (c + 1u) << p.win_lg;
+    W.refills++;
+  } else {
+    W.a_next = e;
+  }
   if (wait) {
     while (!mbar_test(bar, W.phase)) {}
     W.phase ^= 1u;
     W.inflight = 0;
     asm volatile("fence.acq_rel.cta;" ::: "memory");
-    *(volatile uint32_t*)&W.cov_hi = b;
+    *(volatile uint32_t*)&W.cov_hi = e;
   }
   return true;
 }
@@ -976,6 +1030,24 @@ __device__ __forceinline__ void pace(uint64_t target, uint64_t* start_ns, int64_
   *late = (int64_t)(now - target);
 }
 
+// Stall injection (pl_pipeline_inject_stalls; SURVEY §5 fault injection, DESIGN.md R-STALL): the
+// platform stops every SM for ~1.6 ms every few seconds (profiles/r02_pause_control.txt).  With
+// p.inj_len_ns > 0 a node reaching a firing start inside [T0 + j P, T0 + j P + len), j >= 1,
+// sleeps to the window's end -- every node of every stream stops over the same windows, as in
+// the platform's stalls, only more often -- so a rate search can demand zero misses across them.
+__device__ __noinline__ void inject_stall(const DevParams& p, uint64_t T0) {
+  const uint64_t now = gtimer();
+  const uint64_t j = (now - T0) / p.inj_period_ns;
+  if (j == 0) return;
+  const uint64_t we = T0 + j * p.inj_period_ns + p.inj_len_ns;
+  if (now < we) nap_until(we);
+}
+__device__ __forceinline__ void pace_p(const DevParams& p, uint64_t T0, uint64_t target, uint64_t* start_ns,
+                                       int64_t* late, uint64_t* entry_ns = nullptr) {
+  if (p.inj_len_ns) inject_stall(p, T0);
+  pace(target, start_ns, late, entry_ns);
+}
+
 // exclusive scan of per-lane output counts over the node's v lanes (warp shuffles
 // + one named barrier); returns the lane's offset and the group total.
 __device__ __forceinline__ uint32_t group_scan(uint32_t* wtot, uint32_t x, uint32_t* total, int gtid, int v, int bid,
@@ -1113,6 +1185,37 @@ __device__ __forceinline__ void record_lat_ns(const Node& nd, const Ctx& c, uint
   pend_root = NO_ROOT;
 }
 
+// Live ingest (pl_pipeline_live_start; a1): node 0 takes a root only once every
+// DB word that its descendants can read has been delivered -- up to word (p + k + halo) / 16,
+// the extension walks' reach (R-S3) -- so the logical schedule (arrivals a(r) = r tau0) is the
+// oracle's and a late delivery shows up as lateness and measured latency, not as a different
+// schedule.  Slow path only (the caller checks the cached frontier first); the accountant keeps
+// the window sliding while it waits.  A stream that gets no delivery for 20 s proceeds on
+// whatever its ring holds and flags PL_ERR_INGEST_TIMEOUT (the run must end).
+__device__ __noinline__ void live_gate_slow(Shared& sh, const DevParams& p, unsigned char* win, uint32_t need,
+                                            bool acct, bool leader) {
+  WinCtl& W = sh.win;
+  const uint64_t t0 = gtimer();
+  int spins = 0;
+  while (live_front(W, need) < need) {
+    if (acct) win_step(sh, p, win, false);
+    const uint64_t now = gtimer();
+    if (now - t0 > PL_INGEST_TIMEOUT_NS) {
+      atomicOr(&sh.errors, PL_ERR_INGEST_TIMEOUT);
+      atomicMax(&W.front, W.whi);
+      break;
+    }
+    if (++spins > 2) __nanosleep(spins < 16 ? 64 : 256);
+  }
+  if (leader) {
+    sh.ingest_waits++;
+    atomicMax(&sh.ingest_max_ns, (uint32_t)min(gtimer() - t0, (uint64_t)0xffffffffu));
+  }
+}
+__device__ __forceinline__ uint32_t live_need(const Shared& sh, const DevParams& p, uint32_t p_last) {
+  return min(sh.win.whi, (uint32_t)(((uint64_t)p_last + (uint32_t)p.k + p.win_halo) >> 4) + 1u);
+}
+
 // ------------------------------------------------------------------- node loop
 // One warp group of v threads per node, one item per lane.  Measured faster on B200 than
 // one warp with v/32 items per lane: the group's warps run the per-item latency chains in
@@ -1171,6 +1274,12 @@ __device__ void run_node(Ctx& c, Dna dna, int i, int gtid) {
       const Decision d = decide0(nd, R);
       if (d.done) break;
       T = d.T; n = d.n; head = (uint32_t)R.c0;
+      if (p.live && n) {                 // live ingest: the firing's DB words must have been delivered
+        const uint32_t last = (uint32_t)min((int64_t)head + n, nd.X) - 1u;
+        const uint32_t need = live_need(*c.sh, p, (uint32_t)(nd.lo + last));
+        if (vld(&c.sh->win.front) < need)
+          live_gate_slow(*c.sh, p, (unsigned char*)dna.win, need, v > 32 ? gtid == 32 : leader, leader);
+      }
       if (leader) {
         uint32_t ql = d.qlen;
         if (nd.arr) {                    // arrival data: roots arrived by T (binary search), not yet consumed
@@ -1195,7 +1304,7 @@ __device__ void run_node(Ctx& c, Dna dna, int i, int gtid) {
           int64_t late;
           uint64_t entry;
           const uint64_t prev = start_ns;
-          pace(T0 + units_ns(nd, T), &start_ns, &late, &entry);
+          pace_p(p, T0, T0 + units_ns(nd, T), &start_ns, &late, &entry);
           atomicMax(&A.lateness, clamp32(late));
           if (prev) atomicMax(&A.max_loop, clamp32((int64_t)(entry - prev)));
         }
@@ -1203,7 +1312,7 @@ __device__ void run_node(Ctx& c, Dna dna, int i, int gtid) {
         if (leader) tc = clock64();
       } else if (nd.phys && (gtid & 31) == 0) {   // every warp paces itself against %globaltimer
         uint64_t s_ns, entry; int64_t late;
-        pace(T0 + units_ns(nd, T), &s_ns, &late, &entry);
+        pace_p(p, T0, T0 + units_ns(nd, T), &s_ns, &late, &entry);
         if (leader) {
           if (start_ns) atomicMax(&A.max_loop, clamp32((int64_t)(entry - start_ns)));
           start_ns = s_ns; atomicMax(&A.lateness, clamp32(late)); tc = clock64();
@@ -1238,7 +1347,7 @@ __device__ void run_node(Ctx& c, Dna dna, int i, int gtid) {
           int64_t late;
           uint64_t entry;
           const uint64_t prev = start_ns;
-          pace(T0 + units_ns(nd, d.T), &start_ns, &late, &entry);
+          pace_p(p, T0, T0 + units_ns(nd, d.T), &start_ns, &late, &entry);
           atomicMax(&A.lateness, clamp32(late));
           if (prev && !waited) atomicMax(&A.max_loop, clamp32((int64_t)(entry - prev)));
           tc = clock64();
@@ -1620,7 +1729,8 @@ __device__ void cta_setup(Ctx& c, Shared& sh, unsigned char* dsm, const DevParam
   c.X = (int64_t)(c.hi - c.lo);
   c.H = c.X * p.tau;
   c.dsm = dsm;
-  c.dna.db = p.db;
+  c.dna.db = p.live ? p.ring + (size_t)s * (p.ring_mask + 1u) : p.db;
+  c.dna.dbmask = p.live ? p.ring_mask : 0xffffffffu;
   c.dna.nwords = p.db_words;
   c.dna.db_len = p.db_len;
   c.dna.k = p.k;
@@ -1667,10 +1777,11 @@ __device__ void cta_setup(Ctx& c, Shared& sh, unsigned char* dsm, const DevParam
     const uint32_t lg = p.win_lg, K = p.win_cap >> lg;
     const uint32_t c0 = (uint32_t)wlo >> lg;
     const uint32_t c_end = whi > wlo ? (uint32_t)((whi - 1) >> lg) + 1u : c0;
-    // without TMA (unaligned DB) the window holds the first K chunks and never slides
-    const uint32_t c_init = min(c_end, c0 + K);
-    const uint32_t hi0 = whi > wlo ? min((uint32_t)whi, c_init << lg) : (uint32_t)wlo;
-    c.sliding = p.db_tma && c_end > c_init;
+    // without TMA (unaligned DB) the window holds the first K chunks and never slides; live
+    // ingest stages nothing up front -- win_step loads every chunk as it is delivered
+    const uint32_t c_init = p.live ? c0 : min(c_end, c0 + K);
+    const uint32_t hi0 = whi > wlo ? max((uint32_t)wlo, min((uint32_t)whi, c_init << lg)) : (uint32_t)wlo;
+    c.sliding = p.db_tma && (c_end > c_init || p.live);
     c.dna.win_lo = wlo;
     c.dna.win_lo32 = (uint32_t)wlo;
     c.dna.win_n = hi0 - (uint32_t)wlo;
@@ -1688,6 +1799,14 @@ __device__ void cta_setup(Ctx& c, Shared& sh, unsigned char* dsm, const DevParam
       W.phase = 0;
       W.loaded_hi = hi0;
       W.refills = 0;
+      W.c_first = c0;
+      W.a_next = max(c_init << lg, (uint32_t)wlo);
+      W.front = (uint32_t)wlo;
+      W.pub = (uint32_t)wlo;
+      W.src = c.dna.db;
+      W.src_mask = c.dna.dbmask;
+      W.front_ptr = p.live ? p.front + s : nullptr;
+      W.consumed_ptr = p.live ? p.consumed + s : nullptr;
       const uint32_t bar = smem_addr(&sh.mbar);
       const uint32_t bytes = b_qo + b_qp + b_qw + (win_tma ? c.dna.win_n * 4u : 0u);
       asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(bar));
@@ -1725,7 +1844,7 @@ __device__ void cta_setup(Ctx& c, Shared& sh, unsigned char* dsm, const DevParam
   }
   if (tid == 0) {
     sh.max_lat = 0; sh.max_lat_ns = 0; sh.miss_events = 0; sh.miss_events_ns = 0; sh.errors = 0; sh.log_count = 0;
-    sh.agr_bad = 0; sh.agr_ppm = 0;
+    sh.agr_bad = 0; sh.agr_ppm = 0; sh.ingest_waits = 0; sh.ingest_max_ns = 0;
   }
   // per-root records of this stream
   if (p.flags & PL_REC_LATENCY)
@@ -1753,6 +1872,8 @@ __device__ void cta_finish(Ctx& c, Shared& sh, const DevParams& p) {
     S.win_refills = p.k > 0 ? sh.win.refills : 0u;
     S.agr_bad = sh.agr_bad;
     S.agr_ppm = sh.agr_ppm;
+    S.ingest_waits = sh.ingest_waits;
+    S.ingest_max_ns = sh.ingest_max_ns;
     if (p.summary) {                     // device-side reduction for pl_pipeline_summary
       atomicAdd(p.summary + 0, (unsigned long long)c.X);
       atomicAdd(p.summary + 1, (unsigned long long)sh.miss_events);
@@ -1815,6 +1936,8 @@ __device__ void run_monolithic(Ctx& c) {
       if (tid == 0) {
         vst(&c.sh->bnd[0], (uint32_t)(c.lo + b0));
         const uint32_t need_hi = min(c.sh->win.whi, (uint32_t)(((c.lo + b1 + p.k + p.win_halo) >> 4) + 1));
+        if (p.live && vld(&c.sh->win.front) < need_hi)   // live ingest: the block's words must be delivered
+          live_gate_slow(*c.sh, p, (unsigned char*)c.dna.win, need_hi, true, true);
         while (vld(&c.sh->win.cov_hi) < need_hi && win_step(*c.sh, p, (unsigned char*)c.dna.win, true)) {}
       }
       __syncthreads();
@@ -1825,7 +1948,7 @@ __device__ void run_monolithic(Ctx& c) {
     if (phys) {
       if (tid == 0) {
         uint64_t s_ns; int64_t late;
-        pace(c.sh->T0 + (uint64_t)((double)ready * p.ns_per_unit), &s_ns, &late);   // the block is complete in real time
+        pace_p(p, c.sh->T0, c.sh->T0 + (uint64_t)((double)ready * p.ns_per_unit), &s_ns, &late);   // the block is complete in real time
         sh_start_ns = s_ns;
       }
       __syncthreads();

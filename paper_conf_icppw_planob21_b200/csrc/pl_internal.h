@@ -14,6 +14,8 @@
 #define PL_ERR_MATCH_OVERFLOW   2u
 #define PL_ERR_LOG_OVERFLOW     4u
 #define PL_ERR_SEG_OVERFLOW     8u
+#define PL_ERR_INGEST_TIMEOUT  16u      // live ingest: no delivery for PL_INGEST_TIMEOUT_NS (proceeds on stale data)
+#define PL_INGEST_TIMEOUT_NS   20000000000ull
 
 struct DevStage {
   uint32_t kind, max_out;
@@ -62,6 +64,8 @@ struct CtaStats {
   uint32_t win_refills;                 // DB-window chunks loaded after the initial staging
   uint32_t agr_bad;                     // physical: terminal items outside the 5 % latency band (R-AGREE)
   uint32_t agr_ppm;                     // physical: largest relative latency error (ppm)
+  uint32_t ingest_waits;                // live ingest: node-0 firings / blocks that waited for delivery
+  uint32_t ingest_max_ns;               // live ingest: the longest such wait
   uint32_t pad_;
 };
 
@@ -117,6 +121,13 @@ struct DevParams {
   unsigned long long* summary_next;     // the other slot of the double buffer: zeroed by this launch
                                         // (stream order: the previous launch that used it is done)
   const int64_t* arr;                   // per-root arrival times (NULL: r * tau0)
+  uint64_t inj_period_ns, inj_len_ns;   // stall injection (pl_pipeline_inject_stalls; 0 = off)
+  // live ingest (pl_pipeline_live_start): the DB is delivered while the run executes
+  uint32_t live;                        // 1: stream s reads DB word w from ring[s R + (w & ring_mask)]
+  uint32_t ring_mask;                   // R - 1 (R = ring words per stream, a power of 2)
+  const uint32_t* ring;                 // [n_streams][R] device rings, filled by the copy stream
+  const uint32_t* front;                // [n_streams] doorbells: stream s holds words [wlo_s, front[s])
+  uint32_t* consumed;                   // [n_streams] mapped host: slots below consumed[s] may be reused
   DevStage st[PL_MAX_STAGES];
 };
 

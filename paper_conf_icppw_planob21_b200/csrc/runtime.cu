@@ -8,6 +8,8 @@
 #include <cuda_runtime.h>
 
 #include <algorithm>
+#include <chrono>
+#include <thread>
 #include <cmath>
 #include <cstdarg>
 #include <cstdio>
@@ -137,6 +139,19 @@ struct pl_pipeline {
   cudaEvent_t step_ev[2] = {nullptr, nullptr};
   uint32_t step_launch[2] = {0, 0};          // launch index of the run in each buffer
   uint64_t steps = 0;                        // pl_pipeline_step calls since the last finish
+  // live ingest (pl_pipeline_live_start / push_stream / push_all)
+  bool live = false;                         // a live run is executing: pushes go to its rings
+  uint32_t ring_words = 0;                   // R: ring words per stream
+  uint32_t* d_ring = nullptr;                // [S][R] device rings
+  uint32_t* d_front = nullptr;               // [S] doorbells (device)
+  uint32_t* h_consumed = nullptr;            // [S] consumed watermarks (mapped pinned; written by the device)
+  uint32_t* h_stage = nullptr;               // [S][R] pinned mirror of the rings (the copies' sources)
+  uint32_t* h_bell = nullptr;                // [kBells][S] pinned doorbell slots
+  cudaEvent_t bell_ev[16] = {};              // slot j's copy completed
+  uint64_t bell_next = 0;
+  cudaStream_t copy_stream = nullptr;        // non-blocking: copies run beside the executor
+  std::vector<uint32_t> lw_lo, lw_end, lw_hi, lw_front;   // per stream: words [lo, end) pushed by the
+                                             // caller, zero-padded to hi; front = next word to deliver
 };
 
 namespace {
@@ -148,6 +163,14 @@ void free_all(pl_pipeline* pl) {
   for (void* p : ptrs)
     if (p) cudaFree(p);
   if (pl->h_step) cudaFreeHost(pl->h_step);
+  if (pl->d_ring) cudaFree(pl->d_ring);
+  if (pl->d_front) cudaFree(pl->d_front);
+  if (pl->h_consumed) cudaFreeHost(pl->h_consumed);
+  if (pl->h_stage) cudaFreeHost(pl->h_stage);
+  if (pl->h_bell) cudaFreeHost(pl->h_bell);
+  for (cudaEvent_t& e : pl->bell_ev)
+    if (e) cudaEventDestroy(e);
+  if (pl->copy_stream) cudaStreamDestroy(pl->copy_stream);
   for (cudaEvent_t& e : pl->step_ev)
     if (e) cudaEventDestroy(e);
 }
@@ -551,6 +574,7 @@ pl_status pl_pipeline_set_stream(pl_pipeline* pl, void* stream) {
 
 pl_status pl_pipeline_push(pl_pipeline* pl, const void* items, uint64_t n) {
   if (!pl) return fail(PL_EINVAL, "NULL pipeline");
+  if (pl->live) return fail(PL_ESTATE, "a live run is executing: use pl_pipeline_push_stream / push_all");
   if (pl->drained) return fail(PL_ESTATE, "push after drain; call pl_pipeline_rewind");
   if (pl->dna) {
     if (!items) return fail(PL_EINVAL, "DNA push needs items");
@@ -709,8 +733,237 @@ pl_status pl_pipeline_step_finish(pl_pipeline* pl, pl_summary* last, int* has_la
   return PL_OK;
 }
 
+
+// ------------------------------------------------------------------ live ingest
+namespace {
+constexpr uint32_t kBells = 16;
+// Stream s's DB word range [wlo, whi): its roots plus the k-1 overlap and the extension halo on
+// both sides, 16-byte aligned -- the same computation as the executor's cta_setup.
+void stream_words_range(const pl_pipeline* pl, uint32_t s, uint32_t* lo_out, uint32_t* hi_out) {
+  const DevParams& p = pl->dp;
+  const uint64_t total = pl->db_len >= (uint64_t)pl->k ? pl->db_len - pl->k + 1 : 0;
+  const uint64_t S = pl->cfg.n_streams;
+  const uint64_t lo = (total * s) / S, hi = (total * (s + 1)) / S;
+  int64_t wlo = 0, whi = 0;
+  if (p.win_cap > 0 && hi > lo) {
+    wlo = ((int64_t)lo - (int64_t)p.win_halo) >> 4;
+    whi = (((int64_t)hi + p.k + (int64_t)p.win_halo) >> 4) + 1;
+    wlo = wlo < 0 ? 0 : (wlo & ~3ll);
+    whi = (whi + 3) & ~3ll;
+    if (whi > (int64_t)pl->db_alloc_words) whi = (int64_t)pl->db_alloc_words & ~3ll;
+    if (whi < wlo) whi = wlo;
+  }
+  *lo_out = (uint32_t)wlo;
+  *hi_out = (uint32_t)whi;
+}
+
+// Stage words of stream s into its pinned host mirror (slot = word & (R-1), as on the device)
+// and enqueue the copy of that slot range to the device ring.  The mirror's slots are reused on
+// the same condition as the ring's (the device consumed them), which implies the copy was done.
+cudaError_t stage_copy(pl_pipeline* pl, uint32_t s, uint32_t f, const uint32_t* words, uint32_t n) {
+  const uint32_t R = pl->ring_words;
+  uint32_t* h = pl->h_stage + (size_t)s * R + (f & (R - 1));
+  if (words) std::memcpy(h, words, (size_t)n * 4);
+  else std::memset(h, 0, (size_t)n * 4);
+  return cudaMemcpyAsync(pl->d_ring + (size_t)s * R + (f & (R - 1)), h, (size_t)n * 4, cudaMemcpyHostToDevice,
+                         pl->copy_stream);
+}
+
+// Ring the doorbells of streams [s0, s0 + count) behind every copy enqueued so far: their fronts
+// go through a pinned slot (one of kBells, reused once its copy has completed) to d_front.
+cudaError_t ring_bells(pl_pipeline* pl, uint32_t s0, uint32_t count) {
+  const uint32_t S = pl->cfg.n_streams;
+  const uint32_t j = (uint32_t)(pl->bell_next++ % kBells);
+  cudaError_t e = cudaEventSynchronize(pl->bell_ev[j]);
+  if (e != cudaSuccess) return e;
+  uint32_t* slot = pl->h_bell + (size_t)j * S;
+  std::memcpy(slot + s0, pl->lw_front.data() + s0, (size_t)count * 4);
+  e = cudaMemcpyAsync(pl->d_front + s0, slot + s0, (size_t)count * 4, cudaMemcpyHostToDevice, pl->copy_stream);
+  if (e != cudaSuccess) return e;
+  return cudaEventRecord(pl->bell_ev[j], pl->copy_stream);
+}
+
+// Enqueue up to n words of stream s (as many as its ring has room for); *full = the ring had
+// no room for the rest.
+pl_status push_some(pl_pipeline* pl, uint32_t s, const uint32_t*& words, uint64_t& n, bool* full) {
+  const uint32_t R = pl->ring_words;
+  uint32_t& f = pl->lw_front[s];
+  *full = false;
+  auto room = [&]() {
+    const uint32_t cons = std::max<uint32_t>(pl->lw_lo[s], (uint32_t)*(volatile uint32_t*)(pl->h_consumed + s));
+    return (uint64_t)R - (uint64_t)(f - std::min(f, cons));
+  };
+  while (n > 0) {
+    const uint64_t space = room();
+    if (space == 0) { *full = true; break; }
+    const uint32_t piece = (uint32_t)std::min<uint64_t>(std::min<uint64_t>(n, space), R - (f & (R - 1)));
+    CUDA_TRY(stage_copy(pl, s, f, words, piece));
+    f += piece;
+    words += piece;
+    n -= piece;
+    pl->h2d += (uint64_t)piece * 4;
+  }
+  if (n == 0 && f == pl->lw_end[s] && f < pl->lw_hi[s]) {   // the stream's last words: zero-pad to hi
+    const uint32_t pad = pl->lw_hi[s] - f;                    // (<= 11 words past the DB's end)
+    if (room() < pad) { *full = true; return PL_OK; }
+    const uint32_t first = std::min(pad, R - (f & (R - 1)));
+    CUDA_TRY(stage_copy(pl, s, f, nullptr, first));
+    if (pad > first) CUDA_TRY(stage_copy(pl, s, f + first, nullptr, pad - first));
+    f += pad;
+  }
+  return PL_OK;
+}
+
+pl_status push_streams(pl_pipeline* pl, uint32_t s0, uint32_t count, const uint32_t* const* words,
+                       const uint64_t* n, int nonblocking) {
+  if (!pl) return fail(PL_EINVAL, "NULL pipeline");
+  if (!pl->live) return fail(PL_ESTATE, "no live run (pl_pipeline_live_start)");
+  if (!words || !n) return fail(PL_EINVAL, "NULL argument");
+  const uint32_t R = pl->ring_words;
+  for (uint32_t j = 0; j < count; ++j) {
+    const uint32_t s = s0 + j;
+    if (n[j] && !words[j]) return fail(PL_EINVAL, "stream %u: NULL words", s);
+    if (n[j] && (uint64_t)pl->lw_front[s] + n[j] > pl->lw_end[s])
+      return fail(PL_EINVAL, "stream %u: push of %llu words exceeds its range (%u left)", s,
+                  (unsigned long long)n[j], pl->lw_end[s] - std::min(pl->lw_end[s], pl->lw_front[s]));
+    if (nonblocking) {
+      const uint32_t cons = std::max<uint32_t>(pl->lw_lo[s], (uint32_t)*(volatile uint32_t*)(pl->h_consumed + s));
+      const uint64_t used = pl->lw_front[s] - std::min(pl->lw_front[s], cons);
+      if (used + n[j] + 16 > R) return fail(PL_EAGAIN, "stream %u: ring full (%llu of %u words in use)", s,
+                                            (unsigned long long)used, R);
+    }
+  }
+  cudaSetDevice(pl->device);
+  std::vector<const uint32_t*> w(words, words + count);
+  std::vector<uint64_t> left(n, n + count);
+  const auto t_start = std::chrono::steady_clock::now();
+  for (;;) {
+    bool any_full = false, progress = false;
+    for (uint32_t j = 0; j < count; ++j) {
+      const uint32_t s = s0 + j;
+      const uint32_t f0 = pl->lw_front[s];
+      bool full = false;
+      pl_status st = push_some(pl, s, w[j], left[j], &full);
+      if (st != PL_OK) return st;
+      any_full |= full;
+      progress |= pl->lw_front[s] != f0;
+    }
+    if (progress) CUDA_TRY(ring_bells(pl, s0, count));   // behind the data, in copy-stream order
+    if (!any_full) break;
+    if (std::chrono::steady_clock::now() - t_start > std::chrono::seconds(10))
+      return fail(PL_EAGAIN, "live ring full for 10 s: the executor is not consuming");
+    std::this_thread::yield();
+  }
+  return PL_OK;
+}
+}  // namespace
+
+pl_status pl_pipeline_live_start(pl_pipeline* pl, uint32_t ring_words) {
+  if (!pl) return fail(PL_EINVAL, "NULL pipeline");
+  if (!pl->dna) return fail(PL_EINVAL, "live ingest is for DNA pipelines (items are DB words)");
+  if (pl->live) return fail(PL_ESTATE, "a live run is already executing");
+  if (pl->d_arr) return fail(PL_EINVAL, "live ingest takes arrivals at r * tau0 (no arrival array)");
+  cudaSetDevice(pl->device);
+  const uint32_t S = pl->cfg.n_streams;
+  int sms = 0;
+  CUDA_TRY(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, pl->device));
+  const int per_sm = pl->dp.ctas_per_sm > 1 ? pl->dp.ctas_per_sm : 1;
+  if ((int64_t)S > (int64_t)sms * per_sm)
+    return fail(PL_EINVAL, "live ingest needs every stream resident at once (n_streams %u > %d)", S, sms * per_sm);
+  const uint32_t CH = 1u << pl->dp.win_lg;
+  uint32_t R = ring_words ? ring_words : std::max<uint32_t>(4 * pl->dp.win_cap, 1u << 16);
+  if (!is_pow2(R) || R < 2 * pl->dp.win_cap || R < CH)
+    return fail(PL_EINVAL, "ring_words must be a power of 2 >= 2 x the smem window (%u words)", pl->dp.win_cap);
+  if (R != pl->ring_words) {
+    if (pl->d_ring) cudaFree(pl->d_ring);
+    if (pl->h_stage) cudaFreeHost(pl->h_stage);
+    pl->d_ring = nullptr;
+    pl->h_stage = nullptr;
+    pl->ring_words = 0;
+    if (cudaMalloc(&pl->d_ring, (size_t)S * R * 4) != cudaSuccess) return fail(PL_ENOMEM, "live rings (%u x %u words)", S, R);
+    if (cudaHostAlloc((void**)&pl->h_stage, (size_t)S * R * 4, cudaHostAllocDefault) != cudaSuccess)
+      return fail(PL_ENOMEM, "live ring mirror (pinned, %u x %u words)", S, R);
+    pl->ring_words = R;
+  }
+  if (!pl->h_bell) {
+    if (cudaHostAlloc((void**)&pl->h_bell, (size_t)kBells * S * 4, cudaHostAllocDefault) != cudaSuccess)
+      return fail(PL_ENOMEM, "doorbell slots (pinned)");
+    for (uint32_t j = 0; j < kBells; ++j) CUDA_TRY(cudaEventCreateWithFlags(&pl->bell_ev[j], cudaEventDisableTiming));
+  }
+  if (!pl->d_front && cudaMalloc(&pl->d_front, (size_t)S * 4) != cudaSuccess) return fail(PL_ENOMEM, "doorbells");
+  if (!pl->h_consumed && cudaHostAlloc((void**)&pl->h_consumed, (size_t)S * 4, cudaHostAllocMapped) != cudaSuccess)
+    return fail(PL_ENOMEM, "consumed watermarks (pinned)");
+  if (!pl->copy_stream) CUDA_TRY(cudaStreamCreateWithFlags(&pl->copy_stream, cudaStreamNonBlocking));
+  uint32_t* d_cons = nullptr;
+  CUDA_TRY(cudaHostGetDevicePointer((void**)&d_cons, pl->h_consumed, 0));
+  pl->lw_lo.resize(S);
+  pl->lw_end.resize(S);
+  pl->lw_hi.resize(S);
+  pl->lw_front.resize(S);
+  const uint32_t db_words = (uint32_t)((pl->db_len + 15) / 16);
+  for (uint32_t s = 0; s < S; ++s) {
+    stream_words_range(pl, s, &pl->lw_lo[s], &pl->lw_hi[s]);
+    pl->lw_end[s] = std::max(pl->lw_lo[s], std::min(pl->lw_hi[s], db_words));
+    pl->lw_front[s] = pl->lw_lo[s];
+    pl->h_consumed[s] = pl->lw_lo[s];
+  }
+  // make sure no earlier copy on the copy stream is still in flight, then reset the doorbells
+  CUDA_TRY(cudaStreamSynchronize(pl->copy_stream));
+  CUDA_TRY(cudaMemcpy(pl->d_front, pl->lw_front.data(), (size_t)S * 4, cudaMemcpyHostToDevice));
+  DevParams& d = pl->dp;
+  pl->d_db_bound = nullptr;
+  pl->bound_host = false;
+  pl->pushed = pl->db_len;             // the run covers the whole stream; its words arrive by push
+  d.live = 1;
+  d.ring = pl->d_ring;
+  d.ring_mask = R - 1;
+  d.front = pl->d_front;
+  d.consumed = d_cons;
+  pl_status st = pl_pipeline_launch(pl);
+  d.live = 0;                          // later non-live launches (the kernel took its own copy)
+  if (st != PL_OK) return st;
+  pl->live = true;
+  pl->drained = false;
+  return PL_OK;
+}
+
+pl_status pl_pipeline_stream_words(const pl_pipeline* pl, uint32_t stream, uint64_t* word_lo, uint64_t* word_hi) {
+  if (!pl || !word_lo || !word_hi) return fail(PL_EINVAL, "NULL argument");
+  if (!pl->dna) return fail(PL_EINVAL, "stream words exist for DNA pipelines only");
+  if (stream >= pl->cfg.n_streams) return fail(PL_EINVAL, "stream %u >= n_streams %u", stream, pl->cfg.n_streams);
+  uint32_t lo, hi;
+  stream_words_range(pl, stream, &lo, &hi);
+  const uint32_t db_words = (uint32_t)((pl->db_len + 15) / 16);
+  *word_lo = lo;
+  *word_hi = std::max(lo, std::min(hi, db_words));
+  return PL_OK;
+}
+
+pl_status pl_pipeline_push_stream(pl_pipeline* pl, uint32_t stream, const uint32_t* words, uint64_t n,
+                                  int nonblocking) {
+  if (!pl) return fail(PL_EINVAL, "NULL pipeline");
+  if (stream >= pl->cfg.n_streams) return fail(PL_EINVAL, "stream %u >= n_streams %u", stream, pl->cfg.n_streams);
+  return push_streams(pl, stream, 1, &words, &n, nonblocking);
+}
+
+pl_status pl_pipeline_push_all(pl_pipeline* pl, const uint32_t* const* words, const uint64_t* n, int nonblocking) {
+  if (!pl) return fail(PL_EINVAL, "NULL pipeline");
+  return push_streams(pl, 0, pl->cfg.n_streams, words, n, nonblocking);
+}
+
+pl_status pl_pipeline_inject_stalls(pl_pipeline* pl, int64_t period_ns, int64_t len_ns) {
+  if (!pl) return fail(PL_EINVAL, "NULL pipeline");
+  if (len_ns < 0 || (len_ns > 0 && period_ns <= len_ns))
+    return fail(PL_EINVAL, "stall injection needs 0 <= len_ns < period_ns");
+  if (len_ns > 0 && pl->cfg.clock != PL_CLOCK_GLOBALTIMER) return fail(PL_EINVAL, "stall injection needs the physical clock");
+  pl->dp.inj_period_ns = len_ns > 0 ? (uint64_t)period_ns : 1u;
+  pl->dp.inj_len_ns = (uint64_t)len_ns;
+  return PL_OK;
+}
+
 pl_status pl_pipeline_launch(pl_pipeline* pl) {
   if (!pl) return fail(PL_EINVAL, "NULL pipeline");
+  if (pl->live) return fail(PL_ESTATE, "a live run is executing; pl_pipeline_drain ends it");
   cudaSetDevice(pl->device);
   DevParams& d = pl->dp;
   if (pl->dna) {
@@ -740,11 +993,17 @@ pl_status pl_pipeline_launch(pl_pipeline* pl) {
 
 pl_status pl_pipeline_drain(pl_pipeline* pl) {
   if (!pl) return fail(PL_EINVAL, "NULL pipeline");
-  if (!pl->launched) {     // nothing launched since create / rewind: run the pushed stream now
+  if (pl->live) {          // a live run ends once every stream's words were pushed
+    for (uint32_t s = 0; s < pl->cfg.n_streams; ++s)
+      if (pl->lw_front[s] < pl->lw_hi[s])
+        return fail(PL_ESTATE, "live run: stream %u has %u of its %u words; push them all before drain", s,
+                    pl->lw_front[s] - pl->lw_lo[s], pl->lw_hi[s] - pl->lw_lo[s]);
+  } else if (!pl->launched) {     // nothing launched since create / rewind: run the pushed stream now
     pl_status s = pl_pipeline_launch(pl);
     if (s != PL_OK) return s;
   }
   CUDA_TRY(cudaStreamSynchronize(pl->stream));
+  pl->live = false;
   pl->drained = true;
   std::vector<CtaStats> cs(pl->cfg.n_streams);
   CUDA_TRY(cudaMemcpy(cs.data(), pl->d_stats, cs.size() * sizeof(CtaStats), cudaMemcpyDeviceToHost));
@@ -806,6 +1065,8 @@ pl_status pl_pipeline_stats(pl_pipeline* pl, pl_stats* out) {
     out->window_refills += s.win_refills;
     out->latency_outliers += s.agr_bad;
     out->latency_rel_err_max = std::max(out->latency_rel_err_max, (double)s.agr_ppm * 1e-6);
+    out->ingest_waits += s.ingest_waits;
+    out->max_ingest_wait_ns = std::max<int64_t>(out->max_ingest_wait_ns, s.ingest_max_ns);
   }
   unsigned long long mc = 0;
   CUDA_TRY(cudaMemcpy(&mc, pl->d_match_count, 8, cudaMemcpyDeviceToHost));

@@ -133,6 +133,36 @@ class Pipeline:
         check(lib.pl_pipeline_summary(self.h, C.byref(s)), "pl_pipeline_summary")
         return {k: getattr(s, k) for k, _ in s._fields_}
 
+    # -- live ingest (pl_pipeline_live_start / stream_words / push_stream / push_all)
+    def live_start(self, ring_words=0):
+        """Launch a persistent run whose DB words arrive by push_stream / push_all while it runs."""
+        check(lib.pl_pipeline_live_start(self.h, int(ring_words)), "pl_pipeline_live_start")
+
+    def stream_words(self, s):
+        """[word_lo, word_hi) of the packed DB that stream s must be pushed."""
+        lo, hi = C.c_uint64(), C.c_uint64()
+        check(lib.pl_pipeline_stream_words(self.h, int(s), C.byref(lo), C.byref(hi)), "pl_pipeline_stream_words")
+        return lo.value, hi.value
+
+    def push_stream(self, s, words, nonblocking=False):
+        """Append the next words (uint32 array) of stream s; raises PlError(PL_EAGAIN) if the
+        ring is full and nonblocking."""
+        a = np.ascontiguousarray(words, dtype=np.uint32)
+        check(lib.pl_pipeline_push_stream(self.h, int(s), a.ctypes.data, a.shape[0], int(bool(nonblocking))),
+              "pl_pipeline_push_stream")
+
+    def push_all(self, slices, nonblocking=False):
+        """Append slices[s] (uint32 arrays, possibly empty) to every stream s in one call."""
+        arrs = [np.ascontiguousarray(x, dtype=np.uint32) for x in slices]
+        ptrs = (C.c_void_p * len(arrs))(*[a.ctypes.data if a.size else None for a in arrs])
+        ns = (C.c_uint64 * len(arrs))(*[a.shape[0] for a in arrs])
+        check(lib.pl_pipeline_push_all(self.h, ptrs, ns, int(bool(nonblocking))), "pl_pipeline_push_all")
+
+    def inject_stalls(self, period_ns, len_ns):
+        """pl_pipeline_inject_stalls: every node stops over [T0 + j period, T0 + j period + len)
+        of later physical runs (the platform's ~1.6 ms SM stalls, on demand); len_ns=0: off."""
+        check(lib.pl_pipeline_inject_stalls(self.h, int(period_ns), int(len_ns)), "pl_pipeline_inject_stalls")
+
     def launch(self):
         check(lib.pl_pipeline_launch(self.h), "pl_pipeline_launch")
 

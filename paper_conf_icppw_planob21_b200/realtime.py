@@ -16,9 +16,11 @@ from .pipeline import Pipeline, solve_enforced_waits, solve_monolithic
 PHYS = 1  # PL_CLOCK_GLOBALTIMER
 
 
-def _run(cfg, db_dev, n_bases, wl, flags=0, stream=None, over=None):
+def _run(cfg, db_dev, n_bases, wl, flags=0, stream=None, over=None, inject=None):
     pl = Pipeline(cfg, wl, flags=flags, stream=stream, **(over or {}))
     pl.bind_device(db_dev, n_bases)
+    if inject:   # (period_ns, len_ns): pl_pipeline_inject_stalls
+        pl.inject_stalls(*inject)
     pl.drain()
     st = pl.stats()
     pl.close()
@@ -133,7 +135,7 @@ def stalled(st) -> bool:
 
 def find_rate(cfg, wl, db_dev, tries=12, grow=1.15, stream=None, log=None, over=None, policy=0,
               max_lateness_ns=5000, flags=0, solve_deadline=None, max_outliers=None, start=None,
-              stall_retries=2):
+              stall_retries=2, inject=None):
     """Smallest tau0 (ns) at which a physical run (FIXED_WAIT, or THRESHOLD_SLACK with the
     Fig. 1-derived thresholds when policy=1) has zero deadline misses, no queue overflow
     and, unless max_lateness_ns is None, every firing starting within max_lateness_ns of its
@@ -148,7 +150,11 @@ def find_rate(cfg, wl, db_dev, tries=12, grow=1.15, stream=None, log=None, over=
     platform-stall allowance is kept out of it, DESIGN.md R-STALL), while misses count against
     cfg's D.  `start`: the first tau0 tried (default: the smallest Fig. 1-feasible one).  A
     failing run that met a platform stall (stalled()) is repeated up to `stall_retries` times: it
-    says nothing about the rate.  Returns (tau0, w, theta, T, stats)."""
+    says nothing about the rate.  `inject` = (period_ns, len_ns): every trial run carries injected
+    platform-length stalls (pl_pipeline_inject_stalls), and the criterion becomes zero misses
+    ACROSS them -- the pipeline must catch up after each within D (R-STALL); the 5 % outlier
+    bound then cannot apply (a stalled item is late by construction) and is not checked.
+    Returns (tau0, w, theta, T, stats)."""
     from ._pl import PlError
     scfg = cfg if solve_deadline is None else cfg.replace(deadline=int(solve_deadline))
 
@@ -161,17 +167,17 @@ def find_rate(cfg, wl, db_dev, tries=12, grow=1.15, stream=None, log=None, over=
                         policy=policy)
         for attempt in range(stall_retries + 1):
             try:
-                st = _run(c, db_dev, wl.db_len, wl, flags=flags, stream=stream, over=over)
+                st = _run(c, db_dev, wl.db_len, wl, flags=flags, stream=stream, over=over, inject=inject)
                 ok = (st["misses"] == 0 and st["miss_events"] == 0 and st["miss_events_ns"] == 0
                       and st["errors"] == 0)
                 if max_lateness_ns is not None:
                     ok = ok and max(st["max_lateness_ns"]) <= max_lateness_ns
-                if max_outliers is not None:   # north_star 5 % per-item agreement (R-AGREE)
+                if max_outliers is not None and not inject:   # north_star 5 % per-item agreement (R-AGREE)
                     ok = ok and st["latency_outliers"] <= max_outliers
             except PlError:          # device-side overflow reported by drain
                 st, ok = {"misses": -1, "miss_events_ns": -1, "errors": -1, "overruns": [], "max_latency_ns": -1,
                           "max_lateness_ns": []}, False
-            if ok or not stalled(st):
+            if ok or inject or not stalled(st):
                 break
         if log:
             log(dict(tau=tau, w=w, T=T, misses=st["misses"], overruns=st["overruns"], errors=st["errors"],

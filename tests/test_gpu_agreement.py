@@ -41,14 +41,14 @@ def c4():
 
 def _cfg(base, budgets, tau):
     from paper_conf_icppw_planob21_b200 import realtime
-    cfg = base.replace(clock=C.CLOCK_GLOBALTIMER, ns_per_unit=1.0, service_time=budgets, gain=GAINS, deadline=D,
-                       b=C.PAPER_B, policy=C.THRESHOLD_SLACK, slack_guard=max(budgets) + SG)
+    cfg = _cfg_base(base, budgets)
     w, th, T = realtime.solve_at(cfg.replace(deadline=D - SG), tau)
     return cfg.replace(interarrival=tau, wait_time=tuple(w), wait_threshold=tuple(th))
 
 
 def _run_unstalled(cfg, wl, db, over, flags, tries=4):
     from paper_conf_icppw_planob21_b200 import Pipeline, realtime
+    seen = []
     for _ in range(tries):
         pl = Pipeline(cfg, wl, flags=flags, **over)
         pl.bind_device(db.data_ptr(), wl.db_len)
@@ -62,7 +62,22 @@ def _run_unstalled(cfg, wl, db, over, flags, tries=4):
         pl.close()
         if not realtime.stalled(st):
             return out
-    pytest.skip("every run met a platform stall")
+        seen.append(st["max_lateness_ns"])
+    pytest.skip(f"every run met a platform stall (per-node lateness of each run: {seen})")
+
+
+def _tau(base, b):
+    """1.5 x the node-3 island bound u t_3 / v, and at least 1.3 x the smallest Fig. 1-feasible tau0."""
+    from paper_conf_icppw_planob21_b200 import realtime
+    cfg = _cfg_base(base, b)
+    t_min = realtime.min_feasible_tau(cfg.replace(deadline=D - SG))
+    assert t_min is not None, b
+    return max(int(1.5 * 16 * b[3] / 128), int(1.3 * t_min))
+
+
+def _cfg_base(base, budgets):
+    return base.replace(clock=C.CLOCK_GLOBALTIMER, ns_per_unit=1.0, service_time=budgets, gain=GAINS, deadline=D,
+                        b=C.PAPER_B, policy=C.THRESHOLD_SLACK, slack_guard=max(budgets) + SG)
 
 
 def _budgets(c4, flags):
@@ -77,8 +92,8 @@ def test_bench_kernel_every_item_within_5pct(c4):
     """The record-free kernel bench.py times, at 1.5 x the node-3 island bound u t_3 / v."""
     from paper_conf_icppw_planob21_b200._pl import PL_FIXED_SERVICE
     base, wl, db, over = c4
-    b = _budgets(c4, PL_FIXED_SERVICE)
-    tau = int(1.5 * 16 * b[3] / 128)
+    b = _budgets(c4, 0)                 # bench.py calibrates with the record-free kernel, flags 0
+    tau = _tau(base, b)
     g = _run_unstalled(_cfg(base, b, tau), wl, db, over, PL_FIXED_SERVICE)
     st = g["stats"]
     print("budgets", b, "tau0", tau, "lateness", st["max_lateness_ns"], "rel err max", st["latency_rel_err_max"])
@@ -90,16 +105,27 @@ def test_bench_kernel_every_item_within_5pct(c4):
     assert abs(sum(st["busy_ns"]) / model_busy - 1) < 0.05
 
 
-def test_recording_kernel_per_root_and_sampled_streams(c4):
+@pytest.fixture(scope="module")
+def c4q():
+    """c4's shape (148 streams, heavy-tailed islands, 1 kbp query) at a quarter of its length, so
+    that one run (~0.5 s) usually misses the platform's ~1.6 ms SM stalls (every 2-3 s)."""
+    import torch
+    base = C.c4(dna=dict(db_len=25 << 20, q_len=1024, n_planted=1600, heavy_tailed=True))
+    wl = workload_for(base)
+    db = torch.from_numpy(wl.db.view("int32")).cuda()
+    return base, wl, db, dict(match_capacity=1 << 24, spill_capacity=1 << 19)
+
+
+def test_recording_kernel_per_root_and_sampled_streams(c4q):
     """Every root's measured latency against its logical one, element by element; the logical
     schedule of sampled streams against the oracle's DES."""
     from oracle import des
     from oracle import stages as S
-    base, wl, db, over = c4
-    b = _budgets(c4, 7 | 8)
-    tau = int(1.5 * 16 * b[3] / 128)
+    base, wl, db, over = c4q
+    b = _budgets(c4q, 1)                # the recording kernel's own firing times
+    tau = _tau(base, b)
     cfg = _cfg(base, b, tau)
-    g = _run_unstalled(cfg, wl, db, over, 7 | 8)
+    g = _run_unstalled(cfg, wl, db, over, 1 | 8, tries=8)   # per-root latencies, time-triggered delivery
     st = g["stats"]
     assert st["miss_events_ns"] == 0 and st["errors"] == 0
     lu = g["lat"].astype(np.float64)            # units = ns

@@ -99,7 +99,32 @@ def test_physical_replays_logical_schedule(c2wl, budgets, fixed_service):
         assert abs(sum(st["busy_ns"]) / model_busy - 1) < 0.05
 
 
-def test_physical_zero_misses_at_bench_rate(c2wl, budgets):
+def test_injected_stalls_move_time_not_schedule(c2wl, budgets):
+    """pl_pipeline_inject_stalls (R-STALL): every node of every stream stops over the injected
+    windows -- each node's lateness reaches the stall length and measured latencies grow -- while
+    the logical schedule (matches, traces, model latencies, firing log) stays bit-exact."""
+    from paper_conf_icppw_planob21_b200 import Pipeline
+    _, wl = c2wl
+    cfg = _phys_cfg(budgets, _tau_for(budgets, 40))
+    span = (wl.db_len // 148) * cfg.interarrival      # one stream's arrival span (ns)
+    period, length = span // 3, span // 12
+    pl = Pipeline(cfg, wl, flags=7)
+    pl.push(wl.db, wl.db_len)
+    pl.inject_stalls(period, length)
+    pl.drain()
+    g = dict(stats=pl.stats(), matches=pl.results(), trace=pl.trace(), firings=pl.firings())
+    g["lat"], g["lat_ns"] = pl.latency()
+    pl.close()
+    compare(cfg, g, run_oracle_parallel(cfg, wl))
+    st = g["stats"]
+    print("stall", length, "lateness", st["max_lateness_ns"])
+    assert min(st["max_lateness_ns"]) >= 0.8 * length
+    assert (g["lat_ns"] - g["lat"]).max() >= 0.8 * length
+    with pytest.raises(Exception):
+        Pipeline(cfg.replace(clock=C.CLOCK_LOGICAL), wl).inject_stalls(period, length)
+
+
+def test_physical_zero_misses_1p5x_feasible_rate(c2wl, budgets):
     """Zero measured misses at a rate 1.5x above the Fig. 1 feasibility limit of the budgets
     (at least tau0 = 30 ns)."""
     _, wl = c2wl
