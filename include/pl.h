@@ -86,6 +86,12 @@ enum pl_clock { PL_CLOCK_LOGICAL = 0, PL_CLOCK_GLOBALTIMER = 1 };
                                   starts at T >= A_last are dropped).  The paper models an
                                   unbounded stream (L63) and is silent on its end; without
                                   this flag the periodic / threshold rules run to the drain. */
+#define PL_CLUSTER_NODES 32u   /* N4 ("a fixed 1/N fraction of processor
+                                  time", L265): every stream runs on a cluster of N CTAs, node i on
+                                  CTA rank i (an SM of its own), its input queue in that CTA's
+                                  shared memory, written by node i-1 over DSMEM.  FIXED_WAIT and
+                                  THRESHOLD_SLACK, N <= 8, v <= 256; not with live ingest.  Same
+                                  schedule and results as the one-CTA-per-stream executor.      */
 
 typedef struct {
   uint32_t kind;           /* enum pl_stage_kind                                        */

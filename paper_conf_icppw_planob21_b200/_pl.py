@@ -15,6 +15,7 @@ PL_MAX_STAGES = 8
 PL_MAX_U = 16
 PL_OK, PL_EINVAL, PL_ENOMEM, PL_EDEVICE, PL_EINFEASIBLE, PL_ESTATE, PL_EAGAIN, PL_EOVERFLOW = 0, -1, -2, -3, -4, -5, -6, -7
 PL_REC_LATENCY, PL_REC_TRACE, PL_REC_FIRINGS, PL_FIXED_SERVICE, PL_EAGER_DRAIN = 1, 2, 4, 8, 16
+PL_CLUSTER_NODES = 32
 STATUS_NAMES = {0: "PL_OK", -1: "PL_EINVAL", -2: "PL_ENOMEM", -3: "PL_EDEVICE", -4: "PL_EINFEASIBLE",
                 -5: "PL_ESTATE", -6: "PL_EAGAIN", -7: "PL_EOVERFLOW"}
 

@@ -42,6 +42,11 @@ __device__ __forceinline__ void vst(T* p, T v) { *(volatile T*)p = v; }
 // message passing, so no sequentially consistent fence is needed): MEMBAR.ALL.CTA in SASS,
 // where __threadfence_block() emits the costlier MEMBAR.SC.CTA.
 __device__ __forceinline__ void fence_cta() { asm volatile("fence.acq_rel.cta;" ::: "memory"); }
+// queue fences: CTA scope, or cluster scope when the nodes are the CTAs of a cluster (N4)
+__device__ __forceinline__ void fence_q(bool cl) {
+  if (cl) asm volatile("fence.acq_rel.cluster;" ::: "memory");
+  else asm volatile("fence.acq_rel.cta;" ::: "memory");
+}
 
 
 // ------------------------------------------------------------- counter-based RNG
@@ -371,6 +376,9 @@ struct Ctx {
   uint64_t lo, hi;             // roots [lo, hi)
   int64_t X, H;
   bool sliding;                // the stream's DB range exceeds the window ring: refills (win_step)
+  uint32_t stream;             // this CTA's stream (blockIdx.x, or the cluster's index: N4)
+  int rank;                    // N4 (PL_CLUSTER_NODES): this CTA's rank in its cluster = its node; else -1
+  Shared* agg;                 // the stream's aggregates: this CTA's Shared, or rank 0's (DSMEM)
 };
 
 __device__ __forceinline__ uint32_t smem_addr(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
@@ -536,7 +544,9 @@ struct Node {
   int64_t Mcap, B_per;          // FIXED_WAIT + eager: time-triggered slots m < Mcap (m P < A_last);
                                 // the last of them ends at B_per
   uint32_t* troot;              // smem [v]: the current firing's terminal root per lane (or NO_ROOT)
-  uint32_t* bnd;                // smem: Shared::bnd (sliding window only)
+  uint32_t* bnd_me;             // smem: this node's Shared::bnd entry (sliding window only)
+  const uint32_t* bnd_up;       // the upstream node's entry (its CTA's smem under N4)
+  bool cl;                      // N4: queues are in the consumer CTA's smem (cluster-scope fences)
   uint32_t nap_cap_ns;          // physical: longest poll nap of a waiting leader (t_i / 8, >= 256 ns)
   bool sliding;
   __device__ __forceinline__ int64_t arrival(uint32_t root) const {
@@ -570,15 +580,22 @@ __device__ __forceinline__ Node make_node(const Ctx& c, int i) {
   n.segmask = p.segcap - 1;
   n.capg = p.cap_g;
   n.Ein = &c.sh->e[i];
-  const uint64_t sp = (uint64_t)blockIdx.x * p.N;
+  const uint64_t sp = (uint64_t)c.stream * p.N;
   n.in_ent = (const uint2*)(c.dsm + Lo.off_ent[i]);
   n.in_seg = (const Seg*)(c.dsm + Lo.off_seg[i]);
   n.in_spill = p.spill ? p.spill + (sp + i) * p.cap_g : nullptr;
   n.in_mask = p.cap_s[i] ? p.cap_s[i] - 1 : 0;
   const int o = i + 1 < p.N ? i + 1 : i;
-  n.Eout = &c.sh->e[o];
-  n.out_ent = (uint2*)(c.dsm + Lo.off_ent[o]);
-  n.out_seg = (Seg*)(c.dsm + Lo.off_seg[o]);
+  n.cl = c.rank >= 0;
+  if (n.cl && o != i) {   // N4: the edge into node i+1 lives in CTA i+1's shared memory (DSMEM)
+    n.Eout = (EdgeCtl*)__cluster_map_shared_rank(&c.sh->e[o], (unsigned)o);
+    n.out_ent = (uint2*)__cluster_map_shared_rank(c.dsm + Lo.off_ent[o], (unsigned)o);
+    n.out_seg = (Seg*)__cluster_map_shared_rank(c.dsm + Lo.off_seg[o], (unsigned)o);
+  } else {
+    n.Eout = &c.sh->e[o];
+    n.out_ent = (uint2*)(c.dsm + Lo.off_ent[o]);
+    n.out_seg = (Seg*)(c.dsm + Lo.off_seg[o]);
+  }
   n.out_spill = p.spill ? p.spill + (sp + o) * p.cap_g : nullptr;
   n.out_cap = p.cap_s[o];
   const DevStage& s = p.st[i];
@@ -595,7 +612,9 @@ __device__ __forceinline__ Node make_node(const Ctx& c, int i) {
   n.Mcap = (n.eager && n.fixed) ? cdiv(n.A_last, n.dP) : 0;
   n.B_per = n.Mcap > 0 ? (n.Mcap - 1) * n.P + n.t : 0;
   n.troot = (uint32_t*)(c.dsm + Lo.off_troot) + (uint32_t)i * (uint32_t)p.v;
-  n.bnd = c.sh->bnd;
+  n.bnd_me = &c.sh->bnd[i];
+  n.bnd_up = (n.cl && i > 0) ? (const uint32_t*)__cluster_map_shared_rank(&c.sh->bnd[i - 1], (unsigned)(i - 1))
+                             : &c.sh->bnd[i > 0 ? i - 1 : 0];
   {
     const int64_t cap = n.t_ns / 8;
     n.nap_cap_ns = (uint32_t)(cap < 256 ? 256 : (cap > 8192 ? 8192 : cap));
@@ -730,7 +749,7 @@ __device__ __forceinline__ void publish_W(const Node& nd, Leader& L, int64_t w) 
   if (nd.sink) return;
   if (w > L.W_pub) {
     L.W_pub = w;
-    fence_cta();
+    fence_q(nd.cl);
     vst(&nd.Eout->W, w);
   }
 }
@@ -915,13 +934,13 @@ __device__ Decision decide(const Node& nd, Leader& L, bool& waited, uint64_t T0)
     }
     // node i >= 1: read the upstream watermark (and window bound) first, then the published segments
     const int64_t Wup = vld(&nd.Ein->W);
-    const uint32_t bup = nd.sliding ? vld(&nd.bnd[nd.i - 1]) : 0u;
-    fence_cta();
+    const uint32_t bup = nd.sliding ? vld(nd.bnd_up) : 0u;
+    fence_q(nd.cl);
     const uint32_t st = vld(&nd.Ein->seg_tail);
     const uint32_t tail_known = (st != L.segh) ? nd.in_seg[(st - 1) & nd.segmask].end : L.head;
     const bool any = tail_known != L.head;
     // an empty queue: everything this node will still read comes from upstream's future
-    if (nd.sliding && !any && bup > vld(&nd.bnd[nd.i])) vst(&nd.bnd[nd.i], bup);
+    if (nd.sliding && !any && bup > vld(nd.bnd_me)) vst(nd.bnd_me, bup);
     if (nd.fixed) {
       if (nd.eager && L.m >= nd.Mcap) {  // R-DRAIN: work-conserving from A_last on
         const int64_t B = max(max(nd.B_per, L.B), nd.A_last);
@@ -967,7 +986,7 @@ __device__ Decision decide(const Node& nd, Leader& L, bool& waited, uint64_t T0)
       continue;
     }
     const Seg& hs = nd.in_seg[L.segh & nd.segmask];
-    fence_cta();
+    fence_q(nd.cl);
     const uint2 he = load_entry(nd, L.head, L.segh, st, vld(&nd.Ein->spill_end));
     int64_t Tf = nd.arrival(he.x) + nd.D - nd.R;
     if (Tf < hs.ready) Tf = hs.ready;
@@ -1229,7 +1248,7 @@ __device__ __forceinline__ uint32_t live_need(const Shared& sh, const DevParams&
 // REC: per-item records compiled in (parity / tracing runs); the bench kernel has none.
 // (A separate node-0 instantiation was measured: faster alone, 1.33x slower with all nodes
 // running -- the SM's instruction cache holds one ~76 KB node loop, not two.)
-template <bool REC>
+template <bool REC, bool CL>
 __device__ void run_node(Ctx& c, Dna dna, int i, int gtid) {
   const DevParams& p = *c.p;
   const Node nd = make_node(c, i);
@@ -1239,7 +1258,8 @@ __device__ void run_node(Ctx& c, Dna dna, int i, int gtid) {
   const int bidA = 1 + i;
   const int bidB = (i < 7) ? 9 + i : bidA;       // barrier ids 9..15 for the output barrier
   GroupCtl& G = c.sh->g[i];
-  const uint32_t stream = blockIdx.x;
+  const uint32_t stream = c.stream;
+  Shared& AG = CL ? *c.agg : *c.sh;      // the stream's aggregates (N4: rank 0's, over DSMEM)
   const uint32_t rec = REC ? p.flags : (p.flags & PL_FIXED_SERVICE);
   const uint64_t T0 = c.sh->T0;
   NodeAcc& A = c.sh->acc[i];
@@ -1292,7 +1312,7 @@ __device__ void run_node(Ctx& c, Dna dna, int i, int gtid) {
         }
         atomicMax(&A.max_queue, ql);
         publish_W(nd, L, T + nd.t);      // committed: nothing leaves node 0 before T + t_0
-        if (rec & PL_REC_FIRINGS) G.log_idx[par] = atomicAdd(&c.sh->log_count, 1u);
+        if (rec & PL_REC_FIRINGS) G.log_idx[par] = atomicAdd(&AG.log_count, 1u);
         A.d[par][D_STALL] = 0;
         G.out_loc[par] = nd.sink ? LOC_SMEM : reserve_out(nd, L, n * nd.umax, &A.d[par][D_STALL]);
         G.out_base[par] = L.out_tail;
@@ -1331,10 +1351,10 @@ __device__ void run_node(Ctx& c, Dna dna, int i, int gtid) {
         G.head[par] = L.head;
         G.segh[par] = L.segh;
         G.st[par] = vld(&nd.Ein->seg_tail);
-        fence_cta();
+        fence_q(nd.cl);
         G.in_spill_end[par] = vld(&nd.Ein->spill_end);
         if (!d.done) {
-          if (rec & PL_REC_FIRINGS) G.log_idx[par] = atomicAdd(&c.sh->log_count, 1u);
+          if (rec & PL_REC_FIRINGS) G.log_idx[par] = atomicAdd(&AG.log_count, 1u);
           A.d[par][D_STALL] = 0;
           G.out_loc[par] = nd.sink ? LOC_SMEM : reserve_out(nd, L, d.n * nd.umax, &A.d[par][D_STALL]);
           G.out_base[par] = L.out_tail;
@@ -1374,7 +1394,7 @@ __device__ void run_node(Ctx& c, Dna dna, int i, int gtid) {
     }
     if (nd.sliding) {                    // the window's current range, and this node's bound
       win_snap(dna, *c.sh);
-      if (leader && act && !n0) vst(&nd.bnd[i], e[0].x);   // the firing's first (smallest) root
+      if (leader && act && !n0) vst(nd.bnd_me, e[0].x);   // the firing's first (smallest) root
     }
     {   // warp-uniform dispatch to the stage body: direct compare-and-branch chain (a switch
         // compiles to an indirect BRX, measured ~200 cycles per dispatch)
@@ -1400,7 +1420,7 @@ __device__ void run_node(Ctx& c, Dna dna, int i, int gtid) {
       off = group_scan(G.wtot[par], o[0].c, &total, gtid, v, bidA, nd.umax <= 1);                 // B2
     }
     const uint32_t out_loc = G.out_loc[par], out_base = G.out_base[par];   // leader's reservation (B2)
-    if (nd.sliding && n0 && leader) vst(&nd.bnd[0], (uint32_t)(nd.lo + head));   // every lane is past the last firing
+    if (nd.sliding && n0 && leader) vst(nd.bnd_me, (uint32_t)(nd.lo + head));   // every lane is past the last firing
     if (leader) { const long long t2 = clock64(); A.d[par][D_PH2] = (uint32_t)(t2 - tc); tc = t2; }
     if (REC && n0 && pend_root != NO_ROOT)   // node 0: the previous publish time came through B2
       record_lat_ns(nd, c, T0, G.end_ns[par ^ 1], pend_root);
@@ -1409,7 +1429,7 @@ __device__ void run_node(Ctx& c, Dna dna, int i, int gtid) {
       L.head = head + n;
       const uint32_t st = G.st[par];
       while (L.segh != st && (int32_t)(nd.in_seg[L.segh & nd.segmask].end - L.head) <= 0) ++L.segh;
-      fence_cta();
+      fence_q(nd.cl);
       vst(&nd.Ein->head, L.head);
       vst(&nd.Ein->seg_head, L.segh);
     }
@@ -1433,7 +1453,7 @@ __device__ void run_node(Ctx& c, Dna dna, int i, int gtid) {
           if (gtid == 0) { f->start = T; f->node = i; f->n = n; f->first_root = ei.x; f->stream = stream; f->pad = 0; }
           if ((uint32_t)gtid == n - 1) f->last_root = ei.x;
         } else if (gtid == 0) {
-          atomicOr(&c.sh->errors, PL_ERR_LOG_OVERFLOW);
+          atomicOr(&AG.errors, PL_ERR_LOG_OVERFLOW);
         }
       }
     }
@@ -1465,7 +1485,7 @@ __device__ void run_node(Ctx& c, Dna dna, int i, int gtid) {
             mt.len = oi.len; mt.score = oi.score;
             p.matches[mi] = mt;
           } else {
-            atomicOr(&c.sh->errors, PL_ERR_MATCH_OVERFLOW);
+            atomicOr(&AG.errors, PL_ERR_MATCH_OVERFLOW);
           }
         }
       }
@@ -1519,7 +1539,7 @@ __device__ void run_node(Ctx& c, Dna dna, int i, int gtid) {
         sg.loc = out_loc;
         nd.out_seg[L.out_segt & nd.segmask] = sg;
         if (out_loc == LOC_SPILL) vst(&nd.Eout->spill_end, sg.end);
-        fence_cta();
+        fence_q(nd.cl);
         ++L.out_segt;
         L.out_tail += total;
         vst(&nd.Eout->seg_tail, L.out_segt);
@@ -1605,7 +1625,7 @@ __device__ void run_node(Ctx& c, Dna dna, int i, int gtid) {
           const int64_t due = (int64_t)(T0 + units_ns(nd, T + nd.t));
           const int64_t err = (int64_t)en > due ? (int64_t)en - due : due - (int64_t)en;
           const int64_t lsmall = (int64_t)units_ns(nd, T + nd.t - nd.arrival(rx - 1u));
-          atomicMax(&c.sh->agr_ppm, clamp32((int64_t)((float)err * 1e6f / (float)(lsmall > 0 ? lsmall : 1))));
+          atomicMax(&AG.agr_ppm, clamp32((int64_t)((float)err * 1e6f / (float)(lsmall > 0 ? lsmall : 1))));
           // count the items outside the band exactly -- with PL_FIXED_SERVICE only, where the model's
           // completion time is realised and outliers are rare (in publish mode a firing completes
           // early by design and the count would cost a pass over the lanes on every firing)
@@ -1615,7 +1635,7 @@ __device__ void run_node(Ctx& c, Dna dna, int i, int gtid) {
               const uint32_t r = nd.troot[k];
               if (r != NO_ROOT && err * 20 > (int64_t)units_ns(nd, T + nd.t - nd.arrival(r)) + 20 * PL_AGREE_FLOOR_NS) ++m;
             }
-            atomicAdd(&c.sh->agr_bad, m);
+            atomicAdd(&AG.agr_bad, m);
           }
         }
       }
@@ -1637,7 +1657,7 @@ __device__ void run_node(Ctx& c, Dna dna, int i, int gtid) {
         p0.x += dd.x; p0.y += dd.y; p1.x += dd.z; p1.y += dd.w;
         Cp[0] = c0; Cp[1] = c1; Cp[3] = c3; Cp[4] = c4; Pp[0] = p0; Pp[1] = p1;
       }
-      if (n0 && nd.sliding) win_step(*c.sh, p, (unsigned char*)dna.win, false);   // slide the DB window
+      if ((CL || n0) && nd.sliding) win_step(*c.sh, p, (unsigned char*)dna.win, false);   // slide the DB window
     }
     if (n0) {                            // replicated node-0 state, identical in every lane
       R.c0 += n;
@@ -1650,17 +1670,17 @@ __device__ void run_node(Ctx& c, Dna dna, int i, int gtid) {
     }
     par ^= 1;
   }
-  if (nd.sliding && leader) vst(&nd.bnd[i], 0xffffffffu);   // reads nothing more
+  if (nd.sliding && leader) vst(nd.bnd_me, 0xffffffffu);   // reads nothing more
   if (n0) {
     if (leader) publish_W(nd, L, PL_INF64);   // after the last segment was published
     bar_sync(bidA, v);                   // the last publish time is visible to every lane
     if (REC && pend_root != NO_ROOT) record_lat_ns(nd, c, T0, G.end_ns[par ^ 1], pend_root);
   }
   if (leader) {
-    if (A.lmax) atomicMax(&c.sh->max_lat, A.lmax);
-    if (A.lmax_ns) atomicMax(&c.sh->max_lat_ns, A.lmax_ns);
-    if (A.nmiss) atomicAdd(&c.sh->miss_events, A.nmiss);
-    if (A.nmiss_ns) atomicAdd(&c.sh->miss_events_ns, A.nmiss_ns);
+    if (A.lmax) atomicMax(&AG.max_lat, A.lmax);
+    if (A.lmax_ns) atomicMax(&AG.max_lat_ns, A.lmax_ns);
+    if (A.nmiss) atomicAdd(&AG.miss_events, A.nmiss);
+    if (A.nmiss_ns) atomicAdd(&AG.miss_events_ns, A.nmiss_ns);
     CtaStats& S = p.stats[stream];
     S.firings[i] = A.cnt[C_FIRINGS];
     S.empty[i] = n0 ? R.empties : L.empties;
@@ -1718,12 +1738,16 @@ __host__ __device__ inline uint32_t layout_enforced(const DevParams& p, SmemLayo
   return off;
 }
 
-__device__ void cta_setup(Ctx& c, Shared& sh, unsigned char* dsm, const DevParams& p) {
+// rank >= 0: N4 (PL_CLUSTER_NODES) -- this CTA is node `rank` of the stream given by its cluster
+__device__ void cta_setup(Ctx& c, Shared& sh, unsigned char* dsm, const DevParams& p, int rank = -1) {
   SmemLayout Lo;
   layout_enforced(p, &Lo);
-  const uint32_t s = blockIdx.x, tid = threadIdx.x, nt = blockDim.x;
+  const uint32_t s = rank >= 0 ? blockIdx.x / (uint32_t)p.N : blockIdx.x, tid = threadIdx.x, nt = blockDim.x;
   c.p = &p;
   c.sh = &sh;
+  c.stream = s;
+  c.rank = rank;
+  c.agg = rank > 0 ? (Shared*)__cluster_map_shared_rank(&sh, 0u) : &sh;
   c.lo = (p.total_roots * s) / (uint64_t)p.n_streams;
   c.hi = (p.total_roots * (s + 1)) / (uint64_t)p.n_streams;
   c.X = (int64_t)(c.hi - c.lo);
@@ -1837,7 +1861,8 @@ __device__ void cta_setup(Ctx& c, Shared& sh, unsigned char* dsm, const DevParam
         win[(uint32_t)w & (p.win_cap - 1u)] = w < (int64_t)p.db_words ? p.db[w] : 0u;
       }
   }
-  if (tid < PL_MAX_STAGES) sh.bnd[tid] = (uint32_t)c.lo;   // no node reads below its stream's first root
+  // no node reads below its stream's first root; under N4 this CTA's window serves its own node only
+  if (tid < PL_MAX_STAGES) sh.bnd[tid] = (rank < 0 || (int)tid == rank) ? (uint32_t)c.lo : 0xffffffffu;
   if (tid < PL_MAX_STAGES) {
     EdgeCtl& E = sh.e[tid];
     E.head = 0; E.seg_head = 0; E.seg_tail = 0; E.tail = 0; E.W = -1; E.spill_end = 0; E.stalled = 0;
@@ -1846,21 +1871,25 @@ __device__ void cta_setup(Ctx& c, Shared& sh, unsigned char* dsm, const DevParam
     sh.max_lat = 0; sh.max_lat_ns = 0; sh.miss_events = 0; sh.miss_events_ns = 0; sh.errors = 0; sh.log_count = 0;
     sh.agr_bad = 0; sh.agr_ppm = 0; sh.ingest_waits = 0; sh.ingest_max_ns = 0;
   }
-  // per-root records of this stream
-  if (p.flags & PL_REC_LATENCY)
-    for (uint64_t r = c.lo + tid; r < c.hi; r += nt) { p.lat[r] = -1; if (p.lat_ns) p.lat_ns[r] = -1; }
-  if (p.flags & PL_REC_TRACE)
-    for (uint64_t r = c.lo * (p.N + 1) + tid; r < c.hi * (p.N + 1); r += nt) p.trace[r] = 0u;
-  if (tid == 0) {
-    CtaStats& S = p.stats[s];
-    S.n_log = 0;
-    S.t_end = 0;
+  if (rank <= 0) {   // the stream's records and per-stream stats: one CTA of the cluster (N4)
+    if (p.flags & PL_REC_LATENCY)
+      for (uint64_t r = c.lo + tid; r < c.hi; r += nt) { p.lat[r] = -1; if (p.lat_ns) p.lat_ns[r] = -1; }
+    if (p.flags & PL_REC_TRACE)
+      for (uint64_t r = c.lo * (p.N + 1) + tid; r < c.hi * (p.N + 1); r += nt) p.trace[r] = 0u;
+    if (tid == 0) {
+      CtaStats& S = p.stats[s];
+      S.n_log = 0;
+      S.t_end = 0;
+      S.win_refills = 0;
+    }
   }
 }
 
 __device__ void cta_finish(Ctx& c, Shared& sh, const DevParams& p) {
-  if (threadIdx.x == 0) {
-    CtaStats& S = p.stats[blockIdx.x];
+  if (threadIdx.x == 0 && c.rank >= 0 && p.k > 0)   // N4: every CTA's window refills
+    atomicAdd(&p.stats[c.stream].win_refills, sh.win.refills);
+  if (threadIdx.x == 0 && c.rank <= 0) {
+    CtaStats& S = p.stats[c.stream];
     S.miss_events = sh.miss_events;
     S.miss_events_ns = sh.miss_events_ns;
     S.max_lat = (int64_t)sh.max_lat;
@@ -1869,7 +1898,7 @@ __device__ void cta_finish(Ctx& c, Shared& sh, const DevParams& p) {
     S.n_roots = (uint64_t)c.X;
     S.n_log = sh.log_count < p.log_cap ? sh.log_count : p.log_cap;
     S.errors = sh.errors;
-    S.win_refills = p.k > 0 ? sh.win.refills : 0u;
+    if (c.rank < 0) S.win_refills = p.k > 0 ? sh.win.refills : 0u;
     S.agr_bad = sh.agr_bad;
     S.agr_ppm = sh.agr_ppm;
     S.ingest_waits = sh.ingest_waits;
@@ -2083,8 +2112,36 @@ __global__ void __launch_bounds__(MAXT, MINB) pl_exec_enforced(const __grid_cons
   const bool contig = !(p.variant & 4u);
   const int gi = contig ? w / (p.v >> 5) : w % p.N;
   const int gt = (contig ? w % (p.v >> 5) : w / p.N) * 32 + (threadIdx.x & 31);
-  if (w < p.N * (p.v >> 5)) run_node<REC>(c, c.dna, gi, gt);
+  if (w < p.N * (p.v >> 5)) run_node<REC, false>(c, c.dna, gi, gt);
   __syncthreads();
+  cta_finish(c, sh, p);
+}
+
+// N4 (PL_CLUSTER_NODES, "a fixed 1/N fraction of processor time",
+// L265): one stream per cluster of N CTAs, node i = CTA rank i on an SM of its own.  The edge
+// into node i (its smem ring, segment records and control words) lives in CTA i's shared memory;
+// node i-1 writes its outputs and publishes them there over DSMEM, with cluster-scope fences;
+// the stream's aggregates live in rank 0.  Every CTA stages the query index and slides its own
+// DB window behind its own node's bound.  grid = n_streams x N CTAs of v threads.
+template <bool REC>
+__global__ void __launch_bounds__(256, 1) pl_exec_cluster(const __grid_constant__ DevParams p) {
+  extern __shared__ __align__(16) unsigned char dsm[];
+  __shared__ Shared sh;
+  Ctx c;
+  const int rank = (int)__clusterRelativeBlockRank();
+  cta_setup(c, sh, dsm, p, rank);
+  __syncthreads();
+  __cluster_barrier_arrive();            // every CTA's queues are initialised before any remote access
+  __cluster_barrier_wait();
+  if (threadIdx.x == 0 && rank == 0) sh.T0 = gtimer() + (p.clock == PL_CLOCK_GLOBALTIMER ? p.t0_offset_ns : 0u);
+  __cluster_barrier_arrive();
+  __cluster_barrier_wait();
+  if (threadIdx.x == 0 && rank > 0) sh.T0 = vld(&c.agg->T0);   // one time origin per stream
+  __syncthreads();
+  if ((int)threadIdx.x < p.v) run_node<REC, true>(c, c.dna, rank, (int)threadIdx.x);
+  __syncthreads();
+  __cluster_barrier_arrive();            // every node is done: rank 0's aggregates are final, and no
+  __cluster_barrier_wait();              // CTA leaves while another may still access its smem
   cta_finish(c, sh, p);
 }
 
@@ -2114,6 +2171,22 @@ cudaError_t pl_launch(const DevParams& p, unsigned grid, unsigned block, unsigne
   if (mono) {
     if (block <= 512) pl_exec_monolithic<512><<<grid, block, smem, st>>>(p);
     else pl_exec_monolithic<1024><<<grid, block, smem, st>>>(p);
+  } else if (p.flags & PL_CLUSTER_NODES) {   // N4: grid = streams x N CTAs, clusters of N
+    cudaLaunchConfig_t cfg = {};
+    cudaLaunchAttribute at[1];
+    at[0].id = cudaLaunchAttributeClusterDimension;
+    at[0].val.clusterDim.x = (unsigned)p.N;
+    at[0].val.clusterDim.y = 1;
+    at[0].val.clusterDim.z = 1;
+    cfg.gridDim = dim3(grid * (unsigned)p.N);
+    cfg.blockDim = dim3((unsigned)p.v);
+    cfg.dynamicSmemBytes = smem;
+    cfg.stream = st;
+    cfg.attrs = at;
+    cfg.numAttrs = 1;
+    const bool rec = (p.flags & (PL_REC_LATENCY | PL_REC_TRACE | PL_REC_FIRINGS)) != 0;
+    cudaError_t e = rec ? cudaLaunchKernelEx(&cfg, pl_exec_cluster<true>, p) : cudaLaunchKernelEx(&cfg, pl_exec_cluster<false>, p);
+    if (e != cudaSuccess) return e;
   } else {
     // two CTAs (streams) per SM when the grid asks for more streams than there are SMs and
     // the CTA fits twice (<= 512 threads, 64 registers, smem)
@@ -2141,6 +2214,8 @@ cudaError_t pl_kernel_attributes(unsigned max_smem) {
   if ((e = cudaFuncSetAttribute(pl_exec_enforced<512, 1, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, max_smem))) return e;
   if ((e = cudaFuncSetAttribute(pl_exec_enforced<1024, 1, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, max_smem))) return e;
   if ((e = cudaFuncSetAttribute(pl_exec_enforced<1024, 1, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, max_smem))) return e;
+  if ((e = cudaFuncSetAttribute(pl_exec_cluster<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, max_smem))) return e;
+  if ((e = cudaFuncSetAttribute(pl_exec_cluster<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, max_smem))) return e;
   if ((e = cudaFuncSetAttribute(pl_exec_monolithic<512>, cudaFuncAttributeMaxDynamicSharedMemorySize, max_smem))) return e;
   return cudaFuncSetAttribute(pl_exec_monolithic<1024>, cudaFuncAttributeMaxDynamicSharedMemorySize, max_smem);
 }
@@ -2173,6 +2248,7 @@ __global__ void __launch_bounds__(MAXT, 1) pl_stage_batch_kernel(const __grid_co
   c.dna.qw = (const uint32_t*)(dsm + Lo.off_qw);
   c.dna.nqw = (uint32_t)(p.q_len + 15) / 16u;
   c.dna.win = nullptr; c.dna.win_lo = 0; c.dna.win_lo32 = 0; c.dna.win_n = 0; c.dna.win_mask = 0;
+  c.dna.dbmask = 0xffffffffu;
   c.dna.nofast = true; c.dna.s2tab = nullptr;
   c.sliding = false;
   const uint32_t tid = threadIdx.x, v = blockDim.x;

@@ -191,6 +191,11 @@ pl_status validate(const pl_config* c, const pl_workload* wl) {
   if (c->clock > PL_CLOCK_GLOBALTIMER) return fail(PL_EINVAL, "bad clock %u", c->clock);
   if (c->clock == PL_CLOCK_GLOBALTIMER && !(c->ns_per_unit > 0)) return fail(PL_EINVAL, "ns_per_unit must be > 0");
   if (c->n_streams < 1 || c->n_streams > (1u << 20)) return fail(PL_EINVAL, "n_streams %u", c->n_streams);
+  if (c->flags & PL_CLUSTER_NODES) {   // N4: one node per CTA of an N-CTA cluster
+    if (c->policy == PL_MONOLITHIC) return fail(PL_EINVAL, "PL_CLUSTER_NODES: enforced policies only (one processor per node)");
+    if (N > 8) return fail(PL_EINVAL, "PL_CLUSTER_NODES: N = %u exceeds the portable cluster size 8", N);
+    if (v > 256) return fail(PL_EINVAL, "PL_CLUSTER_NODES: v must be <= 256");
+  }
   bool dna = is_dna(c->stages[0].kind);
   for (uint32_t i = 0; i < N; ++i) {
     const pl_stage& s = c->stages[i];
@@ -863,6 +868,7 @@ pl_status pl_pipeline_live_start(pl_pipeline* pl, uint32_t ring_words) {
   if (!pl->dna) return fail(PL_EINVAL, "live ingest is for DNA pipelines (items are DB words)");
   if (pl->live) return fail(PL_ESTATE, "a live run is already executing");
   if (pl->d_arr) return fail(PL_EINVAL, "live ingest takes arrivals at r * tau0 (no arrival array)");
+  if (pl->cfg.flags & PL_CLUSTER_NODES) return fail(PL_EINVAL, "live ingest runs one CTA per stream (not PL_CLUSTER_NODES)");
   cudaSetDevice(pl->device);
   const uint32_t S = pl->cfg.n_streams;
   int sms = 0;
