@@ -235,7 +235,10 @@ pl_status pl_pipeline_set_stream(pl_pipeline* pl, void* stream);
 /* Append n items from HOST memory: for DNA pipelines `items` holds n bases, 2-bit
  * packed, and the running total must stay <= wl->db_len (every push but the last
  * must be a multiple of 16 bases); the copy to HBM is enqueued on the bound stream
- * before the call returns and `items` may be reused immediately.  For random-gain
+ * and `items` may be reused as soon as the call returns (from page-locked memory the
+ * call waits for the copy -- and so for the work queued before it on the stream).
+ * This is the pre-staged path (one run over a finished stream); live ingest during
+ * a run is pl_pipeline_push_stream / push_all (below).  For random-gain
  * pipelines items must be NULL and n counts roots per stream (<= cfg->n_roots).
  * After pl_pipeline_drain: PL_ESTATE until pl_pipeline_rewind.                  */
 pl_status pl_pipeline_push(pl_pipeline* pl, const void* items, uint64_t n);

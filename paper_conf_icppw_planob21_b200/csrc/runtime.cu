@@ -589,6 +589,11 @@ pl_status pl_pipeline_push(pl_pipeline* pl, const void* items, uint64_t n) {
     cudaSetDevice(pl->device);
     const uint64_t words = (n + 15) / 16;
     CUDA_TRY(cudaMemcpyAsync(pl->d_db + pl->pushed / 16, items, words * 4, cudaMemcpyHostToDevice, pl->stream));
+    // pl.h promises `items` may be reused on return: a copy from pageable memory is staged before
+    // cudaMemcpyAsync returns, one from page-locked memory is not -- wait for that one
+    cudaPointerAttributes at;
+    if (cudaPointerGetAttributes(&at, items) != cudaSuccess) cudaGetLastError();
+    else if (at.type == cudaMemoryTypeHost) CUDA_TRY(cudaStreamSynchronize(pl->stream));
     pl->h2d += words * 4;
     pl->pushed += n;
   } else {

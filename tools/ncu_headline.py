@@ -14,7 +14,7 @@ from plgen import dna as G
 from paper_conf_icppw_planob21_b200 import Pipeline, realtime
 from paper_conf_icppw_planob21_b200._pl import PL_FIXED_SERVICE
 
-src = sys.argv[1] if len(sys.argv) > 1 else "profiles/r02_bench_c4_v1.json"
+src = sys.argv[1] if len(sys.argv) > 1 else "profiles/r02_bench_c4_inject.json"
 b = json.load(open(src))["config"]
 budgets, tau, D, SG, gains = tuple(b["budgets_ns"]), b["tau0_ns"], b["deadline_ns"], b["stall_guard_ns"], tuple(b["gains"])
 base = C.c4()
