@@ -571,7 +571,12 @@ def main():
                          "traffic": ncu.get("dram_bytes_per_launch"), "peak_source": pk_src,
                          "algorithmic_bytes_per_launch": bytes_per_launch,
                          "note": "0.25 B per root (2-bit DB) + 24 B per match; the path is not HBM-bound by design"},
-            "issue": {k: ncu[k] for k in ("issue_active_pct", "warp_inst_per_launch", "sm_throughput_pct") if k in ncu},
+            # the executor's issue-slot use from the committed ncu capture of this configuration
+            # (profiles/ncu_summary_<workload>.json): the binding resource of a real-time executor
+            # is issue slots and latency chains, not bytes; util_same_rate compares enforced waiting
+            # with the monolithic baseline at the same (tau0, D)
+            "issue": {k: ncu[k] for k in ("issue_active_pct", "warp_inst_per_launch", "warp_inst_per_root",
+                                          "sm_throughput_pct", "util_same_rate", "source") if k in ncu},
             # the bound that sets the c4 rate: a repeat island turns every seed into u S3 items, which
             # node 3 serves v per t_3, so tau0 >= u t_3 / v during an island
             "rate_bound": {"bound": "node-3 island burst (tau0 >= u t_3 / v)" if c4 else "node-0 service (tau0 >= t_0/v)",
