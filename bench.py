@@ -562,7 +562,13 @@ def main():
             "side": side,
             "per_node": {f"node{i}": {"firings": st["firings"][i], "mean_fire_ns": round(st["busy_ns"][i] / max(1, st["firings"][i])),
                                       "max_fire_ns": st["max_fire_ns"][i], "max_loop_ns": st["max_loop_ns"][i],
-                                      "spilled": st["spilled"][i], "max_queue": st["max_queue"][i]}
+                                      "spilled": st["spilled"][i], "max_queue": st["max_queue"][i],
+                                      # scheduler overhead per firing (north_star): leader-lane clock64
+                                      # cycles deciding (phase 0) and reserving/publishing (3, 5)
+                                      "sched_cycles_per_firing": round(st["phase_cycles"][i][0] / max(1, st["firings"][i])),
+                                      "publish_cycles_per_firing": round((st["phase_cycles"][i][3] + st["phase_cycles"][i][5])
+                                                                         / max(1, st["firings"][i])),
+                                      "stage_scan_cycles_per_firing": round(st["phase_cycles"][i][2] / max(1, st["firings"][i]))}
                          for i in range(st["n_stages"])},
             "clocks": clk,
             "e2e": e2e,

@@ -910,6 +910,20 @@ __device__ __forceinline__ bool nap_until(uint64_t target) {
 // only for the poll that decides the firing; yielded time is usable).
 constexpr uint64_t PL_NAP_LEAD_NS = 768;
 
+// THRESHOLD_SLACK on the physical clock: a node whose next firing cannot start before logical
+// time lb = max(B, min(Tk, W_up)) -- nothing it has queued can fire earlier, and anything its
+// upstream has not yet published is ready at >= W_up -- sleeps until PL_NAP_LEAD_NS before
+// T0 + lb instead of polling every t_i / 8: its upstream's commit publishes W_up one firing
+// ahead, so an idle node behind node 0 sleeps a whole node-0 period at a time (PAPER.md L75/L85:
+// the waiting node's time is yielded).  At most one nap per distinct lb (`napped`); a node that
+// is behind its schedule (T0 + lb already past) polls as before.
+__device__ __forceinline__ bool nap_to(const Node& nd, uint64_t T0, int64_t lb, int64_t& napped) {
+  if (!nd.phys || lb == napped || lb == PL_INF64) return false;
+  napped = lb;
+  const uint64_t due = T0 + units_ns(nd, lb);
+  return due > T0 + PL_NAP_LEAD_NS && nap_until(due - PL_NAP_LEAD_NS);
+}
+
 // A node may commit a firing at T before its upstream watermark passes T once v entries with
 // ready <= T are queued (the firing is full whatever else arrives).  On the logical clock it
 // does so only when the producer is stalled on this queue -- needed for deadlock freedom,
@@ -981,7 +995,9 @@ __device__ Decision decide(const Node& nd, Leader& L, bool& waited, uint64_t T0)
     // THRESHOLD_SLACK
     if (!any) {
       if (Wup == PL_INF64) { d.done = true; return d; }
-      publish_W(nd, L, (Wup > L.B ? Wup : L.B) + nd.t);
+      const int64_t lb = Wup > L.B ? Wup : L.B;
+      publish_W(nd, L, lb + nd.t);
+      if (nap_to(nd, T0, lb, napped)) { waited = true; spins = 0; continue; }
       backoff(spins, nd.phys, nd.nap_cap_ns); waited = true;
       continue;
     }
@@ -1015,6 +1031,7 @@ __device__ Decision decide(const Node& nd, Leader& L, bool& waited, uint64_t T0)
     int64_t lb = Tk < Wup ? Tk : Wup;
     if (lb < L.B) lb = L.B;
     publish_W(nd, L, lb + nd.t);
+    if (nap_to(nd, T0, lb, napped)) { waited = true; spins = 0; continue; }
     backoff(spins, nd.phys, nd.nap_cap_ns); waited = true;
   }
 }

@@ -1,0 +1,76 @@
+"""N3 (PAPER.md L75, L85 — the processor time a waiting node yields can serve other
+work): a compute-bound co-runner kernel (tools/corunner/corunner.cu, its own small library, not
+part of libplgpu.so) runs on a second stream on every SM beside the physical-clock executor.
+
+Co-residence moves time, never the schedule: the executor's matches, traces, model latencies and
+firing log stay bit-exact with the oracle, and the co-runner finishes with its exact result while
+enforced waiting leaves it most of its standalone throughput (profiles/r01_corunner_n3.txt:
+90-97 % at 1-2 co-runner CTAs per SM)."""
+import ctypes
+
+import numpy as np
+import pytest
+
+from plgen import configs as C
+from parity import compare, run_oracle, workload_for
+
+pytestmark = pytest.mark.gpu
+
+ITERS = 4000
+
+
+def _corunner():
+    import os
+    from paper_conf_icppw_planob21_b200.build import build_corunner
+    lib = ctypes.CDLL(build_corunner())
+    assert os.path.exists(lib._name)
+    return lib
+
+
+def _launch(lib, stream, n_ctas, sink):
+    assert lib.pl_corunner_launch(ctypes.c_void_p(stream.cuda_stream), n_ctas, ITERS,
+                                  ctypes.c_void_p(sink.data_ptr())) == 0
+
+
+def test_corunner_beside_enforced_executor():
+    import torch
+    from paper_conf_icppw_planob21_b200 import Pipeline
+    lib = _corunner()
+    cfg = C.c2(n_streams=148, vector_width=64, dna=dict(db_len=1 << 20, q_len=1024, n_planted=64)).replace(
+        clock=C.CLOCK_GLOBALTIMER, ns_per_unit=1.0, service_time=(20_000,) * 4, interarrival=300,
+        deadline=10_000_000, policy=C.THRESHOLD_SLACK, wait_threshold=(64, 64, 50, 5))
+    wl = workload_for(cfg)
+    n_ctas = 148
+    sA, sB = torch.cuda.Stream(), torch.cuda.Stream()
+    # the co-runner alone (its result is the reference for the co-resident run)
+    ref = torch.zeros(n_ctas * 16, dtype=torch.float32, device="cuda")
+    _launch(lib, sB, n_ctas, ref)
+    torch.cuda.synchronize()
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    sink = torch.zeros_like(ref)
+    e0.record(sB)
+    _launch(lib, sB, n_ctas, sink)
+    e1.record(sB)
+    torch.cuda.synchronize()
+    alone_ms = e0.elapsed_time(e1)
+    # beside the executor
+    pl = Pipeline(cfg, wl, flags=7, stream=sA)
+    pl.push(wl.db, wl.db_len)
+    torch.cuda.synchronize()
+    pl.launch()
+    sink2 = torch.zeros_like(ref)
+    f0, f1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    f0.record(sB)
+    _launch(lib, sB, n_ctas, sink2)
+    f1.record(sB)
+    pl.drain()
+    torch.cuda.synchronize()
+    beside_ms = f0.elapsed_time(f1)
+    g = dict(stats=pl.stats(), matches=pl.results(), trace=pl.trace(), firings=pl.firings())
+    g["lat"], g["lat_ns"] = pl.latency()
+    pl.close()
+    compare(cfg, g, run_oracle(cfg, wl))
+    assert torch.equal(sink2, ref) and bool(torch.isfinite(ref).all()) and float(ref.abs().sum()) > 0
+    print("co-runner alone", alone_ms, "ms, beside the executor", beside_ms, "ms; executor hw busy",
+          g["stats"]["hw_busy_fraction"])
+    assert alone_ms / beside_ms > 0.5

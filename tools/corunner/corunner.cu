@@ -16,7 +16,7 @@ __global__ void __launch_bounds__(128) pl_corunner_kernel(uint64_t iters, float*
   float s = 0;
 #pragma unroll
   for (int j = 0; j < 8; ++j) s += a[j];
-  if (s == 12345.f) sink[blockIdx.x] = s;
+  if (threadIdx.x == 0) sink[blockIdx.x] = s;   // the result, so a co-resident run can be checked exactly
 }
 
 extern "C" int pl_corunner_launch(void* stream, uint32_t n_ctas, uint64_t iters, float* sink) {
