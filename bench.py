@@ -86,6 +86,9 @@ def parse():
                     help="rate searches inject a platform-length stall every this many ms "
                          "(pl_pipeline_inject_stalls; default: c4 100, c2 off)")
     ap.add_argument("--inject-ms", type=float, default=1.8, help="length of an injected stall (R-STALL: ~1.6 ms)")
+    ap.add_argument("--probe-t", type=int, default=None,
+                    help="budget probe: every node's budget during the probe (ns; default c4 1000 = all nodes "
+                         "overloaded, sharing the SM as in a catch-up, L69's 1/N share; c2 20000)")
     ap.add_argument("--headroom", type=float, default=1.0,
                     help="operating tau0 = headroom x the fastest stall-free miss-free tau0 (R-STALL: the "
                          "pipeline must catch up after a ~1.6 ms platform stall within D)")
@@ -276,7 +279,7 @@ def main():
     # pipeline recovering from a platform stall runs exactly like that.
     budgets, cal = realtime.calibrate_budgets(base, wl, db_ptr, stream=stream, margin=a.budget_margin,
                                               slack_ns=a.budget_slack, probe_tau=20 if c4 else 100, over=over,
-                                              probe_t=1000 if c4 else 20_000)
+                                              probe_t=a.probe_t or (1000 if c4 else 20_000))
     # misses count against D; the schedules are solved at D - SG (R-STALL) and THRESHOLD_SLACK
     # reserves SG in every R_i on top of the largest budget
     cfg0 = base.replace(clock=1, ns_per_unit=1.0, service_time=budgets, gain=gains, deadline=D,
@@ -540,7 +543,8 @@ def main():
                        "stall_injection_in_rate_search": ({"period_ms": a.inject_period_ms, "len_ms": a.inject_ms}
                                                           if inject else None),
                        "tau0_edge_ns": tau_edge, "edge_items_per_s": world * a.streams * 1e9 / tau_edge,
-                       "b": list(C.PAPER_B), "budgets_ns": list(budgets), "gains": [round(g, 5) for g in gains],
+                       "b": list(C.PAPER_B), "budgets_ns": list(budgets), "budget_probe_t_ns": a.probe_t or (1000 if c4 else 20_000),
+                       "gains": [round(g, 5) for g in gains],
                        "drain": "eager (R-DRAIN)" if not c4 else "periodic (paper rule)",
                        "streams_per_gpu": a.streams, "roots_per_stream": st["roots"] // a.streams,
                        "arrival_span_ms": st["roots"] / a.streams * tau * 1e-6,

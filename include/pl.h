@@ -206,7 +206,11 @@ typedef struct {
                                               before the stream's last completion, clipped to it */
   double   hw_busy_fraction;               /* physical: busy_ns / (N * wall)           */
   int64_t  wall_ns;                        /* max over streams of kernel-side runtime  */
-  uint32_t errors;                         /* PL_EOVERFLOW bits etc.                   */
+  uint32_t errors;                         /* device error bits (PL_EOVERFLOW at drain): 1 spill ring
+                                              full (physical clock), 2 match buffer full, 4 firing
+                                              log full, 8 segment ring full, 16 live ingest: no
+                                              delivery for 20 s, 32 watchdog: a node waited 30 s
+                                              without progress and gave up                 */
   uint32_t launches;                       /* executor launches so far                 */
   uint64_t h2d_bytes;                      /* host->device bytes copied by this handle (cumulative) */
   uint64_t d2h_bytes;                      /* device->host bytes copied by this handle (cumulative) */

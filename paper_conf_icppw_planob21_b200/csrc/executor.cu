@@ -743,7 +743,19 @@ struct Leader {   // leader-private schedule state of one node
   uint32_t out_tail, out_segt;  // producer side of the output edge
   int64_t W_pub;
   uint64_t empties;
+  uint32_t wd;                  // the watchdog fired (PL_ERR_WATCHDOG)
 };
+
+// Watchdog (SURVEY §5 failure detection): a node that keeps waiting -- for its upstream in
+// decide(), or for room downstream in reserve_out() -- for PL_WATCHDOG_NS of %globaltimer gives
+// up: error bit PL_ERR_WATCHDOG, the node ends (decide) or drops the firing's outputs
+// (reserve_out), so a protocol fault or an abandoned live stream ends the run instead of hanging
+// the GPU.  Checked every 256 spins of a wait, cold.
+__device__ __noinline__ bool watchdog_expired(uint64_t& t0) {
+  const uint64_t now = gtimer();
+  if (t0 == 0) { t0 = now; return false; }
+  return now - t0 > PL_WATCHDOG_NS;
+}
 
 __device__ __forceinline__ void publish_W(const Node& nd, Leader& L, int64_t w) {
   if (nd.sink) return;
@@ -937,7 +949,9 @@ __device__ Decision decide(const Node& nd, Leader& L, bool& waited, uint64_t T0)
   d.done = false; d.T = 0; d.n = 0; d.qlen = 0;
   int spins = 0;
   int64_t napped = -1;
+  uint64_t wd0 = 0;
   for (;;) {
+    if ((spins & 255) == 255 && watchdog_expired(wd0)) { L.wd = 1u; publish_W(nd, L, PL_INF64); d.done = true; return d; }
     if (nd.phys && nd.fixed && !(nd.eager && L.m >= nd.Mcap)) {
       const int64_t Tn = L.m * nd.P;
       if (Tn != napped) {
@@ -1042,7 +1056,9 @@ __device__ Decision decide(const Node& nd, Leader& L, bool& waited, uint64_t T0)
 // in physical mode the wait shows up as lateness and, if it matters, as deadline misses.
 __device__ uint32_t reserve_out(const Node& nd, Leader& L, uint32_t worst, uint32_t* stalled) {
   int spins = 0;
+  uint64_t wd0 = 0;
   for (;;) {
+    if ((spins & 255) == 255 && watchdog_expired(wd0)) { L.wd = 2u; return ~0u; }   // outputs dropped
     const uint32_t h = vld(&nd.Eout->head), sh = vld(&nd.Eout->seg_head);
     const bool seg_ok = (L.out_segt - sh) <= nd.segmask;
     const uint32_t need = L.out_tail + worst - h;
@@ -1284,7 +1300,7 @@ __device__ void run_node(Ctx& c, Dna dna, int i, int gtid) {
 
   Leader L;
   L.m = 0; L.B = 0; L.c0 = 0; L.head = 0; L.segh = 0; L.out_tail = 0; L.out_segt = 0;
-  L.W_pub = -1; L.empties = 0;
+  L.W_pub = -1; L.empties = 0; L.wd = 0;
   Rep R;
   R.m = 0; R.B = 0; R.c0 = 0; R.empties = 0; R.qT = 0; R.rT = 0; R.qvalid = false;
   auto clamp32 = [](int64_t x) { return (uint32_t)(x > 0 ? (x < 0xffffffffll ? x : 0xffffffffll) : 0); };
@@ -1688,6 +1704,7 @@ __device__ void run_node(Ctx& c, Dna dna, int i, int gtid) {
     par ^= 1;
   }
   if (nd.sliding && leader) vst(nd.bnd_me, 0xffffffffu);   // reads nothing more
+  if (leader && L.wd) atomicOr(&AG.errors, PL_ERR_WATCHDOG);
   if (n0) {
     if (leader) publish_W(nd, L, PL_INF64);   // after the last segment was published
     bar_sync(bidA, v);                   // the last publish time is visible to every lane

@@ -16,6 +16,8 @@
 #define PL_ERR_SEG_OVERFLOW     8u
 #define PL_ERR_INGEST_TIMEOUT  16u      // live ingest: no delivery for PL_INGEST_TIMEOUT_NS (proceeds on stale data)
 #define PL_INGEST_TIMEOUT_NS   20000000000ull
+#define PL_ERR_WATCHDOG        32u      // a node waited PL_WATCHDOG_NS without progress and gave up
+#define PL_WATCHDOG_NS         30000000000ull
 
 struct DevStage {
   uint32_t kind, max_out;

@@ -501,7 +501,10 @@ pl_status pl_pipeline_create(const pl_config* cfg, const pl_workload* wl, pl_pip
   // one CTA (stream) per SM: the two-per-SM variant (64 registers) spills and measured no gain
   // (tools/streams_scaling.py); it stays selectable through PL_CTAS_PER_SM=2
   d.ctas_per_sm = 1;
-  d.variant = 0;
+  // bit 1: node 0's leader paces and one barrier releases its lanes (instead of every warp
+  // pacing itself): on c4 the executor issues 17 % fewer instructions at the same rate
+  // (ncu, profiles/r02_bench_ab_leader_paced.json); PL_VARIANT overrides the experiment bits
+  d.variant = 1u;
   if (const char* e = getenv("PL_VARIANT")) d.variant = (uint32_t)atoi(e);
   // physical clock: a stream's time origin is set this far after its CTA has staged its
   // inputs, so that every warp group is resident before the first arrival
@@ -1021,7 +1024,7 @@ pl_status pl_pipeline_drain(pl_pipeline* pl) {
   pl->d2h += cs.size() * sizeof(CtaStats);
   uint32_t err = 0;
   for (auto& s : cs) err |= s.errors;
-  if (err) return fail(PL_EOVERFLOW, "device reported overflow bits 0x%x (queue=1 match=2 log=4 seg=8)", err);
+  if (err) return fail(PL_EOVERFLOW, "device reported overflow bits 0x%x (queue=1 match=2 log=4 seg=8 ingest-timeout=16 watchdog=32)", err);
   return PL_OK;
 }
 

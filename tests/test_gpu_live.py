@@ -175,3 +175,14 @@ def test_live_c4_sampled_streams():
         ok = (lat >= 0) & (np.arange(hi2 - lo) * cfg.interarrival + lat < A)
         assert ok.sum() > 5_000
         assert np.array_equal(g["lat"][lo:hi2][ok], lat[ok]), s
+
+
+@pytest.mark.parametrize("db_len,streams", [(6, 2), (64, 4), (1000, 3)])
+def test_live_tiny_and_empty_streams(db_len, streams):
+    """Degenerate live streams: a DB of one root over two streams (stream 0 has no root and no
+    words to push), and streams shorter than a word, a chunk and the halo; bit-exact."""
+    cfg = _dna(C.THRESHOLD_SLACK, db_len=db_len, streams=streams).replace(
+        dna=dict(db_len=db_len, q_len=64, n_planted=0))
+    wl = workload_for(cfg)
+    g = run_live(cfg, wl, slice_words=3)
+    compare(cfg, g, run_oracle(cfg, wl))
