@@ -81,7 +81,7 @@ class pl_stats(C.Structure):
                 ("launches", C.c_uint32), ("h2d_bytes", C.c_uint64), ("d2h_bytes", C.c_uint64),
                 ("window_refills", C.c_uint64), ("latency_outliers", C.c_uint64),
                 ("latency_rel_err_max", C.c_double), ("ingest_waits", C.c_uint64),
-                ("max_ingest_wait_ns", C.c_int64)]
+                ("max_ingest_wait_ns", C.c_int64), ("batched_firings", _A8)]
 
     def as_dict(self):
         N = self.n_stages
