@@ -567,7 +567,6 @@ def main():
             "per_node": {f"node{i}": {"firings": st["firings"][i], "mean_fire_ns": round(st["busy_ns"][i] / max(1, st["firings"][i])),
                                       "max_fire_ns": st["max_fire_ns"][i], "max_loop_ns": st["max_loop_ns"][i],
                                       "spilled": st["spilled"][i], "max_queue": st["max_queue"][i],
-                                      "batched_firings": st["batched_firings"][i],
                                       # scheduler overhead per firing (north_star): leader-lane clock64
                                       # cycles deciding (phase 0) and reserving/publishing (3, 5)
                                       "sched_cycles_per_firing": round(st["phase_cycles"][i][0] / max(1, st["firings"][i])),

@@ -223,9 +223,6 @@ typedef struct {
   double   latency_rel_err_max;            /* largest |err| / logical latency over terminal items      */
   uint64_t ingest_waits;                   /* live ingest: node-0 firings / blocks that waited for words */
   int64_t  max_ingest_wait_ns;             /* live ingest: the longest such wait                        */
-  uint64_t batched_firings[PL_MAX_STAGES]; /* physical clock, catching up: vectors that carried two of
-                                              the node's logical firings (the schedule, outputs and
-                                              every other counter are the two firings')                */
 } pl_stats;
 
 typedef struct pl_pipeline pl_pipeline;

@@ -81,7 +81,7 @@ class pl_stats(C.Structure):
                 ("launches", C.c_uint32), ("h2d_bytes", C.c_uint64), ("d2h_bytes", C.c_uint64),
                 ("window_refills", C.c_uint64), ("latency_outliers", C.c_uint64),
                 ("latency_rel_err_max", C.c_double), ("ingest_waits", C.c_uint64),
-                ("max_ingest_wait_ns", C.c_int64), ("batched_firings", _A8)]
+                ("max_ingest_wait_ns", C.c_int64)]
 
     def as_dict(self):
         N = self.n_stages
@@ -135,7 +135,11 @@ def _load():
                                        C.POINTER(C.c_uint64), C.POINTER(C.c_uint64)]),
     }
     for name, (res, args) in sig.items():
-        fn = getattr(lib, name)
+        fn = getattr(lib, name, None)
+        if fn is None and os.environ.get("PLGPU_LIB"):   # an older experiment build (tools/): skip
+            continue
+        if fn is None:
+            raise ImportError(f"{LIB_PATH} lacks {name}: rebuild it")
         fn.restype = res
         fn.argtypes = args
     return lib

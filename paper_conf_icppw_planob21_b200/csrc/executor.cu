@@ -305,23 +305,15 @@ struct GroupCtl {           // broadcast from a node's leader to its lanes, doub
   uint32_t n[2], head[2], done[2], segh[2], st[2], log_idx[2];
   uint32_t in_spill_end[2]; // input edge: end seq of its last spilled segment
   uint32_t out_base[2], out_loc[2];
-  // catch-up batching (merge_next): a physical firing that carries two logical firings --
-  // lanes [0, n1) the first (start T), lanes [n1, n) the second (start T2); n1 = 0: one firing
-  int64_t  T2[2];
-  uint64_t end2_ns[2];      // delivery time of the second logical firing's terminal items
-  uint32_t n1[2], split[2]; // split: outputs of the first logical firing (set by lane n1)
   alignas(16) uint32_t wtot[2][8];
   alignas(16) uint32_t rmin[8];   // per warp: smallest terminal root of the current firing
   alignas(16) uint32_t rmax[8];   // per warp: largest terminal root + 1 (0: none; physical clock only)
-  alignas(16) uint32_t rmin2[8];  // the same for the second logical firing of a batched one
-  alignas(16) uint32_t rmax2[8];
 };
 // Leader-only per-node accumulators, in smem so that they take no registers in the node loop.
 // 64-bit shared atomics compile to CAS spin loops (ATOMS.CAST.SPIN.64), so the single writer
 // stores per-firing 32-bit deltas (d[]) as it goes and folds everything into the 64-bit sums
 // with one vectorised read-modify-write per firing; maxima use native 32-bit ATOMS.MAX.
-enum { C_FIRINGS, C_CONSUMED, C_PRODUCED, C_ACTIVE, C_BUSY, C_OVERRUNS, C_SPILLED, C_STALLS, C_ACTIVE_E, C_DRAINF,
-       C_BATCHED, C_N };
+enum { C_FIRINGS, C_CONSUMED, C_PRODUCED, C_ACTIVE, C_BUSY, C_OVERRUNS, C_SPILLED, C_STALLS, C_ACTIVE_E, C_DRAINF, C_N };
 enum { D_PH0, D_PH1, D_PH2, D_PH3, D_STALL, D_N = 8 };
 struct NodeAcc {
   alignas(16) unsigned long long cnt[C_N];
@@ -1062,13 +1054,13 @@ __device__ Decision decide(const Node& nd, Leader& L, bool& waited, uint64_t T0)
 // stage runs so that no extra barrier is needed).  Returns the location.  A full queue
 // back-pressures the producer in both clock modes (deadlock-free):
 // in physical mode the wait shows up as lateness and, if it matters, as deadline misses.
-__device__ uint32_t reserve_out(const Node& nd, Leader& L, uint32_t worst, uint32_t* stalled, uint32_t nseg = 1) {
+__device__ uint32_t reserve_out(const Node& nd, Leader& L, uint32_t worst, uint32_t* stalled) {
   int spins = 0;
   uint64_t wd0 = 0;
   for (;;) {
     if ((spins & 255) == 255 && watchdog_expired(wd0)) { L.wd = 2u; return ~0u; }   // outputs dropped
     const uint32_t h = vld(&nd.Eout->head), sh = vld(&nd.Eout->seg_head);
-    const bool seg_ok = (L.out_segt + nseg - 1u - sh) <= nd.segmask;
+    const bool seg_ok = (L.out_segt - sh) <= nd.segmask;
     const uint32_t need = L.out_tail + worst - h;
     if (seg_ok && need <= nd.out_cap) { if (*stalled) vst(&nd.Eout->stalled, 0u); return LOC_SMEM; }
     if (seg_ok && need <= nd.capg) { if (*stalled) vst(&nd.Eout->stalled, 0u); return LOC_SPILL; }
@@ -1276,52 +1268,6 @@ __device__ __forceinline__ uint32_t live_need(const Shared& sh, const DevParams&
   return min(sh.win.whi, (uint32_t)(((uint64_t)p_last + (uint32_t)p.k + p.win_halo) >> 4) + 1u);
 }
 
-// Catch-up batching (physical clock, THRESHOLD_SLACK, nodes >= 1).  After a stall (R-STALL) a
-// node replays its logical firings back to back, each on its own SIMD vector although they are
-// often far from full (θ_3 = 2 on c4: node 3 fires as soon as it is idle).  When the node has
-// decided firing (T1, n1) and is already late for the firing that follows, peek_next computes
-// that next decision now -- decide()'s THRESHOLD_SLACK rules on the state firing (T1, n1) leaves:
-// head + n1, busy until T1 + t_i -- without waiting or publishing; if it is final (the same test
-// decide() applies), due, and both fit in v lanes, the two logical firings run on one vector
-// (lanes [0, n1) and [n1, n)) and publish two segments with their own ready times.  The logical
-// schedule, every output and every statistic are those of the two firings; only the physical
-// catch-up is faster.  Never on the logical clock or with R-DRAIN; PL_VARIANT bit 8 disables it.
-__device__ __forceinline__ bool peek_next(const Node& nd, const Leader& L0, int64_t T1, uint32_t n1, Decision& d2) {
-  Leader L = L0;
-  L.B = T1 + nd.t;
-  L.head = L0.head + n1;
-  const int64_t Wup = vld(&nd.Ein->W);
-  fence_q(nd.cl);
-  const uint32_t st = vld(&nd.Ein->seg_tail);
-  while (L.segh != st && (int32_t)(nd.in_seg[L.segh & nd.segmask].end - L.head) <= 0) ++L.segh;
-  const uint32_t tail_known = (st != L.segh) ? nd.in_seg[(st - 1) & nd.segmask].end : L.head;
-  if (tail_known == L.head) return false;
-  const Seg& hs = nd.in_seg[L.segh & nd.segmask];
-  fence_q(nd.cl);
-  const uint2 he = load_entry(nd, L.head, L.segh, st, vld(&nd.Ein->spill_end));
-  int64_t Tf = nd.arrival(he.x) + nd.D - nd.R;
-  if (Tf < hs.ready) Tf = hs.ready;
-  const uint32_t kth = L.head + nd.theta - 1;
-  const bool th_known = (int32_t)(tail_known - kth) > 0;
-  int64_t Tth = PL_INF64;
-  if (th_known) {
-    for (uint32_t k = L.segh; k != st; ++k) {
-      const Seg& sg = nd.in_seg[k & nd.segmask];
-      if ((int32_t)(sg.end - kth) > 0) { Tth = sg.ready; break; }
-    }
-  }
-  int64_t Tk = Tth < Tf ? Tth : Tf;
-  if (Tk < L.B) Tk = L.B;
-  if (!(th_known || Tk < Wup)) return false;
-  const uint32_t cnt = count_le(nd, L, st, Tk);
-  if (!(Wup > Tk || cnt >= (uint32_t)nd.v)) return false;   // physical clock: early_ok
-  d2.done = false;
-  d2.T = Tk;
-  d2.n = cnt < (uint32_t)nd.v ? cnt : (uint32_t)nd.v;
-  d2.qlen = count_all_le(nd, L, st, Tk);
-  return true;
-}
-
 // ------------------------------------------------------------------- node loop
 // One warp group of v threads per node, one item per lane.  Measured faster on B200 than
 // one warp with v/32 items per lane: the group's warps run the per-item latency chains in
@@ -1360,7 +1306,6 @@ __device__ void run_node(Ctx& c, Dna dna, int i, int gtid) {
   auto clamp32 = [](int64_t x) { return (uint32_t)(x > 0 ? (x < 0xffffffffll ? x : 0xffffffffll) : 0); };
   uint64_t start_ns = 0;
   uint32_t pend_root = NO_ROOT;          // lane: physical terminal event awaiting its end time (REC)
-  bool pend2 = false;                    // ... of the second logical firing of a batched one
   long long tc = 0;
   int par = 0;
   if (leader) {
@@ -1377,8 +1322,6 @@ __device__ void run_node(Ctx& c, Dna dna, int i, int gtid) {
   for (;;) {
     int64_t T;
     uint32_t n, head;                    // n: items consumed (node 0 with arrival data: from the scan)
-    uint32_t n1 = 0;                     // catch-up batching: lanes [0, n1) fire at T, [n1, n) at T2
-    int64_t T2 = 0;
     if (n0) {
       const long long c0 = leader ? clock64() : 0;
       const Decision d = decide0(nd, R);
@@ -1435,30 +1378,18 @@ __device__ void run_node(Ctx& c, Dna dna, int i, int gtid) {
         bool waited = false;             // the decision waited for upstream (no service-time sample)
         const Decision d = decide(nd, L, waited, T0);
         atomicMax(&A.max_queue, d.qlen);
-        uint32_t nb = 0;                 // catch-up batching: the second logical firing's size
-        if (!d.done && nd.phys && !nd.fixed && !nd.eager && !(p.variant & 8u) && d.n < (uint32_t)v &&
-            gtimer() > T0 + units_ns(nd, d.T + nd.t)) {   // late by more than a service time
-          Decision d2;
-          if (peek_next(nd, L, d.T, d.n, d2) && d.n + d2.n <= (uint32_t)v && gtimer() >= T0 + units_ns(nd, d2.T)) {
-            nb = d2.n;
-            G.T2[par] = d2.T;
-            atomicMax(&A.max_queue, d2.qlen);
-          }
-        }
-        G.n1[par] = nb ? d.n : 0u;
         G.done[par] = d.done ? 1u : 0u;
         G.T[par] = d.T;
-        G.n[par] = d.n + nb;
+        G.n[par] = d.n;
         G.head[par] = L.head;
         G.segh[par] = L.segh;
         G.st[par] = vld(&nd.Ein->seg_tail);
         fence_q(nd.cl);
         G.in_spill_end[par] = vld(&nd.Ein->spill_end);
         if (!d.done) {
-          if (rec & PL_REC_FIRINGS) G.log_idx[par] = atomicAdd(&AG.log_count, nb ? 2u : 1u);
+          if (rec & PL_REC_FIRINGS) G.log_idx[par] = atomicAdd(&AG.log_count, 1u);
           A.d[par][D_STALL] = 0;
-          G.out_loc[par] = nd.sink ? LOC_SMEM
-                                   : reserve_out(nd, L, (d.n + nb) * nd.umax, &A.d[par][D_STALL], nb ? 2u : 1u);
+          G.out_loc[par] = nd.sink ? LOC_SMEM : reserve_out(nd, L, d.n * nd.umax, &A.d[par][D_STALL]);
           G.out_base[par] = L.out_tail;
         } else {
           publish_W(nd, L, PL_INF64);
@@ -1478,11 +1409,9 @@ __device__ void run_node(Ctx& c, Dna dna, int i, int gtid) {
       bar_sync(bidA, v);                                               // B1: decision
       if (leader) { const long long t2 = clock64(); A.d[par][D_PH1] = (uint32_t)(t2 - tc); tc = t2; }
       if (REC && pend_root != NO_ROOT)   // deferred physical latency of the previous firing
-        record_lat_ns(nd, c, T0, pend2 ? G.end2_ns[par ^ 1] : G.end_ns[par ^ 1], pend_root);
+        record_lat_ns(nd, c, T0, G.end_ns[par ^ 1], pend_root);
       if (G.done[par]) break;
       T = G.T[par]; n = G.n[par]; head = G.head[par];
-      n1 = G.n1[par];
-      if (n1) T2 = G.T2[par];
     }
     const bool arrmode = n0 && nd.arr != nullptr;
     const bool act = arrmode ? ((uint32_t)gtid < n && R.c0 + gtid < nd.X &&
@@ -1524,7 +1453,6 @@ __device__ void run_node(Ctx& c, Dna dna, int i, int gtid) {
       off = group_scan(G.wtot[par], o[0].c, &total, gtid, v, bidA, nd.umax <= 1);                 // B2
     }
     const uint32_t out_loc = G.out_loc[par], out_base = G.out_base[par];   // leader's reservation (B2)
-    if (n1 && (uint32_t)gtid == n1) G.split[par] = off;   // outputs of the first logical firing
     if (nd.sliding && n0 && leader) vst(nd.bnd_me, (uint32_t)(nd.lo + head));   // every lane is past the last firing
     if (leader) { const long long t2 = clock64(); A.d[par][D_PH2] = (uint32_t)(t2 - tc); tc = t2; }
     if (REC && n0 && pend_root != NO_ROOT)   // node 0: the previous publish time came through B2
@@ -1542,28 +1470,22 @@ __device__ void run_node(Ctx& c, Dna dna, int i, int gtid) {
     const uint2 ei = e[0];
     const LaneOut oi = o[0];
     const bool term = act && (nd.sink || oi.c == 0);
-    const bool second = n1 && (uint32_t)gtid >= n1;   // this lane belongs to the second logical firing
     if (REC && (rec & 7u)) {              // optional per-item records (parity / tracing runs)
-      const int64_t Tl = second ? T2 : T;
       if (act && (rec & PL_REC_TRACE)) {
         atomicAdd(&p.trace[(uint64_t)ei.x * (N + 1) + i], 1u);
         if (nd.sink && oi.c) atomicAdd(&p.trace[(uint64_t)ei.x * (N + 1) + N], oi.c);
       }
       if (term && (rec & PL_REC_LATENCY)) {
-        atomicMax((long long*)&p.lat[ei.x], (long long)(Tl + nd.t - nd.arrival(ei.x)));
-        if (nd.phys) { pend_root = ei.x; pend2 = second; }
+        atomicMax((long long*)&p.lat[ei.x], (long long)(T + nd.t - nd.arrival(ei.x)));
+        if (nd.phys) pend_root = ei.x;
       }
-      const uint32_t f0 = second ? n1 : 0u, f1 = (n1 && !second) ? n1 - 1u : n - 1u;   // this lane's record
-      if (act && (rec & PL_REC_FIRINGS) && ((uint32_t)gtid == f0 || (uint32_t)gtid == f1)) {
-        const uint32_t li = G.log_idx[par] + (second ? 1u : 0u);
+      if (act && (rec & PL_REC_FIRINGS) && (gtid == 0 || (uint32_t)gtid == n - 1)) {
+        const uint32_t li = G.log_idx[par];
         if (li < p.log_cap) {
           pl_firing* f = p.flog + (uint64_t)stream * p.log_cap + li;
-          if ((uint32_t)gtid == f0) {
-            f->start = Tl; f->node = i; f->n = n1 ? (second ? n - n1 : n1) : n; f->first_root = ei.x;
-            f->stream = stream; f->pad = 0;
-          }
-          if ((uint32_t)gtid == f1) f->last_root = ei.x;
-        } else if ((uint32_t)gtid == f0) {
+          if (gtid == 0) { f->start = T; f->node = i; f->n = n; f->first_root = ei.x; f->stream = stream; f->pad = 0; }
+          if ((uint32_t)gtid == n - 1) f->last_root = ei.x;
+        } else if (gtid == 0) {
           atomicOr(&AG.errors, PL_ERR_LOG_OVERFLOW);
         }
       }
@@ -1574,16 +1496,11 @@ __device__ void run_node(Ctx& c, Dna dna, int i, int gtid) {
         // them after the publish (and counts misses root by root only when one exceeds D).
       const uint32_t tr = term ? ei.x : NO_ROOT;
       nd.troot[gtid] = tr;
-      const uint32_t wmin = __reduce_min_sync(0xffffffffu, second ? NO_ROOT : tr);
+      const uint32_t wmin = __reduce_min_sync(0xffffffffu, tr);
       if ((gtid & 31) == 0) G.rmin[gtid >> 5] = wmin;
       if (nd.phys) {                     // the latest-arriving terminal root: smallest logical latency
-        const uint32_t wmax = __reduce_max_sync(0xffffffffu, (term && !second) ? ei.x + 1u : 0u);
+        const uint32_t wmax = __reduce_max_sync(0xffffffffu, term ? ei.x + 1u : 0u);
         if ((gtid & 31) == 0) G.rmax[gtid >> 5] = wmax;
-        if (n1) {                        // a batched firing: the second logical firing's extremes
-          const uint32_t wmin2 = __reduce_min_sync(0xffffffffu, second ? tr : NO_ROOT);
-          const uint32_t wmax2 = __reduce_max_sync(0xffffffffu, (term && second) ? ei.x + 1u : 0u);
-          if ((gtid & 31) == 0) { G.rmin2[gtid >> 5] = wmin2; G.rmax2[gtid >> 5] = wmax2; }
-        }
       }
     }
     if (nd.sink && nd.kind == PL_UNGAPPED_XDROP) {   // matches: one global atomic per warp
@@ -1637,40 +1554,26 @@ __device__ void run_node(Ctx& c, Dna dna, int i, int gtid) {
       ulonglong2* Cp = reinterpret_cast<ulonglong2*>(A.cnt);
       ulonglong2* Pp = reinterpret_cast<ulonglong2*>(A.ph);
       ulonglong2 c2 = Cp[2], p2 = Pp[2];
-      uint64_t en = 0, fire = 0, done_ns = 0;
-      const int64_t Tlast = n1 ? T2 : T;  // a batched firing ends with its second logical firing
+      uint64_t en = 0, fire = 0;
       if (nd.phys) {
         en = gtimer();
-        done_ns = en;
         fire = en - start_ns;
         // PL_FIXED_SERVICE: time-triggered delivery -- the firing holds its processor and delivers
         // its terminal items at start + t_i (L69), or when done if later.  Its outputs are
         // published now: downstream consumes them at logical times >= T + t_i anyway (the
         // segment's ready time), and an early publish only lets its scheduler decide sooner.
-        if (rec & PL_FIXED_SERVICE) en = max(en, T0 + units_ns(nd, Tlast + nd.t));
+        if (rec & PL_FIXED_SERVICE) en = max(en, T0 + units_ns(nd, T + nd.t));
       }
-      // publish: the segment (outputs ready at T + t_i) -- two for a batched firing, split at the
-      // first logical firing's outputs -- then the watermark
+      // publish: the segment (outputs ready at T + t_i), then the watermark
       if (!nd.sink && total > 0 && out_loc != ~0u) {
-        const uint32_t s1 = n1 ? G.split[par] : total;
-        uint32_t ns = 0;
-        if (s1 > 0) {
-          Seg sg;
-          sg.ready = T + nd.t;
-          sg.end = L.out_tail + s1;
-          sg.loc = out_loc;
-          nd.out_seg[(L.out_segt + ns++) & nd.segmask] = sg;
-        }
-        if (s1 < total) {
-          Seg sg;
-          sg.ready = T2 + nd.t;
-          sg.end = L.out_tail + total;
-          sg.loc = out_loc;
-          nd.out_seg[(L.out_segt + ns++) & nd.segmask] = sg;
-        }
-        if (out_loc == LOC_SPILL) vst(&nd.Eout->spill_end, L.out_tail + total);
+        Seg sg;
+        sg.ready = T + nd.t;
+        sg.end = L.out_tail + total;
+        sg.loc = out_loc;
+        nd.out_seg[L.out_segt & nd.segmask] = sg;
+        if (out_loc == LOC_SPILL) vst(&nd.Eout->spill_end, sg.end);
         fence_q(nd.cl);
-        L.out_segt += ns;
+        ++L.out_segt;
         L.out_tail += total;
         vst(&nd.Eout->seg_tail, L.out_segt);
         vst(&nd.Eout->tail, L.out_tail);
@@ -1683,17 +1586,16 @@ __device__ void run_node(Ctx& c, Dna dna, int i, int gtid) {
         const int64_t Bn = ef ? T + nd.t : (n0 ? R.B : L.B);
         publish_W(nd, L, (nd.eager && mn >= nd.Mcap ? max(max(nd.B_per, Bn), nd.A_last) : mn * nd.P) + nd.t);
       } else {
-        L.B = Tlast + nd.t;
+        L.B = T + nd.t;
         publish_W(nd, L, L.B + nd.t);
       }
       if (nd.phys) {
-        G.end_ns[par] = n1 && (rec & PL_FIXED_SERVICE) ? max(done_ns, T0 + units_ns(nd, T + nd.t)) : en;
-        G.end2_ns[par] = en;
+        G.end_ns[par] = en;
         atomicMax(&A.max_fire, clamp32((int64_t)fire));
       }
       // measured busy time, overruns, publish-phase cycles (the leader's slots of the sums)
       c2.x += nd.phys ? (en - start_ns) : 0ull;
-      c2.y += (nd.phys && (int64_t)fire > (n1 ? 2 : 1) * nd.t_ns) ? 1ull : 0ull;   // work outlasted t_i (per logical firing)
+      c2.y += (nd.phys && (int64_t)fire > nd.t_ns) ? 1ull : 0ull;   // work outlasted t_i
       p2.x += ph4;
       p2.y += (uint64_t)(clock64() - t4);
       Cp[2] = c2; Pp[2] = p2;
@@ -1703,78 +1605,70 @@ __device__ void run_node(Ctx& c, Dna dna, int i, int gtid) {
     // deltas A.d[par] were ordered before B4, and the next writes of each come after this
     // warp has reached the next firing's scan barrier (A.d is double-buffered by parity).
     if (v > 32 ? gtid == 32 : leader) {
-      const uint64_t done = nd.phys ? gtimer() : 0ull;   // completion time of the terminal items
-      A.t_end = (n1 ? T2 : T) + nd.t;    // firing starts increase: the last one ends last
-      // one pass per logical firing (two for a batched one): lanes [klo, khi), start Ts
-      for (int sub = 0; sub < (n1 ? 2 : 1); ++sub) {
-        const int64_t Ts = sub ? T2 : T;
-        const uint32_t klo = sub ? n1 : 0u, khi = (n1 && !sub) ? n1 : n;
-        const uint32_t* gmin = sub ? G.rmin2 : G.rmin;
-        const uint32_t* gmax = sub ? G.rmax2 : G.rmax;
-        uint64_t en = done;
-        if (nd.phys && (rec & PL_FIXED_SERVICE)) en = max(en, T0 + units_ns(nd, Ts + nd.t));   // delivery at start + t_i
-        // the smallest terminal root has the largest latency
-        uint32_t rmin;
-        {
-          const uint4 a = *reinterpret_cast<const uint4*>(gmin);
-          rmin = min(min(a.x, a.y), min(a.z, a.w));
-          if (v > 128) {
-            const uint4 b = *reinterpret_cast<const uint4*>(gmin + 4);
-            rmin = min(rmin, min(min(b.x, b.y), min(b.z, b.w)));
-          }
+      uint64_t en = nd.phys ? gtimer() : 0ull;   // completion time of the terminal items
+      if (nd.phys && (rec & PL_FIXED_SERVICE)) en = max(en, T0 + units_ns(nd, T + nd.t));   // delivery at start + t_i
+      A.t_end = T + nd.t;                // firing starts increase: the last one ends last
+      // the smallest terminal root has the largest latency
+      uint32_t rmin;
+      {
+        const uint4 a = *reinterpret_cast<const uint4*>(G.rmin);
+        rmin = min(min(a.x, a.y), min(a.z, a.w));
+        if (v > 128) {
+          const uint4 b = *reinterpret_cast<const uint4*>(G.rmin + 4);
+          rmin = min(rmin, min(min(b.x, b.y), min(b.z, b.w)));
         }
-        if (rmin != NO_ROOT) {
-          const int64_t ar = nd.arrival(rmin);
-          const int64_t lat = Ts + nd.t - ar;
-          atomicMax(&A.lmax, clamp32(lat));
-          if (lat > nd.D) {                // a miss in this firing: count the late items exactly
-            uint32_t m = 0;
-            for (uint32_t k = klo; k < khi; ++k) {
-              const uint32_t r = nd.troot[k];
-              if (r != NO_ROOT && Ts + nd.t - nd.arrival(r) > nd.D) ++m;
-            }
-            atomicAdd(&A.nmiss, m);
+      }
+      if (rmin != NO_ROOT) {
+        const int64_t ar = nd.arrival(rmin);
+        const int64_t lat = T + nd.t - ar;
+        atomicMax(&A.lmax, clamp32(lat));
+        if (lat > nd.D) {                // a miss in this firing: count the late items exactly
+          uint32_t m = 0;
+          for (int k = 0; k < v; ++k) {
+            const uint32_t r = nd.troot[k];
+            if (r != NO_ROOT && T + nd.t - nd.arrival(r) > nd.D) ++m;
           }
-          if (nd.phys) {
-            const int64_t l = (int64_t)en - (int64_t)(T0 + units_ns(nd, ar));
-            atomicMax(&A.lmax_ns, clamp32(l));
-            if (l > nd.D_ns) {
-              uint32_t m = 0;
-              for (uint32_t k = klo; k < khi; ++k) {
-                const uint32_t r = nd.troot[k];
-                if (r != NO_ROOT && (int64_t)en - (int64_t)(T0 + units_ns(nd, nd.arrival(r))) > nd.D_ns) ++m;
-              }
-              atomicAdd(&A.nmiss_ns, m);
+          atomicAdd(&A.nmiss, m);
+        }
+        if (nd.phys) {
+          const int64_t l = (int64_t)en - (int64_t)(T0 + units_ns(nd, ar));
+          atomicMax(&A.lmax_ns, clamp32(l));
+          if (l > nd.D_ns) {
+            uint32_t m = 0;
+            for (int k = 0; k < v; ++k) {
+              const uint32_t r = nd.troot[k];
+              if (r != NO_ROOT && (int64_t)en - (int64_t)(T0 + units_ns(nd, nd.arrival(r))) > nd.D_ns) ++m;
             }
-            // north_star: every item's measured latency within 5 % of the logical-clock prediction
-            // T + t_i - a(r) (floor PL_AGREE_FLOOR_NS, DESIGN.md R-AGREE).  A firing's terminal items
-            // complete together, so the error is common to them -- with PL_FIXED_SERVICE they are
-            // delivered at max(done, start + t_i), the paper's fixed service time (L69) -- and its
-            // relative size is largest for the latest-arriving terminal root.
-            uint32_t rx;
-            {
-              const uint4 a = *reinterpret_cast<const uint4*>(gmax);
-              rx = max(max(a.x, a.y), max(a.z, a.w));
-              if (v > 128) {
-                const uint4 b = *reinterpret_cast<const uint4*>(gmax + 4);
-                rx = max(rx, max(max(b.x, b.y), max(b.z, b.w)));
-              }
+            atomicAdd(&A.nmiss_ns, m);
+          }
+          // north_star: every item's measured latency within 5 % of the logical-clock prediction
+          // T + t_i - a(r) (floor PL_AGREE_FLOOR_NS, DESIGN.md R-AGREE).  A firing's terminal items
+          // complete together, so the error is common to them -- with PL_FIXED_SERVICE they are
+          // delivered at max(done, start + t_i), the paper's fixed service time (L69) -- and its
+          // relative size is largest for the latest-arriving terminal root.
+          uint32_t rx;
+          {
+            const uint4 a = *reinterpret_cast<const uint4*>(G.rmax);
+            rx = max(max(a.x, a.y), max(a.z, a.w));
+            if (v > 128) {
+              const uint4 b = *reinterpret_cast<const uint4*>(G.rmax + 4);
+              rx = max(rx, max(max(b.x, b.y), max(b.z, b.w)));
             }
-            const int64_t due = (int64_t)(T0 + units_ns(nd, Ts + nd.t));
-            const int64_t err = (int64_t)en > due ? (int64_t)en - due : due - (int64_t)en;
-            const int64_t lsmall = (int64_t)units_ns(nd, Ts + nd.t - nd.arrival(rx - 1u));
-            atomicMax(&AG.agr_ppm, clamp32((int64_t)((float)err * 1e6f / (float)(lsmall > 0 ? lsmall : 1))));
-            // count the items outside the band exactly -- with PL_FIXED_SERVICE only, where the model's
-            // completion time is realised and outliers are rare (in publish mode a firing completes
-            // early by design and the count would cost a pass over the lanes on every firing)
-            if ((rec & PL_FIXED_SERVICE) && err * 20 > lsmall + 20 * PL_AGREE_FLOOR_NS) {
-              uint32_t m = 0;
-              for (uint32_t k = klo; k < khi; ++k) {
-                const uint32_t r = nd.troot[k];
-                if (r != NO_ROOT && err * 20 > (int64_t)units_ns(nd, Ts + nd.t - nd.arrival(r)) + 20 * PL_AGREE_FLOOR_NS) ++m;
-              }
-              atomicAdd(&AG.agr_bad, m);
+          }
+          const int64_t due = (int64_t)(T0 + units_ns(nd, T + nd.t));
+          const int64_t err = (int64_t)en > due ? (int64_t)en - due : due - (int64_t)en;
+          const int64_t lsmall = (int64_t)units_ns(nd, T + nd.t - nd.arrival(rx - 1u));
+          atomicMax(&AG.agr_ppm, clamp32((int64_t)((float)err * 1e6f / (float)(lsmall > 0 ? lsmall : 1))));
+          // count the items outside the band exactly -- with PL_FIXED_SERVICE only, where the model's
+          // completion time is realised and outliers are rare (in publish mode a firing completes
+          // early by design and the count would cost a pass over the lanes on every firing)
+          if ((rec & PL_FIXED_SERVICE) && err * 20 > lsmall + 20 * PL_AGREE_FLOOR_NS) {
+            uint32_t m = 0;
+            for (int k = 0; k < v; ++k) {
+              const uint32_t r = nd.troot[k];
+              if (r != NO_ROOT && err * 20 > (int64_t)units_ns(nd, T + nd.t - nd.arrival(r)) + 20 * PL_AGREE_FLOOR_NS) ++m;
             }
+            atomicAdd(&AG.agr_bad, m);
           }
         }
       }
@@ -1784,11 +1678,10 @@ __device__ void run_node(Ctx& c, Dna dna, int i, int gtid) {
         ulonglong2 c0 = Cp[0], c1 = Cp[1], c3 = Cp[3], c4 = Cp[4], p0 = Pp[0], p1 = Pp[1];
         const uint4 dd = *reinterpret_cast<const uint4*>(A.d[par]);
         const uint32_t stl = A.d[par][D_STALL];
-        c0.x += n1 ? 2ull : 1ull;
+        c0.x += 1ull;
         c0.y += n;
         c1.x += total;
-        const unsigned long long ov = (unsigned long long)overlap(T, T + nd.t, 0, nd.H) +
-                                      (n1 ? (unsigned long long)overlap(T2, T2 + nd.t, 0, nd.H) : 0ull);
+        const unsigned long long ov = (unsigned long long)overlap(T, T + nd.t, 0, nd.H);
         c1.y += ov;
         c4.x += (nd.eager && T >= nd.A_last) ? ov : 0ull;   // R-DRAIN firings (FIXED_WAIT window)
         c4.y += (nd.eager && T >= nd.A_last) ? 1ull : 0ull;
@@ -1796,7 +1689,6 @@ __device__ void run_node(Ctx& c, Dna dna, int i, int gtid) {
         c3.y += stl;
         p0.x += dd.x; p0.y += dd.y; p1.x += dd.z; p1.y += dd.w;
         Cp[0] = c0; Cp[1] = c1; Cp[3] = c3; Cp[4] = c4; Pp[0] = p0; Pp[1] = p1;
-        if (n1) A.cnt[C_BATCHED] += 1ull;   // catch-up batching (the accountant is its only writer)
       }
       if ((CL || n0) && nd.sliding) win_step(*c.sh, p, (unsigned char*)dna.win, false);   // slide the DB window
     }
@@ -1843,7 +1735,6 @@ __device__ void run_node(Ctx& c, Dna dna, int i, int gtid) {
     S.overruns[i] = A.cnt[C_OVERRUNS];
     S.stalls[i] = A.cnt[C_STALLS];
     S.drain_firings[i] = A.cnt[C_DRAINF];
-    S.batched[i] = A.cnt[C_BATCHED];
     S.max_queue[i] = A.max_queue;
     S.lateness[i] = (int64_t)A.lateness;
     S.sched_cycles[i] = A.ph[0];
@@ -2224,7 +2115,7 @@ __device__ void run_monolithic(Ctx& c) {
       S.firings[i] = firings[i]; S.empty[i] = 0; S.consumed[i] = consumed[i]; S.produced[i] = produced[i];
       S.active_ne[i] = active[i]; S.active_win[i] = active[i]; S.busy_ns[i] = i == 0 ? busy_ns : 0;
       S.spilled[i] = 0; S.overruns[i] = 0;
-      S.stalls[i] = 0; S.max_queue[i] = 0; S.drain_firings[i] = 0; S.batched[i] = 0;
+      S.stalls[i] = 0; S.max_queue[i] = 0; S.drain_firings[i] = 0;
       S.lateness[i] = 0; S.sched_cycles[i] = 0; S.max_fire_ns[i] = 0; S.max_loop_ns[i] = 0;
       for (int k = 0; k < 6; ++k) S.phase_cycles[i][k] = 0;
     }

@@ -48,7 +48,6 @@ struct CtaStats {
   uint64_t overruns[PL_MAX_STAGES];
   uint64_t stalls[PL_MAX_STAGES];
   uint64_t drain_firings[PL_MAX_STAGES]; // R-DRAIN firings (at T >= A_last)
-  uint64_t batched[PL_MAX_STAGES];      // physical firings that carried two logical ones (catch-up)
   uint32_t max_queue[PL_MAX_STAGES];
   int64_t  lateness[PL_MAX_STAGES];
   uint64_t sched_cycles[PL_MAX_STAGES];

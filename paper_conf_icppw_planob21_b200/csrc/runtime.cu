@@ -1080,7 +1080,6 @@ pl_status pl_pipeline_stats(pl_pipeline* pl, pl_stats* out) {
     out->latency_outliers += s.agr_bad;
     out->latency_rel_err_max = std::max(out->latency_rel_err_max, (double)s.agr_ppm * 1e-6);
     out->ingest_waits += s.ingest_waits;
-    for (uint32_t i = 0; i < N; ++i) out->batched_firings[i] += s.batched[i];
     out->max_ingest_wait_ns = std::max<int64_t>(out->max_ingest_wait_ns, s.ingest_max_ns);
   }
   unsigned long long mc = 0;

@@ -94,3 +94,31 @@ def test_cluster_rejects_monolithic_and_live():
     with pytest.raises(PlError):
         pl.live_start()
     pl.close()
+
+
+@pytest.mark.parametrize("policy", [C.FIXED_WAIT, C.THRESHOLD_SLACK])
+def test_cluster_eight_nodes(policy):
+    """N = 8: clusters of 8 CTAs (the portable maximum), one random-gain node per CTA."""
+    st = [C.Stage(C.BERNOULLI, 0.8, 1), C.Stage(C.POISSON_CAPPED, 1.3, 4), C.Stage(C.BERNOULLI, 0.6, 1),
+          C.Stage(C.FIXED_GAIN, 2.0, 2), C.Stage(C.BERNOULLI, 0.5, 1), C.Stage(C.KEEP_EVERY, 3.0, 1),
+          C.Stage(C.POISSON_CAPPED, 0.9, 3), C.Stage(C.BERNOULLI, 0.7, 1)]
+    cfg = C.Config(name="n8", stages=st, service_time=(40, 55, 30, 45, 25, 35, 50, 20), vector_width=128,
+                   deadline=20_000, interarrival=3, b=(1,) * 8, wait_time=(300, 100, 50, 80, 40, 60, 90, 30),
+                   wait_threshold=(64, 32, 16, 16, 8, 8, 4, 4), policy=policy, n_streams=3, n_roots=3000, seed=5)
+    compare(cfg, run_gpu(cfg, None, flags=7 | CL), run_oracle(cfg, None))
+
+
+@pytest.mark.parametrize("v", [32, 256])
+def test_cluster_vector_widths(v):
+    cfg = _dna(C.THRESHOLD_SLACK, db_len=1 << 15, streams=3).replace(vector_width=v,
+                                                                     wait_threshold=(v, v - 1, v // 2, 4))
+    wl = workload_for(cfg)
+    compare(cfg, run_gpu(cfg, wl, flags=7 | CL), run_oracle(cfg, wl))
+
+
+def test_cluster_poisson_arrivals():
+    from plgen import arrivals as A
+    cfg = _dna(C.THRESHOLD_SLACK, db_len=1 << 15, streams=3)
+    wl = workload_for(cfg)
+    arr = A.poisson(3, A.stream_sizes(wl.db_len - 6 + 1, cfg.n_streams), cfg.interarrival)
+    compare(cfg, run_gpu(cfg, wl, flags=7 | CL, arrivals=arr), run_oracle(cfg, wl, arrivals=arr))

@@ -131,45 +131,6 @@ def test_injected_stalls_move_time_not_schedule(c2wl, budgets):
         Pipeline(cfg.replace(clock=C.CLOCK_LOGICAL), wl).inject_stalls(period, length)
 
 
-@pytest.mark.parametrize("batching", [True, False])
-def test_catchup_batching_keeps_the_schedule(c2wl, budgets, batching):
-    """Catch-up batching (executor.cu peek_next): after an injected stall every node is far
-    behind its schedule, and a late THRESHOLD_SLACK node runs its next two logical firings on one
-    vector when both are due and fit in v lanes.  The schedule, outputs and every counter stay
-    the oracle's, bit-exact with per-root latencies, traces and the firing log; with batching off
-    (PL_VARIANT bit 8) no vector is batched and the results are the same."""
-    import os
-    from paper_conf_icppw_planob21_b200 import Pipeline, solve_enforced_waits
-    _, wl = c2wl
-    cfg = _phys_cfg(budgets, _tau_for(budgets, 40))
-    w, th, T, Tc = solve_enforced_waits(cfg)
-    cfg = cfg.replace(policy=C.THRESHOLD_SLACK, wait_time=None, wait_threshold=tuple(th),
-                      slack_guard=max(cfg.service_time))
-    span = (wl.db_len // 148) * cfg.interarrival
-    old = os.environ.get("PL_VARIANT")
-    os.environ["PL_VARIANT"] = "1" if batching else "9"
-    try:
-        pl = Pipeline(cfg, wl, flags=7)
-    finally:
-        if old is None:
-            del os.environ["PL_VARIANT"]
-        else:
-            os.environ["PL_VARIANT"] = old
-    pl.push(wl.db, wl.db_len)
-    pl.inject_stalls(span // 3, span // 6)
-    pl.drain()
-    g = dict(stats=pl.stats(), matches=pl.results(), trace=pl.trace(), firings=pl.firings())
-    g["lat"], g["lat_ns"] = pl.latency()
-    pl.close()
-    compare(cfg, g, run_oracle_parallel(cfg, wl))
-    st = g["stats"]
-    print("batched", st["batched_firings"][:4], "lateness", st["max_lateness_ns"])
-    if batching:
-        assert sum(st["batched_firings"]) > 0
-    else:
-        assert sum(st["batched_firings"]) == 0
-
-
 def test_physical_zero_misses_1p5x_feasible_rate(c2wl, budgets):
     """Zero measured misses at a rate 1.5x above the Fig. 1 feasibility limit of the budgets
     (at least tau0 = 30 ns)."""
