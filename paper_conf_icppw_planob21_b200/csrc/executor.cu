@@ -68,6 +68,22 @@ __device__ __forceinline__ uint64_t gain_hash(uint64_t seed, uint32_t stage, uin
 // TMA bulk copies as the stream advances (win_step); [win_lo,
 // win_lo + win_n) is this thread's snapshot of the words it holds.  Extensions compare 16
 // bases per step: XOR of two 2-bit-packed 32-bit windows gives a mismatch mask.
+// experiment switches (tools/build_variant.py -D...; defaults = the product build)
+#ifndef PL_WINSTEP_NOINLINE
+#define PL_WINSTEP_NOINLINE 1
+#endif
+#ifndef PL_LIVE_GATE
+#define PL_LIVE_GATE 1
+#endif
+#ifndef PL_WATCHDOG
+#define PL_WATCHDOG 1
+#endif
+#ifndef PL_DBMASK
+#define PL_DBMASK 1
+#endif
+#ifndef PL_INJECT
+#define PL_INJECT 1
+#endif
 #ifndef PL_S3_MSB
 #define PL_S3_MSB 1
 #endif
@@ -97,7 +113,11 @@ struct Dna {
     const uint64_t r = (uint64_t)(w - win_lo);
     if (r < win_n) return win[(uint32_t)w & win_mask];
     if (!(w >= 0 && w < (int64_t)nwords)) return 0u;
+#if PL_DBMASK
     return dbmask == 0xffffffffu ? __ldg(db + w) : __ldcg(db + ((uint32_t)w & dbmask));
+#else
+    return __ldg(db + w);   // experiment: the live ring's mask compiled out
+#endif
   }
   __device__ __forceinline__ uint32_t qww(int64_t w) const { return (w >= 0 && w < (int64_t)nqw) ? qw[w] : 0u; }
   // bases s..s+15 (base s in bits 0-1); s may be negative (out-of-range bases read as 0)
@@ -434,7 +454,12 @@ __device__ __forceinline__ uint32_t live_front(WinCtl& W, uint32_t need) {
 // Live ingest: a chunk loads in 16-byte-aligned pieces as its words are delivered, and the
 // consumed watermark min(floor, a_next) -- nothing below it is read or staged again -- goes to
 // the host, which may then overwrite those ring slots.  Returns whether it made progress.
-__device__ __noinline__ bool win_step(Shared& sh, const DevParams& p, unsigned char* ring, bool wait) {
+#if PL_WINSTEP_NOINLINE
+__device__ __noinline__
+#else
+__device__
+#endif
+bool win_step(Shared& sh, const DevParams& p, unsigned char* ring, bool wait) {
   WinCtl& W = sh.win;
   const uint32_t bar = smem_addr(&sh.mbar_w);
   bool prog = false;
@@ -773,7 +798,9 @@ __device__ __forceinline__ void publish_W(const Node& nd, Leader& L, int64_t w) 
 // firing start by at most t_i / 8, which the time-triggered delivery (PL_FIXED_SERVICE) absorbs
 // while the work itself takes well under t_i.  Measured on c4 (ncu source page): the fixed
 // 256 ns nap made the waiting leaders' polls ~90 % of all instructions issued.
-__device__ __forceinline__ void backoff(int& spins, bool phys = false, uint32_t cap_ns = 256) {
+// The watchdog (above) is checked deep inside a wait only, every 4096 naps, off every firing's
+// path; a waiter whose watchdog expired finds spins < 0.
+__device__ __forceinline__ void backoff(int& spins, uint64_t& wd0, bool phys = false, uint32_t cap_ns = 256) {
   if (spins < (phys ? 2 : 4)) { ++spins; return; }
   if (phys) {
     const int e = spins - 2 < 16 ? spins - 2 : 16;
@@ -783,6 +810,7 @@ __device__ __forceinline__ void backoff(int& spins, bool phys = false, uint32_t 
     __nanosleep(spins < 64 ? 32 : 256);
   }
   ++spins;
+  if (PL_WATCHDOG && (spins & 4095) == 0 && watchdog_expired(wd0)) spins = -(1 << 30);
 }
 
 // number of entries of the input edge with ready <= T among the published ones (stops at v)
@@ -951,7 +979,7 @@ __device__ Decision decide(const Node& nd, Leader& L, bool& waited, uint64_t T0)
   int64_t napped = -1;
   uint64_t wd0 = 0;
   for (;;) {
-    if ((spins & 255) == 255 && watchdog_expired(wd0)) { L.wd = 1u; publish_W(nd, L, PL_INF64); d.done = true; return d; }
+    if (spins < 0) { L.wd = 1u; publish_W(nd, L, PL_INF64); d.done = true; return d; }   // watchdog
     if (nd.phys && nd.fixed && !(nd.eager && L.m >= nd.Mcap)) {
       const int64_t Tn = L.m * nd.P;
       if (Tn != napped) {
@@ -975,7 +1003,7 @@ __device__ Decision decide(const Node& nd, Leader& L, bool& waited, uint64_t T0)
         if (!any) {
           if (Wup == PL_INF64) { d.done = true; return d; }
           publish_W(nd, L, max(B, Wup) + nd.t);
-          backoff(spins, nd.phys, nd.nap_cap_ns); waited = true;
+          backoff(spins, wd0, nd.phys, nd.nap_cap_ns); waited = true;
           continue;
         }
         const int64_t Te = max(B, nd.in_seg[L.segh & nd.segmask].ready);
@@ -984,7 +1012,7 @@ __device__ Decision decide(const Node& nd, Leader& L, bool& waited, uint64_t T0)
         if (Wup > Te || (cnt >= v && early_ok(nd))) {
           d.T = Te; d.n = cnt < v ? cnt : v; d.qlen = count_all_le(nd, L, st, Te); return d;
         }
-        backoff(spins, nd.phys, nd.nap_cap_ns); waited = true;
+        backoff(spins, wd0, nd.phys, nd.nap_cap_ns); waited = true;
         continue;
       }
       const int64_t T = L.m * nd.P;
@@ -1003,7 +1031,7 @@ __device__ Decision decide(const Node& nd, Leader& L, bool& waited, uint64_t T0)
         continue;
       }
       publish_W(nd, L, T + nd.t);
-      backoff(spins, nd.phys, nd.nap_cap_ns); waited = true;
+      backoff(spins, wd0, nd.phys, nd.nap_cap_ns); waited = true;
       continue;
     }
     // THRESHOLD_SLACK
@@ -1012,7 +1040,7 @@ __device__ Decision decide(const Node& nd, Leader& L, bool& waited, uint64_t T0)
       const int64_t lb = Wup > L.B ? Wup : L.B;
       publish_W(nd, L, lb + nd.t);
       if (nap_to(nd, T0, lb, napped)) { waited = true; spins = 0; continue; }
-      backoff(spins, nd.phys, nd.nap_cap_ns); waited = true;
+      backoff(spins, wd0, nd.phys, nd.nap_cap_ns); waited = true;
       continue;
     }
     const Seg& hs = nd.in_seg[L.segh & nd.segmask];
@@ -1046,7 +1074,7 @@ __device__ Decision decide(const Node& nd, Leader& L, bool& waited, uint64_t T0)
     if (lb < L.B) lb = L.B;
     publish_W(nd, L, lb + nd.t);
     if (nap_to(nd, T0, lb, napped)) { waited = true; spins = 0; continue; }
-    backoff(spins, nd.phys, nd.nap_cap_ns); waited = true;
+    backoff(spins, wd0, nd.phys, nd.nap_cap_ns); waited = true;
   }
 }
 
@@ -1058,7 +1086,7 @@ __device__ uint32_t reserve_out(const Node& nd, Leader& L, uint32_t worst, uint3
   int spins = 0;
   uint64_t wd0 = 0;
   for (;;) {
-    if ((spins & 255) == 255 && watchdog_expired(wd0)) { L.wd = 2u; return ~0u; }   // outputs dropped
+    if (spins < 0) { L.wd = 2u; return ~0u; }   // watchdog: outputs dropped
     const uint32_t h = vld(&nd.Eout->head), sh = vld(&nd.Eout->seg_head);
     const bool seg_ok = (L.out_segt - sh) <= nd.segmask;
     const uint32_t need = L.out_tail + worst - h;
@@ -1066,7 +1094,7 @@ __device__ uint32_t reserve_out(const Node& nd, Leader& L, uint32_t worst, uint3
     if (seg_ok && need <= nd.capg) { if (*stalled) vst(&nd.Eout->stalled, 0u); return LOC_SPILL; }
     if (!*stalled) vst(&nd.Eout->stalled, 1u);
     *stalled = 1u;
-    backoff(spins);
+    backoff(spins, wd0);
   }
 }
 
@@ -1096,7 +1124,7 @@ __device__ __noinline__ void inject_stall(const DevParams& p, uint64_t T0) {
 }
 __device__ __forceinline__ void pace_p(const DevParams& p, uint64_t T0, uint64_t target, uint64_t* start_ns,
                                        int64_t* late, uint64_t* entry_ns = nullptr) {
-  if (p.inj_len_ns) inject_stall(p, T0);
+  if (PL_INJECT && p.inj_len_ns) inject_stall(p, T0);
   pace(target, start_ns, late, entry_ns);
 }
 
@@ -1281,7 +1309,9 @@ __device__ __forceinline__ uint32_t live_need(const Shared& sh, const DevParams&
 // REC: per-item records compiled in (parity / tracing runs); the bench kernel has none.
 // (A separate node-0 instantiation was measured: faster alone, 1.33x slower with all nodes
 // running -- the SM's instruction cache holds one ~76 KB node loop, not two.)
-template <bool REC, bool CL>
+// LIVE: the live-ingest instantiation (node 0 gates its firings on delivered words); the other
+// kernels do not carry that code (the node loop is instruction-cache bound: tools/bisect_fire.py)
+template <bool REC, bool CL, bool LIVE = false>
 __device__ void run_node(Ctx& c, Dna dna, int i, int gtid) {
   const DevParams& p = *c.p;
   const Node nd = make_node(c, i);
@@ -1327,7 +1357,7 @@ __device__ void run_node(Ctx& c, Dna dna, int i, int gtid) {
       const Decision d = decide0(nd, R);
       if (d.done) break;
       T = d.T; n = d.n; head = (uint32_t)R.c0;
-      if (p.live && n) {                 // live ingest: the firing's DB words must have been delivered
+      if (LIVE && PL_LIVE_GATE && n) {   // live ingest: the firing's DB words must have been delivered
         const uint32_t last = (uint32_t)min((int64_t)head + n, nd.X) - 1u;
         const uint32_t need = live_need(*c.sh, p, (uint32_t)(nd.lo + last));
         if (vld(&c.sh->win.front) < need)
@@ -2127,7 +2157,7 @@ __device__ void run_monolithic(Ctx& c) {
 
 // FIXED_WAIT / THRESHOLD_SLACK executor: grid = n_streams, block = N*32 threads (one warp
 // per node); up to 4 CTAs (streams) per SM when N <= 4.
-template <int MAXT, int MINB, bool REC>
+template <int MAXT, int MINB, bool REC, bool LIVE = false>
 __global__ void __launch_bounds__(MAXT, MINB) pl_exec_enforced(const __grid_constant__ DevParams p) {
   extern __shared__ __align__(16) unsigned char dsm[];
   __shared__ Shared sh;
@@ -2146,7 +2176,7 @@ __global__ void __launch_bounds__(MAXT, MINB) pl_exec_enforced(const __grid_cons
   const bool contig = !(p.variant & 4u);
   const int gi = contig ? w / (p.v >> 5) : w % p.N;
   const int gt = (contig ? w % (p.v >> 5) : w / p.N) * 32 + (threadIdx.x & 31);
-  if (w < p.N * (p.v >> 5)) run_node<REC, false>(c, c.dna, gi, gt);
+  if (w < p.N * (p.v >> 5)) run_node<REC, false, LIVE>(c, c.dna, gi, gt);
   __syncthreads();
   cta_finish(c, sh, p);
 }
@@ -2226,7 +2256,15 @@ cudaError_t pl_launch(const DevParams& p, unsigned grid, unsigned block, unsigne
     // the CTA fits twice (<= 512 threads, 64 registers, smem)
     // per-item records (parity / tracing) select the REC instantiation; the bench runs without
     const bool rec = (p.flags & (PL_REC_LATENCY | PL_REC_TRACE | PL_REC_FIRINGS)) != 0;
-    if (block <= 512 && p.ctas_per_sm >= 2) {
+    if (p.live) {                        // live ingest: the instantiation with node 0's delivery gate
+      if (block <= 512) {
+        if (rec) pl_exec_enforced<512, 1, true, true><<<grid, block, smem, st>>>(p);
+        else pl_exec_enforced<512, 1, false, true><<<grid, block, smem, st>>>(p);
+      } else {
+        if (rec) pl_exec_enforced<1024, 1, true, true><<<grid, block, smem, st>>>(p);
+        else pl_exec_enforced<1024, 1, false, true><<<grid, block, smem, st>>>(p);
+      }
+    } else if (block <= 512 && p.ctas_per_sm >= 2) {
       if (rec) pl_exec_enforced<512, 2, true><<<grid, block, smem, st>>>(p);
       else pl_exec_enforced<512, 2, false><<<grid, block, smem, st>>>(p);
     } else if (block <= 512) {
@@ -2248,6 +2286,10 @@ cudaError_t pl_kernel_attributes(unsigned max_smem) {
   if ((e = cudaFuncSetAttribute(pl_exec_enforced<512, 1, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, max_smem))) return e;
   if ((e = cudaFuncSetAttribute(pl_exec_enforced<1024, 1, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, max_smem))) return e;
   if ((e = cudaFuncSetAttribute(pl_exec_enforced<1024, 1, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, max_smem))) return e;
+  if ((e = cudaFuncSetAttribute(pl_exec_enforced<512, 1, false, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, max_smem))) return e;
+  if ((e = cudaFuncSetAttribute(pl_exec_enforced<512, 1, true, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, max_smem))) return e;
+  if ((e = cudaFuncSetAttribute(pl_exec_enforced<1024, 1, false, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, max_smem))) return e;
+  if ((e = cudaFuncSetAttribute(pl_exec_enforced<1024, 1, true, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, max_smem))) return e;
   if ((e = cudaFuncSetAttribute(pl_exec_cluster<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, max_smem))) return e;
   if ((e = cudaFuncSetAttribute(pl_exec_cluster<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, max_smem))) return e;
   if ((e = cudaFuncSetAttribute(pl_exec_monolithic<512>, cudaFuncAttributeMaxDynamicSharedMemorySize, max_smem))) return e;
