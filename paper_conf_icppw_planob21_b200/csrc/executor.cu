@@ -586,6 +586,7 @@ __device__ __forceinline__ uint64_t units_ns(const Node& nd, int64_t t) {
   return nd.ns1 ? (uint64_t)t : (uint64_t)((double)t * nd.nspu);
 }
 
+template <bool CL = false>
 __device__ __forceinline__ Node make_node(const Ctx& c, int i) {
   const DevParams& p = *c.p;
   SmemLayout Lo;
@@ -611,7 +612,7 @@ __device__ __forceinline__ Node make_node(const Ctx& c, int i) {
   n.in_spill = p.spill ? p.spill + (sp + i) * p.cap_g : nullptr;
   n.in_mask = p.cap_s[i] ? p.cap_s[i] - 1 : 0;
   const int o = i + 1 < p.N ? i + 1 : i;
-  n.cl = c.rank >= 0;
+  n.cl = CL && c.rank >= 0;   // a compile-time false outside the cluster kernel
   if (n.cl && o != i) {   // N4: the edge into node i+1 lives in CTA i+1's shared memory (DSMEM)
     n.Eout = (EdgeCtl*)__cluster_map_shared_rank(&c.sh->e[o], (unsigned)o);
     n.out_ent = (uint2*)__cluster_map_shared_rank(c.dsm + Lo.off_ent[o], (unsigned)o);
@@ -971,7 +972,7 @@ __device__ __forceinline__ bool nap_to(const Node& nd, uint64_t T0, int64_t lb, 
 // recorded queue peak is the DES's |Q_i| exactly; the physical clock always may.
 __device__ __forceinline__ bool early_ok(const Node& nd) { return nd.phys || vld(&nd.Ein->stalled) != 0u; }
 
-__device__ Decision decide(const Node& nd, Leader& L, bool& waited, uint64_t T0) {
+__device__ __forceinline__ Decision decide(const Node& nd, Leader& L, bool& waited, uint64_t T0) {
   const uint32_t v = (uint32_t)nd.v;
   Decision d;
   d.done = false; d.T = 0; d.n = 0; d.qlen = 0;
@@ -1082,7 +1083,7 @@ __device__ Decision decide(const Node& nd, Leader& L, bool& waited, uint64_t T0)
 // stage runs so that no extra barrier is needed).  Returns the location.  A full queue
 // back-pressures the producer in both clock modes (deadlock-free):
 // in physical mode the wait shows up as lateness and, if it matters, as deadline misses.
-__device__ uint32_t reserve_out(const Node& nd, Leader& L, uint32_t worst, uint32_t* stalled) {
+__device__ __forceinline__ uint32_t reserve_out(const Node& nd, Leader& L, uint32_t worst, uint32_t* stalled) {
   int spins = 0;
   uint64_t wd0 = 0;
   for (;;) {
@@ -1314,7 +1315,7 @@ __device__ __forceinline__ uint32_t live_need(const Shared& sh, const DevParams&
 template <bool REC, bool CL, bool LIVE = false>
 __device__ void run_node(Ctx& c, Dna dna, int i, int gtid) {
   const DevParams& p = *c.p;
-  const Node nd = make_node(c, i);
+  const Node nd = make_node<CL>(c, i);
   const int v = nd.v, N = nd.N;
   const bool n0 = i == 0;
   const bool leader = gtid == 0;
