@@ -220,6 +220,15 @@ class Pipeline:
         a[:, 5] = buf[:n.value, 5].view(np.int32)
         return a[np.lexsort(a.T[::-1])] if len(a) else a
 
+    def results_raw(self):
+        """The match records as an (n, 6) uint32 array in device order (unsorted; score is the
+        int32 bit pattern) -- the cheap form for very large result sets."""
+        n = C.c_uint64()
+        check(lib.pl_pipeline_results(self.h, None, 0, C.byref(n)), "pl_pipeline_results")
+        buf = np.empty((max(1, n.value), 6), dtype=np.uint32)
+        check(lib.pl_pipeline_results(self.h, buf.ctypes.data, n.value, C.byref(n)), "pl_pipeline_results")
+        return buf[:n.value]
+
     def latency(self):
         n = C.c_uint64()
         check(lib.pl_pipeline_latency(self.h, None, None, 0, C.byref(n)), "pl_pipeline_latency")

@@ -46,6 +46,17 @@ def _cfg(base, budgets, tau):
     return cfg.replace(interarrival=tau, wait_time=tuple(w), wait_threshold=tuple(th))
 
 
+def _multiset_digest(rows):
+    """An order-independent digest of match records: the sum (mod 2^64) of a per-record hash."""
+    r = rows.astype(np.uint64)
+    h = np.zeros(len(r), dtype=np.uint64)
+    for j, k in enumerate((0x9E3779B97F4A7C15, 0xBF58476D1CE4E5B9, 0x94D049BB133111EB, 0xD6E8FEB86659FD93,
+                           0xA0761D6478BD642F, 0xE7037ED1A0B428DB)):
+        h = (h ^ r[:, j]) * np.uint64(k)
+        h ^= h >> np.uint64(29)
+    return int(h.sum(dtype=np.uint64)), len(r)
+
+
 def _run_unstalled(cfg, wl, db, over, flags, tries=4):
     from paper_conf_icppw_planob21_b200 import Pipeline, realtime
     seen = []
@@ -59,6 +70,7 @@ def _run_unstalled(cfg, wl, db, over, flags, tries=4):
             out["lat"], out["lat_ns"] = pl.latency()
         if flags & 4:
             out["firings"] = pl.firings()
+        out["digest"] = _multiset_digest(pl.results_raw())
         pl.close()
         if not realtime.stalled(st):
             return out
@@ -103,6 +115,17 @@ def test_bench_kernel_every_item_within_5pct(c4):
     # processor utilisation: measured occupancy vs the logical schedule's t_i per firing
     model_busy = sum(st["firings"][i] * b[i] for i in range(4))
     assert abs(sum(st["busy_ns"]) / model_busy - 1) < 0.05
+    # the match set and per-node counts are pure functions of the data (R-S0..R-S3): the bench
+    # kernel's equal a logical-clock run's (whose schedule tests/test_gpu_c4.py checks vs the oracle)
+    from paper_conf_icppw_planob21_b200 import Pipeline
+    lg = Pipeline(base.replace(wait_time=(993, 2422, 965, 1628)), wl, **over)
+    lg.bind_device(db.data_ptr(), wl.db_len)
+    lg.drain()
+    sl = lg.stats()
+    dl = _multiset_digest(lg.results_raw())
+    lg.close()
+    assert g["digest"] == dl and st["matches"] == sl["matches"] > 0
+    assert st["consumed"] == sl["consumed"] and st["produced"] == sl["produced"]
 
 
 @pytest.fixture(scope="module")
