@@ -142,3 +142,38 @@ def test_c4_sampled_roots_one_by_one(c4run, ctx):
         a, b = np.searchsorted(gp, r), np.searchsorted(gp, r + 1)
         assert np.array_equal(gm[a:b], _rows(items)), r
     assert amplified > 0
+
+
+def test_c5_rank1_workload_sampled_streams():
+    """BASELINE configs[4] (c5): each rank runs c4 on its own DB, seed 4 + rank (bench.py
+    base_config).  Rank 1's workload at full size, logical clock: the first 20 K roots of two
+    streams against the oracle's DES (causal prefix), plus trace conservation over every root."""
+    from oracle import des
+    from oracle import stages as S
+    from paper_conf_icppw_planob21_b200 import Pipeline, solve_enforced_waits
+    base = C.c4(seed=5)
+    w, th, T, Tc = solve_enforced_waits(base.replace(gain=C.TABLE1_G))
+    cfg = base.replace(wait_time=tuple(w))
+    wl = workload_for(cfg)
+    pl = Pipeline(cfg, wl, flags=3, match_capacity=1 << 25, spill_capacity=1 << 19)
+    pl.push(wl.db, wl.db_len)
+    pl.drain()
+    st = pl.stats()
+    lat, _ = pl.latency()
+    tr = pl.trace().reshape(-1, cfg.n_stages + 1)
+    pl.close()
+    for i in range(cfg.n_stages):
+        assert int(tr[:, i].sum()) == st["consumed"][i]
+    assert int(tr[:, cfg.n_stages].sum()) == st["matches"]
+    ctx = S.DnaContext(wl.db, wl.db_len, wl.query, wl.q_len, 6)
+    fns = des.make_stage_fns(cfg, ctx)
+    rng = des.stream_ranges(cfg, ctx.n_roots)
+    for s in (3, 120):
+        lo, hi = rng[s]
+        hi2 = min(hi, lo + 20_000)
+        r = des.simulate_stream(cfg, fns, lo, hi2)
+        ol = np.asarray(r.lat, dtype=np.int64)
+        A = (hi2 - lo) * cfg.interarrival
+        ok = (ol >= 0) & (np.arange(hi2 - lo) * cfg.interarrival + ol < A)
+        assert ok.sum() > 5_000
+        assert np.array_equal(lat[lo:hi2][ok], ol[ok]), s

@@ -131,6 +131,29 @@ def test_injected_stalls_move_time_not_schedule(c2wl, budgets):
         Pipeline(cfg.replace(clock=C.CLOCK_LOGICAL), wl).inject_stalls(period, length)
 
 
+@pytest.mark.parametrize("policy", [C.FIXED_WAIT, C.THRESHOLD_SLACK])
+@pytest.mark.parametrize("tau,D", [(50, 200_000), (400, 1_000_000)])
+def test_c3_sweep_points_physical(c2wl, budgets, policy, tau, D):
+    """BASELINE configs[2] (c2 swept over arrival rate and deadline): two grid points of
+    tools/sweep_c3_dna.py on the physical clock with the GPU's budgets, Fig. 1 waits /
+    thresholds -- the logical schedule bit-exact with the oracle at full c2 size."""
+    from paper_conf_icppw_planob21_b200 import solve_enforced_waits
+    _, wl = c2wl
+    cfg = C.c2(n_streams=148).replace(clock=C.CLOCK_GLOBALTIMER, ns_per_unit=1.0, service_time=budgets,
+                                       interarrival=tau, deadline=D, gain=(0.2234, 1.1469, 0.07856))
+    try:
+        w, th, T, Tc = solve_enforced_waits(cfg)
+    except RuntimeError:
+        pytest.skip("Fig. 1 infeasible at this point for these budgets")
+    if policy == C.FIXED_WAIT:
+        cfg = cfg.replace(wait_time=tuple(w))
+    else:
+        cfg = cfg.replace(policy=policy, wait_threshold=tuple(th), slack_guard=max(budgets))
+    g = run_gpu(cfg, wl, flags=7)
+    compare(cfg, g, run_oracle_parallel(cfg, wl))
+    assert g["stats"]["errors"] == 0
+
+
 def test_physical_zero_misses_1p5x_feasible_rate(c2wl, budgets):
     """Zero measured misses at a rate 1.5x above the Fig. 1 feasibility limit of the budgets
     (at least tau0 = 30 ns)."""
