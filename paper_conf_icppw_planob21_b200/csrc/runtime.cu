@@ -1017,6 +1017,7 @@ pl_status pl_pipeline_drain(pl_pipeline* pl) {
     if (s != PL_OK) return s;
   }
   CUDA_TRY(cudaStreamSynchronize(pl->stream));
+  if (pl->live) pl->pushed = 0;   // the live words went to the rings, not to the handle's DB buffer
   pl->live = false;
   pl->drained = true;
   std::vector<CtaStats> cs(pl->cfg.n_streams);
