@@ -560,6 +560,8 @@ def main():
                           "latency_rel_err_max_without_stall": acc["relerr_clean"],
                           "util_measured_over_model": util_ratio},
             "sustained_items_per_s": world * a.streams * 1e9 / tau,
+            "per_rank": {"items_per_s": value / world, "streams": a.streams,
+                         "workload_seed": f"4 + rank (c5: every rank its own c4 DB)" if c4 else "2 + rank"},
             "window_refills_per_launch": st["window_refills"],
             "utilisation": {"enforced_model": st_all["active_fraction"], "enforced_hw_busy": st["hw_busy_fraction"],
                             "fig1_T": T},
