@@ -31,6 +31,9 @@ __device__ __forceinline__ uint64_t gtimer() {
   asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
   return t;
 }
+// Named barriers (.aligned bar.sync: every warp reaches them converged -- the node loop
+// reconverges its warps after the leader's and the accountant's single-lane work, __syncwarp).
+// The non-.aligned barrier.sync was measured: node 1-3 firings 1.75x slower.
 __device__ __forceinline__ void bar_sync(int id, int n) {
   asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(n) : "memory");
 }
@@ -70,13 +73,16 @@ __device__ __forceinline__ uint64_t gain_hash(uint64_t seed, uint32_t stage, uin
 // bases per step: XOR of two 2-bit-packed 32-bit windows gives a mismatch mask.
 // experiment switches (tools/build_variant.py -D...; defaults = the product build)
 #ifndef PL_WINSTEP_NOINLINE
-#define PL_WINSTEP_NOINLINE 1
+#define PL_WINSTEP_NOINLINE 0   // out of line, the call inside the accountant's divergent branch leaves its warp diverged at the next scan barrier (synccheck)
 #endif
 #ifndef PL_LIVE_GATE
 #define PL_LIVE_GATE 1
 #endif
 #ifndef PL_WATCHDOG
 #define PL_WATCHDOG 1
+#endif
+#ifndef PL_NAP_SHIFT
+#define PL_NAP_SHIFT 2      // long naps sleep rem >> this (a quarter of the remaining time)
 #endif
 #ifndef PL_DBMASK
 #define PL_DBMASK 1
@@ -940,7 +946,7 @@ __device__ __forceinline__ bool nap_until(uint64_t target) {
   if (now >= target) return false;
   while (now < target) {   // __nanosleep may round up to ~2x: nap a quarter of the remaining time
     const uint64_t rem = target - now;
-    __nanosleep(rem > 4096 ? (uint32_t)min(rem >> 2, (uint64_t)(1u << 20)) : (rem > 1024 ? 256u : 64u));
+    __nanosleep(rem > 4096 ? (uint32_t)min(rem >> PL_NAP_SHIFT, (uint64_t)(1u << 20)) : (rem > 1024 ? 256u : 64u));
     now = gtimer();
   }
   return true;
@@ -1104,7 +1110,7 @@ __device__ __forceinline__ void pace(uint64_t target, uint64_t* start_ns, int64_
   if (entry_ns) *entry_ns = now;
   while (now < target) {   // __nanosleep rounds up to powers of two: sleep at most ~rem/4
     const uint64_t rem = target - now;
-    __nanosleep(rem > 4096 ? (uint32_t)min(rem >> 2, (uint64_t)(1u << 20)) : (rem > 1024 ? 256u : (rem > 256 ? 64u : 0u)));
+    __nanosleep(rem > 4096 ? (uint32_t)min(rem >> PL_NAP_SHIFT, (uint64_t)(1u << 20)) : (rem > 1024 ? 256u : (rem > 256 ? 64u : 0u)));
     now = gtimer();
   }
   *start_ns = now;
@@ -1723,6 +1729,7 @@ __device__ void run_node(Ctx& c, Dna dna, int i, int gtid) {
       }
       if ((CL || n0) && nd.sliding) win_step(*c.sh, p, (unsigned char*)dna.win, false);   // slide the DB window
     }
+    __syncwarp();                        // the leader's and the accountant's warps reconverge (bar.sync is .aligned)
     if (n0) {                            // replicated node-0 state, identical in every lane
       R.c0 += n;
       if (nd.fixed) {

@@ -25,3 +25,38 @@ for clock in (0, 1):
     pl.drain()
     print("dna clock", clock, pl.stats()["firings"], flush=True)
     pl.close()
+# round 2: the sliding window (small ring), live ingest (a ring smaller than the stream), the N4
+# cluster executor (DSMEM queues, forced spills), and injected stalls
+import numpy as np  # noqa: E402
+c = cfg.replace(policy=C.THRESHOLD_SLACK, wait_threshold=(128, 127, 99, 10))
+pl = Pipeline(c, wl, flags=7, window_words=256, window_chunk_words=64)
+pl.push(wl.db, wl.db_len)
+pl.drain()
+print("sliding window refills", pl.stats()["window_refills"], flush=True)
+pl.close()
+pl = Pipeline(c, wl, flags=7, window_words=256, window_chunk_words=64)
+pl.live_start(512)
+rng = [pl.stream_words(s) for s in range(c.n_streams)]
+pos = [lo for lo, _ in rng]
+while any(pos[s] < rng[s][1] for s in range(c.n_streams)):
+    sl = []
+    for s in range(c.n_streams):
+        e = min(pos[s] + 61, rng[s][1])
+        sl.append(wl.db[pos[s]:e])
+        pos[s] = e
+    pl.push_all(sl)
+pl.drain()
+print("live ingest", pl.stats()["firings"], flush=True)
+pl.close()
+pl = Pipeline(c, wl, flags=7 | 32, queue_capacity=64)
+pl.push(wl.db, wl.db_len)
+pl.drain()
+print("cluster", pl.stats()["firings"], flush=True)
+pl.close()
+p = c.replace(clock=1, service_time=(4000,) * 4, interarrival=100, deadline=10**7)
+pl = Pipeline(p, wl, flags=7 | 8)
+pl.push(wl.db, wl.db_len)
+pl.inject_stalls(200_000, 50_000)
+pl.drain()
+print("injected stalls", pl.stats()["max_lateness_ns"], flush=True)
+pl.close()
