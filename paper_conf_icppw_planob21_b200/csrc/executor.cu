@@ -81,6 +81,9 @@ __device__ __forceinline__ uint64_t gain_hash(uint64_t seed, uint32_t stage, uin
 #ifndef PL_WATCHDOG
 #define PL_WATCHDOG 1
 #endif
+#ifndef PL_SINK_SPREAD
+#define PL_SINK_SPREAD 0    // the sink's items dealt round-robin over its warps (experiment)
+#endif
 #ifndef PL_NAP_SHIFT
 #define PL_NAP_SHIFT 2      // long naps sleep rem >> this (a quarter of the remaining time)
 #endif
@@ -1451,14 +1454,19 @@ __device__ void run_node(Ctx& c, Dna dna, int i, int gtid) {
       T = G.T[par]; n = G.n[par]; head = G.head[par];
     }
     const bool arrmode = n0 && nd.arr != nullptr;
+    // the item this lane serves: lane order, or -- the sink, whose outputs carry no order (matches,
+    // terminal latencies) -- dealt round-robin over its warps, so that a partial vector's long
+    // extension walks spread over every SMSP instead of filling the first warps (PL_SINK_SPREAD)
+    const uint32_t jt = (PL_SINK_SPREAD && nd.sink && !n0 && v > 32)
+                            ? (uint32_t)((gtid & 31) * (v >> 5) + (gtid >> 5)) : (uint32_t)gtid;
     const bool act = arrmode ? ((uint32_t)gtid < n && R.c0 + gtid < nd.X &&
                                 __ldg(nd.arr + nd.lo + R.c0 + gtid) <= T)
-                             : (uint32_t)gtid < n;
+                             : jt < n;
     uint2 e[1];
     const bool acts[1] = {act};
     LaneOut o[1];
     {
-      const uint32_t ld = act ? (uint32_t)gtid : 0u;   // inactive lanes repeat a valid entry
+      const uint32_t ld = act ? jt : 0u;   // inactive lanes repeat a valid entry
       if (n0) e[0] = make_uint2((uint32_t)(nd.lo + head + ld), 0u);
       else e[0] = load_entry(nd, head + ld, G.segh[par], G.st[par], G.in_spill_end[par]);
     }
@@ -1516,13 +1524,13 @@ __device__ void run_node(Ctx& c, Dna dna, int i, int gtid) {
         atomicMax((long long*)&p.lat[ei.x], (long long)(T + nd.t - nd.arrival(ei.x)));
         if (nd.phys) pend_root = ei.x;
       }
-      if (act && (rec & PL_REC_FIRINGS) && (gtid == 0 || (uint32_t)gtid == n - 1)) {
+      if (act && (rec & PL_REC_FIRINGS) && (jt == 0 || jt == n - 1)) {
         const uint32_t li = G.log_idx[par];
         if (li < p.log_cap) {
           pl_firing* f = p.flog + (uint64_t)stream * p.log_cap + li;
-          if (gtid == 0) { f->start = T; f->node = i; f->n = n; f->first_root = ei.x; f->stream = stream; f->pad = 0; }
-          if ((uint32_t)gtid == n - 1) f->last_root = ei.x;
-        } else if (gtid == 0) {
+          if (jt == 0) { f->start = T; f->node = i; f->n = n; f->first_root = ei.x; f->stream = stream; f->pad = 0; }
+          if (jt == n - 1) f->last_root = ei.x;
+        } else if (jt == 0) {
           atomicOr(&AG.errors, PL_ERR_LOG_OVERFLOW);
         }
       }
