@@ -81,11 +81,14 @@ __device__ __forceinline__ uint64_t gain_hash(uint64_t seed, uint32_t stage, uin
 #ifndef PL_WATCHDOG
 #define PL_WATCHDOG 1
 #endif
+#ifndef PL_S3_PREFETCH
+#define PL_S3_PREFETCH 0    // X-drop walks load the next step's words one step ahead (experiment)
+#endif
 #ifndef PL_SINK_SPREAD
-#define PL_SINK_SPREAD 0    // the sink's items dealt round-robin over its warps (experiment)
+#define PL_SINK_SPREAD 1    // the sink's items dealt round-robin over its warps: c4 node-3 mean firing -6 %, logical run -5 %
 #endif
 #ifndef PL_NAP_SHIFT
-#define PL_NAP_SHIFT 2      // long naps sleep rem >> this (a quarter of the remaining time)
+#define PL_NAP_SHIFT 1      // long naps sleep half the remaining time (__nanosleep: at most 2x): -9 % instructions on c4
 #endif
 #ifndef PL_DBMASK
 #define PL_DBMASK 1
@@ -201,6 +204,11 @@ struct Dna {
     const uint32_t* qp = qw + (sq >> 4);
     uint32_t shd = (uint32_t)(sd & 15) * 2u, shq = (uint32_t)(sq & 15) * 2u;
     uint32_t dc = win[(dw + 1u) & win_mask], qc = qp[1];              // carried word
+#if PL_S3_PREFETCH
+    // the next step's words are loaded one step ahead, off the mismatch loop's dependency chain
+    // (one word past a walk's end at most: the ring index is masked, the query is padded)
+    uint32_t dnx = win[dw & win_mask], qnx = *qp;
+#endif
     int step = -1;
     bool right = false;
     uint32_t limit = ll, d = 0;
@@ -208,9 +216,17 @@ struct Dna {
     for (;;) {
       bool fin = d >= limit;
       if (!fin) {
+#if PL_S3_PREFETCH
+        const uint32_t dn = dnx, qn = qnx;
+        dw += (uint32_t)step;
+        qp += step;
+        dnx = win[dw & win_mask];
+        qnx = *qp;
+#else
         const uint32_t dn = win[dw & win_mask], qn = *qp;
         dw += (uint32_t)step;
         qp += step;
+#endif
         const uint32_t x = right ? (__funnelshift_r(dc, dn, shd) ^ __funnelshift_r(qc, qn, shq))
                                  : (__funnelshift_r(dn, dc, shd) ^ __funnelshift_r(qn, qc, shq));
         dc = dn;
@@ -270,6 +286,10 @@ struct Dna {
         shq = (uint32_t)(sq & 15) * 2u;
         dc = win[dw++ & win_mask];
         qc = *qp++;
+#if PL_S3_PREFETCH
+        dnx = win[dw & win_mask];
+        qnx = *qp;
+#endif
       }
     }
     *br = best;
@@ -947,7 +967,7 @@ __device__ __forceinline__ void advance0(const Node& nd, Rep& r) {
 __device__ __forceinline__ bool nap_until(uint64_t target) {
   uint64_t now = gtimer();
   if (now >= target) return false;
-  while (now < target) {   // __nanosleep may round up to ~2x: nap a quarter of the remaining time
+  while (now < target) {   // __nanosleep sleeps at most 2x its argument: nap rem >> PL_NAP_SHIFT
     const uint64_t rem = target - now;
     __nanosleep(rem > 4096 ? (uint32_t)min(rem >> PL_NAP_SHIFT, (uint64_t)(1u << 20)) : (rem > 1024 ? 256u : 64u));
     now = gtimer();
@@ -1111,7 +1131,7 @@ __device__ __forceinline__ uint32_t reserve_out(const Node& nd, Leader& L, uint3
 __device__ __forceinline__ void pace(uint64_t target, uint64_t* start_ns, int64_t* late, uint64_t* entry_ns = nullptr) {
   uint64_t now = gtimer();
   if (entry_ns) *entry_ns = now;
-  while (now < target) {   // __nanosleep rounds up to powers of two: sleep at most ~rem/4
+  while (now < target) {   // __nanosleep sleeps at most 2x its argument: nap rem >> PL_NAP_SHIFT
     const uint64_t rem = target - now;
     __nanosleep(rem > 4096 ? (uint32_t)min(rem >> PL_NAP_SHIFT, (uint64_t)(1u << 20)) : (rem > 1024 ? 256u : (rem > 256 ? 64u : 0u)));
     now = gtimer();
