@@ -85,7 +85,8 @@ __device__ __forceinline__ uint64_t gain_hash(uint64_t seed, uint32_t stage, uin
 #define PL_S3_PREFETCH 0    // X-drop walks load the next step's words one step ahead (experiment)
 #endif
 #ifndef PL_SINK_SPREAD
-#define PL_SINK_SPREAD 1    // the sink's items dealt round-robin over its warps: c4 node-3 mean firing -6 %, logical run -5 %
+#define PL_SINK_SPREAD 0    // the sink's items dealt round-robin over its warps: c4 node-3 mean firing -6 %, but c2's longest
+                            // node-3 firing +30 % (every warp then iterates the longest walk): rejected
 #endif
 #ifndef PL_NAP_SHIFT
 #define PL_NAP_SHIFT 1      // long naps sleep half the remaining time (__nanosleep: at most 2x): -9 % instructions on c4
