@@ -325,3 +325,20 @@ def test_pipelined_steps_match_oracle():
     assert s["roots"] == roots and s["matches"] == len(o.matches)
     assert pl.results() == [tuple(m) for m in o.matches]
     pl.close()
+
+
+@pytest.mark.parametrize("policy", [C.FIXED_WAIT, C.THRESHOLD_SLACK])
+def test_extreme_gain_tables(policy):
+    """Threshold tables at their edges (the round-1 advisor's prob_to_u64 case): min(Poisson(60), 16)
+    -- every CDF(k < 16) is below 2^-64, so every threshold is 0 and every input emits 16 --
+    a Bernoulli(1e-30) filter that keeps nothing, and Bernoulli(1.0) that keeps everything."""
+    st = [C.Stage(C.BERNOULLI, 1.0, 1), C.Stage(C.POISSON_CAPPED, 60.0, 16), C.Stage(C.BERNOULLI, 1e-30, 1)]
+    cfg = C.Config(name="edge", stages=st, service_time=(40, 55, 30), vector_width=32, deadline=50_000,
+                   interarrival=20, b=(1, 1, 1), wait_time=(60, 20, 300), wait_threshold=(32, 16, 32),
+                   policy=policy, n_streams=2, n_roots=400, seed=9)
+    g = run_gpu(cfg, None)
+    compare(cfg, g, run_oracle(cfg, None))
+    st_ = g["stats"]
+    assert st_["produced"][0] == st_["consumed"][0]                 # Bernoulli(1.0) keeps all
+    assert st_["produced"][1] == 16 * st_["consumed"][1]            # Poisson(60) capped at 16
+    assert st_["produced"][2] == 0                                  # Bernoulli(1e-30) keeps nothing
