@@ -342,3 +342,15 @@ def test_extreme_gain_tables(policy):
     assert st_["produced"][0] == st_["consumed"][0]                 # Bernoulli(1.0) keeps all
     assert st_["produced"][1] == 16 * st_["consumed"][1]            # Poisson(60) capped at 16
     assert st_["produced"][2] == 0                                  # Bernoulli(1e-30) keeps nothing
+
+
+@pytest.mark.parametrize("k,W,X,u", [(7, 8, 20, 16), (4, 12, 8, 5), (5, 8, 35, 16)])
+def test_dna_stage_parameters(k, W, X, u):
+    """The DNA chain off its defaults: k = 7 (the largest direct-address table, 16 K entries),
+    short seeds with a W = 12 window (the checked S2 walk: W > 8) and a small hit cap u = 5, a
+    large X-drop; a query and DB whose lengths are not multiples of 16; bit-exact."""
+    stages = C.dna_stages(k=k, u=u, W=W, X=X, T3=max(2 * k, 20))
+    cfg = C.c2(stages=stages, n_streams=3, dna=dict(db_len=20_011, q_len=3_001, n_planted=10)).replace(
+        policy=C.THRESHOLD_SLACK, wait_threshold=(128, 100, 64, 8))
+    wl = workload_for(cfg)
+    compare(cfg, run_gpu(cfg, wl), run_oracle(cfg, wl))
