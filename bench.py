@@ -89,9 +89,12 @@ def parse():
     ap.add_argument("--probe-t", type=int, default=None,
                     help="budget probe: every node's budget during the probe (ns; default c4 1000 = all nodes "
                          "overloaded, sharing the SM as in a catch-up, L69's 1/N share; c2 20000)")
-    ap.add_argument("--headroom", type=float, default=1.0,
-                    help="operating tau0 = headroom x the fastest stall-free miss-free tau0 (R-STALL: the "
-                         "pipeline must catch up after a ~1.6 ms platform stall within D)")
+    ap.add_argument("--headroom", type=float, default=1.08,
+                    help="operating tau0 = headroom x the fastest tau0 miss-free across injected stalls "
+                         "(R-STALL: the pipeline must catch up after a ~1.6 ms platform stall within D; the "
+                         "injected stalls sample ~20 stream phases per run, a platform stall lands anywhere, "
+                         "and 1.5 %% below the edge the catch-up fails by tens of ms: "
+                         "profiles/r02_bench_c4_edge_miss.json)")
     a = ap.parse_args()
     if a.deadline_ns is None:
         a.deadline_ns = 3_500_000 if a.workload == "c4" else 350_000
