@@ -4,4 +4,4 @@ for rep in 1 2; do
   timeout 300 python tools/probe_c4.py in-tree
   PLGPU_LIB=_variants/x_spread.so timeout 300 python tools/probe_c4.py spread
 done
-bash tools/r02_nap_ab.sh >&2
+bash tools/gpurun/r02_nap_ab.sh >&2

@@ -1,5 +1,5 @@
 """profiles/ncu_summary_<workload>.json for bench.py's `roofline.traffic` and `issue` fields, from
-one `ncu --set full` capture of the headline kernel (tools/r02_evidence.sh) and the util pass
+one `ncu --set full` capture of the headline kernel (tools/gpurun/r02_evidence.sh) and the util pass
 (enforced vs monolithic at the same tau0, D).
 
 usage: python tools/ncu_bench_summary.py <full.ncu-rep> <util.csv> <roots_per_launch> <alg_bytes> <out.json>"""

@@ -1,3 +1,4 @@
+"""Threshold slack-guard sweep: THRESHOLD_SLACK at guards {0, 2e4, 6e4} on the physical clock."""
 import json, sys
 sys.path.insert(0, ".")
 import torch
