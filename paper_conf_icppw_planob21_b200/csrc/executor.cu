@@ -97,6 +97,16 @@ __device__ __forceinline__ uint64_t gain_hash(uint64_t seed, uint32_t stage, uin
 #ifndef PL_INJECT
 #define PL_INJECT 1
 #endif
+#ifndef PL_S3_COOP
+#define PL_S3_COOP 0        // S3 X-drop: serial rounds, then a warp-cooperative finisher for the last long walks;
+                            // bit-exact, but c4 node-3 longest firing x2 (17.5 -> 36 us) and nodes 0-2 +10-20 %: rejected
+#endif
+#ifndef PL_S3_SB
+#define PL_S3_SB 8          // serial 16-base steps per round of the hybrid walk
+#endif
+#ifndef PL_S3_COOPMAX
+#define PL_S3_COOPMAX 4     // unfinished lanes the cooperative finisher takes over
+#endif
 #ifndef PL_S3_MSB
 #define PL_S3_MSB 1
 #endif
@@ -305,6 +315,230 @@ struct Dna {
     const uint32_t* w = qw + (s >> 4);
     return __funnelshift_r(w[0], w[1], (uint32_t)(s & 15) * 2u);
   }
+#if PL_S3_COOP
+  // ---- S3 hybrid walk (PL_S3_COOP): extend2_win's loop made resumable, plus a warp-cooperative
+  // finisher for the few lanes whose walks outlast the serial budget.  A warp of serial walks
+  // iterates as long as its longest lane (repeat islands: one 1 kbp walk holds 31 idle lanes);
+  // the finisher gives such a walk all 32 lanes, 16 steps each.  Scores, X-drop and the
+  // smallest best position are exactly extend()'s (R-S3), so the outputs are unchanged.
+  struct XWalk {
+    uint32_t dw, dc, qc, shd, shq, limit, d;
+    const uint32_t* qp;
+    int step, score, best, db_, bl, dl;
+    bool right, done;
+  };
+  __device__ __forceinline__ void xw_left(XWalk& w, uint32_t p, uint32_t q, uint32_t ll) const {
+    const int32_t sd = (int32_t)p - 16, sq = (int32_t)q - 16;
+    w.dw = (uint32_t)(sd >> 4);
+    w.qp = qw + (sq >> 4);
+    w.shd = (uint32_t)(sd & 15) * 2u;
+    w.shq = (uint32_t)(sq & 15) * 2u;
+    w.dc = win[(w.dw + 1u) & win_mask];
+    w.qc = w.qp[1];
+    w.step = -1;
+    w.right = false;
+    w.done = false;
+    w.limit = ll;
+    w.d = 0;
+    w.score = w.best = w.db_ = 0;
+    w.bl = w.dl = 0;
+  }
+  __device__ __forceinline__ void xw_right(XWalk& w, uint32_t p, uint32_t q, uint32_t rl) const {
+    const int32_t sd = (int32_t)(p + (uint32_t)k), sq = (int32_t)(q + (uint32_t)k);
+    w.dw = (uint32_t)(sd >> 4);
+    w.qp = qw + (sq >> 4);
+    w.shd = (uint32_t)(sd & 15) * 2u;
+    w.shq = (uint32_t)(sq & 15) * 2u;
+    w.dc = win[w.dw++ & win_mask];
+    w.qc = *w.qp++;
+    w.step = 1;
+    w.right = true;
+    w.limit = rl;
+    w.d = 0;
+    w.score = w.best = w.db_ = 0;
+  }
+  // up to `budget` 16-base steps of the left-then-right walk (extend2_win's loop, MSB-first)
+  __device__ __forceinline__ void xw_run(XWalk& w, int budget, uint32_t p, uint32_t q, uint32_t rl, int X) const {
+    for (; budget > 0; --budget) {
+      bool fin = w.d >= w.limit;
+      if (!fin) {
+        const uint32_t dn = win[w.dw & win_mask], qn = *w.qp;
+        w.dw += (uint32_t)w.step;
+        w.qp += w.step;
+        const uint32_t x = w.right ? (__funnelshift_r(w.dc, dn, w.shd) ^ __funnelshift_r(w.qc, qn, w.shq))
+                                   : (__funnelshift_r(dn, w.dc, w.shd) ^ __funnelshift_r(qn, w.qc, w.shq));
+        w.dc = dn;
+        w.qc = qn;
+        const uint32_t n = (w.limit - w.d) < 16u ? (w.limit - w.d) : 16u;
+        uint32_t mm = (x | (x >> 1)) & 0x55555555u;
+        if (w.right) mm = __brev(mm);
+        uint32_t mmv = mm & (0xffffffffu << (32u - 2u * n));
+        int last = 0;
+        while (mmv) {
+          const uint32_t c = __clz(mmv);
+          const int e = (int)(c >> 1);
+          mmv &= 0x7fffffffu >> c;
+          w.score += e - last;
+          if (w.score > w.best) { w.best = w.score; w.db_ = (int)w.d + e; }
+          w.score -= 3;
+          last = e + 1;
+          if (X > 0 && w.score <= w.best - X) { fin = true; break; }
+        }
+        if (!fin) {
+          w.score += (int)n - last;
+          if (w.score > w.best) { w.best = w.score; w.db_ = (int)(w.d + n); }
+          w.d += n;
+        }
+      }
+      if (fin) {
+        if (w.right) { w.done = true; return; }
+        w.bl = w.best;
+        w.dl = w.db_;
+        xw_right(w, p, q, rl);
+      }
+    }
+  }
+  // Lane L's unfinished walk, finished by the whole (converged) warp.  Per round lane j scores
+  // steps d+16j+1 .. d+16j+16 of the current direction: its chunk total, its peak (the
+  // earliest), its lowest trough and its deepest fall below its own running peak.  A warp sum
+  // scan gives each chunk its entering score S_j, a max scan its entering best B_j; chunk j
+  // holds an X-drop iff S_j + trough - B_j <= -X or its own fall <= -X (a fall below the
+  // running best happens only just after a mismatch, and is the larger of the two).  The
+  // first such chunk is replayed serially by its lane from (S_j, B_j); without one the walk
+  // moves on 512 steps.
+  __device__ __forceinline__ void xw_coop(XWalk& w, int L, uint32_t p, uint32_t q, uint32_t rl, int X) const {
+    const unsigned F = 0xffffffffu;
+    const int lane = threadIdx.x & 31;
+    bool right = __shfl_sync(F, (int)w.right, L) != 0;
+    uint32_t d = __shfl_sync(F, w.d, L), limit = __shfl_sync(F, w.limit, L);
+    int S = __shfl_sync(F, w.score, L), B = __shfl_sync(F, w.best, L), P = __shfl_sync(F, w.db_, L);
+    int bl = __shfl_sync(F, w.bl, L), dl = __shfl_sync(F, w.dl, L);
+    const uint32_t pL = __shfl_sync(F, p, L), qL = __shfl_sync(F, q, L), rlL = __shfl_sync(F, rl, L);
+    for (;;) {
+      bool end = d >= limit;   // warp-uniform
+      if (!end) {
+        const uint32_t d0 = d + 16u * (uint32_t)lane;
+        const uint32_t n = d0 < limit ? ((limit - d0) < 16u ? (limit - d0) : 16u) : 0u;
+        uint32_t mm = 0;         // bit 2e: mismatch at step d0 + 1 + e
+        if (n) {
+          if (right) {
+            const uint32_t x = db16w((int32_t)(pL + (uint32_t)k + d0)) ^ q16w((int32_t)(qL + (uint32_t)k + d0));
+            mm = (x | (x >> 1)) & 0x55555555u;
+          } else {
+            const uint32_t x = db16w((int32_t)pL - (int32_t)d0 - 16) ^ q16w((int32_t)qL - (int32_t)d0 - 16);
+            mm = __brev((x | (x >> 1)) & 0x55555555u) >> 1;
+          }
+          mm &= n >= 16u ? 0xffffffffu : ((1u << (2u * n)) - 1u);
+        }
+        int pre = 0, mx = 0, am = 0, mn = 1 << 29, fall = 0, last = 0;
+        for (uint32_t v = mm; v; v &= v - 1) {
+          const int e = (__ffs(v) - 1) >> 1;
+          pre += e - last;
+          if (pre > mx) { mx = pre; am = e; }
+          pre -= 3;
+          last = e + 1;
+          mn = min(mn, pre);
+          fall = min(fall, pre - mx);
+        }
+        pre += (int)n - last;
+        if (pre > mx) { mx = pre; am = (int)n; }
+        int incl = pre;
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+          const int t = __shfl_up_sync(F, incl, o);
+          if (lane >= o) incl += t;
+        }
+        const int Sin = S + incl - pre;
+        const int cand = Sin + mx;
+        int cm = cand;
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+          const int t = __shfl_up_sync(F, cm, o);
+          if (lane >= o) cm = max(cm, t);
+        }
+        const int up = __shfl_up_sync(F, cm, 1);
+        const int Bin = lane ? max(B, up) : B;
+        const bool drop = X > 0 && n && (Sin + mn - Bin <= -X || fall <= -X);
+        const uint32_t db = __ballot_sync(F, drop);
+        const int top = db ? __ffs(db) - 1 : 31;
+        const int V = db ? __shfl_sync(F, Bin, top) : max(B, __shfl_sync(F, cm, 31));
+        int pos = P;
+        if (V > B) {   // the earliest chunk (before the drop's) whose peak is V
+          const uint32_t hit = __ballot_sync(F, cand == V && (!db || lane < top));
+          pos = __shfl_sync(F, (int)d0 + am, __ffs(hit) - 1);
+        }
+        if (db) {
+          int b = V, bp = pos;
+          if (lane == top) {
+            int s = Sin;
+            last = 0;
+            for (uint32_t v = mm; v; v &= v - 1) {
+              const int e = (__ffs(v) - 1) >> 1;
+              s += e - last;
+              if (s > b) { b = s; bp = (int)d0 + e; }
+              s -= 3;
+              last = e + 1;
+              if (s <= b - X) break;
+            }
+          }
+          B = __shfl_sync(F, b, top);
+          P = __shfl_sync(F, bp, top);
+          end = true;
+        } else {
+          S += __shfl_sync(F, incl, 31);
+          B = V;
+          P = pos;
+          d += 512u;
+          end = d >= limit;
+        }
+      }
+      if (end) {
+        if (right) break;
+        bl = B;
+        dl = P;
+        right = true;
+        d = 0;
+        limit = rlL;
+        S = B = P = 0;
+      }
+    }
+    if (lane == L) {
+      w.bl = bl;
+      w.dl = dl;
+      w.best = B;
+      w.db_ = P;
+      w.right = true;
+      w.done = true;
+    }
+  }
+  // Both X-drop walks of every `on` lane (all 32 lanes call it, converged): serial rounds of
+  // PL_S3_SB steps while more than PL_S3_COOPMAX lanes are unfinished, then the finisher.
+  __device__ __forceinline__ void xdrop_hybrid(bool on, uint32_t p, uint32_t q, uint32_t ll, uint32_t rl, int X,
+                                               int* bl, int* dl, int* br, int* dr) const {
+    XWalk w;
+    if (on) xw_left(w, p, q, ll);
+    else w.done = true;
+    for (;;) {
+      if (!w.done) xw_run(w, PL_S3_SB, p, q, rl, X);
+      uint32_t rem = __ballot_sync(0xffffffffu, !w.done);
+      if (!rem) break;
+      if (__popc(rem) <= PL_S3_COOPMAX) {
+        while (rem) {
+          const int L = __ffs(rem) - 1;
+          rem &= rem - 1;
+          xw_coop(w, L, p, q, rl, X);
+        }
+        break;
+      }
+    }
+    if (on) {
+      *bl = w.bl;
+      *dl = w.dl;
+      *br = w.best;
+      *dr = w.db_;
+    }
+  }
+#endif
   // bits 0, 2, .., 14 of x -> bits 0..7
   static __device__ __forceinline__ uint32_t even_bits8(uint32_t x) {
     x &= 0x5555u;
@@ -740,6 +974,36 @@ __device__ __forceinline__ LaneOut stage_count_ext(const Node& nd, const Dna& dn
   }
   return o;
 }
+
+#if PL_S3_COOP
+// S3 for one entry per lane, called by the whole converged warp: walks outside the smem window
+// take the checked per-lane path, the others the hybrid walk (Dna::xdrop_hybrid).
+__device__ __forceinline__ LaneOut stage_xdrop_warp(const Node& nd, const Dna& dna, uint2 e, bool act) {
+  LaneOut o;
+  o.c = 0; o.a = 0; o.score = 0; o.q_start = 0; o.len = 0;
+  const uint32_t q = e.y & 0xffffu;
+  const uint32_t ll = act ? (uint32_t)dna.left_limit(e.x, q) : 0u;
+  const uint32_t rl = act ? (uint32_t)dna.right_limit(e.x, q) : 0u;
+  const int X = nd.ip1;
+  const bool fast = act && dna.in_win(e.x, ll, rl);
+  int dl = 0, dr = 0, bl = 0, br = 0;
+  if (act && !fast) {
+    bl = dna.extend(e.x, q, -1, ll, X, &dl);
+    br = dna.extend(e.x, q, +1, rl, X, &dr);
+  }
+  __syncwarp();
+  dna.xdrop_hybrid(fast, e.x, q, ll, rl, X, &bl, &dl, &br, &dr);
+  const int score = dna.k + bl + br;
+  if (act && score >= nd.ip2) {
+    o.c = 1;
+    o.score = score;
+    o.a = e.x - dl;
+    o.q_start = q - dl;
+    o.len = dna.k + dl + dr;
+  }
+  return o;
+}
+#endif
 
 __device__ __forceinline__ LaneOut stage_count(const Node& nd, const Dna& dna, const DevParams& p, uint2 e) {
   LaneOut o;
@@ -1259,6 +1523,13 @@ __device__ __forceinline__ void stage_batch(const Node& nd, const Dna& dna, cons
       o[j].c = act[j] ? n : 0u;
     }
   } else {   // S2 window filter / S3 x-drop: per item, one shared copy of the code
+#if PL_S3_COOP
+    if (nd.kind == PL_UNGAPPED_XDROP) {   // warp-uniform: the hybrid walk is warp-collective
+#pragma unroll
+      for (int j = 0; j < K; ++j) o[j] = stage_xdrop_warp(nd, dna, e[j], act[j]);
+      return;
+    }
+#endif
 #pragma unroll
     for (int j = 0; j < K; ++j) {
 #if PL_S3_DEBUG
