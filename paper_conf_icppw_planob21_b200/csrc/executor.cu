@@ -2605,90 +2605,167 @@ cudaError_t pl_kernel_attributes(unsigned max_smem) {
 }
 
 // ------------------------------------------------------------- stage batch kernels
-// K-BENCH: one stage over a large batch, vectors of v inputs per CTA iteration, DB read
-// from global memory (no smem window), query index in smem; outputs compacted per vector
-// (block scan) and appended at an atomically reserved offset.
-template <int MAXT>
-__global__ void __launch_bounds__(MAXT, 1) pl_stage_batch_kernel(const __grid_constant__ DevParams p, int stage,
-                                                                 const uint2* in, uint64_t n, uint64_t first_root,
-                                                                 uint2* out, uint64_t cap, unsigned long long* cnt) {
+// K-BENCH (SURVEY K-BENCH; north_star "achieved HBM GB/s of each stage kernel"): one stage over
+// a large device-resident batch at full occupancy, with the executor's own stage bodies
+// (stage_batch<J, KIND>: J = 4 consecutive items per lane, their latency chains interleaved).
+// Each warp takes chunks of 128 consecutive inputs (two coalesced 16-byte loads per lane), scans
+// its lanes' output counts with shuffles and reserves its output range with ONE atomic per chunk;
+// outputs stay in input order within a chunk.  The DB is the extension's "window" in global
+// memory (the whole DB, read-only), so S2 / S3 take the executor's fast in-window walks; only
+// seeds within a walk's reach of the DB ends take the checked ones.  Shared memory holds only
+// the query index, so several CTAs share an SM.
+struct KbLayout { uint32_t qpos, qw, s2, total; };
+__host__ __device__ inline KbLayout layout_kbench(const DevParams& p) {
+  KbLayout L;
+  uint32_t off = 0;
+  const bool dna = p.k > 0;
+  off += dna ? (((1u << (2 * p.k)) + 1u) * 2u + 15u) & ~15u : 0u;   // qoff at 0
+  L.qpos = off;
+  off += dna ? (((uint32_t)(p.q_len - p.k + 1) * 2u) + 15u) & ~15u : 0u;
+  L.qw = off + (dna ? 16u : 0u);                                     // one 16-byte pad on each side
+  off += dna ? 32u + ((((uint32_t)(p.q_len + 15) / 16u) * 4u + 15u) & ~15u) : 0u;
+  L.s2 = off;
+  off += dna ? 256u : 0u;
+  L.total = off > 16u ? off : 16u;
+  return L;
+}
+constexpr int KB_THREADS = 256;
+constexpr int KB_J = 4;
+
+template <int KIND>
+__global__ void __launch_bounds__(KB_THREADS, 4) pl_kbench_kernel(const __grid_constant__ DevParams p, int stage,
+                                                                  const uint2* in, uint64_t n, uint64_t first_root,
+                                                                  uint2* out, uint64_t cap, unsigned long long* cnt) {
   extern __shared__ __align__(16) unsigned char dsm[];
-  __shared__ Shared sh;
-  __shared__ uint32_t wt[32];
-  __shared__ unsigned long long sbase;
-  Ctx c;
-  c.p = &p;
-  c.sh = &sh;
-  c.dsm = dsm;
-  c.lo = 0;
-  c.hi = p.total_roots;
-  c.X = (int64_t)p.total_roots;
-  c.H = c.X * p.tau;
-  SmemLayout Lo;
-  layout_enforced(p, &Lo);
-  c.dna.db = p.db; c.dna.nwords = p.db_words; c.dna.db_len = p.db_len; c.dna.k = p.k; c.dna.q_len = p.q_len;
-  c.dna.qoff = (const uint16_t*)(dsm + Lo.off_qoff);
-  c.dna.qpos = (const uint16_t*)(dsm + Lo.off_qpos);
-  c.dna.qw = (const uint32_t*)(dsm + Lo.off_qw);
-  c.dna.nqw = (uint32_t)(p.q_len + 15) / 16u;
-  c.dna.win = nullptr; c.dna.win_lo = 0; c.dna.win_lo32 = 0; c.dna.win_n = 0; c.dna.win_mask = 0;
-  c.dna.dbmask = 0xffffffffu;
-  c.dna.nofast = true; c.dna.s2tab = nullptr;
-  c.sliding = false;
-  const uint32_t tid = threadIdx.x, v = blockDim.x;
+  const KbLayout Lo = layout_kbench(p);
+  const uint32_t tid = threadIdx.x, nt = blockDim.x;
+  Dna dna;
+  dna.db = p.db; dna.dbmask = 0xffffffffu; dna.nwords = p.db_words; dna.db_len = p.db_len;
+  dna.k = p.k; dna.q_len = p.q_len;
+  dna.win = p.db; dna.win_lo = 0; dna.win_lo32 = 0; dna.win_n = p.db_words; dna.win_mask = 0xffffffffu;
+  dna.nofast = false;
+  dna.qoff = (const uint16_t*)dsm;
+  dna.qpos = (const uint16_t*)(dsm + Lo.qpos);
+  dna.qw = (const uint32_t*)(dsm + Lo.qw);
+  dna.nqw = (uint32_t)(p.q_len + 15) / 16u;
+  dna.s2tab = dsm + Lo.s2;
   if (p.k > 0) {
     const uint32_t nko = (1u << (2 * p.k)) + 1u, nqp = (uint32_t)(p.q_len - p.k + 1);
-    uint16_t* qo = (uint16_t*)(dsm + Lo.off_qoff);
-    uint16_t* qp = (uint16_t*)(dsm + Lo.off_qpos);
-    uint32_t* qw = (uint32_t*)(dsm + Lo.off_qw);
-    for (uint32_t j = tid; j < nko; j += v) qo[j] = p.qoff[j];
-    for (uint32_t j = tid; j < nqp; j += v) qp[j] = p.qpos[j];
-    for (uint32_t j = tid; j < c.dna.nqw; j += v) qw[j] = p.qwords[j];
-    if (tid < 8) qw[tid < 4 ? (int)tid - 4 : (int)(c.dna.nqw + tid - 4u)] = 0u;   // pad words
+    uint16_t* qo = (uint16_t*)dsm;
+    uint16_t* qp = (uint16_t*)(dsm + Lo.qpos);
+    uint32_t* qw = (uint32_t*)(dsm + Lo.qw);
+    for (uint32_t j = tid; j < nko; j += nt) qo[j] = p.qoff[j];
+    for (uint32_t j = tid; j < nqp; j += nt) qp[j] = p.qpos[j];
+    for (uint32_t j = tid; j < dna.nqw; j += nt) qw[j] = p.qwords[j];
+    if (tid < 8) qw[tid < 4 ? (int)tid - 4 : (int)(dna.nqw + tid - 4u)] = 0u;   // pad words
+    for (uint32_t m = tid; m < 256u; m += nt) {   // S2 table (as the executor's)
+      int sc = 0, best = 0;
+      for (int e = 0; e < 8; ++e) {
+        sc += ((m >> e) & 1u) ? -3 : 1;
+        best = sc > best ? sc : best;
+      }
+      (dsm + Lo.s2)[m] = (unsigned char)best;
+    }
   }
-  if (tid == 0) { sh.errors = 0; }
   __syncthreads();
-  const Node nd = make_node(c, stage);
-  const bool sink = stage == p.N - 1;
-  for (uint64_t vec = blockIdx.x; vec * v < n; vec += gridDim.x) {
+  Node nd;
+  nd.i = stage; nd.N = p.N; nd.v = p.v;
+  nd.sink = stage == p.N - 1;
+  const DevStage& sd = p.st[stage];
+  nd.kind = sd.kind; nd.max_out = sd.max_out; nd.cfix = sd.cfix;
+  nd.umax = sd.kind == PL_FIXED_GAIN ? sd.cfix : sd.max_out;
+  nd.ip1 = sd.ip[1]; nd.ip2 = sd.ip[2];
+  const bool xdrop_sink = nd.sink && nd.kind == PL_UNGAPPED_XDROP;
+  const int lane = (int)(tid & 31u);
+  constexpr uint32_t CH = 32u * KB_J;
+  const uint64_t nw = ((uint64_t)gridDim.x * nt) >> 5;
+  uint32_t maxc = 0;
+  for (uint64_t ch = ((uint64_t)blockIdx.x * nt + tid) >> 5; ch * CH < n; ch += nw) {
     const long long c0 = clock64();
-    const uint64_t idx = vec * v + tid;
-    const bool act = idx < n;
-    uint2 e = make_uint2(0u, 0u);
-    if (act) e = stage == 0 ? make_uint2((uint32_t)(first_root + idx), 0u) : __ldg(in + idx);
-    LaneOut o;
-    if (act) o = stage_count(nd, c.dna, p, e);
-    else { o.c = 0; o.a = 0; o.score = 0; o.q_start = 0; o.len = 0; }
-    uint32_t total;
-    const uint32_t off = block_scan(o.c, &total, wt);
-    if (tid == 0) sbase = total ? atomicAdd(cnt, (unsigned long long)total) : 0ull;
-    __syncthreads();
-    const unsigned long long base = sbase;
-    if (act && o.c) {
-      if (sink && nd.kind == PL_UNGAPPED_XDROP) {
-        const unsigned long long mi = base + off;
-        if (mi < p.match_cap) {
+    const uint64_t b = ch * CH + (uint64_t)lane * KB_J;
+    uint2 e[KB_J];
+    bool act[KB_J];
+#pragma unroll
+    for (int j = 0; j < KB_J; ++j) act[j] = b + j < n;
+    if (stage == 0) {
+#pragma unroll
+      for (int j = 0; j < KB_J; ++j) e[j] = make_uint2((uint32_t)(first_root + (act[j] ? b + j : 0)), 0u);
+    } else if (b + KB_J <= n && ((reinterpret_cast<uintptr_t>(in) & 15u) == 0)) {
+      const uint4 x = __ldg(reinterpret_cast<const uint4*>(in + b));
+      const uint4 y = __ldg(reinterpret_cast<const uint4*>(in + b) + 1);
+      e[0] = make_uint2(x.x, x.y); e[1] = make_uint2(x.z, x.w);
+      e[2] = make_uint2(y.x, y.y); e[3] = make_uint2(y.z, y.w);
+    } else {
+#pragma unroll
+      for (int j = 0; j < KB_J; ++j) e[j] = act[j] ? __ldg(in + b + j) : __ldg(in);
+    }
+    LaneOut o[KB_J];
+    stage_batch<KB_J, KIND>(nd, dna, p, e, act, o);
+    uint32_t mine = 0;
+#pragma unroll
+    for (int j = 0; j < KB_J; ++j) mine += o[j].c;
+    uint32_t incl = mine;
+#pragma unroll
+    for (int d = 1; d < 32; d <<= 1) {
+      const uint32_t t = __shfl_up_sync(0xffffffffu, incl, d);
+      if (lane >= d) incl += t;
+    }
+    const uint32_t total = __shfl_sync(0xffffffffu, incl, 31);
+    unsigned long long base = 0;
+    if (lane == 0 && total) base = atomicAdd(cnt, (unsigned long long)total);
+    base = __shfl_sync(0xffffffffu, base, 0) + (incl - mine);
+#pragma unroll
+    for (int j = 0; j < KB_J; ++j) {
+      if (!o[j].c) continue;
+      if (xdrop_sink) {
+        if (base < p.match_cap) {
           pl_match mt;
-          mt.p = e.x; mt.q = e.y & 0xffffu; mt.db_start = o.a; mt.q_start = o.q_start; mt.len = o.len; mt.score = o.score;
-          p.matches[mi] = mt;
+          mt.p = e[j].x; mt.q = e[j].y & 0xffffu; mt.db_start = o[j].a; mt.q_start = o[j].q_start;
+          mt.len = o[j].len; mt.score = o[j].score;
+          p.matches[base] = mt;
         }
-      } else if (!sink) {
-        for (uint32_t j = 0; j < o.c; ++j)
-          if (base + off + j < cap) out[base + off + j] = stage_output(nd, c.dna, e, o, j);
+        ++base;
+      } else if (!nd.sink) {
+        for (uint32_t k = 0; k < o[j].c; ++k, ++base)
+          if (base < cap) out[base] = stage_output_k<KIND>(nd, dna, e[j], o[j], k);
       }
     }
-    __syncthreads();
-    if (tid == 0) atomicMax(cnt + 1, (unsigned long long)(clock64() - c0));
+    maxc = max(maxc, (uint32_t)(clock64() - c0));
   }
+  maxc = __reduce_max_sync(0xffffffffu, maxc);
+  if (lane == 0 && maxc) atomicMax(cnt + 1, (unsigned long long)maxc);
+}
+
+template <int KIND>
+static cudaError_t kbench_launch(const DevParams& p, int stage, const void* in, uint64_t n, uint64_t first_root,
+                                 void* out, uint64_t cap, unsigned long long* cnt, cudaStream_t st) {
+  const uint32_t smem = layout_kbench(p).total;
+  cudaError_t e = cudaFuncSetAttribute(pl_kbench_kernel<KIND>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                       (int)smem);
+  if (e) return e;
+  int per_sm = 0, sms = 0, dev = 0;
+  if ((e = cudaGetDevice(&dev))) return e;
+  if ((e = cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev))) return e;
+  if ((e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, pl_kbench_kernel<KIND>, KB_THREADS, smem))) return e;
+  const uint64_t chunks = (n + 32u * KB_J - 1) / (32u * KB_J);
+  const uint64_t need = (chunks + KB_THREADS / 32 - 1) / (KB_THREADS / 32);
+  const uint64_t full = (uint64_t)sms * (uint64_t)(per_sm > 0 ? per_sm : 1);
+  const unsigned grid = (unsigned)(need < full ? (need ? need : 1) : full);
+  pl_kbench_kernel<KIND><<<grid, KB_THREADS, smem, st>>>(p, stage, (const uint2*)in, n, first_root, (uint2*)out,
+                                                         cap, cnt);
+  return cudaGetLastError();
 }
 
 cudaError_t pl_launch_stage_batch(const DevParams& p, int stage, const void* in, uint64_t n, uint64_t first_root,
-                                  void* out, uint64_t cap, unsigned long long* cnt, unsigned smem, cudaStream_t st) {
-  const unsigned v = (unsigned)p.v;
-  uint64_t vecs = (n + v - 1) / v;
-  unsigned grid = (unsigned)(vecs < 148u * 8u ? (vecs ? vecs : 1) : 148u * 8u);
-  cudaError_t e = cudaFuncSetAttribute(pl_stage_batch_kernel<256>, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024);
-  if (e) return e;
-  pl_stage_batch_kernel<256><<<grid, v, smem, st>>>(p, stage, (const uint2*)in, n, first_root, (uint2*)out, cap, cnt);
-  return cudaGetLastError();
+                                  void* out, uint64_t cap, unsigned long long* cnt, unsigned /*smem*/, cudaStream_t st) {
+  switch (p.st[stage].kind) {
+    case PL_SEED_LOOKUP: return kbench_launch<PL_SEED_LOOKUP>(p, stage, in, n, first_root, out, cap, cnt, st);
+    case PL_HIT_ENUM: return kbench_launch<PL_HIT_ENUM>(p, stage, in, n, first_root, out, cap, cnt, st);
+    case PL_UNGAPPED_WINDOW:
+    case PL_UNGAPPED_XDROP: return kbench_launch<PL_UNGAPPED_WINDOW>(p, stage, in, n, first_root, out, cap, cnt, st);
+    case PL_BERNOULLI: return kbench_launch<PL_BERNOULLI>(p, stage, in, n, first_root, out, cap, cnt, st);
+    case PL_FIXED_GAIN: return kbench_launch<PL_FIXED_GAIN>(p, stage, in, n, first_root, out, cap, cnt, st);
+    case PL_KEEP_EVERY: return kbench_launch<PL_KEEP_EVERY>(p, stage, in, n, first_root, out, cap, cnt, st);
+    default: return kbench_launch<PL_POISSON_CAPPED>(p, stage, in, n, first_root, out, cap, cnt, st);
+  }
 }

@@ -10,12 +10,15 @@ from parity import workload_for
 pytestmark = pytest.mark.gpu
 
 
-@pytest.mark.parametrize("db_len", [1 << 16, 40_003])
-def test_stage_chain_matches_oracle(db_len):
+@pytest.mark.parametrize("db_len,heavy", [(1 << 16, False), (40_003, False), (1 << 18, True), (1 << 20, True)])
+def test_stage_chain_matches_oracle(db_len, heavy):
     import torch
     from paper_conf_icppw_planob21_b200 import Pipeline
     from oracle import stages as S
-    cfg = C.c2(n_streams=1, dna=dict(db_len=db_len, q_len=1024, n_planted=12), wait_time=(0, 0, 0, 0))
+    dna = dict(db_len=db_len, q_len=1024, n_planted=12)
+    if heavy:   # c4's recipe (repeat islands, tandem-repeat query motifs) at a size the oracle runs
+        dna.update(heavy_tailed=True)
+    cfg = C.c2(n_streams=1, dna=dna, wait_time=(0, 0, 0, 0))
     wl = workload_for(cfg)
     pl = Pipeline(cfg, wl, flags=0)
     pl.push(wl.db, wl.db_len)

@@ -23,7 +23,9 @@ R = db_len - 5
 cap = int(R * 0.5) * 2 + (1 << 20)
 a = torch.empty((cap, 2), dtype=torch.int32, device="cuda")
 b = torch.empty((cap, 2), dtype=torch.int32, device="cuda")
-pk = 6459.3
+import os
+with open(os.path.join(os.path.dirname(os.path.dirname(os.path.abspath(__file__))), "MEASURED_PEAKS.json")) as _f:
+    pk = json.load(_f)["hbm_gbs"]
 out = []
 srcs = [(0, R), None, None, None]
 n_in = R
