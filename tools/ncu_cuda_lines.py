@@ -1,6 +1,6 @@
 """Per-CUDA-source-line stall samples and warp instructions from an ncu report captured with
 --import-source on (ncu's own cuda,sass correlation; no nvdisasm needed).
-usage: python tools/ncu_cuda_lines.py <report.ncu-rep> [top]"""
+usage: python tools/ncu_cuda_lines.py <report.ncu-rep> [top] [inst]   (inst: sort by warp instructions)"""
 import csv
 import io
 import subprocess
@@ -32,6 +32,7 @@ for r in rows:
                     a[2][hdr[i][6:]] = a[2].get(hdr[i][6:], 0) + v
 tot = sum(a[0] for a in agg.values())
 print(f"samples {tot}, warp-inst {sum(a[1] for a in agg.values())}")
-for ln, a in sorted(agg.items(), key=lambda kv: -kv[1][0])[:top]:
+key = 1 if len(sys.argv) > 3 and sys.argv[3] == "inst" else 0
+for ln, a in sorted(agg.items(), key=lambda kv: -kv[1][key])[:top]:
     st = " ".join(f"{k}={v}" for k, v in sorted(a[2].items(), key=lambda kv: -kv[1])[:3])
     print(f"{ln:5d} samp {a[0]:6d} ({100 * a[0] / max(1, tot):4.1f}%) inst {a[1]:10d}  {st:45s} | {src.get(ln, '')}")

@@ -60,3 +60,26 @@ pl.inject_stalls(200_000, 50_000)
 pl.drain()
 print("injected stalls", pl.stats()["max_lateness_ns"], flush=True)
 pl.close()
+# K-BENCH stage kernels (pl_kbench_kernel<KIND>): every stage of a heavy-tailed DNA workload
+# whose extension walks reach both DB ends, and a random-gain chain
+import torch  # noqa: E402
+cfg = C.c2(n_streams=1, dna=dict(db_len=40_003, q_len=1024, n_planted=12, heavy_tailed=True), wait_time=(0,) * 4)
+wl = G.make_dna(cfg.seed, **cfg.dna)
+pl = Pipeline(cfg, wl, flags=0)
+pl.push(wl.db, wl.db_len)
+R = wl.db_len - 6 + 1   # k = 6
+bufs = [torch.empty((R * 16, 2), dtype=torch.int32, device="cuda") for _ in range(2)]
+n_in, src = R, 0
+for st in range(4):
+    out = bufs[st % 2].data_ptr() if st < 3 else 0
+    n_out, _ = pl.stage_batch(st, src, n_in, 0, out, R * 16 if st < 3 else 0)
+    print("kbench stage", st, n_in, "->", n_out, flush=True)
+    n_in, src = n_out, out
+pl.close()
+cfg = C.c1(n_streams=1, n_roots=5000, wait_time=(64, 90))
+pl = Pipeline(cfg, None, flags=0)
+pl.push(None, cfg.n_roots)
+buf = torch.empty((5000 * 4, 2), dtype=torch.int32, device="cuda")
+n0, _ = pl.stage_batch(0, 0, 5000, 0, buf.data_ptr(), 5000 * 4)
+print("kbench gain model stage 0", n0, flush=True)
+pl.close()
