@@ -76,6 +76,7 @@ def parse():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-side", action="store_true", help="skip the FIXED_WAIT / MONOLITHIC side measurements")
+    ap.add_argument("--no-stages", action="store_true", help="skip the per-stage K-BENCH kernels (stage_rooflines)")
     ap.add_argument("--budget-margin", type=float, default=1.10,
                     help="t_i = margin x longest measured firing + slack (SURVEY 8(d): x1.1)")
     ap.add_argument("--budget-slack", type=int, default=128)
@@ -169,6 +170,54 @@ def ncu_summary(workload):
             return json.load(f)
     except (OSError, ValueError):
         return {}
+
+
+def stage_rooflines(base, wl, db_ptr, stream, pk, workload, reps=3):
+    """K-BENCH (north_star: "the achieved HBM GB/s of each stage kernel"): every DNA stage over
+    this rank's whole DB through pl_stage_batch (S0 over every root, then each stage over the
+    previous one's outputs), CUDA events on the launching stream, `reps` launches per stage after
+    one warm-up.  Algorithmic bytes: S0 0.25 B per root in + 8 B per output; S1, S2 8 B per input
+    + 8 B per output; S3 8 B per input + 24 B per match.  `dram_bytes` is ncu's traffic of the same
+    launch from the committed capture (profiles/ncu_kbench_<workload>.json), null if absent."""
+    import torch
+    from paper_conf_icppw_planob21_b200 import Pipeline
+    try:
+        with open(os.path.join(ROOT, "profiles", f"ncu_kbench_{workload}.json")) as f:
+            ncu = json.load(f)
+    except (OSError, ValueError):
+        ncu = {}
+    k = base.stages[0].iparam[0]
+    R = wl.db_len - k + 1
+    pl = Pipeline(base.replace(wait_time=(0,) * base.n_stages), wl, flags=0, stream=stream)
+    pl.bind_device(db_ptr, wl.db_len)
+    cap = R + (R >> 1) + (1 << 20)
+    bufs = [torch.empty((cap, 2), dtype=torch.int32, device="cuda") for _ in range(2)]
+    names = ["S0 seed lookup", "S1 hit enumeration", "S2 window filter", "S3 X-drop"]
+    out, n_in, src = [], R, 0
+    for st in range(base.n_stages):
+        dst = bufs[st % 2].data_ptr() if st + 1 < base.n_stages else 0
+        ocap = cap if st + 1 < base.n_stages else 0
+        pl.stage_batch(st, src, n_in, 0, dst, ocap)              # warm-up
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(stream)
+        for _ in range(reps):
+            n_out, _ = pl.stage_batch(st, src, n_in, 0, dst, ocap)
+        e1.record(stream)
+        torch.cuda.synchronize()
+        sec = e0.elapsed_time(e1) * 1e-3 / reps
+        alg = (0.25 if st == 0 else 8.0) * n_in + (24.0 if st + 1 == base.n_stages else 8.0) * n_out
+        rec = {"stage": names[st] if st < 4 else str(st), "inputs": n_in, "outputs": n_out,
+               "us": round(sec * 1e6, 1), "items_per_s": n_in / sec, "algorithmic_GBps": alg / sec / 1e9,
+               "frac_hbm_algorithmic": alg / sec / 1e9 / pk}
+        d = ncu.get(str(st))
+        if d:
+            rec.update(dram_bytes=d["dram_bytes"], dram_GBps_ncu=d["dram_GBps"], frac_hbm_dram_ncu=d["dram_GBps"] / pk,
+                       issue_active_pct=d["issue_active_pct"])
+        out.append(rec)
+        n_in, src = n_out, dst
+    pl.close()
+    return {"kernel": "pl_kbench_kernel<KIND> (pl_stage_batch)", "peak_GBps": pk, "reps": reps, "stages": out,
+            "ncu_source": ncu.get("source")}
 
 
 # --------------------------------------------------------------- oracle legs
@@ -599,6 +648,10 @@ def main():
                            "peak": world * a.streams * 1e9 * v / ((u * budgets[3]) if c4 else budgets[0]),
                            "unit": "items/s"},
             "cpu_baseline": cpu,
+            # per-stage kernels over the same DB, outside the timed region (north_star: HBM GB/s of each
+            # stage kernel against the peak)
+            "stages": (None if a.no_stages else
+                       stage_rooflines(base, wl, db_ptr, stream, pk, a.workload)),
         }
         rb = line["rate_bound"]
         rb["frac"] = rb["achieved"] / rb["peak"]

@@ -42,3 +42,42 @@ def test_stage_chain_matches_oracle(db_len, heavy):
     assert sorted((int(a), int(b) & 0xffff, int(b) >> 16) for a, b in s1) == sorted((p, q, j) for p, j, q in o1)
     assert sorted((int(a), int(b) & 0xffff) for a, b in s2) == sorted((p, q) for p, j, q in o2)
     assert n3 == len(o3) and matches == o3
+
+
+def _gain_chain(cfg, n_roots):
+    """Every stage of a random-gain pipeline through pl_stage_batch (root lineage carried in
+    entry.y), vs the oracle's per-item stage functions (oracle.des.make_stage_fns) on the same
+    seeded hashes; outputs compared as multisets of (root, lineage)."""
+    import torch
+    from paper_conf_icppw_planob21_b200 import Pipeline
+    from oracle import des
+    pl = Pipeline(cfg, None, flags=0)
+    pl.push(None, n_roots)
+    cap = n_roots * 32
+    bufs = [torch.empty((cap, 2), dtype=torch.int32, device="cuda") for _ in range(2)]
+    fns = des.make_stage_fns(cfg, None)
+    ref = [(r, 0, None) for r in range(n_roots)]
+    n_in, src = n_roots, 0
+    for st in range(cfg.n_stages):
+        last = st + 1 == cfg.n_stages
+        dst = 0 if last else bufs[st % 2].data_ptr()
+        n_out, _ = pl.stage_batch(st, src, n_in, 0, dst, 0 if last else cap)
+        ref = [o for e in ref for o in fns[st](e)]
+        assert n_out == len(ref), f"stage {st}: {n_out} outputs, oracle {len(ref)}"
+        if not last:
+            got = bufs[st % 2][:n_out].cpu().numpy().astype(np.uint32)
+            assert sorted((int(a), int(b)) for a, b in got) == sorted((r, l) for r, l, _ in ref), f"stage {st}"
+        n_in, src = n_out, dst
+    pl.close()
+
+
+@pytest.mark.parametrize("n_roots", [1, 127, 4099, 50_000])
+def test_stage_chain_gain_model_blast(n_roots):
+    """Table 1's random-gain model: Bernoulli -> min(Poisson(1.92), 16) -> Bernoulli -> Bernoulli(1)."""
+    _gain_chain(C.gain_model_blast(n_roots=n_roots), n_roots)
+
+
+def test_stage_chain_c1_and_keep_every():
+    """c1 (Bernoulli 0.5 -> fixed gain 2) and c1r (keep every 2nd -> fixed gain 2), ragged tails."""
+    _gain_chain(C.c1(n_roots=10_007), 10_007)
+    _gain_chain(C.c1r(n_roots=333), 333)
