@@ -57,7 +57,7 @@ WORKLOADS = {
 }
 # c4 schedule parameters of the last GPU bench (profiles/r02_bench_c4_v1.json), for the reference arm,
 # which must not load the product library: the oracle simulates the same schedule (1 unit = 1 ns)
-REF_C4 = dict(budgets=(8682, 11921, 6500, 19031), tau0=3193, gains=(0.04995, 8.9465, 0.56093))   # profiles/r02_bench_c4_h108_1.json
+REF_C4 = dict(budgets=(8189, 11146, 6324, 17904), tau0=3141, gains=(0.04995, 8.9465, 0.56093))   # profiles/r02_bench_c4_final.json
 
 
 def parse():

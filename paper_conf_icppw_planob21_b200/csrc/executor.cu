@@ -91,6 +91,10 @@ __device__ __forceinline__ uint64_t gain_hash(uint64_t seed, uint32_t stage, uin
 #ifndef PL_NAP_SHIFT
 #define PL_NAP_SHIFT 1      // long naps sleep half the remaining time (__nanosleep: at most 2x): -9 % instructions on c4
 #endif
+#ifndef PL_NAP_HALF
+#define PL_NAP_HALF 1       // every nap above the spin threshold sleeps half the remaining time (no 256 / 64 ns tiers):
+                            // c3 THRESHOLD_SLACK -9 to -11 % warp instructions per root, c4 budgets and rate unchanged or better
+#endif
 #ifndef PL_DBMASK
 #define PL_DBMASK 1
 #endif
@@ -1234,7 +1238,11 @@ __device__ __forceinline__ bool nap_until(uint64_t target) {
   if (now >= target) return false;
   while (now < target) {   // __nanosleep sleeps at most 2x its argument: nap rem >> PL_NAP_SHIFT
     const uint64_t rem = target - now;
+#if PL_NAP_HALF
+    __nanosleep(rem > 128 ? (uint32_t)min(rem >> 1, (uint64_t)(1u << 20)) : 64u);
+#else
     __nanosleep(rem > 4096 ? (uint32_t)min(rem >> PL_NAP_SHIFT, (uint64_t)(1u << 20)) : (rem > 1024 ? 256u : 64u));
+#endif
     now = gtimer();
   }
   return true;
@@ -1398,7 +1406,11 @@ __device__ __forceinline__ void pace(uint64_t target, uint64_t* start_ns, int64_
   if (entry_ns) *entry_ns = now;
   while (now < target) {   // __nanosleep sleeps at most 2x its argument: nap rem >> PL_NAP_SHIFT
     const uint64_t rem = target - now;
+#if PL_NAP_HALF
+    __nanosleep(rem > 256 ? (uint32_t)min(rem >> 1, (uint64_t)(1u << 20)) : 0u);
+#else
     __nanosleep(rem > 4096 ? (uint32_t)min(rem >> PL_NAP_SHIFT, (uint64_t)(1u << 20)) : (rem > 1024 ? 256u : (rem > 256 ? 64u : 0u)));
+#endif
     now = gtimer();
   }
   *start_ns = now;
