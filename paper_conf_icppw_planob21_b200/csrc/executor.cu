@@ -95,6 +95,9 @@ __device__ __forceinline__ uint64_t gain_hash(uint64_t seed, uint32_t stage, uin
 #define PL_NAP_HALF 1       // every nap above the spin threshold sleeps half the remaining time (no 256 / 64 ns tiers):
                             // c3 THRESHOLD_SLACK -9 to -11 % warp instructions per root, c4 budgets and rate unchanged or better
 #endif
+#ifndef PL_PHYS_SPINS
+#define PL_PHYS_SPINS 2     // physical-clock polls before the first backoff nap
+#endif
 #ifndef PL_DBMASK
 #define PL_DBMASK 1
 #endif
@@ -1100,9 +1103,9 @@ __device__ __forceinline__ void publish_W(const Node& nd, Leader& L, int64_t w) 
 // The watchdog (above) is checked deep inside a wait only, every 4096 naps, off every firing's
 // path; a waiter whose watchdog expired finds spins < 0.
 __device__ __forceinline__ void backoff(int& spins, uint64_t& wd0, bool phys = false, uint32_t cap_ns = 256) {
-  if (spins < (phys ? 2 : 4)) { ++spins; return; }
+  if (spins < (phys ? PL_PHYS_SPINS : 4)) { ++spins; return; }
   if (phys) {
-    const int e = spins - 2 < 16 ? spins - 2 : 16;
+    const int e = spins - PL_PHYS_SPINS < 16 ? spins - PL_PHYS_SPINS : 16;
     const uint32_t ns = 64u << e;
     __nanosleep(ns < cap_ns ? ns : cap_ns);
   } else {
@@ -1251,7 +1254,11 @@ __device__ __forceinline__ bool nap_until(uint64_t target) {
 // A FIXED_WAIT node cannot start firing m before T = m P_i, so on the physical clock it sleeps
 // until this far ahead of T before it polls its upstream (a waiting node then costs issue slots
 // only for the poll that decides the firing; yielded time is usable).
-constexpr uint64_t PL_NAP_LEAD_NS = 768;
+#ifndef PL_NAP_LEAD
+#define PL_NAP_LEAD 768     // 256: c3 THRESHOLD_SLACK -4 % instructions per root, but firings start late: busy/model
+                            // 0.961 on the c4 bench, 0.930 on a FIXED_WAIT c2 replay (test_physical_replays_logical_schedule): rejected
+#endif
+constexpr uint64_t PL_NAP_LEAD_NS = PL_NAP_LEAD;
 
 // THRESHOLD_SLACK on the physical clock: a node whose next firing cannot start before logical
 // time lb = max(B, min(Tk, W_up)) -- nothing it has queued can fire earlier, and anything its
