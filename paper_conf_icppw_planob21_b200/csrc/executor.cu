@@ -95,6 +95,10 @@ __device__ __forceinline__ uint64_t gain_hash(uint64_t seed, uint32_t stage, uin
 #define PL_NAP_HALF 1       // every nap above the spin threshold sleeps half the remaining time (no 256 / 64 ns tiers):
                             // c3 THRESHOLD_SLACK -9 to -11 % warp instructions per root, c4 budgets and rate unchanged or better
 #endif
+#ifndef PL_PUB_WAIT
+#define PL_PUB_WAIT 0       // physical clock: a waiting leader sleeps on its input edge's mbarrier (woken by the
+                            // producer's publication or the nap's time limit) instead of a plain nap
+#endif
 #ifndef PL_PHYS_SPINS
 #define PL_PHYS_SPINS 2     // physical-clock polls before the first backoff nap
 #endif
@@ -589,6 +593,7 @@ struct EdgeCtl {            // queue INTO node i
   int64_t  W;               // producer watermark
   uint32_t spill_end;       // producer: end seq of the last spilled segment
   uint32_t stalled;         // producer: waiting for room in this queue (reserve_out)
+  alignas(8) uint64_t pub_bar;   // PL_PUB_WAIT: mbarrier (count 1) the producer arrives on at every publication
 };
 struct GroupCtl {           // broadcast from a node's leader to its lanes, double-buffered
   int64_t  T[2];            // by firing parity so that no barrier is needed between firings
@@ -1084,12 +1089,37 @@ __device__ __noinline__ bool watchdog_expired(uint64_t& t0) {
   return now - t0 > PL_WATCHDOG_NS;
 }
 
+// PL_PUB_WAIT: the producer's leader arrives on its output edge's mbarrier after every
+// publication (a new watermark or segment); a waiting consumer leader sleeps in
+// mbarrier.try_wait with the nap's length as the time limit, so it resumes at the publication
+// instead of at the end of a nap.  A wake-up hint only: the consumer re-reads the edge with the
+// usual fences either way.  Not under N4 (the edge lives in another CTA's smem).
+__device__ __forceinline__ void pub_signal(const Node& nd) {
+#if PL_PUB_WAIT
+  if (nd.phys && !nd.cl)
+    asm volatile("mbarrier.arrive.release.cta.shared::cta.b64 _, [%0];" ::"r"(smem_addr(&nd.Eout->pub_bar)) : "memory");
+#endif
+}
+// The input edge's current (incomplete) phase parity, read BEFORE the edge is polled: a
+// publication after the poll then completes that phase and the sleep below returns at once
+// (no lost wake-up).  Phase parity 0 is complete iff the current phase is odd.
+__device__ __forceinline__ uint32_t pub_phase(const Node& nd) {
+  uint32_t cur = 0;
+#if PL_PUB_WAIT
+  if (nd.phys && !nd.cl)
+    asm volatile("{ .reg .pred q; mbarrier.test_wait.parity.shared::cta.b64 q, [%1], 0; selp.u32 %0, 1, 0, q; }"
+                 : "=r"(cur) : "r"(smem_addr(&nd.Ein->pub_bar)) : "memory");
+#endif
+  return cur;
+}
+
 __device__ __forceinline__ void publish_W(const Node& nd, Leader& L, int64_t w) {
   if (nd.sink) return;
   if (w > L.W_pub) {
     L.W_pub = w;
     fence_q(nd.cl);
     vst(&nd.Eout->W, w);
+    pub_signal(nd);
   }
 }
 
@@ -1113,6 +1143,27 @@ __device__ __forceinline__ void backoff(int& spins, uint64_t& wd0, bool phys = f
   }
   ++spins;
   if (PL_WATCHDOG && (spins & 4095) == 0 && watchdog_expired(wd0)) spins = -(1 << 30);
+}
+
+// A waiting leader in decide(): every condition it waits for (upstream watermark past T, enough
+// entries) changes only at an upstream publication, so under PL_PUB_WAIT it sleeps on the edge's
+// mbarrier until the phase `ph` (read before its poll) completes, with t_i as a safety limit;
+// otherwise the backoff naps above.
+__device__ __forceinline__ void wait_up(const Node& nd, uint32_t ph, int& spins, uint64_t& wd0) {
+#if PL_PUB_WAIT
+  if (nd.phys && !nd.cl) {
+    const uint32_t ns = min(nd.nap_cap_ns << 3, 1u << 20);
+    uint32_t done;
+    asm volatile("{ .reg .pred q; mbarrier.try_wait.parity.shared::cta.b64 q, [%1], %2, %3; selp.u32 %0, 1, 0, q; }"
+                 : "=r"(done) : "r"(smem_addr(&nd.Ein->pub_bar)), "r"(ph), "r"(ns) : "memory");
+    (void)done;
+    ++spins;
+    if (PL_WATCHDOG && (spins & 4095) == 0 && watchdog_expired(wd0)) spins = -(1 << 30);
+    return;
+  }
+#endif
+  (void)ph;
+  backoff(spins, wd0, nd.phys, nd.nap_cap_ns);
 }
 
 // number of entries of the input edge with ready <= T among the published ones (stops at v)
@@ -1299,6 +1350,7 @@ __device__ __forceinline__ Decision decide(const Node& nd, Leader& L, bool& wait
       }
     }
     // node i >= 1: read the upstream watermark (and window bound) first, then the published segments
+    const uint32_t ph = pub_phase(nd);
     const int64_t Wup = vld(&nd.Ein->W);
     const uint32_t bup = nd.sliding ? vld(nd.bnd_up) : 0u;
     fence_q(nd.cl);
@@ -1313,7 +1365,7 @@ __device__ __forceinline__ Decision decide(const Node& nd, Leader& L, bool& wait
         if (!any) {
           if (Wup == PL_INF64) { d.done = true; return d; }
           publish_W(nd, L, max(B, Wup) + nd.t);
-          backoff(spins, wd0, nd.phys, nd.nap_cap_ns); waited = true;
+          wait_up(nd, ph, spins, wd0); waited = true;
           continue;
         }
         const int64_t Te = max(B, nd.in_seg[L.segh & nd.segmask].ready);
@@ -1322,7 +1374,7 @@ __device__ __forceinline__ Decision decide(const Node& nd, Leader& L, bool& wait
         if (Wup > Te || (cnt >= v && early_ok(nd))) {
           d.T = Te; d.n = cnt < v ? cnt : v; d.qlen = count_all_le(nd, L, st, Te); return d;
         }
-        backoff(spins, wd0, nd.phys, nd.nap_cap_ns); waited = true;
+        wait_up(nd, ph, spins, wd0); waited = true;
         continue;
       }
       const int64_t T = L.m * nd.P;
@@ -1341,7 +1393,7 @@ __device__ __forceinline__ Decision decide(const Node& nd, Leader& L, bool& wait
         continue;
       }
       publish_W(nd, L, T + nd.t);
-      backoff(spins, wd0, nd.phys, nd.nap_cap_ns); waited = true;
+      wait_up(nd, ph, spins, wd0); waited = true;
       continue;
     }
     // THRESHOLD_SLACK
@@ -1350,7 +1402,7 @@ __device__ __forceinline__ Decision decide(const Node& nd, Leader& L, bool& wait
       const int64_t lb = Wup > L.B ? Wup : L.B;
       publish_W(nd, L, lb + nd.t);
       if (nap_to(nd, T0, lb, napped)) { waited = true; spins = 0; continue; }
-      backoff(spins, wd0, nd.phys, nd.nap_cap_ns); waited = true;
+      wait_up(nd, ph, spins, wd0); waited = true;
       continue;
     }
     const Seg& hs = nd.in_seg[L.segh & nd.segmask];
@@ -1384,7 +1436,7 @@ __device__ __forceinline__ Decision decide(const Node& nd, Leader& L, bool& wait
     if (lb < L.B) lb = L.B;
     publish_W(nd, L, lb + nd.t);
     if (nap_to(nd, T0, lb, napped)) { waited = true; spins = 0; continue; }
-    backoff(spins, wd0, nd.phys, nd.nap_cap_ns); waited = true;
+    wait_up(nd, ph, spins, wd0); waited = true;
   }
 }
 
@@ -1933,6 +1985,7 @@ __device__ void run_node(Ctx& c, Dna dna, int i, int gtid) {
         L.out_tail += total;
         vst(&nd.Eout->seg_tail, L.out_segt);
         vst(&nd.Eout->tail, L.out_tail);
+        pub_signal(nd);
       }
       if (nd.fixed) {
         ++L.m;
@@ -2257,6 +2310,9 @@ __device__ void cta_setup(Ctx& c, Shared& sh, unsigned char* dsm, const DevParam
   if (tid < PL_MAX_STAGES) {
     EdgeCtl& E = sh.e[tid];
     E.head = 0; E.seg_head = 0; E.seg_tail = 0; E.tail = 0; E.W = -1; E.spill_end = 0; E.stalled = 0;
+#if PL_PUB_WAIT
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(smem_addr(&E.pub_bar)) : "memory");
+#endif
   }
   if (tid == 0) {
     sh.max_lat = 0; sh.max_lat_ns = 0; sh.miss_events = 0; sh.miss_events_ns = 0; sh.errors = 0; sh.log_count = 0;
