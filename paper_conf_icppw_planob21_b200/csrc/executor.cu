@@ -97,7 +97,9 @@ __device__ __forceinline__ uint64_t gain_hash(uint64_t seed, uint32_t stage, uin
 #endif
 #ifndef PL_PUB_WAIT
 #define PL_PUB_WAIT 0       // physical clock: a waiting leader sleeps on its input edge's mbarrier (woken by the
-                            // producer's publication or the nap's time limit) instead of a plain nap
+                            // producer's publication or the nap's time limit) instead of a plain nap; parity-exact
+                            // (110 physical/live/window tests) but no fewer instructions at the c3 points
+                            // (37.2 vs 37.0 per root) and the c4 edge no faster: rejected (profiles/r02_ab/pub_wait.txt)
 #endif
 #ifndef PL_PHYS_SPINS
 #define PL_PHYS_SPINS 2     // physical-clock polls before the first backoff nap
