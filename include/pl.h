@@ -393,11 +393,13 @@ pl_status pl_solve_monolithic(const pl_config* cfg, uint32_t* M_out, double* T_o
  * Consumes n device-resident entries {root, aux} (uint2: aux = q | j<<16 for DNA hits,
  * lineage for random gains); for stage 0 `in_dev` is ignored and the roots are
  * first_root .. first_root+n-1.  Outputs of non-sink stages are appended to out_dev
- * (device, capacity cap entries): in input order within each chunk of 128 consecutive
- * inputs (one warp's), chunks in any order.  The last DNA stage writes pl_match records to
+ * (device, capacity cap entries): in input order within each warp's chunk of consecutive
+ * inputs, chunks in any order.  The last DNA stage writes pl_match records to
  * the pipeline's match buffer (read with pl_pipeline_results).  *n_out = outputs produced;
  * *max_vec_cycles (may be NULL) = longest per-chunk clock64 duration.  The kernel runs at
- * full occupancy (256-thread CTAs, the query index in smem, the executor's stage bodies).
+ * full occupancy (256-thread CTAs, the query index in smem): S0 rolls k-mers over 16-byte DB
+ * loads (first_root a multiple of 64, 4 <= k <= 8; else per item), S1 writes its outputs
+ * through smem as contiguous runs, the other stages run the executor's stage bodies.
  * Needs a pushed or bound DB for DNA.  PL_EOVERFLOW: more outputs than cap (the first cap
  * are written).                                                                        */
 pl_status pl_stage_batch(pl_pipeline* pl, uint32_t stage, const void* in_dev, uint64_t n, uint64_t first_root,

@@ -2691,7 +2691,7 @@ cudaError_t pl_kernel_attributes(unsigned max_smem) {
 // memory (the whole DB, read-only), so S2 / S3 take the executor's fast in-window walks; only
 // seeds within a walk's reach of the DB ends take the checked ones.  Shared memory holds only
 // the query index, so several CTAs share an SM.
-struct KbLayout { uint32_t qpos, qw, s2, total; };
+struct KbLayout { uint32_t qpos, qw, s2, hit, total; };
 __host__ __device__ inline KbLayout layout_kbench(const DevParams& p) {
   KbLayout L;
   uint32_t off = 0;
@@ -2703,11 +2703,94 @@ __host__ __device__ inline KbLayout layout_kbench(const DevParams& p) {
   off += dna ? 32u + ((((uint32_t)(p.q_len + 15) / 16u) * 4u + 15u) & ~15u) : 0u;
   L.s2 = off;
   off += dna ? 256u : 0u;
+  L.hit = off;                                                       // S0: one bit per k-mer (has hits)
+  off += dna ? ((((1u << (2 * p.k)) + 31u) / 32u) * 4u + 15u) & ~15u : 0u;
   L.total = off > 16u ? off : 16u;
   return L;
 }
 constexpr int KB_THREADS = 256;
 constexpr int KB_J = 4;
+constexpr int KB_KMAX = 8;
+constexpr uint32_t KB_S1_U = 16;   // S1 staging: outputs per input a warp slice holds
+
+// S0 over consecutive roots (K-BENCH fast path; north_star "coalesced 128-bit loads"): a lane
+// takes 64 consecutive roots, i.e. 4 DB words loaded as one 16-byte vector plus the next lane's
+// first word (a shuffle), rolls the k-mer key base by base (key = (key << 2 | base) mod 4^k,
+// the first base most significant as in R-S0) and tests it in a smem bitmap of the k-mers that
+// occur in the query (bit set iff qoff[key + 1] > qoff[key]).  Hits become a 64-bit lane mask,
+// a shuffle scan and one atomic per warp place them, in root order within the warp's 2048 roots.
+// k is a template parameter (4..8; the root index of each base is then a constant) and only a
+// lane holding the batch's end checks the root bound.  Requires first_root % 64 == 0 and a
+// 16-byte-aligned DB (else the per-item path).
+template <int K, bool TAIL>
+__device__ __forceinline__ uint64_t s0_roll64(const uint32_t (&wd)[5], const uint32_t* hitbm, uint64_t lim) {
+  constexpr uint32_t kmask = (1u << (2 * K)) - 1u;
+  uint32_t lo = 0, hi = 0, key = 0;
+#pragma unroll
+  for (int b = 0; b < 64 + K - 1; ++b) {
+    key = ((key << 2) | ((wd[b >> 4] >> ((b & 15) * 2)) & 3u)) & kmask;
+    const int j = b - K + 1;                                           // the root whose k-mer ends at base b
+    if (j >= 0) {
+      const uint32_t bit = (hitbm[key >> 5] >> (key & 31u)) & 1u;
+      const uint32_t ok = TAIL ? (bit & ((uint64_t)j < lim ? 1u : 0u)) : bit;
+      if (j < 32) lo |= ok << j; else hi |= ok << (j - 32);
+    }
+  }
+  return ((uint64_t)hi << 32) | lo;
+}
+template <int K>
+__device__ __forceinline__ uint64_t s0_roll(const uint32_t (&wd)[5], const uint32_t* hitbm, uint64_t lim) {
+  return lim >= 64 ? s0_roll64<K, false>(wd, hitbm, lim) : s0_roll64<K, true>(wd, hitbm, lim);
+}
+
+__device__ __forceinline__ void kbench_s0_rolling(const DevParams& p, const uint32_t* hitbm, uint64_t n,
+                                                  uint64_t first_root, uint2* out, uint64_t cap,
+                                                  unsigned long long* cnt) {
+  const int lane = (int)(threadIdx.x & 31u);
+  const uint64_t nw = ((uint64_t)gridDim.x * blockDim.x) >> 5;
+  uint32_t maxc = 0;
+  for (uint64_t ch = ((uint64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5; ch * 2048u < n; ch += nw) {
+    const long long c0 = clock64();
+    const uint64_t j0 = ch * 2048u + (uint64_t)lane * 64u;            // local index of the lane's first root
+    const uint64_t r0 = first_root + j0;
+    const uint64_t w0 = r0 >> 4;
+    uint4 W = make_uint4(0u, 0u, 0u, 0u);
+    if (w0 + 3 < p.db_words) W = __ldg(reinterpret_cast<const uint4*>(p.db + w0));
+    else {
+      if (w0 < p.db_words) W.x = __ldg(p.db + w0);
+      if (w0 + 1 < p.db_words) W.y = __ldg(p.db + w0 + 1);
+      if (w0 + 2 < p.db_words) W.z = __ldg(p.db + w0 + 2);
+    }
+    uint32_t nx = __shfl_down_sync(0xffffffffu, W.x, 1);
+    if (lane == 31) nx = (w0 + 4 < p.db_words) ? __ldg(p.db + w0 + 4) : 0u;
+    const uint32_t wd[5] = {W.x, W.y, W.z, W.w, nx};
+    const uint64_t lim = n > j0 ? n - j0 : 0;                          // valid roots of this lane
+    uint64_t hits = 0;
+    switch (p.k) {
+      case 4: hits = s0_roll<4>(wd, hitbm, lim); break;
+      case 5: hits = s0_roll<5>(wd, hitbm, lim); break;
+      case 6: hits = s0_roll<6>(wd, hitbm, lim); break;
+      case 7: hits = s0_roll<7>(wd, hitbm, lim); break;
+      default: hits = s0_roll<8>(wd, hitbm, lim); break;
+    }
+    const uint32_t mine = (uint32_t)__popcll(hits);
+    uint32_t incl = mine;
+#pragma unroll
+    for (int d = 1; d < 32; d <<= 1) {
+      const uint32_t t = __shfl_up_sync(0xffffffffu, incl, d);
+      if (lane >= d) incl += t;
+    }
+    const uint32_t total = __shfl_sync(0xffffffffu, incl, 31);
+    unsigned long long base = 0;
+    if (lane == 0 && total) base = atomicAdd(cnt, (unsigned long long)total);
+    base = __shfl_sync(0xffffffffu, base, 0) + (incl - mine);
+    for (uint64_t m = hits; m; m &= m - 1, ++base)
+      if (base < cap) out[base] = make_uint2((uint32_t)(r0 + (uint64_t)(__ffsll((long long)m) - 1)), 0u);
+    maxc = max(maxc, (uint32_t)(clock64() - c0));
+  }
+  maxc = __reduce_max_sync(0xffffffffu, maxc);
+  if (lane == 0 && maxc) atomicMax(cnt + 1, (unsigned long long)maxc);
+}
 
 template <int KIND>
 __global__ void __launch_bounds__(KB_THREADS, 4) pl_kbench_kernel(const __grid_constant__ DevParams p, int stage,
@@ -2735,6 +2818,13 @@ __global__ void __launch_bounds__(KB_THREADS, 4) pl_kbench_kernel(const __grid_c
     for (uint32_t j = tid; j < nqp; j += nt) qp[j] = p.qpos[j];
     for (uint32_t j = tid; j < dna.nqw; j += nt) qw[j] = p.qwords[j];
     if (tid < 8) qw[tid < 4 ? (int)tid - 4 : (int)(dna.nqw + tid - 4u)] = 0u;   // pad words
+    uint32_t* hb = (uint32_t*)(dsm + Lo.hit);      // S0 bitmap: k-mers that occur in the query
+    for (uint32_t w = tid; w < (nko - 1u + 31u) / 32u; w += nt) {
+      uint32_t bits = 0;
+      for (uint32_t b = 0; b < 32u && w * 32u + b < nko - 1u; ++b)
+        bits |= (p.qoff[w * 32u + b + 1u] > p.qoff[w * 32u + b] ? 1u : 0u) << b;
+      hb[w] = bits;
+    }
     for (uint32_t m = tid; m < 256u; m += nt) {   // S2 table (as the executor's)
       int sc = 0, best = 0;
       for (int e = 0; e < 8; ++e) {
@@ -2745,6 +2835,12 @@ __global__ void __launch_bounds__(KB_THREADS, 4) pl_kbench_kernel(const __grid_c
     }
   }
   __syncthreads();
+  if constexpr (KIND == PL_SEED_LOOKUP) {
+    if (p.k >= 4 && p.k <= KB_KMAX && (first_root & 63u) == 0 && (reinterpret_cast<uintptr_t>(p.db) & 15u) == 0) {
+      kbench_s0_rolling(p, (const uint32_t*)(dsm + Lo.hit), n, first_root, out, cap, cnt);
+      return;
+    }
+  }
   Node nd;
   nd.i = stage; nd.N = p.N; nd.v = p.v;
   nd.sink = stage == p.N - 1;
@@ -2754,6 +2850,45 @@ __global__ void __launch_bounds__(KB_THREADS, 4) pl_kbench_kernel(const __grid_c
   nd.ip1 = sd.ip[1]; nd.ip2 = sd.ip[2];
   const bool xdrop_sink = nd.sink && nd.kind == PL_UNGAPPED_XDROP;
   const int lane = (int)(tid & 31u);
+  if constexpr (KIND == PL_HIT_ENUM) {
+    // S1 amplifies (up to u outputs per input): one input per lane, the warp's outputs staged in its
+    // own smem slice in output order, then written as contiguous 8-byte runs (scattered per-lane
+    // runs cost ~4 partial-sector L2 writes per output)
+    if (!nd.sink && nd.umax <= KB_S1_U) {
+      uint2* wbuf = reinterpret_cast<uint2*>(dsm + Lo.total) + (tid >> 5) * (32u * KB_S1_U);
+      const uint64_t nw1 = ((uint64_t)gridDim.x * nt) >> 5;
+      uint32_t maxc1 = 0;
+      for (uint64_t ch = ((uint64_t)blockIdx.x * nt + tid) >> 5; ch * 32u < n; ch += nw1) {
+        const long long c0 = clock64();
+        const uint64_t idx = ch * 32u + (uint64_t)lane;
+        uint2 ea[1];
+        bool aa[1] = {idx < n};
+        ea[0] = aa[0] ? __ldg(in + idx) : __ldg(in);
+        LaneOut oa[1];
+        stage_batch<1, PL_HIT_ENUM>(nd, dna, p, ea, aa, oa);
+        const uint32_t mine = oa[0].c;
+        uint32_t incl = mine;
+#pragma unroll
+        for (int d = 1; d < 32; d <<= 1) {
+          const uint32_t t = __shfl_up_sync(0xffffffffu, incl, d);
+          if (lane >= d) incl += t;
+        }
+        const uint32_t total = __shfl_sync(0xffffffffu, incl, 31);
+        unsigned long long base = 0;
+        if (lane == 0 && total) base = atomicAdd(cnt, (unsigned long long)total);
+        base = __shfl_sync(0xffffffffu, base, 0);
+        for (uint32_t k = 0; k < mine; ++k) wbuf[incl - mine + k] = stage_output_k<PL_HIT_ENUM>(nd, dna, ea[0], oa[0], k);
+        __syncwarp();
+        for (uint32_t t = (uint32_t)lane; t < total; t += 32u)
+          if (base + t < cap) out[base + t] = wbuf[t];
+        __syncwarp();
+        maxc1 = max(maxc1, (uint32_t)(clock64() - c0));
+      }
+      maxc1 = __reduce_max_sync(0xffffffffu, maxc1);
+      if (lane == 0 && maxc1) atomicMax(cnt + 1, (unsigned long long)maxc1);
+      return;
+    }
+  }
   constexpr uint32_t CH = 32u * KB_J;
   const uint64_t nw = ((uint64_t)gridDim.x * nt) >> 5;
   uint32_t maxc = 0;
@@ -2816,7 +2951,8 @@ __global__ void __launch_bounds__(KB_THREADS, 4) pl_kbench_kernel(const __grid_c
 template <int KIND>
 static cudaError_t kbench_launch(const DevParams& p, int stage, const void* in, uint64_t n, uint64_t first_root,
                                  void* out, uint64_t cap, unsigned long long* cnt, cudaStream_t st) {
-  const uint32_t smem = layout_kbench(p).total;
+  const uint32_t smem = layout_kbench(p).total +
+                        (KIND == PL_HIT_ENUM ? (uint32_t)(KB_THREADS / 32) * 32u * KB_S1_U * 8u : 0u);
   cudaError_t e = cudaFuncSetAttribute(pl_kbench_kernel<KIND>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                        (int)smem);
   if (e) return e;

@@ -81,3 +81,28 @@ def test_stage_chain_c1_and_keep_every():
     """c1 (Bernoulli 0.5 -> fixed gain 2) and c1r (keep every 2nd -> fixed gain 2), ragged tails."""
     _gain_chain(C.c1(n_roots=10_007), 10_007)
     _gain_chain(C.c1r(n_roots=333), 333)
+
+
+@pytest.mark.parametrize("first_root", [0, 64, 37, 1 << 12])
+def test_s0_first_root_paths(first_root):
+    """S0 through pl_stage_batch from an arbitrary first root: the rolling-k-mer path (first_root a
+    multiple of 64) and the per-item path (otherwise) both equal the oracle's S0 on every root, in
+    root order (the kernel keeps input order within a warp's chunk; chunks are sorted here)."""
+    import torch
+    from paper_conf_icppw_planob21_b200 import Pipeline
+    from oracle import stages as S
+    cfg = C.c2(n_streams=1, dna=dict(db_len=40_003, q_len=1024, n_planted=12, heavy_tailed=True),
+               wait_time=(0, 0, 0, 0))
+    wl = workload_for(cfg)
+    pl = Pipeline(cfg, wl, flags=0)
+    pl.push(wl.db, wl.db_len)
+    R = wl.db_len - 6 + 1
+    n = R - first_root
+    buf = torch.empty((n + 64, 2), dtype=torch.int32, device="cuda")
+    n0, _ = pl.stage_batch(0, 0, n, first_root, buf.data_ptr(), n + 64)
+    got = buf[:n0].cpu().numpy().astype(np.uint32)
+    pl.close()
+    ctx = S.DnaContext(wl.db, wl.db_len, wl.query, wl.q_len, 6)
+    ref = [p for p in range(first_root, R) if S.s0_seed_lookup(ctx, (p, 0, None))]
+    assert n0 == len(ref)
+    assert sorted(int(a) for a, _ in got) == ref and all(int(b) == 0 for _, b in got)
