@@ -400,7 +400,8 @@ pl_status pl_solve_monolithic(const pl_config* cfg, uint32_t* M_out, double* T_o
  * full occupancy (256-thread CTAs, the query index in smem): S0 rolls k-mers over 16-byte DB
  * loads (first_root a multiple of 64, 4 <= k <= 8; else per item), S1 writes its outputs
  * through smem as contiguous runs, the other stages run the executor's stage bodies.
- * Needs a pushed or bound DB for DNA.  PL_EOVERFLOW: more outputs than cap (the first cap
+ * Needs a pushed or bound DB for DNA; PL_EINVAL if stage 0's roots first_root .. first_root+n-1
+ * reach past the DB's last k-mer.  PL_EOVERFLOW: more outputs than cap (the first cap
  * are written).                                                                        */
 pl_status pl_stage_batch(pl_pipeline* pl, uint32_t stage, const void* in_dev, uint64_t n, uint64_t first_root,
                          void* out_dev, uint64_t cap, uint64_t* n_out, uint64_t* max_vec_cycles);

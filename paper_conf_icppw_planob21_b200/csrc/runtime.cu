@@ -1240,6 +1240,9 @@ pl_status pl_stage_batch(pl_pipeline* pl, uint32_t stage, const void* in_dev, ui
   } else {
     d.total_roots = first_root + n;
   }
+  if (stage == 0 && pl->dna && first_root + n > d.total_roots)
+    return fail(PL_EINVAL, "roots %llu..%llu beyond the DB's %llu roots", (unsigned long long)first_root,
+                (unsigned long long)(first_root + n), (unsigned long long)d.total_roots);
   d.win_cap = 0;
   d.match_count = pl->d_match_count;
   d.summary = nullptr;

@@ -106,3 +106,22 @@ def test_s0_first_root_paths(first_root):
     ref = [p for p in range(first_root, R) if S.s0_seed_lookup(ctx, (p, 0, None))]
     assert n0 == len(ref)
     assert sorted(int(a) for a, _ in got) == ref and all(int(b) == 0 for _, b in got)
+
+
+def test_s0_roots_past_db_end_rejected():
+    """pl_stage_batch refuses stage-0 roots beyond the DB's last k-mer (PL_EINVAL), which would
+    otherwise read k-mers of the zero padding."""
+    import torch
+    from paper_conf_icppw_planob21_b200 import Pipeline
+    from paper_conf_icppw_planob21_b200._pl import PlError
+    cfg = C.c2(n_streams=1, dna=dict(db_len=1 << 14, q_len=1024, n_planted=4), wait_time=(0, 0, 0, 0))
+    wl = workload_for(cfg)
+    pl = Pipeline(cfg, wl, flags=0)
+    pl.push(wl.db, wl.db_len)
+    R = wl.db_len - 6 + 1
+    buf = torch.empty((R + 64, 2), dtype=torch.int32, device="cuda")
+    n_ok, _ = pl.stage_batch(0, 0, R, 0, buf.data_ptr(), R + 64)
+    with pytest.raises(PlError):
+        pl.stage_batch(0, 0, R, 1, buf.data_ptr(), R + 64)
+    pl.close()
+    assert n_ok >= 0
