@@ -95,6 +95,9 @@ __device__ __forceinline__ uint64_t gain_hash(uint64_t seed, uint32_t stage, uin
 #define PL_NAP_HALF 1       // every nap above the spin threshold sleeps half the remaining time (no 256 / 64 ns tiers):
                             // c3 THRESHOLD_SLACK -9 to -11 % warp instructions per root, c4 budgets and rate unchanged or better
 #endif
+#ifndef PL_S3_TAB
+#define PL_S3_TAB 0         // S3 X-drop walks 8 steps per table lookup ([deficit][mismatch byte] transitions in smem)
+#endif
 #ifndef PL_PUB_WAIT
 #define PL_PUB_WAIT 0       // physical clock: a waiting leader sleeps on its input edge's mbarrier (woken by the
                             // producer's publication or the nap's time limit) instead of a plain nap; parity-exact
@@ -140,6 +143,8 @@ struct Dna {
   uint32_t win_mask;
   bool nofast;             // experiment switch (PL_VARIANT & 16): always the checked walk
   const uint8_t* s2tab;    // smem: max(0, max prefix score) of an 8-step walk by mismatch pattern
+  const uint16_t* xtab;    // smem (PL_S3_TAB): 8-step X-drop transitions [deficit][mismatch byte] (xdrop_tab_entry)
+  int xtab_X;              // the X the table was built for (0: no table)
   const uint32_t* qw;      // query words (smem), nqw valid words
   uint32_t nqw;
   const uint16_t* qoff;    // smem
@@ -314,6 +319,92 @@ struct Dna {
         dnx = win[dw & win_mask];
         qnx = *qp;
 #endif
+      }
+    }
+    *br = best;
+    *dr = db_;
+  }
+  // PL_S3_TAB: one 8-step chunk of an X-drop walk (+1 match / -3 mismatch, R-S3) entered with the
+  // running best `def` above the score: bit e of m = mismatch at the chunk's step e + 1.  Entry:
+  // bits 0-3 the best's rise (0..8), 4-7 the chunk step where the new best is first reached,
+  // 8-13 the deficit after the chunk, bit 14 = the walk X-drops inside the chunk (score <= best - X
+  // right after a mismatch; the best at that point is the walk's result).  Exactly extend()'s
+  // arithmetic, 8 steps at a time.
+  static __host__ __device__ __forceinline__ uint16_t xdrop_tab_entry(uint32_t def, uint32_t m, int X) {
+    int s = -(int)def, b = 0, bpos = 0;
+    for (int e = 0; e < 8; ++e) {
+      if ((m >> e) & 1u) {
+        s -= 3;
+        if (s <= b - X) return (uint16_t)(b | (bpos << 4) | (1 << 14));
+      } else {
+        s += 1;
+        if (s > b) { b = s; bpos = e + 1; }
+      }
+    }
+    return (uint16_t)(b | (bpos << 4) | ((b - s) << 8));
+  }
+  // extend2_win with the mismatch loop replaced by two table steps per 16-base word: the word's
+  // mismatch mask is compressed to 16 bits (bit j = step d+1+j), steps past the walk's limit are
+  // marked as mismatches (they never raise the best, and a drop among them ends the walk where
+  // the limit would), and each byte is one lookup.  Needs xtab_X == X (1..63) and in_win.
+  __device__ __forceinline__ void extend2_tab(uint32_t p, uint32_t q, uint32_t ll, uint32_t rl, int* bl,
+                                              int* dl, int* br, int* dr) const {
+    int32_t sd = (int32_t)p - 16, sq = (int32_t)q - 16;
+    uint32_t dw = (uint32_t)(sd >> 4);
+    const uint32_t* qp = qw + (sq >> 4);
+    uint32_t shd = (uint32_t)(sd & 15) * 2u, shq = (uint32_t)(sq & 15) * 2u;
+    uint32_t dc = win[(dw + 1u) & win_mask], qc = qp[1];
+    int step = -1;
+    bool right = false;
+    uint32_t limit = ll, d = 0, def = 0;
+    int best = 0, db_ = 0;
+    for (;;) {
+      bool fin = d >= limit;
+      if (!fin) {
+        const uint32_t dn = win[dw & win_mask], qn = *qp;
+        dw += (uint32_t)step;
+        qp += step;
+        const uint32_t x = right ? (__funnelshift_r(dc, dn, shd) ^ __funnelshift_r(qc, qn, shq))
+                                 : (__funnelshift_r(dn, dc, shd) ^ __funnelshift_r(qn, qc, shq));
+        dc = dn;
+        qc = qn;
+        uint32_t mm = (x | (x >> 1)) & 0x55555555u;   // bit 2e: mismatch at window position e
+        if (!right) mm = __brev(mm) >> 1;             // left: window position 15-e is step d+1+e
+        mm = (mm | (mm >> 1)) & 0x33333333u;
+        mm = (mm | (mm >> 2)) & 0x0f0f0f0fu;
+        mm = (mm | (mm >> 4)) & 0x00ff00ffu;
+        mm = (mm | (mm >> 8)) & 0x0000ffffu;          // bit j: mismatch at step d+1+j
+        const uint32_t n = (limit - d) < 16u ? (limit - d) : 16u;
+        mm |= (0xffffu << n) & 0xffffu;
+        uint32_t t = xtab[(def << 8) | (mm & 0xffu)];
+        if (t & 15u) { best += (int)(t & 15u); db_ = (int)d + (int)((t >> 4) & 15u); }
+        if (t & 0x4000u) fin = true;
+        else {
+          def = (t >> 8) & 63u;
+          t = xtab[(def << 8) | (mm >> 8)];
+          if (t & 15u) { best += (int)(t & 15u); db_ = (int)d + 8 + (int)((t >> 4) & 15u); }
+          if (t & 0x4000u) fin = true;
+          else { def = (t >> 8) & 63u; d += n; }
+        }
+      }
+      if (fin) {
+        if (right) break;
+        *bl = best;
+        *dl = db_;
+        right = true;
+        step = 1;
+        limit = rl;
+        d = 0;
+        def = 0;
+        best = db_ = 0;
+        sd = (int32_t)(p + (uint32_t)k);
+        sq = (int32_t)(q + (uint32_t)k);
+        dw = (uint32_t)(sd >> 4);
+        qp = qw + (sq >> 4);
+        shd = (uint32_t)(sd & 15) * 2u;
+        shq = (uint32_t)(sq & 15) * 2u;
+        dc = win[dw++ & win_mask];
+        qc = *qp++;
       }
     }
     *br = best;
@@ -858,6 +949,16 @@ struct Node {
 };
 
 __host__ __device__ inline uint32_t layout_enforced(const DevParams& p, SmemLayout* L);
+// PL_S3_TAB: the X of the DNA sink's X-drop when its transition table is built (1..63), else 0
+__host__ __device__ inline int xtab_X(const DevParams& p) {
+#if PL_S3_TAB
+  if (p.k > 0 && p.N > 0 && p.st[p.N - 1].kind == PL_UNGAPPED_XDROP && p.st[p.N - 1].ip[1] >= 1 &&
+      p.st[p.N - 1].ip[1] <= 63)
+    return p.st[p.N - 1].ip[1];
+#endif
+  (void)p;
+  return 0;
+}
 
 // logical time units -> ns of %globaltimer (physical clock)
 __device__ __forceinline__ uint64_t units_ns(const Node& nd, int64_t t) {
@@ -969,6 +1070,10 @@ __device__ __forceinline__ LaneOut stage_count_ext(const Node& nd, const Dna& dn
     return o;
   }
   if (dna.in_win(e.x, ll, rl)) {
+#if PL_S3_TAB
+    if (X > 0 && X == dna.xtab_X) dna.extend2_tab(e.x, q, ll, rl, &bl, &dl, &br, &dr);
+    else
+#endif
     dna.extend2_win(e.x, q, ll, rl, X, &bl, &dl, &br, &dr);
   } else {
     bl = dna.extend(e.x, q, -1, ll, X, &dl);
@@ -2180,6 +2285,8 @@ __host__ __device__ inline uint32_t layout_enforced(const DevParams& p, SmemLayo
   off += p.win_cap * 4u;
   L->off_s2 = off;                // S2 table (Dna::s2_best8): 256 bytes
   off += dna ? 256u : 0u;
+  L->off_xt = off;                // S3 transition table (PL_S3_TAB): 256 x X entries of 2 bytes
+  off += (uint32_t)xtab_X(p) * 512u;
   L->total = off;
   return off;
 }
@@ -2218,6 +2325,13 @@ __device__ void cta_setup(Ctx& c, Shared& sh, unsigned char* dsm, const DevParam
   if (s == 0 && tid < 8 && p.summary_next) p.summary_next[tid] = 0ull;   // the next launch's summary slot
   c.dna.nofast = (p.variant & 16u) != 0;
   c.dna.s2tab = dsm + Lo.off_s2;
+  {
+    const int XT = xtab_X(p);
+    c.dna.xtab = (const uint16_t*)(dsm + Lo.off_xt);
+    c.dna.xtab_X = XT;
+    for (uint32_t m = tid; m < 256u * (uint32_t)XT; m += nt)
+      ((uint16_t*)(dsm + Lo.off_xt))[m] = Dna::xdrop_tab_entry(m >> 8, m & 255u, XT);
+  }
   if (p.k > 0)   // S2 table: max(0, max prefix) of the 8-step +1/-3 walk, bit e = mismatch at step e+1
     for (uint32_t m = tid; m < 256u; m += nt) {
       int sc = 0, best = 0;
@@ -2691,7 +2805,7 @@ cudaError_t pl_kernel_attributes(unsigned max_smem) {
 // memory (the whole DB, read-only), so S2 / S3 take the executor's fast in-window walks; only
 // seeds within a walk's reach of the DB ends take the checked ones.  Shared memory holds only
 // the query index, so several CTAs share an SM.
-struct KbLayout { uint32_t qpos, qw, s2, hit, total; };
+struct KbLayout { uint32_t qpos, qw, s2, hit, xt, total; };
 __host__ __device__ inline KbLayout layout_kbench(const DevParams& p) {
   KbLayout L;
   uint32_t off = 0;
@@ -2705,6 +2819,8 @@ __host__ __device__ inline KbLayout layout_kbench(const DevParams& p) {
   off += dna ? 256u : 0u;
   L.hit = off;                                                       // S0: one bit per k-mer (has hits)
   off += dna ? ((((1u << (2 * p.k)) + 31u) / 32u) * 4u + 15u) & ~15u : 0u;
+  L.xt = off;                                                        // S3 transitions (PL_S3_TAB)
+  off += (uint32_t)xtab_X(p) * 512u;
   L.total = off > 16u ? off : 16u;
   return L;
 }
@@ -2809,6 +2925,10 @@ __global__ void __launch_bounds__(KB_THREADS, 4) pl_kbench_kernel(const __grid_c
   dna.qw = (const uint32_t*)(dsm + Lo.qw);
   dna.nqw = (uint32_t)(p.q_len + 15) / 16u;
   dna.s2tab = dsm + Lo.s2;
+  dna.xtab = (const uint16_t*)(dsm + Lo.xt);
+  dna.xtab_X = xtab_X(p);
+  for (uint32_t m = tid; m < 256u * (uint32_t)dna.xtab_X; m += nt)
+    ((uint16_t*)(dsm + Lo.xt))[m] = Dna::xdrop_tab_entry(m >> 8, m & 255u, dna.xtab_X);
   if (p.k > 0) {
     const uint32_t nko = (1u << (2 * p.k)) + 1u, nqp = (uint32_t)(p.q_len - p.k + 1);
     uint16_t* qo = (uint16_t*)dsm;

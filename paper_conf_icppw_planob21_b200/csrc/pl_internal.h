@@ -138,7 +138,7 @@ struct SmemLayout {
   uint32_t off_ent[PL_MAX_STAGES];      // uint2 rings, edge into node i (i >= 1)
   uint32_t off_seg[PL_MAX_STAGES];
   uint32_t off_troot;                   // [N][v] u32: terminal root per lane of the current firing
-  uint32_t off_qoff, off_qpos, off_qw, off_win, off_s2;
+  uint32_t off_qoff, off_qpos, off_qw, off_win, off_s2, off_xt;
   uint32_t total;
 };
 
