@@ -90,6 +90,9 @@ def parse():
     ap.add_argument("--probe-t", type=int, default=None,
                     help="budget probe: every node's budget during the probe (ns; default c4 1000 = all nodes "
                          "overloaded, sharing the SM as in a catch-up, L69's 1/N share; c2 20000)")
+    ap.add_argument("--lat-margin", type=float, default=0.85,
+                    help="rate search across injected stalls: a trial also needs its largest measured latency "
+                         "<= lat_margin x D (near the edge the worst latency is not monotone in tau0)")
     ap.add_argument("--headroom", type=float, default=1.08,
                     help="operating tau0 = headroom x the fastest tau0 miss-free across injected stalls "
                          "(R-STALL: the pipeline must catch up after a ~1.6 ms platform stall within D; the "
@@ -359,7 +362,8 @@ def main():
     tau, w, th, T, st_ok = realtime.find_rate(cfg, wl, db_ptr, stream=stream, log=log, policy=1, over=over,
                                               max_lateness_ns=None, grow=1.5 if c4 else 1.15, tries=16,
                                               flags=PL_FIXED_SERVICE, solve_deadline=D - SG, max_outliers=0,
-                                              inject=inject)
+                                              inject=inject,
+                                              max_latency_ns=int(a.lat_margin * D) if inject else None)
     # the operating point: headroom over the edge the search found on stall-free runs, so that
     # the pipeline catches up after a platform stall within D (R-STALL); confirmed by --confirm
     # runs with zero measured misses whether or not they meet a stall, and zero latency
@@ -592,7 +596,8 @@ def main():
                                            f"outliers on stall-free runs ({tau_edge} ns)")) +
                                           f"; then {a.confirm} confirmation runs without injection: zero misses, and "
                                           f"zero latency outliers in those without a platform stall (tries: {confirm_log})",
-                       "stall_injection_in_rate_search": ({"period_ms": a.inject_period_ms, "len_ms": a.inject_ms}
+                       "stall_injection_in_rate_search": ({"period_ms": a.inject_period_ms, "len_ms": a.inject_ms,
+                                                           "max_latency_frac_of_D": a.lat_margin}
                                                           if inject else None),
                        "tau0_edge_ns": tau_edge, "edge_items_per_s": world * a.streams * 1e9 / tau_edge,
                        "b": list(C.PAPER_B), "budgets_ns": list(budgets), "budget_probe_t_ns": a.probe_t or (1000 if c4 else 20_000),

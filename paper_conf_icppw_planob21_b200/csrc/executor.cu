@@ -96,7 +96,8 @@ __device__ __forceinline__ uint64_t gain_hash(uint64_t seed, uint32_t stage, uin
                             // c3 THRESHOLD_SLACK -9 to -11 % warp instructions per root, c4 budgets and rate unchanged or better
 #endif
 #ifndef PL_S3_TAB
-#define PL_S3_TAB 0         // S3 X-drop walks 8 steps per table lookup ([deficit][mismatch byte] transitions in smem)
+#define PL_S3_TAB 1         // S3 X-drop walks 8 steps per table lookup ([deficit][mismatch byte] transitions in smem):
+                            // K-BENCH S3 2.54 -> 1.27 ms, c4 node-3 longest probe firing 16.4 -> 10.5 us, bit-exact
 #endif
 #ifndef PL_PUB_WAIT
 #define PL_PUB_WAIT 0       // physical clock: a waiting leader sleeps on its input edge's mbarrier (woken by the

@@ -135,7 +135,7 @@ def stalled(st) -> bool:
 
 def find_rate(cfg, wl, db_dev, tries=12, grow=1.15, stream=None, log=None, over=None, policy=0,
               max_lateness_ns=5000, flags=0, solve_deadline=None, max_outliers=None, start=None,
-              stall_retries=2, inject=None):
+              stall_retries=2, inject=None, max_latency_ns=None):
     """Smallest tau0 (ns) at which a physical run (FIXED_WAIT, or THRESHOLD_SLACK with the
     Fig. 1-derived thresholds when policy=1) has zero deadline misses, no queue overflow
     and, unless max_lateness_ns is None, every firing starting within max_lateness_ns of its
@@ -154,6 +154,9 @@ def find_rate(cfg, wl, db_dev, tries=12, grow=1.15, stream=None, log=None, over=
     platform-length stalls (pl_pipeline_inject_stalls), and the criterion becomes zero misses
     ACROSS them -- the pipeline must catch up after each within D (R-STALL); the 5 % outlier
     bound then cannot apply (a stalled item is late by construction) and is not checked.
+    `max_latency_ns`: a run also needs its largest measured latency within this bound (a margin
+    under D: near the edge the worst latency across stalls is not monotone in tau0, and a run that
+    just clears D says little about the next one).  
     Returns (tau0, w, theta, T, stats)."""
     from ._pl import PlError
     scfg = cfg if solve_deadline is None else cfg.replace(deadline=int(solve_deadline))
@@ -172,6 +175,8 @@ def find_rate(cfg, wl, db_dev, tries=12, grow=1.15, stream=None, log=None, over=
                       and st["errors"] == 0)
                 if max_lateness_ns is not None:
                     ok = ok and max(st["max_lateness_ns"]) <= max_lateness_ns
+                if max_latency_ns is not None:
+                    ok = ok and st["max_latency_ns"] <= max_latency_ns
                 if max_outliers is not None and not inject:   # north_star 5 % per-item agreement (R-AGREE)
                     ok = ok and st["latency_outliers"] <= max_outliers
             except PlError:          # device-side overflow reported by drain
