@@ -80,7 +80,10 @@ def parse():
     ap.add_argument("--budget-margin", type=float, default=1.10,
                     help="t_i = margin x longest measured firing + slack (SURVEY 8(d): x1.1)")
     ap.add_argument("--budget-slack", type=int, default=128)
-    ap.add_argument("--refine", type=int, default=2, help="budget refinement rounds at the operating point")
+    ap.add_argument("--refine", type=int, default=None,
+                    help="budget refinement rounds at the operating point (default c2: 2; c4: 0 -- on c4 the "
+                         "refinement runs at the fastest stall-free rate, far below the injected-stall edge, where "
+                         "back-pressure inflates node 2's loop time to twice its firing: profiles/r02_ab/bench_c4_refine0_*.json)")
     ap.add_argument("--confirm", type=int, default=3,
                     help="confirmation runs the operating point must pass (else +10 %% and retry)")
     ap.add_argument("--inject-period-ms", type=float, default=None,
@@ -102,6 +105,8 @@ def parse():
     a = ap.parse_args()
     if a.deadline_ns is None:
         a.deadline_ns = 3_500_000 if a.workload == "c4" else 350_000
+    if a.refine is None:
+        a.refine = 0 if a.workload == "c4" else 2
     if a.inject_period_ms is None:
         a.inject_period_ms = 100.0 if a.workload == "c4" else 0.0
     if a.stall_guard_ns is None:
