@@ -57,7 +57,7 @@ WORKLOADS = {
 }
 # c4 schedule parameters of the last GPU bench (profiles/r02_bench_c4_v1.json), for the reference arm,
 # which must not load the product library: the oracle simulates the same schedule (1 unit = 1 ns)
-REF_C4 = dict(budgets=(8189, 11146, 6324, 17904), tau0=3141, gains=(0.04995, 8.9465, 0.56093))   # profiles/r02_bench_c4_final.json
+REF_C4 = dict(budgets=(8330, 12343, 6113, 12660), tau0=2625, gains=(0.04995, 8.9465, 0.56093))   # profiles/r02_bench_c4_final.json
 
 
 def parse():
@@ -651,11 +651,12 @@ def main():
             # with the monolithic baseline at the same (tau0, D)
             "issue": {k: ncu[k] for k in ("issue_active_pct", "warp_inst_per_launch", "warp_inst_per_root",
                                           "sm_throughput_pct", "util_same_rate", "source") if k in ncu},
-            # the bound that sets the c4 rate: a repeat island turns every seed into u S3 items, which
-            # node 3 serves v per t_3, so tau0 >= u t_3 / v during an island
-            "rate_bound": {"bound": "node-3 island burst (tau0 >= u t_3 / v)" if c4 else "node-0 service (tau0 >= t_0/v)",
+            # the bound that sets the c4 rate: a repeat island turns every seed into u S2 items (and up
+            # to u S3 items), which nodes 2 and 3 serve v per t_i, so tau0 >= u max(t_2, t_3) / v there
+            "rate_bound": {"bound": ("island burst at nodes 2-3 (tau0 >= u max(t_2, t_3) / v: a repeat-island seed "
+                                     "becomes u S2 items and up to u S3 items)") if c4 else "node-0 service (tau0 >= t_0/v)",
                            "achieved": world * a.streams * 1e9 / tau,
-                           "peak": world * a.streams * 1e9 * v / ((u * budgets[3]) if c4 else budgets[0]),
+                           "peak": world * a.streams * 1e9 * v / ((u * max(budgets[2], budgets[3])) if c4 else budgets[0]),
                            "unit": "items/s"},
             "cpu_baseline": cpu,
             # per-stage kernels over the same DB, outside the timed region (north_star: HBM GB/s of each
