@@ -99,6 +99,10 @@ __device__ __forceinline__ uint64_t gain_hash(uint64_t seed, uint32_t stage, uin
 #define PL_S3_TAB 1         // S3 X-drop walks 8 steps per table lookup ([deficit][mismatch byte] transitions in smem):
                             // K-BENCH S3 2.54 -> 1.27 ms, c4 node-3 longest probe firing 16.4 -> 10.5 us, bit-exact
 #endif
+#ifndef PL_S3_TAB2
+#define PL_S3_TAB2 0        // experiment: the left and right table walks advanced together (two chains per lane);
+                            // bit-exact but node 3's longest c4 probe firing 10.6 -> 17.9 us, bench 4.9e7: rejected
+#endif
 #ifndef PL_PUB_WAIT
 #define PL_PUB_WAIT 0       // physical clock: a waiting leader sleeps on its input edge's mbarrier (woken by the
                             // producer's publication or the nap's time limit) instead of a plain nap; parity-exact
@@ -411,6 +415,72 @@ struct Dna {
     *br = best;
     *dr = db_;
   }
+#if PL_S3_TAB2
+  // PL_S3_TAB2 (experiment): extend2_tab with the left and right walks advanced together, one word
+  // of each per iteration -- two independent table chains per lane instead of one after the other
+  struct TWalk {
+    uint32_t dw, shd, shq, dc, qc, limit, d, def;
+    const uint32_t* qp;
+    int best, db_;
+    bool fin;
+  };
+  __device__ __forceinline__ void tw_step(TWalk& w, bool right) const {
+    const uint32_t dn = win[w.dw & win_mask], qn = *w.qp;
+    w.dw += right ? 1u : 0xffffffffu;
+    w.qp += right ? 1 : -1;
+    const uint32_t x = right ? (__funnelshift_r(w.dc, dn, w.shd) ^ __funnelshift_r(w.qc, qn, w.shq))
+                             : (__funnelshift_r(dn, w.dc, w.shd) ^ __funnelshift_r(qn, w.qc, w.shq));
+    w.dc = dn;
+    w.qc = qn;
+    uint32_t mm = (x | (x >> 1)) & 0x55555555u;
+    if (!right) mm = __brev(mm) >> 1;
+    mm = (mm | (mm >> 1)) & 0x33333333u;
+    mm = (mm | (mm >> 2)) & 0x0f0f0f0fu;
+    mm = (mm | (mm >> 4)) & 0x00ff00ffu;
+    mm = (mm | (mm >> 8)) & 0x0000ffffu;
+    const uint32_t n = (w.limit - w.d) < 16u ? (w.limit - w.d) : 16u;
+    mm |= (0xffffu << n) & 0xffffu;
+    uint32_t t = xtab[(w.def << 8) | (mm & 0xffu)];
+    if (t & 15u) { w.best += (int)(t & 15u); w.db_ = (int)w.d + (int)((t >> 4) & 15u); }
+    if (t & 0x4000u) { w.fin = true; return; }
+    w.def = (t >> 8) & 63u;
+    t = xtab[(w.def << 8) | (mm >> 8)];
+    if (t & 15u) { w.best += (int)(t & 15u); w.db_ = (int)w.d + 8 + (int)((t >> 4) & 15u); }
+    if (t & 0x4000u) { w.fin = true; return; }
+    w.def = (t >> 8) & 63u;
+    w.d += n;
+    if (w.d >= w.limit) w.fin = true;
+  }
+  __device__ __forceinline__ void extend2_tab2(uint32_t p, uint32_t q, uint32_t ll, uint32_t rl, int* bl,
+                                               int* dl, int* br, int* dr) const {
+    TWalk L, R;
+    {
+      const int32_t sd = (int32_t)p - 16, sq = (int32_t)q - 16;
+      L.dw = (uint32_t)(sd >> 4);
+      L.qp = qw + (sq >> 4);
+      L.shd = (uint32_t)(sd & 15) * 2u;
+      L.shq = (uint32_t)(sq & 15) * 2u;
+      L.dc = win[(L.dw + 1u) & win_mask];
+      L.qc = L.qp[1];
+      L.limit = ll; L.d = 0; L.def = 0; L.best = 0; L.db_ = 0; L.fin = ll == 0;
+    }
+    {
+      const int32_t sd = (int32_t)(p + (uint32_t)k), sq = (int32_t)(q + (uint32_t)k);
+      R.dw = (uint32_t)(sd >> 4);
+      R.qp = qw + (sq >> 4);
+      R.shd = (uint32_t)(sd & 15) * 2u;
+      R.shq = (uint32_t)(sq & 15) * 2u;
+      R.dc = win[R.dw++ & win_mask];
+      R.qc = *R.qp++;
+      R.limit = rl; R.d = 0; R.def = 0; R.best = 0; R.db_ = 0; R.fin = rl == 0;
+    }
+    while (!(L.fin && R.fin)) {
+      if (!L.fin) tw_step(L, false);
+      if (!R.fin) tw_step(R, true);
+    }
+    *bl = L.best; *dl = L.db_; *br = R.best; *dr = R.db_;
+  }
+#endif
   // 16 bases starting at s (s >= win_lo * 16, in the window) / at query position s >= -16
   __device__ __forceinline__ uint32_t db16w(int32_t s) const {
     const uint32_t w = (uint32_t)(s >> 4);
@@ -1072,8 +1142,13 @@ __device__ __forceinline__ LaneOut stage_count_ext(const Node& nd, const Dna& dn
   }
   if (dna.in_win(e.x, ll, rl)) {
 #if PL_S3_TAB
+#if PL_S3_TAB2
+    if (X > 0 && X == dna.xtab_X) dna.extend2_tab2(e.x, q, ll, rl, &bl, &dl, &br, &dr);
+    else
+#else
     if (X > 0 && X == dna.xtab_X) dna.extend2_tab(e.x, q, ll, rl, &bl, &dl, &br, &dr);
     else
+#endif
 #endif
     dna.extend2_win(e.x, q, ll, rl, X, &bl, &dl, &br, &dr);
   } else {
